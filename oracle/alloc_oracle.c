@@ -1,0 +1,521 @@
+/*
+ * oracle/alloc_oracle.c -- O2: the SEQUENTIAL Gallatin allocator (CPU).
+ *
+ * TEST INFRASTRUCTURE ONLY.  Only tests/, __graft_entry__.smoke() and
+ * bench.py's cpu_baseline / --impl reference legs may load this code.  It
+ * shares no code, header, table or constant with the CUDA path and never
+ * calls it.  Its trees are O1 textbook vEB trees (veb_oracle.c).
+ *
+ * It implements, one request at a time and in the paper's order, the policy
+ * of PAPER.md S4-S5 (P = /root/reference/PAPER.md line):
+ *   - heap of 16 MB segments; segment tree, bit=1 <=> free;
+ *     segments for blocks taken from the FRONT by successor(0);
+ *   - one block tree per block size; a segment formatted for tree t
+ *     holds nb(t) = 256 >> t blocks (256 blocks at 16 B slices,
+ *     128 at 32 B); blocks leave and return through a constant-size
+ *     per-segment ring queue, i.e. FIFO; the segment leaves its block
+ *     tree when its last block is handed out and rejoins when a block comes
+ *     back (reading A-16: on avail 0 -> 1); when every block is back
+ *     the segment returns to the segment tree;
+ *   - slices: a block holds 4096 slices of 1/4096 of the block, slice
+ *     sizes 16 B..4096 B, tree id = log2(size) - log2(16);
+ *     slices are handed out in order by a counter (Alg.3 P:212-
+ *     213: valid = idx < 4096), address offset(blockId*4096 + idx);
+ *   - block buffer: NSLOT(c) = max(slot_min, slot_base >> c) live blocks per
+ *     class, slot chosen by the request's key mod NSLOT(c) (reading
+ *     A-6); an exhausted block is replaced by the request that finds it
+ *     exhausted (Alg.3, reading A-7); optional prefetch: the request
+ *     that takes index theta fetches the next block early (not in the paper;
+ *     theta = 0 is the paper's behaviour);
+ *   - requests in (4 KB, 16 MB): one whole block of tree max(0, ceil(log2
+ *     size) - 16) whose free counter is preset to 4095 so that Alg.4's rule
+ *      returns it on its one free (reading A-2);
+ *   - requests >= 16 MB: k = ceil(size / 16 MB) contiguous segments from the
+ *     END of the segment tree, first fit via predecessor search (P:111-113,
+ *     P:138, reading A-17: the highest start), tree id = 9 + k;
+ *   - free (Alg.4): segment = offset / 16 MB (reading A-10);
+ *     tree id < 9: block = (offset in segment) >> log2(block size) (P:239,
+ *     reading A-11), free counter += 1, the free that completes 4096 returns
+ *     the block (reading A-14); otherwise the k segments are
+ *     re-inserted into the segment tree.
+ *   - drain (reading A-15/SURVEY A15): retire every block-buffer slot, the
+ *     unissued remainder of its block counted as freed.
+ *
+ * Canonical metadata image: see include/gallatin.h, "Snapshot image"; this
+ * file writes the same documented layout from its own state.
+ */
+#include <stdint.h>
+#include <stdlib.h>
+#include <string.h>
+
+/* ---- O1 (veb_oracle.c) ---- */
+typedef struct oracle_veb oracle_veb;
+oracle_veb *oracle_veb_create(unsigned k);
+void oracle_veb_destroy(oracle_veb *h);
+int oracle_veb_member(const oracle_veb *h, uint64_t x);
+int oracle_veb_insert(oracle_veb *h, uint64_t x);
+int oracle_veb_delete(oracle_veb *h, uint64_t x);
+uint64_t oracle_veb_successor(const oracle_veb *h, uint64_t x);
+uint64_t oracle_veb_predecessor(const oracle_veb *h, uint64_t x);
+
+#define NONE64 UINT64_MAX
+/* The paper's constants, restated (not shared with the CUDA path). */
+#define SEGMENT_BYTES (16ULL << 20)   /* P:134 "16MB regions"              */
+#define SLICES_PER_BLOCK 4096ULL
+#define MIN_SLICE 16ULL               /* P:184 "16 B"                     */
+#define MAX_SLICE 4096ULL             /* P:184 "4096 B"                   */
+#define NUM_BLOCK_TREES 9u            /* 16 B..4 KB slices -> 64 KB..16 MB blocks (A-1) */
+#define MAX_BLOCKS_PER_SEGMENT 256u
+#define TREE_FREE 0xFFFFFFFFu         /* segment in the segment tree       */
+#define TREE_CONT 0xFFFFFFFEu         /* non-first segment of a large alloc */
+#define GID_NONE 0xFFFFFFFFu
+#define IMAGE_MAGIC 0x47414C4C494D4731ULL
+
+static uint64_t ceil_log2(uint64_t x) { uint64_t r = 0; while ((1ULL << r) < x) r++; return r; }
+static uint32_t nb_of(uint32_t t) { return MAX_BLOCKS_PER_SEGMENT >> t; }
+static uint64_t block_bytes(uint32_t t) { return SEGMENT_BYTES / nb_of(t); }
+
+typedef struct { uint16_t e[256]; uint32_t head, count; } ring_t;   /* FIFO */
+typedef struct { uint64_t key, val; } kv_t;
+
+typedef struct o2 {
+    uint64_t nseg;
+    unsigned slot_base, slot_min, theta;
+    unsigned nslot[NUM_BLOCK_TREES], slot_off[NUM_BLOCK_TREES], nslot_total;
+    uint32_t *tree;               /* memoryTable.ids           */
+    int32_t *avail;               /* blocks currently in the ring       */
+    ring_t *ring;
+    uint32_t *freecnt;            /* per block free counter     */
+    oracle_veb *segfree;          /* segment tree               */
+    oracle_veb *btree[NUM_BLOCK_TREES];  /* block trees         */
+    uint64_t *slot;               /* (cnt << 32) | gid                  */
+    uint32_t *next;               /* prefetched block or GID_NONE       */
+    uint64_t err;                 /* out-of-heap / non-allocated segment frees */
+    /* oracle-only bookkeeping for the invariant checks */
+    kv_t *live; uint64_t live_cap, live_n;
+    uint64_t usable_live;
+    uint64_t violations;          /* bit mask, see o2_violations()      */
+} o2_t;
+
+enum { V_FRONT_FIRST = 1, V_BACK_FIRST = 2, V_BAD_FREE = 4, V_OVERLAP = 8,
+       V_ALIGN = 16, V_HEAP = 32, V_ACCOUNT = 64, V_TREES = 128, V_RING = 256 };
+
+/* ------------------------------------------------ live-allocation map --- */
+static uint64_t mix(uint64_t x) { x ^= x >> 33; x *= 0xff51afd7ed558ccdULL; x ^= x >> 33; return x; }
+static void live_grow(o2_t *a);
+static void live_put(o2_t *a, uint64_t k, uint64_t v) {
+    if (2 * (a->live_n + 1) > a->live_cap) live_grow(a);
+    uint64_t m = a->live_cap - 1, i = mix(k) & m;
+    while (a->live[i].key != NONE64) i = (i + 1) & m;
+    a->live[i].key = k; a->live[i].val = v; a->live_n++;
+}
+static void live_grow(o2_t *a) {
+    kv_t *old = a->live; uint64_t oc = a->live_cap;
+    a->live_cap = oc ? oc * 2 : 1024;
+    a->live = (kv_t *)malloc(a->live_cap * sizeof(kv_t));
+    for (uint64_t i = 0; i < a->live_cap; i++) a->live[i].key = NONE64;
+    a->live_n = 0;
+    for (uint64_t i = 0; i < oc; i++) if (old[i].key != NONE64) live_put(a, old[i].key, old[i].val);
+    free(old);
+}
+static int live_take(o2_t *a, uint64_t k, uint64_t *v) {
+    if (!a->live_cap) return 0;
+    uint64_t m = a->live_cap - 1, i = mix(k) & m;
+    while (a->live[i].key != NONE64) {
+        if (a->live[i].key == k) {
+            *v = a->live[i].val;
+            /* backward-shift deletion */
+            uint64_t j = i;
+            for (;;) {
+                j = (j + 1) & m;
+                if (a->live[j].key == NONE64) break;
+                uint64_t h = mix(a->live[j].key) & m;
+                if ((j > i && (h <= i || h > j)) || (j < i && (h <= i && h > j))) {
+                    a->live[i] = a->live[j]; i = j;
+                }
+            }
+            a->live[i].key = NONE64; a->live_n--;
+            return 1;
+        }
+        i = (i + 1) & m;
+    }
+    return 0;
+}
+
+/* ---------------------------------------------------------- lifecycle --- */
+o2_t *o2_create(uint64_t nseg, unsigned slot_base, unsigned slot_min, unsigned theta) {
+    if (nseg < 1 || nseg > (1ULL << 22) || theta >= SLICES_PER_BLOCK || slot_base < 1) return NULL;
+    o2_t *a = (o2_t *)calloc(1, sizeof(o2_t));
+    a->nseg = nseg; a->slot_base = slot_base; a->slot_min = slot_min; a->theta = theta;
+    unsigned off = 0;
+    for (unsigned c = 0; c < NUM_BLOCK_TREES; c++) {
+        unsigned n = slot_base >> c;                  /* halving per class */
+        if (n < slot_min) n = slot_min;               /* "capped at four"  */
+        if (n < 1) n = 1;
+        a->nslot[c] = n; a->slot_off[c] = off; off += n;
+    }
+    a->nslot_total = off;
+    a->tree = (uint32_t *)malloc(nseg * sizeof(uint32_t));
+    a->avail = (int32_t *)calloc(nseg, sizeof(int32_t));
+    a->ring = (ring_t *)calloc(nseg, sizeof(ring_t));
+    a->freecnt = (uint32_t *)calloc(nseg * MAX_BLOCKS_PER_SEGMENT, sizeof(uint32_t));
+    unsigned k = (unsigned)ceil_log2(nseg); if (k < 1) k = 1;
+    a->segfree = oracle_veb_create(k);
+    for (unsigned t = 0; t < NUM_BLOCK_TREES; t++) a->btree[t] = oracle_veb_create(k);
+    for (uint64_t s = 0; s < nseg; s++) { a->tree[s] = TREE_FREE; oracle_veb_insert(a->segfree, s); }
+    a->slot = (uint64_t *)malloc(a->nslot_total * sizeof(uint64_t));
+    a->next = (uint32_t *)malloc(a->nslot_total * sizeof(uint32_t));
+    for (unsigned i = 0; i < a->nslot_total; i++) {
+        a->slot[i] = (SLICES_PER_BLOCK << 32) | GID_NONE;   /* empty: exhausted, no block */
+        a->next[i] = GID_NONE;
+    }
+    return a;
+}
+
+void o2_destroy(o2_t *a) {
+    if (!a) return;
+    free(a->tree); free(a->avail); free(a->ring); free(a->freecnt);
+    oracle_veb_destroy(a->segfree);
+    for (unsigned t = 0; t < NUM_BLOCK_TREES; t++) oracle_veb_destroy(a->btree[t]);
+    free(a->slot); free(a->next); free(a->live);
+    free(a);
+}
+
+unsigned o2_nslot(const o2_t *a, unsigned c) { return c < NUM_BLOCK_TREES ? a->nslot[c] : 0; }
+uint64_t o2_errors(const o2_t *a) { return a->err; }
+uint64_t o2_violations(const o2_t *a) { return a->violations; }
+uint64_t o2_live_count(const o2_t *a) { return a->live_n; }
+uint64_t o2_usable_live(const o2_t *a) { return a->usable_live; }
+
+/* --------------------------------------------- Alg.1 getSegment (front) --- */
+/* successor(0) on the segment tree, claim it, format it for tree t, hand it
+ * to block tree t. */
+static int get_segment(o2_t *a, uint32_t t) {
+    uint64_t s = oracle_veb_successor(a->segfree, 0);
+    if (s == NONE64 || s >= a->nseg) return 0;            /* "All segments in use" */
+    /* front-first invariant: every segment below s is in use */
+    for (uint64_t i = 0; i < s; i++) if (a->tree[i] == TREE_FREE) a->violations |= V_FRONT_FIRST;
+    oracle_veb_delete(a->segfree, s);                      /* claimIndex          */
+    uint32_t nb = nb_of(t);
+    a->tree[s] = t;                                         /* initSegment         */
+    a->avail[s] = (int32_t)nb;
+    ring_t *r = &a->ring[s];
+    r->head = 0; r->count = nb;
+    for (uint32_t j = 0; j < 256; j++) r->e[j] = j < nb ? (uint16_t)j : 0xFFFF;
+    oracle_veb_insert(a->btree[t], s);                     /* "broadcast availability" */
+    return 1;
+}
+
+/* --------------------------------------------------- Alg.2 getBlock --- */
+static uint32_t get_block(o2_t *a, uint32_t t) {
+    uint64_t s = oracle_veb_successor(a->btree[t], 0);     /* findSegment        */
+    if (s == NONE64) {
+        if (!get_segment(a, t)) return GID_NONE;           /* "No allocations left" */
+        s = oracle_veb_successor(a->btree[t], 0);
+    }
+    ring_t *r = &a->ring[s];
+    uint32_t j = r->e[r->head];                            /* ring dequeue */
+    r->e[r->head] = 0xFFFF;
+    r->head = (r->head + 1) & 255; r->count--;
+    a->avail[s]--;
+    if (a->avail[s] == 0) oracle_veb_delete(a->btree[t], s);  /* no over-subscription */
+    return (uint32_t)(s * MAX_BLOCKS_PER_SEGMENT + j);
+}
+
+/* ------------------------------------------ block / segment return --- */
+static void return_block(o2_t *a, uint64_t s, uint32_t j, uint32_t t) {
+    ring_t *r = &a->ring[s];
+    r->e[(r->head + r->count) & 255] = (uint16_t)j;        /* ring enqueue       */
+    r->count++;
+    a->avail[s]++;
+    if ((uint32_t)a->avail[s] == nb_of(t)) {               /* every block back  */
+        a->tree[s] = TREE_FREE; a->avail[s] = 0;
+        r->head = 0; r->count = 0;
+        for (int i = 0; i < 256; i++) r->e[i] = 0xFFFF;
+        oracle_veb_delete(a->btree[t], s);
+        oracle_veb_insert(a->segfree, s);                   /* back to segment tree */
+    } else if (a->avail[s] == 1) {
+        oracle_veb_insert(a->btree[t], s);                  /* re-added (A-16)    */
+    }
+}
+
+static void block_freed(o2_t *a, uint32_t gid, uint32_t count) {
+    a->freecnt[gid] += count;
+    if (a->freecnt[gid] == SLICES_PER_BLOCK) {              /* P:250 (== 4095 before) */
+        a->freecnt[gid] = 0;
+        uint64_t s = gid / MAX_BLOCKS_PER_SEGMENT;
+        return_block(a, s, gid % MAX_BLOCKS_PER_SEGMENT, a->tree[s]);
+    }
+}
+
+/* ------------------------------------------ claimMultiple (back) --- */
+/* Highest start i with [i, i+k) all free: walk down with predecessor (P:112,
+ * P:138, reading A-17). */
+static uint64_t claim_multiple(o2_t *a, uint64_t k) {
+    if (k > a->nseg) return NONE64;
+    uint64_t x = a->nseg - 1;
+    for (;;) {
+        uint64_t y = oracle_veb_predecessor(a->segfree, x);
+        if (y == NONE64) return NONE64;
+        uint64_t run = 1;
+        while (run < k && y >= run && oracle_veb_member(a->segfree, y - run)) run++;
+        if (run >= k) {
+            uint64_t i = y - k + 1;
+            /* back-first invariant: no free window starts above i */
+            for (uint64_t j = i + 1; j + k <= a->nseg; j++) {
+                uint64_t m = 0;
+                while (m < k && a->tree[j + m] == TREE_FREE) m++;
+                if (m == k) a->violations |= V_BACK_FIRST;
+            }
+            for (uint64_t m = 0; m < k; m++) oracle_veb_delete(a->segfree, i + m);
+            a->tree[i] = NUM_BLOCK_TREES + (uint32_t)k;
+            for (uint64_t m = 1; m < k; m++) a->tree[i + m] = TREE_CONT;   /* A-18 */
+            return i;
+        }
+        if (y < run + 1) return NONE64;
+        x = y - run - 1;  /* y - run is in use; continue below it */
+        if (x == NONE64) return NONE64;
+    }
+}
+
+/* ------------------------------------------------------------ malloc --- */
+static uint64_t slice_addr(uint32_t gid, uint32_t c, uint64_t idx) {
+    uint64_t s = gid / MAX_BLOCKS_PER_SEGMENT, j = gid % MAX_BLOCKS_PER_SEGMENT;
+    uint64_t slice = MIN_SLICE << c;
+    /* offset(blockId*4096 + idx), blockId in units of this class's block */
+    return s * SEGMENT_BYTES + (j * SLICES_PER_BLOCK + idx) * slice;
+}
+
+static uint64_t malloc_slice(o2_t *a, uint32_t c, uint64_t key) {
+    unsigned i = a->slot_off[c] + (unsigned)(key % a->nslot[c]);
+    for (;;) {
+        uint64_t cnt = a->slot[i] >> 32;
+        uint32_t gid = (uint32_t)a->slot[i];
+        if (cnt < SLICES_PER_BLOCK) {                       /* valid = idx < 4096 */
+            a->slot[i] = ((cnt + 1) << 32) | gid;
+            uint64_t off = slice_addr(gid, c, cnt);
+            if (a->theta && cnt == a->theta && a->next[i] == GID_NONE)
+                a->next[i] = get_block(a, c);               /* prefetch (ours) */
+            return off;
+        }
+        /* exhausted: this request replaces the block (Alg.3) */
+        uint32_t nbk = a->next[i];
+        a->next[i] = GID_NONE;
+        if (nbk == GID_NONE) nbk = get_block(a, c);
+        if (nbk == GID_NONE) {
+            a->slot[i] = (SLICES_PER_BLOCK << 32) | GID_NONE;
+            return NONE64;                                   /* nullptr */
+        }
+        a->slot[i] = (uint64_t)nbk;                          /* (cnt 0, gid)     */
+    }
+}
+
+static uint64_t class_usable(uint64_t size, uint32_t *kind, uint32_t *cls) {
+    if (size <= MAX_SLICE) {
+        uint64_t c = ceil_log2(size); c = c < 4 ? 0 : c - 4;
+        *kind = 0; *cls = (uint32_t)c; return MIN_SLICE << c;
+    }
+    if (size < SEGMENT_BYTES) {
+        uint64_t t = ceil_log2(size); t = t < 16 ? 0 : t - 16;
+        *kind = 1; *cls = (uint32_t)t; return block_bytes((uint32_t)t);
+    }
+    uint64_t k = (size + SEGMENT_BYTES - 1) / SEGMENT_BYTES;
+    *kind = 2; *cls = (uint32_t)k; return k * SEGMENT_BYTES;
+}
+
+/* Usable bytes a request of `size` receives (A-1..A-4); 0 for size 0. */
+uint64_t o2_usable_size(uint64_t size) {
+    if (size == 0) return 0;
+    uint32_t kind, cls;
+    return class_usable(size, &kind, &cls);
+}
+
+uint64_t o2_malloc(o2_t *a, uint64_t size, uint64_t key) {
+    if (size == 0) return NONE64;                            /* reading A-4 */
+    uint32_t kind, cls;
+    uint64_t usable = class_usable(size, &kind, &cls);
+    uint64_t off;
+    if (kind == 0) {
+        off = malloc_slice(a, cls, key);
+    } else if (kind == 1) {
+        uint32_t gid = get_block(a, cls);
+        if (gid == GID_NONE) return NONE64;
+        a->freecnt[gid] = SLICES_PER_BLOCK - 1;              /* one free returns it (A-2) */
+        off = (uint64_t)(gid / MAX_BLOCKS_PER_SEGMENT) * SEGMENT_BYTES +
+              (uint64_t)(gid % MAX_BLOCKS_PER_SEGMENT) * block_bytes(cls);
+    } else {
+        uint64_t i = claim_multiple(a, cls);
+        if (i == NONE64) return NONE64;
+        off = i * SEGMENT_BYTES;
+    }
+    if (off == NONE64) return NONE64;
+    /* invariants on the new allocation */
+    if (off + usable > a->nseg * SEGMENT_BYTES) a->violations |= V_HEAP;
+    uint64_t align = usable < SEGMENT_BYTES ? usable : SEGMENT_BYTES;
+    if (off % align) a->violations |= V_ALIGN;
+    live_put(a, off, usable);
+    a->usable_live += usable;
+    return off;
+}
+
+/* ------------------------------------------------------- Alg.4 free --- */
+void o2_free(o2_t *a, uint64_t off) {
+    if (off == NONE64) return;                               /* free(NULL) */
+    if (off >= a->nseg * SEGMENT_BYTES) { a->err++; return; }
+    uint64_t usable;
+    if (live_take(a, off, &usable)) a->usable_live -= usable;
+    else a->violations |= V_BAD_FREE;
+    uint64_t s = off / SEGMENT_BYTES;
+    uint32_t t = a->tree[s];
+    if (t < NUM_BLOCK_TREES) {
+        uint32_t j = (uint32_t)((off % SEGMENT_BYTES) / block_bytes(t));
+        block_freed(a, (uint32_t)(s * MAX_BLOCKS_PER_SEGMENT + j), 1);
+    } else if (t != TREE_FREE && t != TREE_CONT) {
+        uint64_t k = t - NUM_BLOCK_TREES;
+        for (uint64_t m = 0; m < k; m++) {
+            a->tree[s + m] = TREE_FREE; a->avail[s + m] = 0;
+            oracle_veb_insert(a->segfree, s + m);
+        }
+    } else {
+        a->err++;
+    }
+}
+
+/* Retire every block-buffer slot in class-major, slot-ascending order: the
+ * unissued remainder of the current block is counted as freed; a prefetched
+ * block is returned whole. */
+void o2_drain(o2_t *a) {
+    for (unsigned i = 0; i < a->nslot_total; i++) {
+        uint64_t cnt = a->slot[i] >> 32;
+        uint32_t gid = (uint32_t)a->slot[i];
+        a->slot[i] = (SLICES_PER_BLOCK << 32) | GID_NONE;
+        if (gid != GID_NONE && cnt < SLICES_PER_BLOCK)
+            block_freed(a, gid, (uint32_t)(SLICES_PER_BLOCK - cnt));
+        uint32_t nx = a->next[i];
+        a->next[i] = GID_NONE;
+        if (nx != GID_NONE) block_freed(a, nx, (uint32_t)SLICES_PER_BLOCK);
+    }
+}
+
+/* Replay: kinds[i] 0 = malloc(args[i]) with slot key keys[i], out[i] = offset
+ * (UINT64_MAX = NULL); 1 = free(out[args[i]]); 2 = drain. */
+void o2_replay(o2_t *a, const uint8_t *kinds, const uint64_t *args, const uint64_t *keys,
+               uint64_t n, uint64_t *out) {
+    for (uint64_t i = 0; i < n; i++) {
+        if (kinds[i] == 0) out[i] = o2_malloc(a, args[i], keys[i]);
+        else if (kinds[i] == 1) { o2_free(a, out[args[i]]); out[i] = 0; }
+        else { o2_drain(a); out[i] = 0; }
+    }
+}
+
+/* Bulk helpers for timing the oracle on a workload (one thread, in order):
+ * malloc every size (key = i / keydiv, i.e. the request's warp), then free
+ * every returned offset in the same order. */
+void o2_malloc_batch(o2_t *a, const uint64_t *sizes, uint64_t n, uint64_t keydiv, uint64_t *out) {
+    for (uint64_t i = 0; i < n; i++) out[i] = o2_malloc(a, sizes[i], keydiv ? i / keydiv : 0);
+}
+void o2_free_batch(o2_t *a, const uint64_t *offs, uint64_t n) {
+    for (uint64_t i = 0; i < n; i++) o2_free(a, offs[i]);
+}
+
+/* -------------------------------------------------- invariant check --- */
+static int cmp_kv(const void *x, const void *y) {
+    const kv_t *p = (const kv_t *)x, *q = (const kv_t *)y;
+    return p->key < q->key ? -1 : p->key > q->key;
+}
+
+/* Full structural check; returns the accumulated violation mask. */
+uint64_t o2_check(o2_t *a) {
+    /* live allocations never overlap (sort and scan) */
+    kv_t *v = (kv_t *)malloc((a->live_n + 1) * sizeof(kv_t));
+    uint64_t n = 0, sum = 0;
+    for (uint64_t i = 0; i < a->live_cap; i++) if (a->live[i].key != NONE64) v[n++] = a->live[i];
+    qsort(v, n, sizeof(kv_t), cmp_kv);
+    for (uint64_t i = 0; i < n; i++) {
+        sum += v[i].val;
+        if (i + 1 < n && v[i].key + v[i].val > v[i + 1].key) a->violations |= V_OVERLAP;
+    }
+    free(v);
+    if (sum != a->usable_live) a->violations |= V_ACCOUNT;
+    /* trees agree with the memory table */
+    for (uint64_t s = 0; s < a->nseg; s++) {
+        uint32_t t = a->tree[s];
+        int fr = oracle_veb_member(a->segfree, s);
+        if (fr != (t == TREE_FREE)) a->violations |= V_TREES;
+        for (uint32_t b = 0; b < NUM_BLOCK_TREES; b++) {
+            int want = (t == b) && a->avail[s] > 0;
+            if (oracle_veb_member(a->btree[b], s) != want) a->violations |= V_TREES;
+        }
+        if (t < NUM_BLOCK_TREES) {
+            ring_t *r = &a->ring[s];
+            if (r->count != (uint32_t)a->avail[s] || a->avail[s] < 0 || (uint32_t)a->avail[s] > nb_of(t))
+                a->violations |= V_RING;
+            uint8_t seen[256] = {0};
+            for (uint32_t q = 0; q < r->count; q++) {
+                uint16_t j = r->e[(r->head + q) & 255];
+                if (j >= nb_of(t) || seen[j]++) a->violations |= V_RING;
+            }
+        } else if (a->avail[s] != 0) {
+            a->violations |= V_RING;
+        }
+    }
+    return a->violations;
+}
+
+/* ------------------------------------------------------------- image --- */
+static uint64_t tree_words(uint64_t nbits, uint64_t *wpl, unsigned *levels) {
+    uint64_t w = (nbits + 63) / 64, total = 0;
+    unsigned L = 0;
+    for (;;) { wpl[L++] = w; total += w; if (w == 1) break; w = (w + 63) / 64; }
+    *levels = L;
+    return total;
+}
+
+static void tree_image(const oracle_veb *t, uint64_t nbits, uint64_t *out) {
+    uint64_t wpl[16]; unsigned L;
+    uint64_t total = tree_words(nbits, wpl, &L);
+    memset(out, 0, total * sizeof(uint64_t));
+    for (uint64_t x = oracle_veb_successor(t, 0); x != NONE64 && x < nbits;
+         x = oracle_veb_successor(t, x + 1))
+        out[x >> 6] |= 1ULL << (x & 63);
+    uint64_t bp = 0, b = wpl[0];
+    for (unsigned l = 1; l < L; l++) {
+        for (uint64_t c = 0; c < wpl[l - 1]; c++) if (out[bp + c]) out[b + (c >> 6)] |= 1ULL << (c & 63);
+        bp = b; b += wpl[l];
+    }
+}
+
+uint64_t o2_image_words(const o2_t *a) {
+    uint64_t wpl[16]; unsigned L;
+    uint64_t W = tree_words(a->nseg, wpl, &L);
+    return 8 + 10 * W + a->nseg * (1 + 65 + 128) + 2ULL * a->nslot_total;
+}
+
+/* Canonical image; layout documented in include/gallatin.h. */
+uint64_t o2_image(const o2_t *a, uint64_t *out, uint64_t cap) {
+    uint64_t need = o2_image_words(a);
+    if (cap < need) return 0;
+    uint64_t wpl[16]; unsigned L;
+    uint64_t W = tree_words(a->nseg, wpl, &L);
+    uint64_t *p = out;
+    p[0] = IMAGE_MAGIC; p[1] = a->nseg; p[2] = L; p[3] = W; p[4] = a->nslot_total;
+    p[5] = a->err; p[6] = 0; p[7] = 0;
+    p += 8;
+    tree_image(a->segfree, a->nseg, p); p += W;
+    for (unsigned t = 0; t < NUM_BLOCK_TREES; t++) { tree_image(a->btree[t], a->nseg, p); p += W; }
+    for (uint64_t s = 0; s < a->nseg; s++) *p++ = ((uint64_t)a->tree[s] << 32) | (uint32_t)a->avail[s];
+    for (uint64_t s = 0; s < a->nseg; s++) {
+        const ring_t *r = &a->ring[s];
+        *p++ = r->count;
+        uint16_t e[256];
+        for (uint32_t q = 0; q < 256; q++) e[q] = q < r->count ? r->e[(r->head + q) & 255] : 0xFFFF;
+        for (uint32_t q = 0; q < 64; q++)
+            *p++ = (uint64_t)e[4 * q] | ((uint64_t)e[4 * q + 1] << 16) |
+                   ((uint64_t)e[4 * q + 2] << 32) | ((uint64_t)e[4 * q + 3] << 48);
+    }
+    for (uint64_t g = 0; g < a->nseg * MAX_BLOCKS_PER_SEGMENT; g += 2)
+        *p++ = (uint64_t)a->freecnt[g] | ((uint64_t)a->freecnt[g + 1] << 32);
+    for (unsigned i = 0; i < a->nslot_total; i++) *p++ = a->slot[i];
+    for (unsigned i = 0; i < a->nslot_total; i++) *p++ = a->next[i];
+    return need;
+}
