@@ -1,0 +1,201 @@
+/*
+ * gallatin.h -- C-ABI of libgallatin.so, the B200 (sm_100a) Gallatin hot path.
+ *
+ * Source of the operations: "Gallatin: A General-Purpose GPU Memory Manager",
+ * McCoy & Pandey, PPoPP'24 (PAPER.md; P:n = line n).  The paper gives "a
+ * standard malloc/free interface" over one cudaMalloc'd heap,
+ * excluded-from-timing construction, a reset between runs,
+ * nullptr on exhaustion and a concurrent vEB tree with
+ * insert / delete / successor / predecessor / query.
+ *
+ * Conventions (every entry point):
+ *   - Return value: GALLATIN_OK (0) or a negative GALLATIN_ERR_* code.  Device
+ *     pointer arguments are not dereferenced on the host; bad device pointers
+ *     surface as GALLATIN_ERR_CUDA from a later call (asynchronous errors).
+ *   - `stream` is a cudaStream_t passed as void* (NULL = legacy default
+ *     stream).  Bulk calls are asynchronous on it and return after the launch.
+ *   - "d_" arrays are caller-owned DEVICE memory, "h_" arrays caller-owned
+ *     HOST memory (pinned or pageable).  Sizes are element counts.
+ *   - The library owns the heap and all metadata.  A pointer returned by the
+ *     allocator is owned by the caller until it is freed.
+ *   - One allocator per process (the paper's global variant), on the
+ *     device current at gallatin_init.  Host calls are thread-compatible, not
+ *     thread-safe.  Device calls (bulk kernels, device header) are fully
+ *     concurrent with each other.
+ */
+#ifndef GALLATIN_H_
+#define GALLATIN_H_
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+enum {
+    GALLATIN_OK = 0,
+    GALLATIN_ERR_INVALID = -1,   /* bad argument (size, count, universe, NULL)       */
+    GALLATIN_ERR_CUDA = -2,      /* a CUDA runtime call or kernel launch failed       */
+    GALLATIN_ERR_STATE = -3,     /* not initialized / already initialized             */
+    GALLATIN_ERR_NOMEM = -4      /* cudaMalloc of heap/metadata failed (init only)    */
+};
+
+/* ------------------------------------------------------------ allocator --- */
+
+/* Tuning knobs (all optional: zero selects the default).
+ *   heap_bytes : rounded DOWN to a multiple of 16 MiB, >= 1 segment.
+ *   slot_base  : block-buffer slots of the 16 B class; class c gets
+ *                max(slot_min, slot_base >> c).  Default = #SMs (148).
+ *   slot_min   : lower cap, default 4 ("capped at four").
+ *   theta      : prefetch threshold: the request that takes slice index theta
+ *                of a buffered block fetches the next block into the slot's
+ *                side field (0 = off = the paper; not in the paper).
+ *   fence_free : 1 (default) = a release fence per freeing team before its
+ *                free-counter atomic; 2 = none
+ *                (measurement only: frees then do not order user data).
+ */
+typedef struct gallatin_config {
+    uint64_t heap_bytes;
+    uint32_t slot_base;
+    uint32_t slot_min;
+    uint32_t theta;
+    uint32_t fence_free;
+    uint32_t reserved[4];
+} gallatin_config_t;
+
+int gallatin_init(uint64_t heap_bytes);                 /* defaults for the rest */
+int gallatin_init_ex(const gallatin_config_t *cfg);
+int gallatin_destroy(void);                             /* frees heap + metadata; every
+                                                           outstanding pointer dies   */
+int gallatin_is_initialized(void);                      /* 1 / 0 */
+
+/* Bulk malloc (Alg. 3 -> 2 -> 1): d_ptrs[i] = malloc(d_sizes[i]) by
+ * one GPU thread per request.  Size 0 and exhaustion give NULL.  Sizes
+ * <= 4096 B are slices (16 B .. 4 KB powers of two); (4 KB, 16 MB)
+ * whole blocks; >= 16 MB whole contiguous segments. */
+int gallatin_malloc(const uint64_t *d_sizes, void **d_ptrs, uint64_t n, void *stream);
+
+/* Bulk free (Alg. 4).  NULL entries are ignored.  A pointer outside
+ * the heap or into an unallocated segment increments the device error counter
+ * (gallatin_stats); other foreign, interior or double frees are undefined. */
+int gallatin_free(void *const *d_ptrs, uint64_t n, void *stream);
+
+/* Same two calls with HOST arrays: copies the inputs to the device, runs the
+ * kernel on `stream`, copies the results back and synchronizes the stream. */
+int gallatin_malloc_host(const uint64_t *h_sizes, uint64_t *h_ptrs, uint64_t n, void *stream);
+int gallatin_free_host(const uint64_t *h_ptrs, uint64_t n, void *stream);
+
+/* Pristine state (the paper resets before every run).  Invalidates
+ * every outstanding pointer.  Asynchronous on `stream`. */
+int gallatin_reset(void *stream);
+
+/* Quiescent only (no malloc/free in flight): retire every block-buffer slot;
+ * the unissued remainder of each buffered block is freed, prefetched blocks
+ * are returned.  After every user pointer is freed, drain restores the
+ * pristine image.  Runs sequentially (one thread) in slot order. */
+int gallatin_drain(void *stream);
+
+/* Serialized replay (test hook, one GPU thread, in order): kinds[i] 0 =
+ * malloc(args[i]) with block-buffer slot key keys[i] (instead of %smid); 1 =
+ * free(result of op args[i]); 2 = drain.  d_out[i] = pointer OFFSET from the
+ * heap base for mallocs (UINT64_MAX = NULL), 0 otherwise. */
+int gallatin_replay(const uint8_t *d_kinds, const uint64_t *d_args, const uint64_t *d_keys,
+                    uint64_t n, uint64_t *d_out, void *stream);
+
+typedef struct gallatin_stats {
+    uint64_t heap_base;          /* device address of segment 0 (16 MiB aligned)   */
+    uint64_t heap_bytes;
+    uint64_t num_segments;
+    uint64_t free_segments;      /* bits set in the segment tree                    */
+    uint64_t tree_segments[9];   /* segments formatted for each block tree          */
+    uint64_t large_segments;     /* segments held by >= 16 MB allocations           */
+    uint64_t errors;             /* device error counter (bad frees)                */
+    uint32_t nslot[9];           /* block-buffer slots per class                    */
+    uint32_t theta, fence_free;
+} gallatin_stats_t;
+int gallatin_stats(gallatin_stats_t *out);               /* synchronizes the device */
+
+/* Snapshot image (synchronizes the device).  A flat array of uint64 words:
+ *   [0] magic 0x47414C4C494D4731  [1] nseg  [2] tree levels L  [3] W = words
+ *   per tree  [4] S = total slots  [5] error counter  [6],[7] 0
+ *   then: segment tree (W words: level 0 first; bit = segment free)
+ *         9 block trees (9*W; bit s of tree t = segment s formatted for t
+ *           with blocks available)
+ *         memory table (nseg words: tree id << 32 | (uint32) available blocks;
+ *           tree id 0..8 block tree, 9+k first of k segments, 0xFFFFFFFE
+ *           continuation, 0xFFFFFFFF free)
+ *         ring queues (nseg x 65 words: [count] then 256 uint16 block ids in
+ *           FIFO order, 0xFFFF padded, 4 per word little-endian)
+ *         block free counters (nseg*256 uint32, 2 per word)
+ *         block-buffer slots (S words: issued-count << 32 | block id,
+ *           0xFFFFFFFF = none; class-major)
+ *         prefetched block per slot (S words; 0xFFFFFFFF = none)
+ * gallatin_snapshot_words() gives the length. */
+int gallatin_snapshot_words(uint64_t *words);
+int gallatin_snapshot(uint64_t *h_out, uint64_t cap_words, uint64_t *len_words);
+
+/* Device view for the header-only device API (include/gallatin/device.cuh). */
+struct gallatin_device_view;
+int gallatin_get_device_view(struct gallatin_device_view *out, uint64_t out_bytes);
+uint64_t gallatin_device_view_bytes(void);
+
+/* Test harness kernels (not timed by the paper; "checks the correctness
+ * of allocated memory"):
+ *   stamp  : every request i writes the uint32 value i over ceil(size/4) words.
+ *   verify : separate launch, L1-bypassing loads; adds the number of words not
+ *            equal to i to *d_bad (uint64).
+ *   usable : for every non-NULL pointer, the usable size read from the memory
+ *            table (slice 16<<t, block 64K<<t, or k segments); adds the sum to
+ *            *d_sum and the count of pointers whose table entry contradicts
+ *            their request (wrong class, not aligned, outside the heap) to
+ *            *d_bad. d_usable (nullable) receives the per-pointer value. */
+int gallatin_stamp(void *const *d_ptrs, const uint64_t *d_sizes, uint64_t n, void *stream);
+int gallatin_verify(void *const *d_ptrs, const uint64_t *d_sizes, uint64_t n,
+                    uint64_t *d_bad, void *stream);
+int gallatin_usable(void *const *d_ptrs, const uint64_t *d_sizes, uint64_t n,
+                    uint64_t *d_usable, uint64_t *d_sum, uint64_t *d_bad, void *stream);
+
+/* ------------------------------------------------------ standalone vEB --- */
+/* The paper's GPU vEB tree: 64-bit bitmap nodes, no min/max, a
+ * fixed height ceil(log64 u); a concurrent set over [0, 2^universe_log2).
+ * Every node operation is one 64-bit atomic.  Keys >= 2^universe_log2 are
+ * ignored by insert/delete (out 0) and have no successor (UINT64_MAX). */
+typedef struct veb veb_t;
+int veb_create(uint32_t universe_log2 /* 1..32 */, veb_t **out);
+int veb_destroy(veb_t *h);
+int veb_clear(veb_t *h, void *stream);
+/* d_out[i] = 1 iff key i was newly added / was present (exactly one of several
+ * equal keys in a batch reports 1).  d_out may be NULL. */
+int veb_insert(veb_t *h, const uint64_t *d_keys, uint8_t *d_out, uint64_t n, void *stream);
+int veb_delete(veb_t *h, const uint64_t *d_keys, uint8_t *d_out, uint64_t n, void *stream);
+int veb_member(veb_t *h, const uint64_t *d_keys, uint8_t *d_out, uint64_t n, void *stream);
+/* succ(x) = min{y in S, y >= x}; pred(x) = max{y in S, y <= x};
+ * UINT64_MAX when none.  Query batches read the tree through the read-only
+ * path: no insert/delete may run on the same tree concurrently (different
+ * streams) with a query batch. */
+int veb_successor(veb_t *h, const uint64_t *d_q, uint64_t *d_out, uint64_t n, void *stream);
+int veb_predecessor(veb_t *h, const uint64_t *d_q, uint64_t *d_out, uint64_t n, void *stream);
+/* Image (all levels, level 0 first; bit = element / child non-empty); syncs. */
+int veb_words(const veb_t *h, uint64_t *words);
+int veb_snapshot(const veb_t *h, uint64_t *h_out, uint64_t cap_words, uint64_t *len_words);
+
+/* ------------------------------------------------------ measurement ----- */
+/* Peak probes; each returns the kernel time of one
+ * launch in *ms (CUDA events on `stream`) and the operation count in *ops.
+ *   kind 1: distinct-address 64-bit atomicAdd with return, over `param` words
+ *   kind 2: hot-address atomicAdd with return, one lane per warp, `param` lines
+ *   kind 3: as 2 with red (no return)
+ *   kind 4: bump ceiling: per warp one atomicAdd(32) on `param` lines and
+ *           __shfl_sync + 16 B of HBM I/O per lane (the allocator's lower bound)
+ *   kind 5: fence.acq_rel.gpu per warp (ops = warps)
+ *   kind 6: HBM copy of `param` bytes (ops = bytes moved, read + write)
+ * `n` = threads launched. */
+int gallatin_probe(int kind, uint64_t n, uint64_t param, double *ms, double *ops, void *stream);
+
+const char *gallatin_version(void);
+const char *gallatin_error_string(int code);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* GALLATIN_H_ */

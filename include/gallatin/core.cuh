@@ -1,0 +1,384 @@
+// gallatin/core.cuh -- the allocator's device code (one copy, used by the bulk
+// kernels of libgallatin.so and by user kernels through gallatin/device.cuh).
+//
+// PAPER.md (P = line): segments of 16 MB in a segment tree (S4.1, P:132-143,
+// Alg. 1), blocks of 4096 slices in per-size block trees (S4.2, P:170-180,
+// Alg. 2), slices handed out by a counter from a per-SM block buffer with
+// warp coalescing (S4.3, Alg. 3), frees through per-block counters
+// and segment re-insertion (S5, Alg. 4).  Differences from the
+// paper's own GPU design are listed in DESIGN.md ("Deviations") and marked
+// [dev] here.
+#pragma once
+#include <stdint.h>
+
+#include "gallatin/bittree.cuh"
+#include "gallatin/ptx.cuh"
+#include "gallatin/view.h"
+
+namespace gallatin {
+namespace core {
+
+using View = gallatin_device_view;
+
+constexpr uint32_t kSegLog2 = 24;                   // 16 MB segments
+constexpr uint64_t kSegBytes = 1ull << kSegLog2;
+constexpr uint32_t kSlices = 4096;                  // slices per block
+constexpr uint32_t kSliceLog2 = 12;
+constexpr uint32_t kMinSliceLog2 = 4;               // 16 B
+constexpr uint64_t kMaxSlice = 4096;                // 4096 B
+constexpr uint32_t kTrees = GALLATIN_NUM_TREES;     // block trees 64 KB..16 MB
+constexpr uint32_t kMaxBlocks = 256;                // blocks per segment
+constexpr uint32_t kTreeFree = 0xFFFFFFFFu;
+constexpr uint32_t kTreeCont = 0xFFFFFFFEu;
+constexpr uint32_t kGidNone = 0xFFFFFFFFu;
+constexpr uint32_t kAvailBias = 0x80000000u;
+constexpr uint16_t kRingEmpty = 0xFFFF;
+constexpr uint64_t kSlotEmpty = ((uint64_t)kSlices << 32) | kGidNone;
+
+__device__ __forceinline__ uint32_t nb_of(uint32_t t) { return kMaxBlocks >> t; }
+
+// ---- memory-table word {tree id : 32 | available blocks + 2^31 : 32} --------
+// [dev] The paper keeps the tree id and the ring queue separately and
+// re-checks the id with ldcv after taking a block (Alg.2).  Packing
+// the id with the ring's reservation count lets one fetch-add reserve a block
+// and validate the id at once; every update of the word is a fetch-add (or
+// the one CAS that retires a full segment), so concurrent updates commute.
+__device__ __forceinline__ uint32_t sw_tree(uint64_t w) { return (uint32_t)(w >> 32); }
+__device__ __forceinline__ int32_t sw_avail(uint64_t w) { return (int32_t)((uint32_t)w - kAvailBias); }
+__device__ __forceinline__ uint64_t sw_make(uint32_t tree, int32_t avail) {
+    return ((uint64_t)tree << 32) | (uint32_t)((uint32_t)avail + kAvailBias);
+}
+__device__ __forceinline__ uint64_t sw_retree(uint32_t from, uint32_t to) {
+    return (uint64_t)(uint32_t)(to - from) << 32;
+}
+// block tree t holds segment s  <=>  s is formatted for t and has a block
+__device__ __forceinline__ bool sw_in_tree(uint64_t w, uint32_t t) { return sw_tree(w) == t && sw_avail(w) > 0; }
+
+__device__ __forceinline__ BitTree seg_tree(const View &v) {
+    BitTree b;
+    b.w = v.seg_tree;
+    b.nbits = v.nseg;
+    b.levels = v.tree_levels;
+#pragma unroll
+    for (int i = 0; i < kMaxLevels; i++) b.off[i] = v.level_off[i];
+    return b;
+}
+__device__ __forceinline__ BitTree block_tree(const View &v, uint32_t t) {
+    BitTree b = seg_tree(v);
+    b.w = v.block_trees + (uint64_t)t * v.tree_words;
+    return b;
+}
+
+// Make block-tree t's bit for segment s equal its predicate (the derived-bit
+// reconcile loop of DESIGN.md "Quiescent exactness").
+__device__ inline void btree_reconcile(const View &v, uint32_t t, uint64_t s) {
+    const BitTree bt = block_tree(v, t);
+    uint64_t *leaf = bt.w + bt.off[0] + (s >> 6);
+    const uint64_t bit = 1ull << (s & 63);
+    bool flipped = false;
+    ptx::fence_sc();
+    for (;;) {
+        const bool in = sw_in_tree(ptx::ld_relaxed(v.seg_word + s), t);
+        const uint64_t old = in ? ptx::atom_or(leaf, bit) : ptx::atom_and(leaf, ~bit);
+        flipped |= in ? (old == 0) : (old == bit);
+        ptx::fence_sc();
+        if (sw_in_tree(ptx::ld_relaxed(v.seg_word + s), t) == in) break;
+    }
+    if (flipped) bt_reconcile_up(bt, 0, s >> 6);
+}
+
+__device__ void try_free_segment(const View &v, uint64_t s, uint32_t t);
+
+// Every thread whose RMW on seg_word[s] changed a block-tree predicate repairs
+// that bit; the RMW that brings a segment back to "all blocks home" retires it.
+__device__ inline void seg_after_rmw(const View &v, uint64_t s, uint64_t old, uint64_t now) {
+    const uint32_t to = sw_tree(old), tn = sw_tree(now);
+    if (to < kTrees && sw_in_tree(old, to) != sw_in_tree(now, to)) btree_reconcile(v, to, s);
+    if (tn < kTrees && tn != to && sw_in_tree(old, tn) != sw_in_tree(now, tn)) btree_reconcile(v, tn, s);
+    if (tn < kTrees && tn == to && sw_avail(now) == (int32_t)nb_of(tn) && sw_avail(old) < sw_avail(now))
+        try_free_segment(v, s, tn);
+}
+
+// "When all blocks are returned, the segment is freed and re-added to the
+// segment tree".
+__device__ inline void try_free_segment(const View &v, uint64_t s, uint32_t t) {
+    const uint64_t full = sw_make(t, (int32_t)nb_of(t));
+    if (ptx::atom_cas(v.seg_word + s, full, sw_make(kTreeFree, 0)) != full) return;
+    // No block of s is out or in flight: reset its ring.
+    ptx::st_relaxed(v.q_head + s, 0u);
+    ptx::st_relaxed(v.q_tail + s, 0u);
+    uint4 *e = reinterpret_cast<uint4 *>(v.q_entries + s * kMaxBlocks);
+#pragma unroll 4
+    for (int i = 0; i < (int)(kMaxBlocks * sizeof(uint16_t) / sizeof(uint4)); i++)
+        e[i] = make_uint4(0xFFFFFFFFu, 0xFFFFFFFFu, 0xFFFFFFFFu, 0xFFFFFFFFu);
+    ptx::fence_acq_rel();
+    btree_reconcile(v, t, s);
+    bt_insert(seg_tree(v), s);
+}
+
+// ---- Alg. 1 GetSegment(treeId < numBlockTrees) ----------------
+__device__ inline bool get_segment(const View &v, uint32_t t) {
+    const BitTree st = seg_tree(v);
+    for (;;) {
+        uint64_t s = bt_successor<false>(st, 0);           // front first
+        if (s == kNone) {
+            s = bt_scan_first(st);                         // confirm before failing
+            if (s == kNone) return false;                  // "All segments in use"
+        }
+        if (!bt_delete(st, s)) continue;                   // claimIndex lost
+        ptx::fence_acq_rel();
+        // initSegment: the ring holds blocks 0..nb-1 in order
+        const uint32_t nb = nb_of(t);
+        uint16_t *e = v.q_entries + s * kMaxBlocks;
+        if (nb >= 4) {
+            uint64_t *e4 = reinterpret_cast<uint64_t *>(e);
+            for (uint32_t q = 0; q < nb / 4; q++) {
+                const uint64_t j = 4ull * q;
+                e4[q] = j | ((j + 1) << 16) | ((j + 2) << 32) | ((j + 3) << 48);
+            }
+        } else {
+            for (uint32_t j = 0; j < nb; j++) e[j] = (uint16_t)j;
+        }
+        ptx::st_relaxed(v.q_head + s, 0u);
+        ptx::st_relaxed(v.q_tail + s, nb);
+        ptx::fence_acq_rel();
+        // "broadcast availability": the table word, then block tree t
+        const uint64_t delta = sw_retree(kTreeFree, t) + nb;
+        const uint64_t old = ptx::atom_add(v.seg_word + s, delta);
+        seg_after_rmw(v, s, old, old + delta);
+        return true;
+    }
+}
+
+// ---- Alg. 2 GetBlock(treeId) ---------------------------------
+// Returns a global block id gid = segment*256 + block, or kGidNone.
+__device__ inline uint32_t get_block(const View &v, uint32_t t) {
+    const BitTree bt = block_tree(v, t);
+    ptx::Backoff bo;
+    for (;;) {
+        const uint64_t s = bt_successor<false>(bt, 0);     // findSegment
+        if (s != kNone) {
+            // reserve one block of s and validate its tree id in one RMW [dev]
+            const uint64_t old = ptx::atom_add(v.seg_word + s, ~0ull);
+            if (sw_tree(old) == t && sw_avail(old) > 0) {
+                seg_after_rmw(v, s, old, old - 1);         // last block out: leave tree
+                // getBlock from the segment's ring queue
+                const uint32_t pos = atomicAdd(v.q_head + s, 1u) & (kMaxBlocks - 1);
+                uint16_t *slotp = v.q_entries + s * kMaxBlocks + pos;
+                uint16_t j;
+                ptx::Backoff wb;
+                while ((j = ptx::ld_relaxed(slotp)) == kRingEmpty) wb.pause();   // enqueue in flight
+                ptx::st_relaxed(slotp, kRingEmpty);
+                ptx::fence_acq_rel();
+                return (uint32_t)(s * kMaxBlocks + j);
+            }
+            // stale hint (P:158-161's failure case): undo, repair, retry
+            seg_after_rmw(v, s, old, old - 1);
+            const uint64_t o2 = ptx::atom_add(v.seg_word + s, 1ull);
+            seg_after_rmw(v, s, o2, o2 + 1);
+            btree_reconcile(v, t, s);
+            bo.pause();
+            continue;
+        }
+        // no formatted segment has a block: format one (Alg.2).
+        // [dev] one formatter per tree at a time (a token) instead of every
+        // waiting thread formatting its own segment.
+        uint32_t *tok = v.fmt_token + t * 32;
+        if (atomicCAS(tok, 0u, 1u) == 0u) {
+            bool ok = true;
+            if (bt_successor<false>(bt, 0) == kNone) ok = get_segment(v, t);
+            ptx::fence_acq_rel();
+            atomicExch(tok, 0u);
+            if (!ok && bt_scan_first(bt) == kNone) return kGidNone;   // "No allocations left"
+            continue;
+        }
+        while (ptx::ld_relaxed(tok) != 0u && bt_successor<false>(bt, 0) == kNone) bo.pause();
+    }
+}
+
+// ---- block return (Alg.4; ring enqueue P:178) --------------------
+__device__ inline void return_block(const View &v, uint32_t gid) {
+    const uint64_t s = gid / kMaxBlocks;
+    const uint32_t pos = atomicAdd(v.q_tail + s, 1u) & (kMaxBlocks - 1);
+    uint16_t *slotp = v.q_entries + s * kMaxBlocks + pos;
+    ptx::Backoff wb;
+    while (ptx::ld_relaxed(slotp) != kRingEmpty) wb.pause();   // previous lap's dequeue in flight
+    ptx::st_relaxed(slotp, (uint16_t)(gid % kMaxBlocks));
+    ptx::fence_acq_rel();
+    const uint64_t old = ptx::atom_add(v.seg_word + s, 1ull);
+    seg_after_rmw(v, s, old, old + 1);
+}
+
+// n slices of block gid came back; the team completing 4096 returns it
+// (reading A-14 of "== 4095").
+__device__ inline void block_freed(const View &v, uint32_t gid, uint32_t n) {
+    const uint32_t old = atomicAdd(v.block_free + gid, n);
+    if (old + n == kSlices) {
+        atomicExch(v.block_free + gid, 0u);
+        ptx::fence_acq_rel();
+        return_block(v, gid);
+    }
+}
+
+// ---- addresses -------------------------------------------------------------
+__device__ __forceinline__ void *slice_ptr(const View &v, uint32_t gid, uint32_t c, uint32_t idx) {
+    // offset(blockId*4096 + idx): block j of segment s is 2^(16+c) B
+    const uint64_t s = gid / kMaxBlocks, j = gid % kMaxBlocks;
+    return reinterpret_cast<void *>(v.heap + (s << kSegLog2) + (j << (16 + c)) + ((uint64_t)idx << (kMinSliceLog2 + c)));
+}
+__device__ __forceinline__ uint64_t *slot_word(const View &v, uint32_t si) { return v.slots + (uint64_t)si * 16; }
+__device__ __forceinline__ uint32_t *slot_next(const View &v, uint32_t si) {
+    return reinterpret_cast<uint32_t *>(v.slots + (uint64_t)si * 16 + 1);
+}
+
+// Replace an exhausted buffered block (Alg.3): the prefetched block
+// if there is one, else GetBlock.  On exhaustion the slot is left empty.
+__device__ inline bool refill_slot(const View &v, uint32_t si, uint32_t c) {
+    uint32_t b = kGidNone;
+    if (v.theta) b = atomicExch(slot_next(v, si), kGidNone);
+    if (b == kGidNone) b = get_block(v, c);
+    if (b == kGidNone) {
+        ptx::atom_exch(slot_word(v, si), kSlotEmpty);
+        return false;
+    }
+    ptx::atom_exch(slot_word(v, si), (uint64_t)b);        // {issued 0, block b}
+    return true;
+}
+
+// [dev] prefetch: the request that takes index theta fetches the next block.
+__device__ inline void prefetch_slot(const View &v, uint32_t si, uint32_t c) {
+    const uint32_t b = get_block(v, c);
+    if (b == kGidNone) return;
+    if (atomicCAS(slot_next(v, si), kGidNone, b) != kGidNone) block_freed(v, b, kSlices);   // raced: give it back
+}
+
+// ---- Alg. 3 MALLOC.Slice ---------------------------------------
+// The lanes of a warp asking the same slot form a team (reading A-8);
+// the leader does ONE atomicAdd on the slot word {issued:32 | block:32} that
+// returns the block and the first slice index together [dev: the paper reads
+// the buffer, then adds on the block's counter]; __shfl_sync broadcasts it;
+// lane r takes index old+r, valid iff < 4096.  The lane that draws
+// index 4096 replaces the block (reading A-7); other lanes past the
+// end wait for the replacement and retry.
+__device__ inline void *malloc_slice(const View &v, uint32_t c, uint32_t key) {
+    const uint32_t si = v.slot_off[c] + key % v.nslot[c];
+    uint64_t *sw = slot_word(v, si);
+    const uint32_t lane = ptx::lane_id();
+    for (;;) {
+        const unsigned act = __activemask();
+        const unsigned peers = __match_any_sync(act, si);
+        const uint32_t leader = (uint32_t)__ffs((int)peers) - 1;
+        const uint32_t rank = (uint32_t)__popc(peers & ptx::lanemask_lt());
+        uint64_t old = 0;
+        if (lane == leader) old = ptx::atom_add(sw, (uint64_t)__popc(peers) << 32);
+        old = __shfl_sync(peers, old, (int)leader);
+        const uint32_t cnt = (uint32_t)(old >> 32), gid = (uint32_t)old;
+        const uint32_t idx = cnt + rank;
+        if (idx < kSlices) {
+            if (v.theta && idx == v.theta) prefetch_slot(v, si, c);
+            return slice_ptr(v, gid, c, idx);
+        }
+        if (idx == kSlices) {
+            if (!refill_slot(v, si, c)) return nullptr;            // nullptr
+            continue;
+        }
+        ptx::Backoff bo;
+        while ((uint32_t)(ptx::ld_relaxed(sw) >> 32) > kSlices) bo.pause();
+    }
+}
+
+// (4 KB, 16 MB): one whole block of the smallest fitting tree; its counter is
+// preset to 4095 so that Alg.4's rule returns it on its one free (reading A-2).
+__device__ inline void *malloc_block(const View &v, uint32_t t) {
+    const uint32_t gid = get_block(v, t);
+    if (gid == kGidNone) return nullptr;
+    atomicExch(v.block_free + gid, kSlices - 1);
+    const uint64_t s = gid / kMaxBlocks, j = gid % kMaxBlocks;
+    return reinterpret_cast<void *>(v.heap + (s << kSegLog2) + (j << (16 + t)));
+}
+
+// >= 16 MB: Alg.1 with treeId >= numBlockTrees: claimMultiple from the back
+// (P:110-113); tree id = numBlockTrees + numSegments.
+__device__ inline void *malloc_large(const View &v, uint64_t k) {
+    if (k > v.nseg) return nullptr;
+    const BitTree st = seg_tree(v);
+    ptx::Backoff bo;
+    uint64_t i;
+    int misses = 0;
+    for (;;) {
+        i = bt_find_highest_run(st, k);
+        if (i == kNone) {
+            if (++misses > 2) return nullptr;
+            bo.pause();
+            continue;
+        }
+        if (bt_claim_range(st, i, k)) break;
+        bo.pause();
+    }
+    ptx::fence_acq_rel();
+    ptx::atom_add(v.seg_word + i, sw_retree(kTreeFree, kTrees + (uint32_t)k));
+    for (uint64_t m = 1; m < k; m++) ptx::atom_add(v.seg_word + i + m, sw_retree(kTreeFree, kTreeCont));
+    ptx::fence_acq_rel();
+    return reinterpret_cast<void *>(v.heap + (i << kSegLog2));
+}
+
+// Classify (A1): slices 16 B..4 KB by ceil(log2), blocks, segments.
+__device__ inline void *malloc_impl(const View &v, uint64_t size, uint32_t key) {
+    if (size == 0) return nullptr;
+    if (size <= kMaxSlice) {
+        const uint32_t c = size <= 16 ? 0u : (uint32_t)(64 - __clzll((long long)(size - 1))) - kMinSliceLog2;
+        return malloc_slice(v, c, key);
+    }
+    if (size < kSegBytes) {
+        const uint32_t t = size <= 65536 ? 0u : (uint32_t)(64 - __clzll((long long)(size - 1))) - 16;
+        return malloc_block(v, t);
+    }
+    const uint64_t k = (size >> kSegLog2) + ((size & (kSegBytes - 1)) != 0);
+    return malloc_large(v, k);
+}
+
+// ---- Alg. 4 FREE -----------------------------------------------
+__device__ inline void free_impl(const View &v, void *p) {
+    if (p == nullptr) return;
+    const uint64_t off = reinterpret_cast<uint64_t>(p) - v.heap;
+    if (off >= (v.nseg << kSegLog2)) { atomicAdd(v.err, 1ull); return; }
+    const uint64_t s = off >> kSegLog2;
+    const uint32_t t = sw_tree(ptx::ld_relaxed(v.seg_word + s));   // ldcv(ids[segment])
+    if (t < kTrees) {
+        // locateBlock; frees of one block coalesce
+        const uint32_t gid = (uint32_t)(s * kMaxBlocks + ((off & (kSegBytes - 1)) >> (16 + t)));
+        const unsigned act = __activemask();
+        const unsigned peers = __match_any_sync(act, gid);
+        const uint32_t leader = (uint32_t)__ffs((int)peers) - 1;
+        if (v.fence_free != 2) __syncwarp(peers);
+        if (ptx::lane_id() == leader) {
+            if (v.fence_free != 2) ptx::fence_acq_rel();     // release the team's writes
+            block_freed(v, gid, (uint32_t)__popc(peers));
+        }
+        return;
+    }
+    if (t == kTreeFree || t == kTreeCont) { atomicAdd(v.err, 1ull); return; }
+    // segment allocation: return the k segments to the segment tree
+    const uint64_t k = t - kTrees;
+    ptx::fence_acq_rel();
+    ptx::atom_add(v.seg_word + s, sw_retree(t, kTreeFree));
+    for (uint64_t m = 1; m < k; m++) ptx::atom_add(v.seg_word + s + m, sw_retree(kTreeCont, kTreeFree));
+    ptx::fence_acq_rel();
+    bt_insert_range(seg_tree(v), s, k);
+}
+
+// Quiescent drain: retire every slot in class-major order; the unissued
+// remainder of a buffered block counts as freed, a prefetched block is
+// returned whole.
+__device__ inline void drain_slots(const View &v) {
+    for (uint32_t si = 0; si < v.nslot_total; si++) {
+        const uint64_t w = ptx::atom_exch(slot_word(v, si), kSlotEmpty);
+        const uint32_t cnt = (uint32_t)(w >> 32), gid = (uint32_t)w;
+        if (gid != kGidNone && cnt < kSlices) block_freed(v, gid, kSlices - cnt);
+        const uint32_t nx = atomicExch(slot_next(v, si), kGidNone);
+        if (nx != kGidNone) block_freed(v, nx, kSlices);
+    }
+}
+
+}  // namespace core
+}  // namespace gallatin

@@ -1,0 +1,54 @@
+/*
+ * gallatin/view.h -- the device view: where every piece of allocator state
+ * lives in HBM.  A plain C struct, passed by value to the bulk kernels and
+ * copied into __constant__ memory by the device-header binding.
+ *
+ * Layout (P = PAPER.md line):
+ *   heap        nseg x 16 MiB, base aligned to 16 MiB
+ *   seg_tree    W words: 64-ary bitmap levels, level 0 first, bit = free
+ *   block_trees 9 x W words (tree t at t*W): bit s = segment s formatted for
+ *               tree t with blocks available
+ *   seg_word    nseg x u64 {tree id:32 | available blocks + 2^31:32}: the
+ *               memory table's ids fused with the ring's
+ *               reservation count
+ *   q_head/tail nseg x u32 ring counters; q_entries nseg x 256 x u16 block ids
+ *               (the per-segment ring queue)
+ *   block_free  nseg x 256 x u32 free counters
+ *   slots       S x 128 B lines: word 0 = {issued count:32 | block id:32},
+ *               word 1 = prefetched block id (block buffer)
+ *   fmt_token   9 x 128 B lines: one formatter per block tree
+ *   err         u64 error counter (bad frees)
+ */
+#ifndef GALLATIN_VIEW_H_
+#define GALLATIN_VIEW_H_
+#include <stdint.h>
+
+#define GALLATIN_NUM_TREES 9
+#define GALLATIN_MAX_LEVELS 8
+
+struct gallatin_device_view {
+    uint64_t heap;              /* device address of segment 0                */
+    uint64_t nseg;
+    uint64_t *seg_tree;
+    uint64_t *block_trees;
+    uint64_t *seg_word;
+    uint32_t *q_head;
+    uint32_t *q_tail;
+    uint16_t *q_entries;
+    uint32_t *block_free;
+    uint64_t *slots;            /* 16 words (128 B) per slot                  */
+    uint32_t *fmt_token;        /* 32 words (128 B) per tree                  */
+    unsigned long long *err;
+    uint32_t tree_levels;       /* L                                           */
+    uint32_t tree_words;        /* W                                           */
+    uint32_t level_off[GALLATIN_MAX_LEVELS];
+    uint32_t nslot[GALLATIN_NUM_TREES];
+    uint32_t slot_off[GALLATIN_NUM_TREES];
+    uint32_t nslot_total;
+    uint32_t theta;             /* 0 = no prefetch                            */
+    uint32_t fence_free;        /* 1 = release fence per freeing team, 2 = none */
+    uint32_t reserved;
+};
+typedef struct gallatin_device_view gallatin_device_view_t;
+
+#endif

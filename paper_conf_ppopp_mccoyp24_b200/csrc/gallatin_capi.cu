@@ -1,0 +1,543 @@
+// gallatin_capi.cu -- libgallatin.so: the C-ABI of include/gallatin.h.
+//
+// Host plumbing (heap + metadata in HBM, reset, snapshot, stats) and the bulk
+// kernels: one GPU thread per request, each running the same device code a
+// user kernel gets from include/gallatin/device.cuh (one thread per
+// allocation, 1M+ threads).
+#include <cuda_runtime.h>
+#include <stdint.h>
+#include <stdio.h>
+#include <string.h>
+
+#include <vector>
+
+#include "gallatin.h"
+#include "gallatin/core.cuh"
+
+using namespace gallatin;
+using core::View;
+
+namespace {
+
+constexpr int kThreads = 256;
+
+struct State {
+    bool init = false;
+    int device = 0;
+    gallatin_config_t cfg{};
+    void *heap_raw = nullptr;
+    void *meta = nullptr;
+    uint64_t meta_bytes = 0;
+    View v{};
+    void *scratch = nullptr;
+    uint64_t scratch_bytes = 0;
+};
+State g;
+
+#define CUDA_TRY(x)                                                                 \
+    do {                                                                            \
+        cudaError_t e_ = (x);                                                       \
+        if (e_ != cudaSuccess) {                                                    \
+            fprintf(stderr, "gallatin: %s failed: %s\n", #x, cudaGetErrorString(e_)); \
+            return GALLATIN_ERR_CUDA;                                               \
+        }                                                                           \
+    } while (0)
+
+inline cudaStream_t S(void *s) { return reinterpret_cast<cudaStream_t>(s); }
+inline unsigned grid_for(uint64_t n) { return (unsigned)((n + kThreads - 1) / kThreads); }
+inline uint64_t align_up(uint64_t x, uint64_t a) { return (x + a - 1) / a * a; }
+
+int launch_status() {
+    cudaError_t e = cudaGetLastError();
+    if (e != cudaSuccess) {
+        fprintf(stderr, "gallatin: launch failed: %s\n", cudaGetErrorString(e));
+        return GALLATIN_ERR_CUDA;
+    }
+    return GALLATIN_OK;
+}
+
+// ------------------------------------------------------------ kernels ----
+__global__ void k_reset(View v) {
+    const uint64_t W = v.tree_words, nseg = v.nseg;
+    const uint64_t S = v.nslot_total;
+    const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
+    uint64_t total = nseg * 128;
+    if (S * 16 > total) total = S * 16;
+    if (9 * W > total) total = 9 * W;
+    if (9 * 32 > total) total = 9 * 32;
+    for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < total; i += stride) {
+        if (i < W) {
+            // pristine segment tree: every segment free, summaries consistent
+            uint32_t lvl = 0;
+            while (lvl + 1 < v.tree_levels && i >= v.level_off[lvl + 1]) lvl++;
+            const uint64_t word = i - v.level_off[lvl];
+            const uint64_t nbits = lvl == 0 ? nseg : (uint64_t)(v.level_off[lvl] - v.level_off[lvl - 1]);
+            const uint64_t lo = word * 64;
+            const uint64_t cnt = nbits > lo ? (nbits - lo < 64 ? nbits - lo : 64) : 0;
+            v.seg_tree[i] = cnt == 64 ? ~0ull : ((1ull << cnt) - 1);
+        }
+        if (i < 9 * W) v.block_trees[i] = 0;
+        if (i < nseg) {
+            v.seg_word[i] = core::sw_make(core::kTreeFree, 0);
+            v.q_head[i] = 0;
+            v.q_tail[i] = 0;
+        }
+        if (i < nseg * 64) reinterpret_cast<uint64_t *>(v.q_entries)[i] = ~0ull;
+        if (i < nseg * 128) reinterpret_cast<uint64_t *>(v.block_free)[i] = 0;
+        if (i < S * 16) {
+            const uint64_t w = i % 16;
+            v.slots[i] = w == 0 ? core::kSlotEmpty : (w == 1 ? (uint64_t)core::kGidNone : 0);
+        }
+        if (i < 9 * 32) v.fmt_token[i] = 0;
+        if (i == 0) *v.err = 0;
+    }
+}
+
+__global__ void __launch_bounds__(kThreads) k_bulk_malloc(View v, const uint64_t *__restrict__ sizes,
+                                                          void **__restrict__ ptrs, uint64_t n) {
+    const uint64_t i = blockIdx.x * (uint64_t)kThreads + threadIdx.x;
+    if (i >= n) return;
+    ptrs[i] = core::malloc_impl(v, sizes[i], ptx::smid());
+}
+
+__global__ void __launch_bounds__(kThreads) k_bulk_free(View v, void *const *__restrict__ ptrs, uint64_t n) {
+    const uint64_t i = blockIdx.x * (uint64_t)kThreads + threadIdx.x;
+    if (i >= n) return;
+    core::free_impl(v, ptrs[i]);
+}
+
+__global__ void k_replay(View v, const uint8_t *kinds, const uint64_t *args, const uint64_t *keys, uint64_t n,
+                         uint64_t *out) {
+    for (uint64_t i = 0; i < n; i++) {
+        const uint8_t k = kinds[i];
+        if (k == 0) {
+            void *p = core::malloc_impl(v, args[i], (uint32_t)keys[i]);
+            out[i] = p ? reinterpret_cast<uint64_t>(p) - v.heap : ~0ull;
+        } else if (k == 1) {
+            const uint64_t o = out[args[i]];
+            core::free_impl(v, o == ~0ull ? nullptr : reinterpret_cast<void *>(v.heap + o));
+            out[i] = 0;
+        } else {
+            core::drain_slots(v);
+            out[i] = 0;
+        }
+    }
+}
+
+__global__ void k_drain(View v) { core::drain_slots(v); }
+
+// -- correctness harness ("checks the correctness of allocated memory")
+__global__ void k_stamp(void *const *ptrs, const uint64_t *sizes, uint64_t n) {
+    const uint64_t warp = (blockIdx.x * (uint64_t)blockDim.x + threadIdx.x) >> 5;
+    const uint32_t lane = threadIdx.x & 31;
+    for (uint32_t a = 0; a < 32; a++) {
+        const uint64_t i = warp * 32 + a;
+        if (i >= n) break;
+        uint32_t *p = reinterpret_cast<uint32_t *>(ptrs[i]);
+        if (!p) continue;
+        const uint64_t words = (sizes[i] + 3) / 4, n16 = words / 4;
+        const uint32_t val = (uint32_t)i;
+        uint4 *q = reinterpret_cast<uint4 *>(p);
+        for (uint64_t w = lane; w < n16; w += 32) q[w] = make_uint4(val, val, val, val);
+        for (uint64_t w = n16 * 4 + lane; w < words; w += 32) p[w] = val;
+    }
+}
+
+__global__ void k_verify(void *const *ptrs, const uint64_t *sizes, uint64_t n, unsigned long long *bad) {
+    const uint64_t warp = (blockIdx.x * (uint64_t)blockDim.x + threadIdx.x) >> 5;
+    const uint32_t lane = threadIdx.x & 31;
+    unsigned long long mine = 0;
+    for (uint32_t a = 0; a < 32; a++) {
+        const uint64_t i = warp * 32 + a;
+        if (i >= n) break;
+        const uint32_t *p = reinterpret_cast<const uint32_t *>(ptrs[i]);
+        if (!p) continue;
+        const uint64_t words = (sizes[i] + 3) / 4, n16 = words / 4;
+        const uint32_t val = (uint32_t)i;
+        const uint4 *q = reinterpret_cast<const uint4 *>(p);
+        for (uint64_t w = lane; w < n16; w += 32) {
+            const uint4 x = __ldcg(q + w);
+            mine += (x.x != val) + (x.y != val) + (x.z != val) + (x.w != val);
+        }
+        for (uint64_t w = n16 * 4 + lane; w < words; w += 32) mine += __ldcg(p + w) != val;
+    }
+    for (int o = 16; o; o >>= 1) mine += __shfl_down_sync(0xFFFFFFFFu, mine, o);
+    if (lane == 0 && mine) atomicAdd(bad, mine);
+}
+
+__global__ void k_usable(View v, void *const *ptrs, const uint64_t *sizes, uint64_t n, uint64_t *usable,
+                         unsigned long long *sum, unsigned long long *bad) {
+    const uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
+    if (i >= n) return;
+    const uint64_t p = reinterpret_cast<uint64_t>(ptrs[i]);
+    uint64_t u = 0;
+    bool wrong = false;
+    if (p) {
+        const uint64_t off = p - v.heap, req = sizes[i];
+        if (off >= (v.nseg << core::kSegLog2)) {
+            wrong = true;
+        } else {
+            const uint32_t t = core::sw_tree(ptx::ld_relaxed(v.seg_word + (off >> core::kSegLog2)));
+            if (req <= core::kMaxSlice) {
+                const uint32_t c = req <= 16 ? 0u : (uint32_t)(64 - __clzll((long long)(req - 1))) - 4;
+                u = t < core::kTrees ? (16ull << t) : 0;
+                wrong = t != c;
+            } else if (req < core::kSegBytes) {
+                const uint32_t tb = req <= 65536 ? 0u : (uint32_t)(64 - __clzll((long long)(req - 1))) - 16;
+                u = t < core::kTrees ? (65536ull << t) : 0;
+                wrong = t != tb;
+            } else {
+                const uint64_t k = (req >> core::kSegLog2) + ((req & (core::kSegBytes - 1)) != 0);
+                u = (t >= core::kTrees && t < core::kTreeCont) ? ((uint64_t)(t - core::kTrees) << core::kSegLog2) : 0;
+                wrong = t != core::kTrees + k;
+            }
+            if (u == 0 || (off & ((u < core::kSegBytes ? u : core::kSegBytes) - 1)) || u < req) wrong = true;
+            if (off + u > (v.nseg << core::kSegLog2)) wrong = true;
+        }
+    }
+    if (usable) usable[i] = u;
+    if (u) atomicAdd(sum, (unsigned long long)u);
+    if (wrong) atomicAdd(bad, 1ull);
+}
+
+// ------------------------------------------------------- host helpers ----
+uint64_t image_words(const View &v) {
+    return 8 + 10ull * v.tree_words + v.nseg * (1 + 65 + 128) + 2ull * v.nslot_total;
+}
+
+struct HostCopy {
+    std::vector<uint64_t> seg_tree, block_trees, seg_word, slots;
+    std::vector<uint32_t> q_head, q_tail, block_free;
+    std::vector<uint16_t> q_entries;
+    unsigned long long err = 0;
+};
+
+int copy_state(HostCopy &h) {
+    const View &v = g.v;
+    const uint64_t W = v.tree_words, nseg = v.nseg;
+    h.seg_tree.resize(W);
+    h.block_trees.resize(9 * W);
+    h.seg_word.resize(nseg);
+    h.q_head.resize(nseg);
+    h.q_tail.resize(nseg);
+    h.q_entries.resize(nseg * 256);
+    h.block_free.resize(nseg * 256);
+    h.slots.resize((uint64_t)v.nslot_total * 16);
+    CUDA_TRY(cudaDeviceSynchronize());
+    CUDA_TRY(cudaMemcpy(h.seg_tree.data(), v.seg_tree, W * 8, cudaMemcpyDeviceToHost));
+    CUDA_TRY(cudaMemcpy(h.block_trees.data(), v.block_trees, 9 * W * 8, cudaMemcpyDeviceToHost));
+    CUDA_TRY(cudaMemcpy(h.seg_word.data(), v.seg_word, nseg * 8, cudaMemcpyDeviceToHost));
+    CUDA_TRY(cudaMemcpy(h.q_head.data(), v.q_head, nseg * 4, cudaMemcpyDeviceToHost));
+    CUDA_TRY(cudaMemcpy(h.q_tail.data(), v.q_tail, nseg * 4, cudaMemcpyDeviceToHost));
+    CUDA_TRY(cudaMemcpy(h.q_entries.data(), v.q_entries, nseg * 512, cudaMemcpyDeviceToHost));
+    CUDA_TRY(cudaMemcpy(h.block_free.data(), v.block_free, nseg * 1024, cudaMemcpyDeviceToHost));
+    CUDA_TRY(cudaMemcpy(h.slots.data(), v.slots, h.slots.size() * 8, cudaMemcpyDeviceToHost));
+    CUDA_TRY(cudaMemcpy(&h.err, v.err, 8, cudaMemcpyDeviceToHost));
+    return GALLATIN_OK;
+}
+
+int free_all() {
+    if (g.heap_raw) cudaFree(g.heap_raw);
+    if (g.meta) cudaFree(g.meta);
+    if (g.scratch) cudaFree(g.scratch);
+    g = State{};
+    return GALLATIN_OK;
+}
+
+}  // namespace
+
+// ================================================================ C-ABI ====
+extern "C" {
+
+const char *gallatin_version(void) { return "gallatin-b200 0.1 (sm_100a)"; }
+
+const char *gallatin_error_string(int code) {
+    switch (code) {
+    case GALLATIN_OK: return "ok";
+    case GALLATIN_ERR_INVALID: return "invalid argument";
+    case GALLATIN_ERR_CUDA: return "CUDA error";
+    case GALLATIN_ERR_STATE: return "bad allocator state";
+    case GALLATIN_ERR_NOMEM: return "out of device memory";
+    default: return "unknown";
+    }
+}
+
+int gallatin_is_initialized(void) { return g.init ? 1 : 0; }
+
+int gallatin_init_ex(const gallatin_config_t *cfg_in) {
+    if (g.init) return GALLATIN_ERR_STATE;
+    if (!cfg_in) return GALLATIN_ERR_INVALID;
+    gallatin_config_t cfg = *cfg_in;
+    const uint64_t nseg = cfg.heap_bytes >> core::kSegLog2;
+    if (nseg < 1 || nseg > (1ull << 22)) return GALLATIN_ERR_INVALID;
+    int dev = 0, sms = 148;
+    CUDA_TRY(cudaGetDevice(&dev));
+    CUDA_TRY(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev));
+    if (!cfg.slot_base) cfg.slot_base = (uint32_t)sms;      // one slot per SM
+    if (!cfg.slot_min) cfg.slot_min = 4;                     // "capped at four"
+    if (!cfg.fence_free) cfg.fence_free = 1;
+    if (cfg.theta >= core::kSlices) return GALLATIN_ERR_INVALID;
+
+    View v{};
+    v.nseg = nseg;
+    uint32_t levels = 0;
+    const uint64_t W = bittree_geometry(nseg, &levels, v.level_off);
+    v.tree_levels = levels;
+    v.tree_words = (uint32_t)W;
+    uint32_t off = 0;
+    for (uint32_t c = 0; c < core::kTrees; c++) {
+        uint32_t n = cfg.slot_base >> c;
+        if (n < cfg.slot_min) n = cfg.slot_min;
+        if (n < 1) n = 1;
+        v.nslot[c] = n;
+        v.slot_off[c] = off;
+        off += n;
+    }
+    v.nslot_total = off;
+    v.theta = cfg.theta;
+    v.fence_free = cfg.fence_free;
+
+    // metadata: one allocation, 256 B aligned sections
+    uint64_t sz[11] = {W * 8, 9 * W * 8, nseg * 8, nseg * 4, nseg * 4, nseg * 512, nseg * 1024,
+                       (uint64_t)off * 128, 9 * 128, 128, 0};
+    uint64_t total = 0, offs[11];
+    for (int i = 0; i < 10; i++) { offs[i] = total; total += align_up(sz[i], 256); }
+    void *meta = nullptr;
+    if (cudaMalloc(&meta, total) != cudaSuccess) { cudaGetLastError(); return GALLATIN_ERR_NOMEM; }
+    void *heap = nullptr;
+    if (cudaMalloc(&heap, (nseg << core::kSegLog2) + core::kSegBytes) != cudaSuccess) {
+        cudaGetLastError();
+        cudaFree(meta);
+        return GALLATIN_ERR_NOMEM;
+    }
+    char *m = static_cast<char *>(meta);
+    v.seg_tree = reinterpret_cast<uint64_t *>(m + offs[0]);
+    v.block_trees = reinterpret_cast<uint64_t *>(m + offs[1]);
+    v.seg_word = reinterpret_cast<uint64_t *>(m + offs[2]);
+    v.q_head = reinterpret_cast<uint32_t *>(m + offs[3]);
+    v.q_tail = reinterpret_cast<uint32_t *>(m + offs[4]);
+    v.q_entries = reinterpret_cast<uint16_t *>(m + offs[5]);
+    v.block_free = reinterpret_cast<uint32_t *>(m + offs[6]);
+    v.slots = reinterpret_cast<uint64_t *>(m + offs[7]);
+    v.fmt_token = reinterpret_cast<uint32_t *>(m + offs[8]);
+    v.err = reinterpret_cast<unsigned long long *>(m + offs[9]);
+    v.heap = align_up(reinterpret_cast<uint64_t>(heap), core::kSegBytes);   // 16 MiB aligned base
+
+    g.init = true;
+    g.device = dev;
+    g.cfg = cfg;
+    g.heap_raw = heap;
+    g.meta = meta;
+    g.meta_bytes = total;
+    g.v = v;
+    const int rc = gallatin_reset(nullptr);
+    if (rc != GALLATIN_OK) { free_all(); return rc; }
+    CUDA_TRY(cudaDeviceSynchronize());
+    return GALLATIN_OK;
+}
+
+int gallatin_init(uint64_t heap_bytes) {
+    gallatin_config_t cfg{};
+    cfg.heap_bytes = heap_bytes;
+    return gallatin_init_ex(&cfg);
+}
+
+int gallatin_destroy(void) {
+    if (!g.init) return GALLATIN_ERR_STATE;
+    cudaDeviceSynchronize();
+    return free_all();
+}
+
+int gallatin_reset(void *stream) {
+    if (!g.init) return GALLATIN_ERR_STATE;
+    uint64_t n = g.v.nseg * 128;
+    if ((uint64_t)g.v.nslot_total * 16 > n) n = (uint64_t)g.v.nslot_total * 16;
+    unsigned grid = grid_for(n);
+    if (grid > 148 * 16) grid = 148 * 16;
+    k_reset<<<grid, kThreads, 0, S(stream)>>>(g.v);
+    return launch_status();
+}
+
+int gallatin_malloc(const uint64_t *d_sizes, void **d_ptrs, uint64_t n, void *stream) {
+    if (!g.init) return GALLATIN_ERR_STATE;
+    if (n == 0) return GALLATIN_OK;
+    if (!d_sizes || !d_ptrs || n > (1ull << 40)) return GALLATIN_ERR_INVALID;
+    k_bulk_malloc<<<grid_for(n), kThreads, 0, S(stream)>>>(g.v, d_sizes, d_ptrs, n);
+    return launch_status();
+}
+
+int gallatin_free(void *const *d_ptrs, uint64_t n, void *stream) {
+    if (!g.init) return GALLATIN_ERR_STATE;
+    if (n == 0) return GALLATIN_OK;
+    if (!d_ptrs || n > (1ull << 40)) return GALLATIN_ERR_INVALID;
+    k_bulk_free<<<grid_for(n), kThreads, 0, S(stream)>>>(g.v, d_ptrs, n);
+    return launch_status();
+}
+
+static int ensure_scratch(uint64_t bytes) {
+    if (g.scratch_bytes >= bytes) return GALLATIN_OK;
+    if (g.scratch) cudaFree(g.scratch);
+    g.scratch = nullptr;
+    g.scratch_bytes = 0;
+    if (cudaMalloc(&g.scratch, bytes) != cudaSuccess) { cudaGetLastError(); return GALLATIN_ERR_NOMEM; }
+    g.scratch_bytes = bytes;
+    return GALLATIN_OK;
+}
+
+int gallatin_malloc_host(const uint64_t *h_sizes, uint64_t *h_ptrs, uint64_t n, void *stream) {
+    if (!g.init) return GALLATIN_ERR_STATE;
+    if (n == 0) return GALLATIN_OK;
+    if (!h_sizes || !h_ptrs) return GALLATIN_ERR_INVALID;
+    int rc = ensure_scratch(16 * n);
+    if (rc) return rc;
+    uint64_t *d_sizes = static_cast<uint64_t *>(g.scratch);
+    void **d_ptrs = reinterpret_cast<void **>(d_sizes + n);
+    CUDA_TRY(cudaMemcpyAsync(d_sizes, h_sizes, 8 * n, cudaMemcpyHostToDevice, S(stream)));
+    rc = gallatin_malloc(d_sizes, d_ptrs, n, stream);
+    if (rc) return rc;
+    CUDA_TRY(cudaMemcpyAsync(h_ptrs, d_ptrs, 8 * n, cudaMemcpyDeviceToHost, S(stream)));
+    CUDA_TRY(cudaStreamSynchronize(S(stream)));
+    return GALLATIN_OK;
+}
+
+int gallatin_free_host(const uint64_t *h_ptrs, uint64_t n, void *stream) {
+    if (!g.init) return GALLATIN_ERR_STATE;
+    if (n == 0) return GALLATIN_OK;
+    if (!h_ptrs) return GALLATIN_ERR_INVALID;
+    int rc = ensure_scratch(16 * n);
+    if (rc) return rc;
+    void **d_ptrs = static_cast<void **>(g.scratch);
+    CUDA_TRY(cudaMemcpyAsync(d_ptrs, h_ptrs, 8 * n, cudaMemcpyHostToDevice, S(stream)));
+    rc = gallatin_free(d_ptrs, n, stream);
+    if (rc) return rc;
+    CUDA_TRY(cudaStreamSynchronize(S(stream)));
+    return GALLATIN_OK;
+}
+
+int gallatin_drain(void *stream) {
+    if (!g.init) return GALLATIN_ERR_STATE;
+    k_drain<<<1, 1, 0, S(stream)>>>(g.v);
+    return launch_status();
+}
+
+int gallatin_replay(const uint8_t *d_kinds, const uint64_t *d_args, const uint64_t *d_keys, uint64_t n,
+                    uint64_t *d_out, void *stream) {
+    if (!g.init) return GALLATIN_ERR_STATE;
+    if (n == 0) return GALLATIN_OK;
+    if (!d_kinds || !d_args || !d_keys || !d_out) return GALLATIN_ERR_INVALID;
+    k_replay<<<1, 1, 0, S(stream)>>>(g.v, d_kinds, d_args, d_keys, n, d_out);
+    return launch_status();
+}
+
+int gallatin_snapshot_words(uint64_t *words) {
+    if (!g.init) return GALLATIN_ERR_STATE;
+    if (!words) return GALLATIN_ERR_INVALID;
+    *words = image_words(g.v);
+    return GALLATIN_OK;
+}
+
+int gallatin_snapshot(uint64_t *out, uint64_t cap, uint64_t *len) {
+    if (!g.init) return GALLATIN_ERR_STATE;
+    const View &v = g.v;
+    const uint64_t need = image_words(v);
+    if (len) *len = need;
+    if (!out || cap < need) return GALLATIN_ERR_INVALID;
+    HostCopy h;
+    int rc = copy_state(h);
+    if (rc) return rc;
+    uint64_t *p = out;
+    p[0] = 0x47414C4C494D4731ull;
+    p[1] = v.nseg;
+    p[2] = v.tree_levels;
+    p[3] = v.tree_words;
+    p[4] = v.nslot_total;
+    p[5] = h.err;
+    p[6] = 0;
+    p[7] = 0;
+    p += 8;
+    memcpy(p, h.seg_tree.data(), v.tree_words * 8ull);
+    p += v.tree_words;
+    memcpy(p, h.block_trees.data(), 9ull * v.tree_words * 8);
+    p += 9ull * v.tree_words;
+    for (uint64_t s = 0; s < v.nseg; s++) {
+        const uint64_t w = h.seg_word[s];
+        *p++ = (w & 0xFFFFFFFF00000000ull) | (uint32_t)((uint32_t)w - core::kAvailBias);
+    }
+    for (uint64_t s = 0; s < v.nseg; s++) {
+        const uint32_t cnt = h.q_tail[s] - h.q_head[s];
+        *p++ = cnt;
+        uint16_t e[256];
+        for (uint32_t q = 0; q < 256; q++) e[q] = q < cnt ? h.q_entries[s * 256 + ((h.q_head[s] + q) & 255)] : 0xFFFF;
+        for (uint32_t q = 0; q < 64; q++)
+            *p++ = (uint64_t)e[4 * q] | ((uint64_t)e[4 * q + 1] << 16) | ((uint64_t)e[4 * q + 2] << 32) |
+                   ((uint64_t)e[4 * q + 3] << 48);
+    }
+    memcpy(p, h.block_free.data(), v.nseg * 1024);
+    p += v.nseg * 128;
+    for (uint32_t i = 0; i < v.nslot_total; i++) *p++ = h.slots[(uint64_t)i * 16];
+    for (uint32_t i = 0; i < v.nslot_total; i++) *p++ = (uint32_t)h.slots[(uint64_t)i * 16 + 1];
+    return GALLATIN_OK;
+}
+
+int gallatin_stats(gallatin_stats_t *out) {
+    if (!g.init) return GALLATIN_ERR_STATE;
+    if (!out) return GALLATIN_ERR_INVALID;
+    HostCopy h;
+    int rc = copy_state(h);
+    if (rc) return rc;
+    memset(out, 0, sizeof(*out));
+    const View &v = g.v;
+    out->heap_base = v.heap;
+    out->heap_bytes = v.nseg << core::kSegLog2;
+    out->num_segments = v.nseg;
+    for (uint64_t s = 0; s < v.nseg; s++) {
+        if ((h.seg_tree[s >> 6] >> (s & 63)) & 1) out->free_segments++;
+        const uint32_t t = (uint32_t)(h.seg_word[s] >> 32);
+        if (t < core::kTrees) out->tree_segments[t]++;
+        else if (t != core::kTreeFree) out->large_segments++;
+    }
+    out->errors = h.err;
+    for (int c = 0; c < 9; c++) out->nslot[c] = v.nslot[c];
+    out->theta = v.theta;
+    out->fence_free = v.fence_free;
+    return GALLATIN_OK;
+}
+
+uint64_t gallatin_device_view_bytes(void) { return sizeof(gallatin_device_view); }
+
+int gallatin_get_device_view(struct gallatin_device_view *out, uint64_t out_bytes) {
+    if (!g.init) return GALLATIN_ERR_STATE;
+    if (!out || out_bytes != sizeof(gallatin_device_view)) return GALLATIN_ERR_INVALID;
+    *out = g.v;
+    return GALLATIN_OK;
+}
+
+int gallatin_stamp(void *const *d_ptrs, const uint64_t *d_sizes, uint64_t n, void *stream) {
+    if (n == 0) return GALLATIN_OK;
+    if (!d_ptrs || !d_sizes) return GALLATIN_ERR_INVALID;
+    const uint64_t threads = (n + 31) / 32 * 32;
+    k_stamp<<<grid_for(threads), kThreads, 0, S(stream)>>>(d_ptrs, d_sizes, n);
+    return launch_status();
+}
+
+int gallatin_verify(void *const *d_ptrs, const uint64_t *d_sizes, uint64_t n, uint64_t *d_bad, void *stream) {
+    if (n == 0) return GALLATIN_OK;
+    if (!d_ptrs || !d_sizes || !d_bad) return GALLATIN_ERR_INVALID;
+    const uint64_t threads = (n + 31) / 32 * 32;
+    k_verify<<<grid_for(threads), kThreads, 0, S(stream)>>>(d_ptrs, d_sizes, n,
+                                                           reinterpret_cast<unsigned long long *>(d_bad));
+    return launch_status();
+}
+
+int gallatin_usable(void *const *d_ptrs, const uint64_t *d_sizes, uint64_t n, uint64_t *d_usable, uint64_t *d_sum,
+                    uint64_t *d_bad, void *stream) {
+    if (!g.init) return GALLATIN_ERR_STATE;
+    if (n == 0) return GALLATIN_OK;
+    if (!d_ptrs || !d_sizes || !d_sum || !d_bad) return GALLATIN_ERR_INVALID;
+    k_usable<<<grid_for(n), kThreads, 0, S(stream)>>>(g.v, d_ptrs, d_sizes, n, d_usable,
+                                                     reinterpret_cast<unsigned long long *>(d_sum),
+                                                     reinterpret_cast<unsigned long long *>(d_bad));
+    return launch_status();
+}
+
+}  // extern "C"

@@ -1,0 +1,191 @@
+"""GPU parity of the allocator (C-ABI gallatin_*) against O2 and the paper's invariants.
+
+* Serialized replay (one GPU thread, slot key = the op's key): every pointer
+  offset and the final metadata image equal O2's bit-exactly.
+* Concurrent bulk runs (address assignment is nondeterministic, reading A-30):
+  stamp-and-verify finds 0 overwritten words, the sorted pointers never
+  overlap, every pointer is aligned and in the heap, the usable bytes read from
+  the memory table equal the closed form and O2's accounting, and free-all +
+  drain restores the pristine image bit-exactly (== O2's == analytic).
+"""
+import numpy as np
+import pytest
+import torch
+
+import oracle
+import workload_gen as wg
+from helpers import SEG, class_size, diff_images, pristine_image
+
+pytestmark = pytest.mark.gpu
+NONE = (1 << 64) - 1
+
+
+def _dev(a, dtype=np.uint64):
+    a = np.ascontiguousarray(a, dtype=dtype)
+    return torch.from_numpy(a.view(np.int64) if a.dtype.itemsize == 8 else a).cuda()
+
+
+def _u64(t):
+    return t.cpu().numpy().view(np.uint64)
+
+
+@pytest.fixture()
+def G():
+    import paper_conf_ppopp_mccoyp24_b200 as G
+    yield G
+    if G.gallatin_is_initialized():
+        G.gallatin_destroy()
+
+
+def _replay_case(G, nseg, theta, kinds, args, keys, slot_base=16, slot_min=2):
+    G.gallatin_init(nseg * SEG, slot_base=slot_base, slot_min=slot_min, theta=theta)
+    out = _u64(G.gallatin_replay(_dev(kinds, np.uint8), _dev(args), _dev(keys)))
+    o2 = oracle.Allocator(nseg, slot_base=slot_base, slot_min=slot_min, theta=theta)
+    want = o2.replay(kinds, args, keys)
+    bad = np.nonzero(out != want)[0]
+    assert len(bad) == 0, f"{len(bad)} ops differ; first op {bad[0]} kind {kinds[bad[0]]} size {args[bad[0]]}: " \
+                          f"gpu {out[bad[0]]:#x} oracle {want[bad[0]]:#x}"
+    msg = diff_images(G.gallatin_snapshot(), o2.image())
+    assert not msg, msg
+    G.gallatin_destroy()
+    return out
+
+
+@pytest.mark.parametrize("seed,nseg,theta", [(1, 4, 0), (2, 8, 0), (3, 6, 2048), (4, 64, 0), (5, 5, 100),
+                                             (6, 16, 0), (7, 3, 4095)])
+def test_serialized_replay_matches_oracle(cuda_ok, G, seed, nseg, theta):
+    """Mixed slices / blocks / multi-segment allocations, interleaved frees,
+    drains and OOM on 3-64 segment heaps (SURVEY 8(c) "Scope of serialized replay")."""
+    kinds, args, keys = wg.replay_ops(6000, seed + 100, p_free=0.45, p_drain=0.003, nkeys=64)
+    _replay_case(G, nseg, theta, kinds, args, keys)
+
+
+def test_serialized_replay_block_boundaries(cuda_ok, G):
+    """Exactly-full blocks, exhausted slots, refill and prefetch edges with a
+    single slot per class (every request hits the same slot)."""
+    n = 3 * 4096 + 7
+    kinds = np.zeros(n, dtype=np.uint8)
+    args = np.full(n, 16, dtype=np.uint64)
+    keys = np.zeros(n, dtype=np.uint64)
+    kinds2 = np.concatenate([kinds, np.ones(4096, dtype=np.uint8), np.array([2], dtype=np.uint8)])
+    args2 = np.concatenate([args, np.arange(4096, dtype=np.uint64), np.array([0], dtype=np.uint64)])
+    keys2 = np.concatenate([keys, np.zeros(4097, dtype=np.uint64)])
+    for theta in (0, 1, 4095):
+        _replay_case(G, 2, theta, kinds2, args2, keys2, slot_base=1, slot_min=1)
+
+
+def _bulk_round(G, nseg, sizes, check_accounting=True):
+    """malloc -> stamp -> verify -> usable/overlap checks -> free; returns #NULL."""
+    d_sizes = _dev(sizes)
+    ptrs = G.gallatin_malloc(d_sizes)
+    torch.cuda.synchronize()
+    p = _u64(ptrs)
+    null = p == 0
+    st = G.gallatin_stats()
+    base = st["heap_base"]
+    G.gallatin_stamp(ptrs, d_sizes)
+    assert G.gallatin_verify(ptrs, d_sizes) == 0, "stamp-verify found overwritten words"
+    usable = torch.empty_like(ptrs)
+    usum, ubad = G.gallatin_usable(ptrs, d_sizes, usable)
+    assert ubad == 0, f"{ubad} pointers contradict their size class / alignment"
+    if check_accounting:
+        want = int(sum(class_size(int(s)) * int(c) for s, c in zip(*np.unique(sizes[~null], return_counts=True))))
+        assert usum == want, f"usable {usum} != closed form {want}"
+    # no overlap: sort live pointers, each ends before the next begins
+    live = ~null
+    order = np.argsort(p[live])
+    sp, su = p[live][order], _u64(usable)[live][order]
+    assert np.all(sp[:-1] + su[:-1] <= sp[1:]), "overlapping allocations"
+    assert np.all((sp - np.uint64(base)) < np.uint64(nseg * SEG))
+    G.gallatin_free(ptrs)
+    torch.cuda.synchronize()
+    return int(null.sum())
+
+
+def _assert_pristine(G, nseg):
+    G.gallatin_drain()
+    img = G.gallatin_snapshot()
+    S = int(img[4])
+    msg = diff_images(img, pristine_image(nseg, S))
+    assert not msg, msg
+
+
+def test_config1_concurrent(cuda_ok, G):
+    """BASELINE configs[0]: 64 MB heap, 2^16 threads malloc 16 B then free."""
+    nseg = 4
+    G.gallatin_init(nseg * SEG)
+    sizes = wg.single_sizes(16, 1 << 16)
+    assert _bulk_round(G, nseg, sizes) == 0
+    _assert_pristine(G, nseg)
+    # accounting equals O2's on the same sizes
+    o2 = oracle.Allocator(nseg)
+    o2.malloc_batch(sizes)
+    assert o2.usable_live == (1 << 16) * 16
+
+
+@pytest.mark.parametrize("size", wg.SLICE_SIZES)
+def test_config2_single_size_reduced(cuda_ok, G, size):
+    """BASELINE configs[1] shape at 2^20 threads on the 16 GB heap."""
+    nseg = 1024
+    G.gallatin_init(nseg * SEG)
+    for rep in range(2):                     # second round: warm (no reset)
+        assert _bulk_round(G, nseg, wg.single_sizes(size, 1 << 20)) == 0
+        _assert_pristine(G, nseg)
+
+
+def test_config3_mixed_reduced(cuda_ok, G):
+    """BASELINE configs[2] shape: random 16 B-4 KB plus 1-64 MB large
+    allocations (p = 2^-12) at 2^20 threads on a 64 GB heap."""
+    nseg = 4096
+    G.gallatin_init(nseg * SEG)
+    sizes = wg.mixed_sizes(1 << 20)
+    assert (sizes > 4096).sum() > 100
+    assert _bulk_round(G, nseg, sizes) == 0
+    _assert_pristine(G, nseg)
+    sizes_b = wg.mixed_sizes(1 << 20, seed=wg.cell_seed(3, 1), exact_pow2=False, p_large=2.0 ** -10)
+    assert _bulk_round(G, nseg, sizes_b) == 0
+    _assert_pristine(G, nseg)
+
+
+def test_oom_capacity_and_recovery(cuda_ok, G):
+    """A 4-segment heap asked for 4x its capacity: NULLs, no overlap, and after
+    freeing everything the heap is pristine (P:274 nullptr on exhaustion)."""
+    nseg = 4
+    G.gallatin_init(nseg * SEG)
+    sizes = wg.single_sizes(1024, 1 << 18)          # 256 MiB requested, 64 MiB heap
+    nulls = _bulk_round(G, nseg, sizes, check_accounting=False)
+    assert nulls >= (1 << 18) - nseg * SEG // 1024
+    _assert_pristine(G, nseg)
+    sizes = wg.mixed_sizes(1 << 16, p_large=2.0 ** -6)
+    _bulk_round(G, nseg, sizes, check_accounting=False)
+    _assert_pristine(G, nseg)
+
+
+def test_bad_frees_counted(cuda_ok, G):
+    G.gallatin_init(4 * SEG)
+    base = G.gallatin_stats()["heap_base"]
+    bad = np.array([base + 9 * SEG, base + 2 * SEG + 64, 0], dtype=np.uint64)   # outside; FREE segment; NULL
+    G.gallatin_free(_dev(bad))
+    torch.cuda.synchronize()
+    assert G.gallatin_stats()["errors"] == 2
+
+
+def test_host_buffer_api(cuda_ok, G):
+    nseg = 16
+    G.gallatin_init(nseg * SEG)
+    sizes = wg.mixed_sizes(1 << 14, p_large=0.0)
+    p = G.gallatin_malloc_host(sizes)
+    assert np.all(p != 0)
+    o = np.sort(p)
+    assert len(np.unique(o)) == len(o)
+    G.gallatin_free_host(p)
+    _assert_pristine(G, nseg)
+
+
+def test_reset_restores_pristine(cuda_ok, G):
+    nseg = 8
+    G.gallatin_init(nseg * SEG)
+    G.gallatin_malloc(_dev(wg.mixed_sizes(1 << 14, p_large=2.0 ** -8)))
+    G.gallatin_reset()
+    img = G.gallatin_snapshot()
+    assert not diff_images(img, pristine_image(nseg, int(img[4])))

@@ -1,0 +1,138 @@
+"""GPU parity of the concurrent vEB bitmap tree (C-ABI veb_*) against O1.
+
+BASELINE north_star: "vEB successor/insert/delete results for the same op
+batches" bit-exact vs the CPU oracle; final level words bit-exact (SURVEY
+8(c): leaf words = O1 membership, summaries = OR reduction at quiescence).
+"""
+import numpy as np
+import pytest
+import torch
+
+import oracle
+import workload_gen as wg
+from oracle import NONE, OV_DELETE, OV_INSERT, OV_MEMBER, OV_PRED, OV_SUCC
+
+pytestmark = pytest.mark.gpu
+
+
+def _dev(a):
+    return torch.from_numpy(np.ascontiguousarray(a, dtype=np.uint64).view(np.int64)).cuda()
+
+
+def _u64(t):
+    return t.cpu().numpy().view(np.uint64)
+
+
+def _run_batches(k, batches):
+    """Apply the same homogeneous batches to the GPU tree and to O1; compare
+    every per-op output and the final image."""
+    import paper_conf_ppopp_mccoyp24_b200 as G
+    g = G.Veb(k)
+    o = oracle.Veb(k)
+    for op, keys in batches:
+        d = _dev(keys)
+        want = o.batch(op, keys)
+        if op == OV_INSERT:
+            got = g.insert(d).cpu().numpy().astype(np.uint64)
+        elif op == OV_DELETE:
+            got = g.delete(d).cpu().numpy().astype(np.uint64)
+        elif op == OV_MEMBER:
+            got = g.member(d).cpu().numpy().astype(np.uint64)
+        elif op == OV_SUCC:
+            got = _u64(g.successor(d))
+        else:
+            got = _u64(g.predecessor(d))
+        bad = np.nonzero(got != want)[0]
+        assert len(bad) == 0, f"op {op}: {len(bad)} mismatches, e.g. key {keys[bad[:3]]} got {got[bad[:3]]} want {want[bad[:3]]}"
+    torch.cuda.synchronize()
+    img_g, img_o = g.snapshot(), o.image()
+    assert np.array_equal(img_g, img_o), f"image differs at words {np.nonzero(img_g != img_o)[0][:8]}"
+    g.close()
+
+
+def test_config1_veb_parity(cuda_ok):
+    """BASELINE configs[0]: 2^16 random insert / successor / delete on a 2^20
+    universe, plus pred/member of the same queries."""
+    w = wg.veb_workload(20, 1 << 16)
+    _run_batches(20, [
+        (OV_SUCC, w["succ1"]),                     # empty tree: all none
+        (OV_INSERT, w["insert"]),
+        (OV_SUCC, w["succ1"]),
+        (OV_PRED, w["succ1"]),
+        (OV_MEMBER, w["succ1"]),
+        (OV_DELETE, w["delete"]),
+        (OV_SUCC, w["succ2"]),
+        (OV_PRED, w["succ2"]),
+    ])
+
+
+@pytest.mark.parametrize("k", [1, 3, 6, 7, 12, 13, 18, 19, 24])
+def test_universe_sizes(cuda_ok, k):
+    """Every level count (1..5) incl. partial top words; dense and sparse sets."""
+    u = 1 << k
+    n = min(u, 1 << 15)
+    seed = wg.cell_seed(1, 200 + k)
+    ins = wg.distinct_below(seed, n, u)
+    q = np.concatenate([wg.uniform_below(seed ^ 1, 4096, u), np.array([0, u - 1, u, u + 7], dtype=np.uint64)])
+    dele = ins[: n // 2]
+    _run_batches(k, [(OV_INSERT, ins), (OV_SUCC, q), (OV_PRED, q), (OV_DELETE, dele), (OV_SUCC, q),
+                     (OV_PRED, q), (OV_MEMBER, q), (OV_DELETE, ins), (OV_SUCC, q)])
+
+
+def test_universe_2_32_sampled(cuda_ok):
+    k = 32
+    seed = wg.cell_seed(1, 232)
+    ins = np.unique(wg.uniform_below(seed, 1 << 14, 1 << 32))
+    q = wg.uniform_below(seed ^ 9, 1 << 14, 1 << 32)
+    _run_batches(k, [(OV_INSERT, ins), (OV_SUCC, q), (OV_PRED, q), (OV_DELETE, ins[::3]), (OV_SUCC, q)])
+
+
+def test_duplicate_keys_exactly_one_reports(cuda_ok):
+    """Reading A-23: with repeated keys in one batch, exactly one op per
+    distinct key reports 'newly added' / 'was present'."""
+    import paper_conf_ppopp_mccoyp24_b200 as G
+    k = 16
+    rng = np.random.Generator(np.random.PCG64(3))
+    keys = rng.integers(0, 1 << 12, size=1 << 16).astype(np.uint64)     # heavy duplication
+    g = G.Veb(k)
+    got = g.insert(_dev(keys)).cpu().numpy()
+    uniq = np.unique(keys)
+    per_key = np.bincount(keys.astype(np.int64), weights=got, minlength=1 << 12)
+    assert got.sum() == len(uniq) and np.all(per_key[uniq.astype(np.int64)] == 1)
+    o = oracle.Veb(k)
+    o.batch(OV_INSERT, keys)
+    assert np.array_equal(g.snapshot(), o.image())
+    got = g.delete(_dev(keys)).cpu().numpy()
+    per_key = np.bincount(keys.astype(np.int64), weights=got, minlength=1 << 12)
+    assert got.sum() == len(uniq) and np.all(per_key[uniq.astype(np.int64)] == 1)
+    assert not g.snapshot().any()
+
+
+def test_concurrent_insert_delete_quiescent_exact(cuda_ok):
+    """Inserts and deletes of disjoint key sets racing on different streams
+    hammer the same leaf words; at quiescence every summary word must equal the
+    OR of its children and the leaves must equal the set semantics."""
+    import paper_conf_ppopp_mccoyp24_b200 as G
+    k = 14
+    u = 1 << k
+    g = G.Veb(k)
+    evens = np.arange(0, u, 2, dtype=np.uint64)
+    odds = np.arange(1, u, 2, dtype=np.uint64)
+    g.insert(_dev(odds), want_out=False)
+    torch.cuda.synchronize()
+    s1, s2 = torch.cuda.Stream(), torch.cuda.Stream()
+    de, do = _dev(evens), _dev(odds)
+    for _ in range(20):
+        with torch.cuda.stream(s1):
+            g.insert(de, want_out=False, stream=s1.cuda_stream)
+        with torch.cuda.stream(s2):
+            g.delete(do, want_out=False, stream=s2.cuda_stream)
+        torch.cuda.synchronize()
+        with torch.cuda.stream(s1):
+            g.delete(de, want_out=False, stream=s1.cuda_stream)
+        with torch.cuda.stream(s2):
+            g.insert(do, want_out=False, stream=s2.cuda_stream)
+        torch.cuda.synchronize()
+    o = oracle.Veb(k)
+    o.batch(OV_INSERT, odds)
+    assert np.array_equal(g.snapshot(), o.image())
