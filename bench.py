@@ -1,0 +1,468 @@
+#!/usr/bin/env python
+"""Benchmark of the Gallatin hot path on B200 (BASELINE.json metric:
+"malloc+free ops/s per B200 (single/mixed size); vEB successor ops/s").
+
+Workload at N=1: BASELINE configs[1], the single-size sweep (PAPER.md S6.5,
+P:309-315) on a 16 GB heap: one STEP = for every slice size s in 16 B..4 KB,
+reset the allocator, n_s = min(2^24, 8 GiB / s) threads each malloc(s)
+(bulk kernel), then the same threads free.  value = (malloc + free ops) / time.
+The line also carries the mixed-size cell (configs[2] shape, 2^22 threads on a
+64 GB heap) and the vEB successor throughput (configs[0] tree, 2^24 queries).
+
+Multi-GPU: one process per GPU (torchrun), independent per-GPU heaps ("replicas
+only"); value = all ranks' ops / max-over-ranks time.
+
+--impl reference times the CPU oracle (oracle/, O2) on a bounded sample of the
+same workload (the reference arm of this tier: a deliberately slow program).
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import numpy as np  # noqa: E402
+
+SEG = 1 << 24
+HEAP_C2 = 16 << 30
+HEAP_C3 = 64 << 30
+SIZES = [16 << i for i in range(9)]
+
+
+def cells_c2(scale: int = 1):
+    """(size, threads) of the sweep: 2^20..2^24 threads, capped so that s*n <= 8 GiB
+    (the feasible cells of SURVEY 8(d) C2); the largest feasible n per size."""
+    return [(s, min(1 << 24, (8 << 30) // s) // scale) for s in SIZES]
+
+
+# ------------------------------------------------------------------ clocks ---
+class ClockSampler:
+    """nvidia-smi clocks + throttle reasons sampled DURING the timed region."""
+    FIELDS = ("clocks.sm,clocks.max.sm,clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+              "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, index: int):
+        self.index = index
+        self.rows: list[list[str]] = []
+        self.proc = None
+        self.thread = None
+
+    def start(self):
+        try:
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", "-i", str(self.index), f"--query-gpu={self.FIELDS}", "--format=csv,noheader,nounits",
+                 "-lms", "100"], stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+        except Exception:
+            self.proc = None
+            return
+        self.thread = threading.Thread(target=self._read, daemon=True)
+        self.thread.start()
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.rows.append([x.strip() for x in line.split(",")])
+
+    def stop(self) -> dict:
+        if self.proc is None:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        time.sleep(0.25)
+        self.proc.terminate()
+        try:
+            self.proc.wait(timeout=5)
+        except Exception:
+            self.proc.kill()
+        if self.thread:
+            self.thread.join(timeout=2)
+        rows = [r for r in self.rows if len(r) >= 6 and r[0].replace(".", "").isdigit()]
+        if not rows:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["no samples"], "samples": 0}
+        sm = [float(r[0]) for r in rows]
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = sorted({names[i] for r in rows for i in range(4) if r[2 + i].lower().startswith("active")})
+        return {"sm_mhz": statistics.median(sm), "sm_max_mhz": float(rows[0][1]), "reasons": reasons,
+                "samples": len(rows)}
+
+
+# ------------------------------------------------------------- distributed ---
+def dist_setup(ngpus: int):
+    rank = int(os.environ.get("RANK", "0"))
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    if world != ngpus and world > 1:
+        raise SystemExit(f"--gpus {ngpus} but WORLD_SIZE={world}")
+    return rank, world, local
+
+
+class Dist:
+    def __init__(self, rank, world, backend):
+        self.rank, self.world = rank, world
+        self.pg = None
+        if world > 1:
+            import torch.distributed as dist
+            dist.init_process_group(backend)
+            self.pg = dist
+
+    def barrier(self):
+        if self.pg:
+            self.pg.barrier()
+
+    def max(self, x: float) -> float:
+        if not self.pg:
+            return x
+        import torch
+        t = torch.tensor([x], dtype=torch.float64, device="cuda" if torch.cuda.is_available() else "cpu")
+        self.pg.all_reduce(t, op=self.pg.ReduceOp.MAX)
+        return float(t.item())
+
+    def sum(self, x: float) -> float:
+        if not self.pg:
+            return x
+        import torch
+        t = torch.tensor([x], dtype=torch.float64, device="cuda" if torch.cuda.is_available() else "cpu")
+        self.pg.all_reduce(t, op=self.pg.ReduceOp.SUM)
+        return float(t.item())
+
+    def close(self):
+        if self.pg:
+            self.pg.destroy_process_group()
+
+
+def peaks_file() -> dict:
+    try:
+        return json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))
+    except Exception:
+        return {}
+
+
+# ------------------------------------------------------------- our arm -------
+def run_ours(args, rank, world, local):
+    import torch
+    import paper_conf_ppopp_mccoyp24_b200 as G
+
+    torch.cuda.set_device(local)
+    d = Dist(rank, world, "nccl")
+    stream = torch.cuda.current_stream()
+    cells = cells_c2(args.scale)
+
+    G.gallatin_init(HEAP_C2)
+    size_t = [torch.full((n,), s, dtype=torch.int64, device="cuda") for s, n in cells]
+    nmax = max(n for _, n in cells)
+    ptrs = torch.empty(nmax, dtype=torch.int64, device="cuda")
+    ops_per_step = sum(2 * n for _, n in cells)
+
+    ev = {"m0": [], "m1": [], "f0": [], "f1": []}
+
+    def step(record: bool):
+        for (s, n), st in zip(cells, size_t):
+            p = ptrs[:n]
+            G.gallatin_reset()
+            if record:
+                e = torch.cuda.Event(enable_timing=True); e.record(stream); ev["m0"].append(e)
+            G.gallatin_malloc(st, p)
+            if record:
+                e = torch.cuda.Event(enable_timing=True); e.record(stream); ev["m1"].append(e)
+                e = torch.cuda.Event(enable_timing=True); e.record(stream); ev["f0"].append(e)
+            G.gallatin_free(p)
+            if record:
+                e = torch.cuda.Event(enable_timing=True); e.record(stream); ev["f1"].append(e)
+
+    # correctness gate on the bench's own launch configuration (untimed): the
+    # first cell's pointers stamp/verify clean and the heap drains to pristine
+    for w in range(max(args.warmup, 3)):
+        step(False)
+    torch.cuda.synchronize()
+    (s0, n0), st0 = cells[0], size_t[0]
+    G.gallatin_reset()
+    G.gallatin_malloc(st0, ptrs[:n0])
+    G.gallatin_stamp(ptrs[:n0], st0)
+    bad = G.gallatin_verify(ptrs[:n0], st0)
+    G.gallatin_free(ptrs[:n0])
+    torch.cuda.synchronize()
+    if bad:
+        raise SystemExit(f"stamp-verify failed: {bad} words")
+
+    clk = ClockSampler(local)
+    d.barrier()
+    torch.cuda.synchronize()
+    clk.start()
+    t0 = torch.cuda.Event(enable_timing=True)
+    t1 = torch.cuda.Event(enable_timing=True)
+    t0.record(stream)
+    for _ in range(args.steps):
+        step(True)
+    t1.record(stream)
+    torch.cuda.synchronize()
+    clocks = clk.stop()
+    d.barrier()
+    ms_local = t0.elapsed_time(t1)
+    ms = d.max(ms_local)
+    total_ops = d.sum(ops_per_step * args.steps)
+    value = total_ops / (ms / 1e3)
+
+    # per-kernel times (the roofline's dominant kernel)
+    m_ms = [a.elapsed_time(b) for a, b in zip(ev["m0"], ev["m1"])]
+    f_ms = [a.elapsed_time(b) for a, b in zip(ev["f0"], ev["f1"])]
+    nsum = sum(n for _, n in cells) * args.steps
+    malloc_ops_s = nsum / (sum(m_ms) / 1e3)
+    free_ops_s = nsum / (sum(f_ms) / 1e3)
+    per_cell = {}
+    for i, (s, n) in enumerate(cells):
+        mm = statistics.median(m_ms[i::len(cells)])
+        fm = statistics.median(f_ms[i::len(cells)])
+        per_cell[str(s)] = {"n": n, "malloc_ms": round(mm, 4), "free_ms": round(fm, 4),
+                            "malloc_ops_s": n / mm * 1e3, "free_ops_s": n / fm * 1e3}
+    dominant = "malloc" if sum(m_ms) >= sum(f_ms) else "free"
+    bytes_per_op = 16 if dominant == "malloc" else 8
+    kern_ms = sum(m_ms) if dominant == "malloc" else sum(f_ms)
+    achieved = nsum * bytes_per_op / (kern_ms / 1e3) / 1e9
+    pk = peaks_file()
+    hbm_peak = pk.get("hbm_gbs")
+    peak_src = "MEASURED_PEAKS.json hbm_gbs"
+    if not hbm_peak:
+        hbm_peak, peak_src = 6650.0, "B200_PROFILING.md fallback"
+    traffic = None
+    tf = os.path.join(ROOT, "profiles", "traffic.json")
+    if os.path.exists(tf):
+        try:
+            traffic = json.load(open(tf)).get(f"k_bulk_{dominant}")
+        except Exception:
+            traffic = None
+
+    extras = {}
+    if not args.no_extras:
+        extras = run_extras(args, G, torch, stream)
+
+    # e2e through the C-ABI with HOST buffers (pinned), copies inside the timed region
+    e2e = run_e2e(args, G, torch, cells)
+
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu:
+        cpu = cpu_baseline(args)
+
+    G.gallatin_destroy()
+    if rank == 0:
+        line = {
+            "metric": "malloc+free ops/s per B200 (single-size sweep 16 B-4 KB)",
+            "value": value, "unit": "ops/s", "n_gpus": world, "steps": args.steps, "warmup": max(args.warmup, 3),
+            "ms_per_step": ms / args.steps, "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
+            "dtype": "u64", "data": "synthetic",
+            "config": {"workload": "BASELINE configs[1]: single-size sweep 16 B-4 KB, n_s=min(2^24, 8GiB/s) threads, "
+                                   "16 GiB heap, reset+malloc+free per size" + (f" (1/{args.scale} scale)" if args.scale > 1 else ""),
+                       "heap_bytes": HEAP_C2, "cells": [[s, n] for s, n in cells],
+                       "ops_per_step": ops_per_step, "parallelism": f"replicas x{world}",
+                       "l2": "no flush: each step reads %.2f GiB of sizes + writes/reads the pointer array (> 126 MB L2)" % (
+                           sum(8 * n for _, n in cells) / 2 ** 30)},
+            "malloc_ops_s": malloc_ops_s, "free_ops_s": free_ops_s, "per_size": per_cell,
+            "roofline": {"bound": "hbm", "kernel": f"k_bulk_{dominant}", "achieved": achieved, "peak": hbm_peak,
+                         "unit": "GB/s", "frac": achieved / hbm_peak, "traffic": traffic,
+                         "algorithmic_bytes_per_op": bytes_per_op, "peak_source": peak_src},
+            "clocks": clocks,
+            "e2e": e2e,
+            "gpu_launches": 27 * args.steps,
+            "cpu_baseline": cpu,
+        }
+        line.update(extras)
+        print(json.dumps(line))
+    d.close()
+
+
+def run_extras(args, G, torch, stream):
+    """Mixed-size cell, vEB successor throughput, peak probes (not part of `value`)."""
+    import workload_gen as wg
+    out = {}
+    # --- vEB successor (configs[0] tree, 2^24 queries) ---
+    w = wg.veb_workload(20, 1 << 16)
+    v = G.Veb(20)
+    keys = torch.from_numpy(w["insert"].view(np.int64)).cuda()
+    nq = (1 << 24) // args.scale
+    q = torch.from_numpy(wg.uniform_below(wg.cell_seed(1, 7), nq, 1 << 20).view(np.int64)).cuda()
+    res = torch.empty_like(q)
+    v.insert(keys, want_out=False)
+    for _ in range(3):
+        v.successor(q, res)
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    reps = 20
+    e0.record(stream)
+    for _ in range(reps):
+        v.successor(q, res)
+    e1.record(stream)
+    torch.cuda.synchronize()
+    succ_ms = e0.elapsed_time(e1) / reps
+    # insert/delete throughput on the same universe
+    dk = torch.from_numpy(w["delete"].view(np.int64)).cuda()
+    v.clear()
+    e0.record(stream)
+    v.insert(keys, want_out=False)
+    e1.record(stream)
+    torch.cuda.synchronize()
+    ins_ms = e0.elapsed_time(e1)
+    e0.record(stream)
+    v.delete(dk, want_out=False)
+    e1.record(stream)
+    torch.cuda.synchronize()
+    del_ms = e0.elapsed_time(e1)
+    v.close()
+    out["veb"] = {"successor_ops_s": nq / succ_ms * 1e3, "successor_queries": nq, "successor_ms": succ_ms,
+                  "insert_ops_s": len(w["insert"]) / ins_ms * 1e3, "delete_ops_s": len(w["delete"]) / del_ms * 1e3,
+                  "universe": "2^20", "keys": len(w["insert"]),
+                  "successor_hbm_gbs": nq * 16 / succ_ms / 1e6}
+
+    # --- mixed-size cell (configs[2] shape) on its own 64 GiB heap ---
+    G.gallatin_destroy()
+    G.gallatin_init(HEAP_C3)
+    n = (1 << 22) // args.scale
+    sizes = torch.from_numpy(wg.mixed_sizes(n).view(np.int64)).cuda()
+    p = torch.empty_like(sizes)
+    mm, fm = [], []
+    for it in range(8):
+        G.gallatin_reset()
+        a, b, c = (torch.cuda.Event(enable_timing=True) for _ in range(3))
+        a.record(stream)
+        G.gallatin_malloc(sizes, p)
+        b.record(stream)
+        G.gallatin_free(p)
+        c.record(stream)
+        torch.cuda.synchronize()
+        if it >= 3:
+            mm.append(a.elapsed_time(b))
+            fm.append(b.elapsed_time(c))
+    m, f = statistics.median(mm), statistics.median(fm)
+    out["mixed"] = {"threads": n, "malloc_ops_s": n / m * 1e3, "free_ops_s": n / f * 1e3,
+                    "combined_ops_s": 2 * n / (m + f) * 1e3, "malloc_ms": m, "free_ms": f,
+                    "workload": "BASELINE configs[2]: 16 B-4 KB powers of two + p=2^-12 large 1-64 MB, 64 GiB heap"}
+    G.gallatin_destroy()
+    G.gallatin_init(HEAP_C2)
+
+    # --- peak probes ---
+    pk = {}
+    nt = 1 << 24
+    ms, ops = G.gallatin_probe(1, nt, 1 << 21)
+    pk["atom_distinct_ops_s"] = ops / ms * 1e3
+    for lines in (4, 37, 148):
+        ms, ops = G.gallatin_probe(2, nt, lines)
+        pk[f"atom_hot{lines}_ops_s"] = ops / ms * 1e3
+    ms, ops = G.gallatin_probe(4, nt, 148)
+    pk["bump_ceiling_ops_s"] = ops / ms * 1e3
+    ms, ops = G.gallatin_probe(5, nt, 1)
+    pk["fence_per_warp_ops_s"] = ops / ms * 1e3
+    ms, ops = G.gallatin_probe(6, 1 << 24, 1 << 30)
+    pk["hbm_copy_gbs"] = ops / ms / 1e6
+    out["probes"] = pk
+    return out
+
+
+def run_e2e(args, G, torch, cells):
+    """Same metric through gallatin_malloc_host / gallatin_free_host: the sizes are
+    copied host->device, the pointers device->host (malloc) and host->device (free)."""
+    host = []
+    for s, n in cells:
+        hs = torch.full((n,), s, dtype=torch.int64, pin_memory=True).numpy().view(np.uint64)
+        hp = torch.empty(n, dtype=torch.int64, pin_memory=True).numpy().view(np.uint64)
+        host.append((hs, hp))
+    steps = max(1, min(args.steps, 5))
+    for (hs, hp) in host:                                 # warm-up
+        G.gallatin_reset()
+        torch.cuda.synchronize()
+        G.gallatin_malloc_host(hs, hp)
+        G.gallatin_free_host(hp)
+    torch.cuda.synchronize()
+    t = time.perf_counter()
+    for _ in range(steps):
+        for (hs, hp) in host:
+            G.gallatin_reset()
+            G.gallatin_malloc_host(hs, hp)
+            G.gallatin_free_host(hp)
+    torch.cuda.synchronize()
+    dt = time.perf_counter() - t
+    ops = sum(2 * n for _, n in cells) * steps
+    return {"value": ops / dt, "unit": "ops/s", "h2d_bytes_per_step": sum(16 * n for _, n in cells),
+            "d2h_bytes_per_step": sum(8 * n for _, n in cells), "steps": steps,
+            "api": "gallatin_malloc_host/gallatin_free_host (pinned host arrays)"}
+
+
+# ---------------------------------------------------------- CPU oracle ------
+def cpu_sample(scale_div: int):
+    """The bounded oracle sample: every cell at 1/scale_div of its threads."""
+    return [(s, max(1, n // scale_div)) for s, n in cells_c2()]
+
+
+def time_oracle(cells, steps: int):
+    import oracle
+    import workload_gen as wg
+    os.sched_setaffinity(0, {sorted(os.sched_getaffinity(0))[0]})   # one host core
+    sizes = [wg.single_sizes(s, n) for s, n in cells]
+    total = 0.0
+    ops = 0
+    for _ in range(steps):
+        for (s, n), sz in zip(cells, sizes):
+            a = oracle.Allocator(HEAP_C2 // SEG)       # fresh = the paper's reset
+            t = time.perf_counter()
+            offs = a.malloc_batch(sz, keydiv=32)
+            a.free_batch(offs)
+            total += time.perf_counter() - t
+            ops += 2 * n
+            a.close()
+    return ops, total
+
+
+def cpu_baseline(args):
+    div = 8
+    cells = cpu_sample(div)
+    ops, sec = time_oracle(cells, 1)
+    return {"value": ops / sec, "unit": "ops/s", "cores": 1, "kind": "oracle",
+            "sample": f"O2 (oracle/alloc_oracle.c) on every cell of the sweep at 1/{div} of its threads "
+                      f"({ops // 2} mallocs + frees), one pinned host core", "seconds": sec}
+
+
+def run_reference(args, rank, world):
+    if rank != 0:
+        return
+    div = 8
+    cells = cpu_sample(div)
+    steps = max(1, min(args.steps, 3))
+    for _ in range(min(args.warmup, 1)):
+        time_oracle(cells[:1], 1)
+    ops, sec = time_oracle(cells, steps)
+    value = ops / sec
+    line = {
+        "impl": "reference",
+        "metric": "malloc+free ops/s per B200 (single-size sweep 16 B-4 KB)",
+        "value": value, "unit": "ops/s", "n_gpus": world, "steps": steps, "warmup": args.warmup,
+        "ms_per_step": sec / steps * 1e3, "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
+        "dtype": "u64", "data": "synthetic",
+        "config": {"workload": "BASELINE configs[1]: single-size sweep 16 B-4 KB, 16 GiB heap; the CPU oracle "
+                               f"runs each cell at 1/{div} of its threads", "cells": [[s, n] for s, n in cells]},
+        "cpu_baseline": {"value": value, "unit": "ops/s", "cores": 1, "kind": "oracle",
+                         "sample": f"every cell at 1/{div} of its threads, {steps} step(s), one pinned host core"},
+        "e2e": {"value": value, "unit": "ops/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }
+    print(json.dumps(line))
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=20)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--scale", type=int, default=1, help="divide every thread count (debug only)")
+    ap.add_argument("--no-extras", action="store_true")
+    ap.add_argument("--no-cpu", action="store_true")
+    args = ap.parse_args()
+    rank, world, local = dist_setup(args.gpus)
+    if args.impl == "reference":
+        run_reference(args, rank, world)
+        return
+    run_ours(args, rank, world, local)
+
+
+if __name__ == "__main__":
+    main()
