@@ -47,20 +47,27 @@ enum {
  *   slot_base  : block-buffer slots of the 16 B class; class c gets
  *                max(slot_min, slot_base >> c).  Default = #SMs (148).
  *   slot_min   : lower cap, default 4 ("capped at four").
- *   theta      : prefetch threshold: the request that takes slice index theta
- *                of a buffered block fetches the next block into the slot's
- *                side field (0 = off = the paper; not in the paper).
+ *   run_max    : a slot holds a RUN of up to run_max consecutive blocks (1..128,
+ *                default 16); the run starts at one block and doubles on every
+ *                refill of the slot.  1 = the paper's one-block buffer.
+ *   run_bytes  : and at most run_bytes per run (default min(64 MiB, heap/64)).
+ *   format_ahead: 1 (default) = the reservation that leaves a segment with
+ *                fewer than nb/4 blocks formats the next segment of its tree;
+ *                2 = off (the paper: format on demand).
  *   fence_free : 1 (default) = a release fence per freeing team before its
  *                free-counter atomic; 2 = none
  *                (measurement only: frees then do not order user data).
- */
+ * (run_max = 1, format_ahead = 2 reproduce the paper's policy exactly; the
+ *  run/format-ahead policy is DESIGN.md "Deviations" 5.) */
 typedef struct gallatin_config {
     uint64_t heap_bytes;
+    uint64_t run_bytes;
     uint32_t slot_base;
     uint32_t slot_min;
-    uint32_t theta;
+    uint32_t run_max;
+    uint32_t format_ahead;
     uint32_t fence_free;
-    uint32_t reserved[4];
+    uint32_t reserved[3];
 } gallatin_config_t;
 
 int gallatin_init(uint64_t heap_bytes);                 /* defaults for the rest */
@@ -89,10 +96,11 @@ int gallatin_free_host(const uint64_t *h_ptrs, uint64_t n, void *stream);
  * every outstanding pointer.  Asynchronous on `stream`. */
 int gallatin_reset(void *stream);
 
-/* Quiescent only (no malloc/free in flight): retire every block-buffer slot;
- * the unissued remainder of each buffered block is freed, prefetched blocks
- * are returned.  After every user pointer is freed, drain restores the
- * pristine image.  Runs sequentially (one thread) in slot order. */
+/* Quiescent only (no malloc/free in flight): retire every block-buffer slot
+ * (sequentially, class-major slot order) -- the unissued remainder of every
+ * block of its run is freed -- then return every formatted segment whose
+ * blocks are all home to the segment tree.  After every user pointer is freed,
+ * drain restores the pristine image. */
 int gallatin_drain(void *stream);
 
 /* Serialized replay (test hook, one GPU thread, in order): kinds[i] 0 =
@@ -110,8 +118,10 @@ typedef struct gallatin_stats {
     uint64_t tree_segments[9];   /* segments formatted for each block tree          */
     uint64_t large_segments;     /* segments held by >= 16 MB allocations           */
     uint64_t errors;             /* device error counter (bad frees)                */
+    uint64_t run_bytes;          /* effective configuration ...                     */
     uint32_t nslot[9];           /* block-buffer slots per class                    */
-    uint32_t theta, fence_free;
+    uint32_t run_cap[9];         /* max blocks per run per class                    */
+    uint32_t slot_base, slot_min, run_max, format_ahead, fence_free;
 } gallatin_stats_t;
 int gallatin_stats(gallatin_stats_t *out);               /* synchronizes the device */
 
@@ -127,9 +137,9 @@ int gallatin_stats(gallatin_stats_t *out);               /* synchronizes the dev
  *         ring queues (nseg x 65 words: [count] then 256 uint16 block ids in
  *           FIFO order, 0xFFFF padded, 4 per word little-endian)
  *         block free counters (nseg*256 uint32, 2 per word)
- *         block-buffer slots (S words: issued-count << 32 | block id,
- *           0xFFFFFFFF = none; class-major)
- *         prefetched block per slot (S words; 0xFFFFFFFF = none)
+ *         block-buffer slots (S words, class-major: issued count << 32 |
+ *           run length << 24 | first block of the run as a linear index in
+ *           units of the class's block size; empty = 0x0000000000FFFFFF)
  * gallatin_snapshot_words() gives the length. */
 int gallatin_snapshot_words(uint64_t *words);
 int gallatin_snapshot(uint64_t *h_out, uint64_t cap_words, uint64_t *len_words);

@@ -33,7 +33,7 @@ constexpr uint32_t kTreeCont = 0xFFFFFFFEu;
 constexpr uint32_t kGidNone = 0xFFFFFFFFu;
 constexpr uint32_t kAvailBias = 0x80000000u;
 constexpr uint16_t kRingEmpty = 0xFFFF;
-constexpr uint64_t kSlotEmpty = ((uint64_t)kSlices << 32) | kGidNone;
+constexpr uint32_t kMaxRun = 128;                   // blocks per slot run (8-bit field)
 
 __device__ __forceinline__ uint32_t nb_of(uint32_t t) { return kMaxBlocks >> t; }
 
@@ -71,17 +71,17 @@ __device__ __forceinline__ BitTree block_tree(const View &v, uint32_t t) {
 
 // Make block-tree t's bit for segment s equal its predicate (the derived-bit
 // reconcile loop of DESIGN.md "Quiescent exactness").
-__device__ inline void btree_reconcile(const View &v, uint32_t t, uint64_t s) {
+__device__ __noinline__ void btree_reconcile(const View &v, uint32_t t, uint64_t s) {
     const BitTree bt = block_tree(v, t);
     uint64_t *leaf = bt.w + bt.off[0] + (s >> 6);
     const uint64_t bit = 1ull << (s & 63);
     bool flipped = false;
-    ptx::fence_sc();
+    ptx::fence_acq_rel();
     for (;;) {
         const bool in = sw_in_tree(ptx::ld_relaxed(v.seg_word + s), t);
         const uint64_t old = in ? ptx::atom_or(leaf, bit) : ptx::atom_and(leaf, ~bit);
         flipped |= in ? (old == 0) : (old == bit);
-        ptx::fence_sc();
+        ptx::fence_acq_rel();
         if (sw_in_tree(ptx::ld_relaxed(v.seg_word + s), t) == in) break;
     }
     if (flipped) bt_reconcile_up(bt, 0, s >> 6);
@@ -91,7 +91,7 @@ __device__ void try_free_segment(const View &v, uint64_t s, uint32_t t);
 
 // Every thread whose RMW on seg_word[s] changed a block-tree predicate repairs
 // that bit; the RMW that brings a segment back to "all blocks home" retires it.
-__device__ inline void seg_after_rmw(const View &v, uint64_t s, uint64_t old, uint64_t now) {
+__device__ __forceinline__ void seg_after_rmw(const View &v, uint64_t s, uint64_t old, uint64_t now) {
     const uint32_t to = sw_tree(old), tn = sw_tree(now);
     if (to < kTrees && sw_in_tree(old, to) != sw_in_tree(now, to)) btree_reconcile(v, to, s);
     if (tn < kTrees && tn != to && sw_in_tree(old, tn) != sw_in_tree(now, tn)) btree_reconcile(v, tn, s);
@@ -101,7 +101,7 @@ __device__ inline void seg_after_rmw(const View &v, uint64_t s, uint64_t old, ui
 
 // "When all blocks are returned, the segment is freed and re-added to the
 // segment tree".
-__device__ inline void try_free_segment(const View &v, uint64_t s, uint32_t t) {
+__device__ __noinline__ void try_free_segment(const View &v, uint64_t s, uint32_t t) {
     const uint64_t full = sw_make(t, (int32_t)nb_of(t));
     if (ptx::atom_cas(v.seg_word + s, full, sw_make(kTreeFree, 0)) != full) return;
     // No block of s is out or in flight: reset its ring.
@@ -117,87 +117,40 @@ __device__ inline void try_free_segment(const View &v, uint64_t s, uint32_t t) {
 }
 
 // ---- Alg. 1 GetSegment(treeId < numBlockTrees) ----------------
-__device__ inline bool get_segment(const View &v, uint32_t t) {
+// successor(0) on the segment tree + claimIndex, front first
+// (P:138).  Returns the claimed segment or kNone when every segment is in use.
+__device__ __noinline__ uint64_t claim_front(const View &v) {
     const BitTree st = seg_tree(v);
     for (;;) {
-        uint64_t s = bt_successor<false>(st, 0);           // front first
+        uint64_t s = bt_successor<false>(st, 0);
         if (s == kNone) {
             s = bt_scan_first(st);                         // confirm before failing
-            if (s == kNone) return false;                  // "All segments in use"
+            if (s == kNone) return kNone;                  // "All segments in use"
         }
-        if (!bt_delete(st, s)) continue;                   // claimIndex lost
-        ptx::fence_acq_rel();
-        // initSegment: the ring holds blocks 0..nb-1 in order
-        const uint32_t nb = nb_of(t);
-        uint16_t *e = v.q_entries + s * kMaxBlocks;
-        if (nb >= 4) {
-            uint64_t *e4 = reinterpret_cast<uint64_t *>(e);
-            for (uint32_t q = 0; q < nb / 4; q++) {
-                const uint64_t j = 4ull * q;
-                e4[q] = j | ((j + 1) << 16) | ((j + 2) << 32) | ((j + 3) << 48);
-            }
-        } else {
-            for (uint32_t j = 0; j < nb; j++) e[j] = (uint16_t)j;
+        if (bt_delete(st, s)) {
+            ptx::fence_acq_rel();
+            return s;
         }
-        ptx::st_relaxed(v.q_head + s, 0u);
-        ptx::st_relaxed(v.q_tail + s, nb);
-        ptx::fence_acq_rel();
-        // "broadcast availability": the table word, then block tree t
-        const uint64_t delta = sw_retree(kTreeFree, t) + nb;
-        const uint64_t old = ptx::atom_add(v.seg_word + s, delta);
-        seg_after_rmw(v, s, old, old + delta);
-        return true;
     }
 }
 
-// ---- Alg. 2 GetBlock(treeId) ---------------------------------
-// Returns a global block id gid = segment*256 + block, or kGidNone.
-__device__ inline uint32_t get_block(const View &v, uint32_t t) {
-    const BitTree bt = block_tree(v, t);
-    ptx::Backoff bo;
-    for (;;) {
-        const uint64_t s = bt_successor<false>(bt, 0);     // findSegment
-        if (s != kNone) {
-            // reserve one block of s and validate its tree id in one RMW [dev]
-            const uint64_t old = ptx::atom_add(v.seg_word + s, ~0ull);
-            if (sw_tree(old) == t && sw_avail(old) > 0) {
-                seg_after_rmw(v, s, old, old - 1);         // last block out: leave tree
-                // getBlock from the segment's ring queue (P:157, P:178)
-                const uint32_t pos = atomicAdd(v.q_head + s, 1u) & (kMaxBlocks - 1);
-                uint16_t *slotp = v.q_entries + s * kMaxBlocks + pos;
-                uint16_t j;
-                ptx::Backoff wb;
-                while ((j = ptx::ld_relaxed(slotp)) == kRingEmpty) wb.pause();   // enqueue in flight
-                ptx::st_relaxed(slotp, kRingEmpty);
-                ptx::fence_acq_rel();
-                return (uint32_t)(s * kMaxBlocks + j);
-            }
-            // stale hint (P:158-161's failure case): undo, repair, retry
-            seg_after_rmw(v, s, old, old - 1);
-            const uint64_t o2 = ptx::atom_add(v.seg_word + s, 1ull);
-            seg_after_rmw(v, s, o2, o2 + 1);
-            btree_reconcile(v, t, s);
-            bo.pause();
-            continue;
-        }
-        // no formatted segment has a block: format one (Alg.2).
-        // [dev] one formatter per tree at a time (a token) instead of every
-        // waiting thread formatting its own segment.
-        uint32_t *tok = v.fmt_token + t * 32;
-        if (atomicCAS(tok, 0u, 1u) == 0u) {
-            bool ok = true;
-            if (bt_successor<false>(bt, 0) == kNone) ok = get_segment(v, t);
-            ptx::fence_acq_rel();
-            atomicExch(tok, 0u);
-            if (!ok && bt_scan_first(bt) == kNone) return kGidNone;   // "No allocations left"
-            continue;
-        }
-        while (ptx::ld_relaxed(tok) != 0u && bt_successor<false>(bt, 0) == kNone) bo.pause();
-    }
+// initSegment for tree t: blocks [keep, nb) go into the ring in order
+// and the segment joins block tree t ("broadcast availability");
+// blocks [0, keep) belong to the caller.
+__device__ __noinline__ void format_segment(const View &v, uint64_t s, uint32_t t, uint32_t keep) {
+    const uint32_t nb = nb_of(t);
+    uint16_t *e = v.q_entries + s * kMaxBlocks;
+    for (uint32_t j = keep; j < nb; j++) e[j - keep] = (uint16_t)j;
+    ptx::st_relaxed(v.q_head + s, 0u);
+    ptx::st_relaxed(v.q_tail + s, nb - keep);
+    ptx::fence_acq_rel();
+    const uint64_t delta = sw_retree(kTreeFree, t) + (nb - keep);
+    const uint64_t old = ptx::atom_add(v.seg_word + s, delta);
+    seg_after_rmw(v, s, old, old + delta);
 }
 
 // ---- block return (Alg.4; ring enqueue P:178) --------------------
-__device__ inline void return_block(const View &v, uint32_t gid) {
+__device__ __noinline__ void return_block(const View &v, uint32_t gid) {
     const uint64_t s = gid / kMaxBlocks;
     const uint32_t pos = atomicAdd(v.q_tail + s, 1u) & (kMaxBlocks - 1);
     uint16_t *slotp = v.q_entries + s * kMaxBlocks + pos;
@@ -211,7 +164,7 @@ __device__ inline void return_block(const View &v, uint32_t gid) {
 
 // n slices of block gid came back; the team completing 4096 returns it
 // (reading A-14 of "== 4095").
-__device__ inline void block_freed(const View &v, uint32_t gid, uint32_t n) {
+__device__ __forceinline__ void block_freed(const View &v, uint32_t gid, uint32_t n) {
     const uint32_t old = atomicAdd(v.block_free + gid, n);
     if (old + n == kSlices) {
         atomicExch(v.block_free + gid, 0u);
@@ -220,46 +173,170 @@ __device__ inline void block_freed(const View &v, uint32_t gid, uint32_t n) {
     }
 }
 
-// ---- addresses -------------------------------------------------------------
-__device__ __forceinline__ void *slice_ptr(const View &v, uint32_t gid, uint32_t c, uint32_t idx) {
-    // offset(blockId*4096 + idx): block j of segment s is 2^(16+c) B
-    const uint64_t s = gid / kMaxBlocks, j = gid % kMaxBlocks;
-    return reinterpret_cast<void *>(v.heap + (s << kSegLog2) + (j << (16 + c)) + ((uint64_t)idx << (kMinSliceLog2 + c)));
-}
-__device__ __forceinline__ uint64_t *slot_word(const View &v, uint32_t si) { return v.slots + (uint64_t)si * 16; }
-__device__ __forceinline__ uint32_t *slot_next(const View &v, uint32_t si) {
-    return reinterpret_cast<uint32_t *>(v.slots + (uint64_t)si * 16 + 1);
+__device__ __forceinline__ uint32_t gid_of(uint32_t t, uint64_t linear) {
+    const uint32_t sh = 8 - t;                              // log2 nb(t)
+    return (uint32_t)(((linear >> sh) << 8) | (linear & ((1u << sh) - 1)));
 }
 
-// Replace an exhausted buffered block (Alg.3): the prefetched block
-// if there is one, else GetBlock.  On exhaustion the slot is left empty.
-__device__ inline bool refill_slot(const View &v, uint32_t si, uint32_t c) {
-    uint32_t b = kGidNone;
-    if (v.theta) b = atomicExch(slot_next(v, si), kGidNone);
-    if (b == kGidNone) b = get_block(v, c);
-    if (b == kGidNone) {
+// [dev] format one more segment for tree t when the current one runs low, so
+// that refills rarely wait for a format (one formatter per tree; skipped if
+// the formatter token is busy).
+__device__ __noinline__ void format_ahead(const View &v, uint32_t t) {
+    uint32_t *tok = v.fmt_token + t * 32;
+    if (atomicCAS(tok, 0u, 1u) != 0u) return;
+    const uint64_t s = claim_front(v);
+    if (s != kNone) format_segment(v, s, t, 0);
+    ptx::fence_acq_rel();
+    atomicExch(tok, 0u);
+}
+
+// ---- Alg. 2 GetBlock(treeId), for a RUN of blocks [dev] --------
+// Returns the number of consecutive blocks obtained (0 = exhausted) and the
+// first one's linear index (segment * nb + block) in *first.
+__device__ __noinline__ uint32_t get_run(const View &v, uint32_t t, uint32_t want, uint32_t *first) {
+    const BitTree bt = block_tree(v, t);
+    const uint32_t nb = nb_of(t);
+    ptx::Backoff bo;
+    uint64_t from = 0;
+    for (;;) {
+        const uint64_t s = bt_successor<false>(bt, from);    // findSegment
+        if (s != kNone) {
+            // reserve up to `want` blocks of s and validate its tree id in one RMW
+            const uint64_t dec = (uint64_t)(-(int64_t)want);
+            const uint64_t old = ptx::atom_add(v.seg_word + s, dec);
+            const int32_t a = sw_avail(old);
+            if (sw_tree(old) == t && a > 0) {
+                const uint32_t got = (uint32_t)a < want ? (uint32_t)a : want;
+                seg_after_rmw(v, s, old, old + dec);
+                if (got < want) {                               // give back the excess
+                    const uint64_t o2 = ptx::atom_add(v.seg_word + s, (uint64_t)(want - got));
+                    seg_after_rmw(v, s, o2, o2 + (want - got));
+                }
+                const uint32_t low = nb / 4;
+                if (v.format_ahead && (uint32_t)a >= low && (uint32_t)a - got < low &&
+                    bt_successor<false>(bt, s + 1) == kNone)
+                    format_ahead(v, t);
+                // getBlock from the segment's ring queue (P:157, P:178)
+                const uint32_t pos = atomicAdd(v.q_head + s, got);
+                uint16_t *ring = v.q_entries + s * kMaxBlocks;
+                uint16_t e[kMaxRun];
+                uint32_t p = 1;
+                for (uint32_t q = 0; q < got; q++) {
+                    uint16_t *ep = ring + ((pos + q) & (kMaxBlocks - 1));
+                    uint16_t j;
+                    ptx::Backoff wb;
+                    while ((j = ptx::ld_relaxed(ep)) == kRingEmpty) wb.pause();   // enqueue in flight
+                    ptx::st_relaxed(ep, kRingEmpty);
+                    e[q] = j;
+                    if (q == p && j == e[0] + q) p++;          // consecutive prefix
+                }
+                ptx::fence_acq_rel();
+                for (uint32_t q = p; q < got; q++) return_block(v, (uint32_t)(s * kMaxBlocks + e[q]));
+                *first = (uint32_t)(s * nb + e[0]);
+                return p;
+            }
+            // stale hint (P:158-161's failure case): undo, repair, look further
+            seg_after_rmw(v, s, old, old + dec);
+            const uint64_t o2 = ptx::atom_add(v.seg_word + s, (uint64_t)want);
+            seg_after_rmw(v, s, o2, o2 + want);
+            btree_reconcile(v, t, s);
+            from = s + 1;
+            continue;
+        }
+        if (from != 0) {                                      // re-scan from the front once more
+            from = 0;
+            bo.pause();
+            continue;
+        }
+        if (want >= nb) {
+            // the run covers whole segments: take fresh ones privately [dev]
+            const uint64_t s0 = claim_front(v);
+            if (s0 == kNone) return 0;                        // "No allocations left"
+            const BitTree st = seg_tree(v);
+            uint32_t k = 1;
+            while (k < want / nb && s0 + k < v.nseg && bt_delete(st, s0 + k)) k++;
+            ptx::fence_acq_rel();
+            for (uint32_t q = 0; q < k; q++) ptx::atom_add(v.seg_word + s0 + q, sw_retree(kTreeFree, t));
+            ptx::fence_acq_rel();
+            *first = (uint32_t)(s0 * nb);
+            return k * nb;
+        }
+        // Alg.2: format a segment; [dev] one formatter per tree
+        uint32_t *tok = v.fmt_token + t * 32;
+        if (atomicCAS(tok, 0u, 1u) == 0u) {
+            if (bt_successor<false>(bt, 0) != kNone) {        // someone published meanwhile
+                atomicExch(tok, 0u);
+                continue;
+            }
+            const uint64_t s1 = claim_front(v);
+            if (s1 != kNone) format_segment(v, s1, t, want);
+            ptx::fence_acq_rel();
+            atomicExch(tok, 0u);
+            if (s1 == kNone) {
+                if (bt_scan_first(bt) == kNone) return 0;     // "No allocations left"
+                continue;
+            }
+            *first = (uint32_t)(s1 * nb);
+            return want;
+        }
+        while (ptx::ld_relaxed(tok) != 0u && bt_successor<false>(bt, 0) == kNone) bo.pause();
+    }
+}
+
+// ---- addresses -------------------------------------------------------------
+__device__ __forceinline__ uint64_t *slot_word(const View &v, uint32_t si) { return v.slots + (uint64_t)si * 16; }
+
+constexpr uint32_t kRunNone = 0xFFFFFFu;
+constexpr uint64_t kSlotEmpty = kRunNone;                 // issued 0, run 0: refill on first use
+
+// Replace an exhausted run (Alg.3): the run doubles up to the class cap.
+__device__ __noinline__ bool refill_slot(const View &v, uint32_t si, uint32_t c, uint32_t m_prev) {
+    const uint32_t cap = v.run_cap[c];
+    const uint32_t want = m_prev == 0 ? 1u : (2 * m_prev < cap ? 2 * m_prev : cap);
+    uint32_t first = 0;
+    const uint32_t got = get_run(v, c, want, &first);
+    if (got == 0) {
         ptx::atom_exch(slot_word(v, si), kSlotEmpty);
         return false;
     }
-    ptx::atom_exch(slot_word(v, si), (uint64_t)b);        // {issued 0, block b}
+    ptx::atom_exch(slot_word(v, si), ((uint64_t)got << 24) | first);
     return true;
 }
 
-// [dev] prefetch: the request that takes index theta fetches the next block.
-__device__ inline void prefetch_slot(const View &v, uint32_t si, uint32_t c) {
-    const uint32_t b = get_block(v, c);
-    if (b == kGidNone) return;
-    if (atomicCAS(slot_next(v, si), kGidNone, b) != kGidNone) block_freed(v, b, kSlices);   // raced: give it back
+__device__ __forceinline__ void *slice_ptr(const View &v, uint32_t c, uint64_t first, uint64_t idx) {
+    // offset(blockId*4096 + idx) with the run's blocks contiguous
+    return reinterpret_cast<void *>(v.heap + (first << (16 + c)) + (idx << (kMinSliceLog2 + c)));
+}
+
+__device__ __forceinline__ uint32_t slice_class(uint64_t size) {
+    return size <= 16 ? 0u : (uint32_t)(64 - __clzll((long long)(size - 1))) - kMinSliceLog2;
+}
+__device__ __forceinline__ uint32_t block_class(uint64_t size) {
+    return size <= 65536 ? 0u : (uint32_t)(64 - __clzll((long long)(size - 1))) - 16;
+}
+
+// After a team RMW returned `old` and this lane drew idx >= the run's end:
+// refill (the lane that drew exactly the end) or wait for the refill.
+// Returns false if the refill found no memory.
+__device__ __noinline__ bool slot_exhausted(const View &v, uint32_t si, uint32_t c, uint64_t old, uint32_t idx) {
+    const uint32_t m = (uint32_t)(old >> 24) & 0xFF;
+    if (idx == (m << kSliceLog2)) return refill_slot(v, si, c, m);
+    ptx::Backoff bo;
+    for (;;) {
+        const uint64_t w = ptx::ld_relaxed(slot_word(v, si));
+        if ((uint32_t)(w >> 32) <= ((((uint32_t)(w >> 24)) & 0xFF) << kSliceLog2)) return true;
+        bo.pause();
+    }
 }
 
 // ---- Alg. 3 MALLOC.Slice ---------------------------------------
 // The lanes of a warp asking the same slot form a team (reading A-8);
-// the leader does ONE atomicAdd on the slot word {issued:32 | block:32} that
-// returns the block and the first slice index together [dev: the paper reads
-// the buffer, then adds on the block's counter]; __shfl_sync broadcasts it;
-// lane r takes index old+r, valid iff < 4096.  The lane that draws
-// index 4096 replaces the block (reading A-7); other lanes past the
-// end wait for the replacement and retry.
+// the leader does ONE atomicAdd on the slot word {issued:32 | run:8 |
+// first:24} that returns the run and the first slice index together [dev: the
+// paper reads the buffer, then adds on the block's counter]; __shfl_sync
+// broadcasts it; lane r takes index old+r, valid iff < 4096 * run.
+// The lane that draws the end replaces the run (reading A-7);
+// lanes past it wait for the replacement and retry.
 __device__ inline void *malloc_slice(const View &v, uint32_t c, uint32_t key) {
     const uint32_t si = v.slot_off[c] + key % v.nslot[c];
     uint64_t *sw = slot_word(v, si);
@@ -272,34 +349,24 @@ __device__ inline void *malloc_slice(const View &v, uint32_t c, uint32_t key) {
         uint64_t old = 0;
         if (lane == leader) old = ptx::atom_add(sw, (uint64_t)__popc(peers) << 32);
         old = __shfl_sync(peers, old, (int)leader);
-        const uint32_t cnt = (uint32_t)(old >> 32), gid = (uint32_t)old;
-        const uint32_t idx = cnt + rank;
-        if (idx < kSlices) {
-            if (v.theta && idx == v.theta) prefetch_slot(v, si, c);
-            return slice_ptr(v, gid, c, idx);
-        }
-        if (idx == kSlices) {
-            if (!refill_slot(v, si, c)) return nullptr;            // nullptr
-            continue;
-        }
-        ptx::Backoff bo;
-        while ((uint32_t)(ptx::ld_relaxed(sw) >> 32) > kSlices) bo.pause();
+        const uint32_t idx = (uint32_t)(old >> 32) + rank;
+        if (idx < ((((uint32_t)(old >> 24)) & 0xFF) << kSliceLog2)) return slice_ptr(v, c, old & kRunNone, idx);
+        if (!slot_exhausted(v, si, c, old, idx)) return nullptr;   // nullptr
     }
 }
 
 // (4 KB, 16 MB): one whole block of the smallest fitting tree; its counter is
 // preset to 4095 so that Alg.4's rule returns it on its one free (reading A-2).
-__device__ inline void *malloc_block(const View &v, uint32_t t) {
-    const uint32_t gid = get_block(v, t);
-    if (gid == kGidNone) return nullptr;
-    atomicExch(v.block_free + gid, kSlices - 1);
-    const uint64_t s = gid / kMaxBlocks, j = gid % kMaxBlocks;
-    return reinterpret_cast<void *>(v.heap + (s << kSegLog2) + (j << (16 + t)));
+__device__ __noinline__ void *malloc_block(const View &v, uint32_t t) {
+    uint32_t first = 0;
+    if (get_run(v, t, 1, &first) == 0) return nullptr;
+    atomicExch(v.block_free + gid_of(t, first), kSlices - 1);
+    return reinterpret_cast<void *>(v.heap + ((uint64_t)first << (16 + t)));
 }
 
 // >= 16 MB: Alg.1 with treeId >= numBlockTrees: claimMultiple from the back
 // (P:110-113); tree id = numBlockTrees + numSegments.
-__device__ inline void *malloc_large(const View &v, uint64_t k) {
+__device__ __noinline__ void *malloc_large(const View &v, uint64_t k) {
     if (k > v.nseg) return nullptr;
     const BitTree st = seg_tree(v);
     ptx::Backoff bo;
@@ -325,16 +392,20 @@ __device__ inline void *malloc_large(const View &v, uint64_t k) {
 // Classify (A1): slices 16 B..4 KB by ceil(log2), blocks, segments.
 __device__ inline void *malloc_impl(const View &v, uint64_t size, uint32_t key) {
     if (size == 0) return nullptr;
-    if (size <= kMaxSlice) {
-        const uint32_t c = size <= 16 ? 0u : (uint32_t)(64 - __clzll((long long)(size - 1))) - kMinSliceLog2;
-        return malloc_slice(v, c, key);
-    }
-    if (size < kSegBytes) {
-        const uint32_t t = size <= 65536 ? 0u : (uint32_t)(64 - __clzll((long long)(size - 1))) - 16;
-        return malloc_block(v, t);
-    }
+    if (size <= kMaxSlice) return malloc_slice(v, slice_class(size), key);
+    if (size < kSegBytes) return malloc_block(v, block_class(size));
     const uint64_t k = (size >> kSegLog2) + ((size & (kSegBytes - 1)) != 0);
     return malloc_large(v, k);
+}
+
+// segment allocation: return the k segments to the segment tree
+__device__ __noinline__ void free_large(const View &v, uint64_t s, uint32_t t) {
+    const uint64_t k = t - kTrees;
+    ptx::fence_acq_rel();
+    ptx::atom_add(v.seg_word + s, sw_retree(t, kTreeFree));
+    for (uint64_t m = 1; m < k; m++) ptx::atom_add(v.seg_word + s + m, sw_retree(kTreeCont, kTreeFree));
+    ptx::fence_acq_rel();
+    bt_insert_range(seg_tree(v), s, k);
 }
 
 // ---- Alg. 4 FREE -----------------------------------------------
@@ -358,26 +429,33 @@ __device__ inline void free_impl(const View &v, void *p) {
         return;
     }
     if (t == kTreeFree || t == kTreeCont) { atomicAdd(v.err, 1ull); return; }
-    // segment allocation: return the k segments to the segment tree
-    const uint64_t k = t - kTrees;
-    ptx::fence_acq_rel();
-    ptx::atom_add(v.seg_word + s, sw_retree(t, kTreeFree));
-    for (uint64_t m = 1; m < k; m++) ptx::atom_add(v.seg_word + s + m, sw_retree(kTreeCont, kTreeFree));
-    ptx::fence_acq_rel();
-    bt_insert_range(seg_tree(v), s, k);
+    free_large(v, s, t);
 }
 
-// Quiescent drain: retire every slot in class-major order; the unissued
-// remainder of a buffered block counts as freed, a prefetched block is
-// returned whole.
+// Quiescent drain, part 1 (one thread): retire every slot in class-major
+// order; the unissued remainder of every block of its run counts as freed.
 __device__ inline void drain_slots(const View &v) {
-    for (uint32_t si = 0; si < v.nslot_total; si++) {
-        const uint64_t w = ptx::atom_exch(slot_word(v, si), kSlotEmpty);
-        const uint32_t cnt = (uint32_t)(w >> 32), gid = (uint32_t)w;
-        if (gid != kGidNone && cnt < kSlices) block_freed(v, gid, kSlices - cnt);
-        const uint32_t nx = atomicExch(slot_next(v, si), kGidNone);
-        if (nx != kGidNone) block_freed(v, nx, kSlices);
+    for (uint32_t c = 0; c < kTrees; c++) {
+        for (uint32_t q = 0; q < v.nslot[c]; q++) {
+            const uint64_t w = ptx::atom_exch(slot_word(v, v.slot_off[c] + q), kSlotEmpty);
+            const uint64_t cnt = w >> 32;
+            const uint32_t m = (uint32_t)(w >> 24) & 0xFF;
+            const uint64_t first = w & kRunNone;
+            for (uint32_t k = 0; k < m; k++) {
+                const uint64_t lo = (uint64_t)k << kSliceLog2;
+                const uint64_t issued = cnt <= lo ? 0 : (cnt - lo > kSlices ? kSlices : cnt - lo);
+                if (issued < kSlices) block_freed(v, gid_of(c, first + k), (uint32_t)(kSlices - issued));
+            }
+        }
     }
+}
+
+// Quiescent drain, part 2: a segment whose blocks are all home (formatted
+// ahead, never used) goes back to the segment tree.
+__device__ inline void retire_idle(const View &v, uint64_t s) {
+    const uint64_t w = ptx::ld_relaxed(v.seg_word + s);
+    const uint32_t t = sw_tree(w);
+    if (t < kTrees && sw_avail(w) == (int32_t)nb_of(t)) try_free_segment(v, s, t);
 }
 
 }  // namespace core

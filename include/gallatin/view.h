@@ -14,8 +14,10 @@
  *   q_head/tail nseg x u32 ring counters; q_entries nseg x 256 x u16 block ids
  *               (the per-segment ring queue)
  *   block_free  nseg x 256 x u32 free counters
- *   slots       S x 128 B lines: word 0 = {issued count:32 | block id:32},
- *               word 1 = prefetched block id (block buffer)
+ *   slots       S x 128 B lines: word 0 = {issued count:32 | run length:8 |
+ *               first block:24} (block buffer; a run = consecutive
+ *               blocks, first block as a linear index in units of the class's
+ *               block size)
  *   fmt_token   9 x 128 B lines: one formatter per block tree
  *   err         u64 error counter (bad frees)
  */
@@ -45,9 +47,9 @@ struct gallatin_device_view {
     uint32_t nslot[GALLATIN_NUM_TREES];
     uint32_t slot_off[GALLATIN_NUM_TREES];
     uint32_t nslot_total;
-    uint32_t theta;             /* 0 = no prefetch                            */
+    uint32_t run_cap[GALLATIN_NUM_TREES];  /* max blocks per slot run, per class */
+    uint32_t format_ahead;      /* 1 = format the next segment at nb/4 left   */
     uint32_t fence_free;        /* 1 = release fence per freeing team, 2 = none */
-    uint32_t reserved;
 };
 typedef struct gallatin_device_view gallatin_device_view_t;
 

@@ -21,12 +21,21 @@
  *     sizes 16 B..4096 B, tree id = log2(size) - log2(16);
  *     slices are handed out in order by a counter (Alg.3 P:212-
  *     213: valid = idx < 4096), address offset(blockId*4096 + idx);
- *   - block buffer: NSLOT(c) = max(slot_min, slot_base >> c) live blocks per
- *     class, slot chosen by the request's key mod NSLOT(c) (reading
- *     A-6); an exhausted block is replaced by the request that finds it
- *     exhausted (Alg.3, reading A-7); optional prefetch: the request
- *     that takes index theta fetches the next block early (not in the paper;
- *     theta = 0 is the paper's behaviour);
+ *   - block buffer: NSLOT(c) = max(slot_min, slot_base >> c) slots per class
+ *     (P:195), slot chosen by the request's key mod NSLOT(c) (reading A-6); an
+ *     exhausted slot is refilled by the request that finds it exhausted
+ *     (Alg.3, reading A-7).
+ *   - [ours, DESIGN.md "Deviations"] a slot holds a RUN of m consecutive
+ *     blocks (a contiguous address range) handed out slice by slice in order;
+ *     m starts at 1 and doubles on each refill of the slot up to a cap.  With
+ *     cap 1 and format_ahead off this is exactly the paper's one-block buffer.
+ *     A run comes from the lowest segment of the block tree (up to m of its
+ *     ring entries, keeping the longest consecutive prefix and re-enqueueing
+ *     the rest), else from fresh segments: when m covers whole segments the
+ *     run takes them privately (no ring, no block tree), otherwise one segment
+ *     is formatted with the run's blocks removed and the rest published.
+ *     format_ahead: the reservation that takes a segment below nb/4 available
+ *     blocks formats one more segment for the tree.
  *   - requests in (4 KB, 16 MB): one whole block of tree max(0, ceil(log2
  *     size) - 16) whose free counter is preset to 4095 so that Alg.4's rule
  *      returns it on its one free (reading A-2);
@@ -38,8 +47,9 @@
  *     reading A-11), free counter += 1, the free that completes 4096 returns
  *     the block (reading A-14); otherwise the k segments are
  *     re-inserted into the segment tree.
- *   - drain (reading A-15/SURVEY A15): retire every block-buffer slot, the
- *     unissued remainder of its block counted as freed.
+ *   - drain (reading A-15/SURVEY A15, R-1): retire every block-buffer slot,
+ *     the unissued remainder of its run counted as freed; then retire the
+ *     segments whose blocks are all home.
  *
  * Canonical metadata image: see include/gallatin.h, "Snapshot image"; this
  * file writes the same documented layout from its own state.
@@ -80,7 +90,8 @@ typedef struct { uint64_t key, val; } kv_t;
 
 typedef struct o2 {
     uint64_t nseg;
-    unsigned slot_base, slot_min, theta;
+    unsigned slot_base, slot_min, run_max, format_ahead;
+    uint64_t run_bytes;
     unsigned nslot[NUM_BLOCK_TREES], slot_off[NUM_BLOCK_TREES], nslot_total;
     uint32_t *tree;               /* memoryTable.ids           */
     int32_t *avail;               /* blocks currently in the ring       */
@@ -88,8 +99,7 @@ typedef struct o2 {
     uint32_t *freecnt;            /* per block free counter     */
     oracle_veb *segfree;          /* segment tree               */
     oracle_veb *btree[NUM_BLOCK_TREES];  /* block trees         */
-    uint64_t *slot;               /* (cnt << 32) | gid                  */
-    uint32_t *next;               /* prefetched block or GID_NONE       */
+    uint64_t *slot;               /* cnt << 32 | m << 24 | first block  */
     uint64_t err;                 /* out-of-heap / non-allocated segment frees */
     /* oracle-only bookkeeping for the invariant checks */
     kv_t *live; uint64_t live_cap, live_n;
@@ -143,10 +153,18 @@ static int live_take(o2_t *a, uint64_t k, uint64_t *v) {
 }
 
 /* ---------------------------------------------------------- lifecycle --- */
-o2_t *o2_create(uint64_t nseg, unsigned slot_base, unsigned slot_min, unsigned theta) {
-    if (nseg < 1 || nseg > (1ULL << 22) || theta >= SLICES_PER_BLOCK || slot_base < 1) return NULL;
+#define RUN_NONE 0xFFFFFFu
+#define SLOT_EMPTY ((uint64_t)RUN_NONE)            /* cnt 0, m 0: refill on first use */
+static uint64_t slot_make(uint64_t cnt, uint32_t m, uint32_t first) {
+    return (cnt << 32) | ((uint64_t)m << 24) | first;
+}
+
+o2_t *o2_create(uint64_t nseg, unsigned slot_base, unsigned slot_min, unsigned run_max,
+                uint64_t run_bytes, unsigned format_ahead) {
+    if (nseg < 1 || nseg > (1ULL << 16) || slot_base < 1 || run_max < 1 || run_max > 128) return NULL;
     o2_t *a = (o2_t *)calloc(1, sizeof(o2_t));
-    a->nseg = nseg; a->slot_base = slot_base; a->slot_min = slot_min; a->theta = theta;
+    a->nseg = nseg; a->slot_base = slot_base; a->slot_min = slot_min;
+    a->run_max = run_max; a->run_bytes = run_bytes; a->format_ahead = format_ahead;
     unsigned off = 0;
     for (unsigned c = 0; c < NUM_BLOCK_TREES; c++) {
         unsigned n = slot_base >> c;                  /* halving per class */
@@ -162,13 +180,12 @@ o2_t *o2_create(uint64_t nseg, unsigned slot_base, unsigned slot_min, unsigned t
     unsigned k = (unsigned)ceil_log2(nseg); if (k < 1) k = 1;
     a->segfree = oracle_veb_create(k);
     for (unsigned t = 0; t < NUM_BLOCK_TREES; t++) a->btree[t] = oracle_veb_create(k);
-    for (uint64_t s = 0; s < nseg; s++) { a->tree[s] = TREE_FREE; oracle_veb_insert(a->segfree, s); }
-    a->slot = (uint64_t *)malloc(a->nslot_total * sizeof(uint64_t));
-    a->next = (uint32_t *)malloc(a->nslot_total * sizeof(uint32_t));
-    for (unsigned i = 0; i < a->nslot_total; i++) {
-        a->slot[i] = (SLICES_PER_BLOCK << 32) | GID_NONE;   /* empty: exhausted, no block */
-        a->next[i] = GID_NONE;
+    for (uint64_t s = 0; s < nseg; s++) {
+        a->tree[s] = TREE_FREE; oracle_veb_insert(a->segfree, s);
+        for (int i = 0; i < 256; i++) a->ring[s].e[i] = 0xFFFF;
     }
+    a->slot = (uint64_t *)malloc(a->nslot_total * sizeof(uint64_t));
+    for (unsigned i = 0; i < a->nslot_total; i++) a->slot[i] = SLOT_EMPTY;
     return a;
 }
 
@@ -177,7 +194,7 @@ void o2_destroy(o2_t *a) {
     free(a->tree); free(a->avail); free(a->ring); free(a->freecnt);
     oracle_veb_destroy(a->segfree);
     for (unsigned t = 0; t < NUM_BLOCK_TREES; t++) oracle_veb_destroy(a->btree[t]);
-    free(a->slot); free(a->next); free(a->live);
+    free(a->slot); free(a->live);
     free(a);
 }
 
@@ -187,48 +204,57 @@ uint64_t o2_violations(const o2_t *a) { return a->violations; }
 uint64_t o2_live_count(const o2_t *a) { return a->live_n; }
 uint64_t o2_usable_live(const o2_t *a) { return a->usable_live; }
 
-/* --------------------------------------------- Alg.1 getSegment (front) --- */
-/* successor(0) on the segment tree, claim it, format it for tree t, hand it
- * to block tree t. */
-static int get_segment(o2_t *a, uint32_t t) {
-    uint64_t s = oracle_veb_successor(a->segfree, 0);
-    if (s == NONE64 || s >= a->nseg) return 0;            /* "All segments in use" */
-    /* front-first invariant: every segment below s is in use */
-    for (uint64_t i = 0; i < s; i++) if (a->tree[i] == TREE_FREE) a->violations |= V_FRONT_FIRST;
-    oracle_veb_delete(a->segfree, s);                      /* claimIndex          */
-    uint32_t nb = nb_of(t);
-    a->tree[s] = t;                                         /* initSegment         */
-    a->avail[s] = (int32_t)nb;
-    ring_t *r = &a->ring[s];
-    r->head = 0; r->count = nb;
-    for (uint32_t j = 0; j < 256; j++) r->e[j] = j < nb ? (uint16_t)j : 0xFFFF;
-    oracle_veb_insert(a->btree[t], s);                     /* "broadcast availability" */
-    return 1;
+/* Largest run (in blocks of tree t) a slot may hold: run_max blocks and
+ * run_bytes bytes, at least one block. */
+static uint32_t run_cap(const o2_t *a, uint32_t t) {
+    uint64_t by = a->run_bytes / block_bytes(t);
+    uint64_t m = a->run_max < by ? a->run_max : by;
+    return m < 1 ? 1 : (uint32_t)m;
 }
 
-/* --------------------------------------------------- Alg.2 getBlock --- */
-static uint32_t get_block(o2_t *a, uint32_t t) {
-    uint64_t s = oracle_veb_successor(a->btree[t], 0);     /* findSegment        */
-    if (s == NONE64) {
-        if (!get_segment(a, t)) return GID_NONE;           /* "No allocations left" */
-        s = oracle_veb_successor(a->btree[t], 0);
-    }
-    ring_t *r = &a->ring[s];
-    uint32_t j = r->e[r->head];                            /* ring dequeue */
+/* ------------------------------------------------ ring queue --- */
+static uint16_t ring_pop(ring_t *r) {
+    uint16_t j = r->e[r->head];
     r->e[r->head] = 0xFFFF;
     r->head = (r->head + 1) & 255; r->count--;
-    a->avail[s]--;
-    if (a->avail[s] == 0) oracle_veb_delete(a->btree[t], s);  /* no over-subscription */
-    return (uint32_t)(s * MAX_BLOCKS_PER_SEGMENT + j);
+    return j;
+}
+static void ring_push(ring_t *r, uint16_t j) {
+    r->e[(r->head + r->count) & 255] = j;
+    r->count++;
+}
+
+/* --------------------------------------------- Alg.1 getSegment (front) --- */
+/* successor(0) on the segment tree and claimIndex; front-first
+ * invariant: every segment below the claimed one is in use. */
+static uint64_t claim_front(o2_t *a) {
+    uint64_t s = oracle_veb_successor(a->segfree, 0);
+    if (s == NONE64 || s >= a->nseg) return NONE64;        /* "All segments in use" */
+    for (uint64_t i = 0; i < s; i++) if (a->tree[i] == TREE_FREE) a->violations |= V_FRONT_FIRST;
+    oracle_veb_delete(a->segfree, s);
+    return s;
+}
+
+/* initSegment for tree t: blocks [keep, nb) go into the ring and the
+ * segment joins block tree t ("broadcast availability"); blocks
+ * [0, keep) are handed to the caller. */
+static void format_segment(o2_t *a, uint64_t s, uint32_t t, uint32_t keep) {
+    uint32_t nb = nb_of(t);
+    a->tree[s] = t;
+    a->avail[s] = (int32_t)(nb - keep);
+    ring_t *r = &a->ring[s];
+    r->head = 0; r->count = 0;
+    for (uint32_t j = 0; j < 256; j++) r->e[j] = 0xFFFF;
+    for (uint32_t j = keep; j < nb; j++) ring_push(r, (uint16_t)j);
+    if (a->avail[s] > 0) oracle_veb_insert(a->btree[t], s);
 }
 
 /* ------------------------------------------ block / segment return --- */
 static void return_block(o2_t *a, uint64_t s, uint32_t j, uint32_t t) {
-    ring_t *r = &a->ring[s];
-    r->e[(r->head + r->count) & 255] = (uint16_t)j;        /* ring enqueue       */
-    r->count++;
+    ring_push(&a->ring[s], (uint16_t)j);                   /* ring enqueue       */
     a->avail[s]++;
     if ((uint32_t)a->avail[s] == nb_of(t)) {               /* every block back  */
+        ring_t *r = &a->ring[s];
         a->tree[s] = TREE_FREE; a->avail[s] = 0;
         r->head = 0; r->count = 0;
         for (int i = 0; i < 256; i++) r->e[i] = 0xFFFF;
@@ -246,6 +272,59 @@ static void block_freed(o2_t *a, uint32_t gid, uint32_t count) {
         uint64_t s = gid / MAX_BLOCKS_PER_SEGMENT;
         return_block(a, s, gid % MAX_BLOCKS_PER_SEGMENT, a->tree[s]);
     }
+}
+
+/* --------------------------------------------------- Alg.2 getBlock --- */
+/* A run of up to `want` consecutive blocks of tree t.  Returns the number of
+ * blocks (0 = no memory) and the first block's linear index in *first
+ * (segment * nb + block). */
+static uint32_t get_run(o2_t *a, uint32_t t, uint32_t want, uint32_t *first) {
+    uint32_t nb = nb_of(t);
+    uint64_t s = oracle_veb_successor(a->btree[t], 0);     /* findSegment */
+    if (s != NONE64) {
+        ring_t *r = &a->ring[s];
+        uint32_t av = (uint32_t)a->avail[s];
+        uint32_t got = want < av ? want : av;              /* reserve */
+        uint32_t low = nb / 4;
+        a->avail[s] -= (int32_t)got;
+        if (a->avail[s] == 0) oracle_veb_delete(a->btree[t], s);   /* no over-subscription */
+        if (a->format_ahead && av >= low && av - got < low &&
+            oracle_veb_successor(a->btree[t], s + 1) == NONE64) {
+            uint64_t f = claim_front(a);                      /* format one segment ahead */
+            if (f != NONE64) format_segment(a, f, t, 0);
+        }
+        uint16_t e[256] = {0};
+        for (uint32_t q = 0; q < got; q++) e[q] = ring_pop(r);      /* getBlock */
+        uint32_t p = 1;
+        while (p < got && e[p] == e[0] + p) p++;                   /* consecutive prefix */
+        for (uint32_t q = p; q < got; q++) return_block(a, s, e[q], t);
+        *first = (uint32_t)(s * nb + e[0]);
+        return p;
+    }
+    if (want >= nb) {
+        /* the run covers whole segments: take up to want/nb consecutive free
+         * segments from the front, privately (no ring, no block tree) */
+        uint64_t s0 = claim_front(a);
+        if (s0 == NONE64) return 0;                           /* "No allocations left" */
+        uint32_t k = 1;
+        while (k < want / nb && s0 + k < a->nseg && oracle_veb_member(a->segfree, s0 + k)) {
+            oracle_veb_delete(a->segfree, s0 + k);
+            k++;
+        }
+        for (uint32_t q = 0; q < k; q++) format_segment(a, s0 + q, t, nb);
+        *first = (uint32_t)(s0 * nb);
+        return k * nb;
+    }
+    uint64_t s1 = claim_front(a);                             /* Alg.2 -> getSegment */
+    if (s1 == NONE64) return 0;
+    format_segment(a, s1, t, want);
+    *first = (uint32_t)(s1 * nb);
+    return want;
+}
+
+static uint32_t gid_of(uint32_t t, uint64_t linear) {
+    uint32_t nb = nb_of(t);
+    return (uint32_t)((linear / nb) * MAX_BLOCKS_PER_SEGMENT + linear % nb);
 }
 
 /* ------------------------------------------ claimMultiple (back) --- */
@@ -279,34 +358,31 @@ static uint64_t claim_multiple(o2_t *a, uint64_t k) {
 }
 
 /* ------------------------------------------------------------ malloc --- */
-static uint64_t slice_addr(uint32_t gid, uint32_t c, uint64_t idx) {
-    uint64_t s = gid / MAX_BLOCKS_PER_SEGMENT, j = gid % MAX_BLOCKS_PER_SEGMENT;
-    uint64_t slice = MIN_SLICE << c;
-    /* offset(blockId*4096 + idx), blockId in units of this class's block */
-    return s * SEGMENT_BYTES + (j * SLICES_PER_BLOCK + idx) * slice;
+/* offset(blockId*4096 + idx): slices of a run are consecutive; the
+ * run's first block has linear index `first` in units of the class's block. */
+static uint64_t slice_addr(uint32_t first, uint32_t c, uint64_t idx) {
+    return (uint64_t)first * block_bytes(c) + idx * (MIN_SLICE << c);
 }
 
 static uint64_t malloc_slice(o2_t *a, uint32_t c, uint64_t key) {
     unsigned i = a->slot_off[c] + (unsigned)(key % a->nslot[c]);
     for (;;) {
         uint64_t cnt = a->slot[i] >> 32;
-        uint32_t gid = (uint32_t)a->slot[i];
-        if (cnt < SLICES_PER_BLOCK) {                       /* valid = idx < 4096 */
-            a->slot[i] = ((cnt + 1) << 32) | gid;
-            uint64_t off = slice_addr(gid, c, cnt);
-            if (a->theta && cnt == a->theta && a->next[i] == GID_NONE)
-                a->next[i] = get_block(a, c);               /* prefetch (ours) */
-            return off;
+        uint32_t m = (uint32_t)(a->slot[i] >> 24) & 0xFF;
+        uint32_t first = (uint32_t)a->slot[i] & RUN_NONE;
+        if (cnt < SLICES_PER_BLOCK * m) {                   /* valid = idx < 4096 (per block) */
+            a->slot[i] = slot_make(cnt + 1, m, first);
+            return slice_addr(first, c, cnt);
         }
-        /* exhausted: this request replaces the block (Alg.3) */
-        uint32_t nbk = a->next[i];
-        a->next[i] = GID_NONE;
-        if (nbk == GID_NONE) nbk = get_block(a, c);
-        if (nbk == GID_NONE) {
-            a->slot[i] = (SLICES_PER_BLOCK << 32) | GID_NONE;
+        /* exhausted: this request replaces the run (Alg.3) */
+        uint32_t cap = run_cap(a, c);
+        uint32_t want = m == 0 ? 1 : (2 * m < cap ? 2 * m : cap);
+        uint32_t got = get_run(a, c, want, &first);
+        if (!got) {
+            a->slot[i] = SLOT_EMPTY;
             return NONE64;                                   /* nullptr */
         }
-        a->slot[i] = (uint64_t)nbk;                          /* (cnt 0, gid)     */
+        a->slot[i] = slot_make(0, got, first);
     }
 }
 
@@ -338,11 +414,11 @@ uint64_t o2_malloc(o2_t *a, uint64_t size, uint64_t key) {
     if (kind == 0) {
         off = malloc_slice(a, cls, key);
     } else if (kind == 1) {
-        uint32_t gid = get_block(a, cls);
-        if (gid == GID_NONE) return NONE64;
+        uint32_t first;
+        if (!get_run(a, cls, 1, &first)) return NONE64;
+        uint32_t gid = gid_of(cls, first);
         a->freecnt[gid] = SLICES_PER_BLOCK - 1;              /* one free returns it (A-2) */
-        off = (uint64_t)(gid / MAX_BLOCKS_PER_SEGMENT) * SEGMENT_BYTES +
-              (uint64_t)(gid % MAX_BLOCKS_PER_SEGMENT) * block_bytes(cls);
+        off = (uint64_t)first * block_bytes(cls);
     } else {
         uint64_t i = claim_multiple(a, cls);
         if (i == NONE64) return NONE64;
@@ -382,18 +458,35 @@ void o2_free(o2_t *a, uint64_t off) {
 }
 
 /* Retire every block-buffer slot in class-major, slot-ascending order: the
- * unissued remainder of the current block is counted as freed; a prefetched
- * block is returned whole. */
+ * unissued remainder of each block of its run is counted as freed.  Then
+ * every segment whose blocks are all home (formatted ahead and never used)
+ * goes back to the segment tree, in segment order. */
 void o2_drain(o2_t *a) {
-    for (unsigned i = 0; i < a->nslot_total; i++) {
-        uint64_t cnt = a->slot[i] >> 32;
-        uint32_t gid = (uint32_t)a->slot[i];
-        a->slot[i] = (SLICES_PER_BLOCK << 32) | GID_NONE;
-        if (gid != GID_NONE && cnt < SLICES_PER_BLOCK)
-            block_freed(a, gid, (uint32_t)(SLICES_PER_BLOCK - cnt));
-        uint32_t nx = a->next[i];
-        a->next[i] = GID_NONE;
-        if (nx != GID_NONE) block_freed(a, nx, (uint32_t)SLICES_PER_BLOCK);
+    for (unsigned c = 0; c < NUM_BLOCK_TREES; c++) {
+        for (unsigned q = 0; q < a->nslot[c]; q++) {
+            unsigned i = a->slot_off[c] + q;
+            uint64_t cnt = a->slot[i] >> 32;
+            uint32_t m = (uint32_t)(a->slot[i] >> 24) & 0xFF;
+            uint32_t first = (uint32_t)a->slot[i] & RUN_NONE;
+            a->slot[i] = SLOT_EMPTY;
+            for (uint32_t k = 0; k < m; k++) {
+                uint64_t lo = SLICES_PER_BLOCK * k;
+                uint64_t issued = cnt <= lo ? 0 : (cnt - lo > SLICES_PER_BLOCK ? SLICES_PER_BLOCK : cnt - lo);
+                if (issued < SLICES_PER_BLOCK)
+                    block_freed(a, gid_of(c, (uint64_t)first + k), (uint32_t)(SLICES_PER_BLOCK - issued));
+            }
+        }
+    }
+    for (uint64_t s = 0; s < a->nseg; s++) {
+        uint32_t t = a->tree[s];
+        if (t < NUM_BLOCK_TREES && (uint32_t)a->avail[s] == nb_of(t)) {
+            ring_t *r = &a->ring[s];
+            a->tree[s] = TREE_FREE; a->avail[s] = 0;
+            r->head = 0; r->count = 0;
+            for (int i = 0; i < 256; i++) r->e[i] = 0xFFFF;
+            oracle_veb_delete(a->btree[t], s);
+            oracle_veb_insert(a->segfree, s);
+        }
     }
 }
 
@@ -488,7 +581,7 @@ static void tree_image(const oracle_veb *t, uint64_t nbits, uint64_t *out) {
 uint64_t o2_image_words(const o2_t *a) {
     uint64_t wpl[16]; unsigned L;
     uint64_t W = tree_words(a->nseg, wpl, &L);
-    return 8 + 10 * W + a->nseg * (1 + 65 + 128) + 2ULL * a->nslot_total;
+    return 8 + 10 * W + a->nseg * (1 + 65 + 128) + (uint64_t)a->nslot_total;
 }
 
 /* Canonical image; layout documented in include/gallatin.h. */
@@ -516,6 +609,5 @@ uint64_t o2_image(const o2_t *a, uint64_t *out, uint64_t cap) {
     for (uint64_t g = 0; g < a->nseg * MAX_BLOCKS_PER_SEGMENT; g += 2)
         *p++ = (uint64_t)a->freecnt[g] | ((uint64_t)a->freecnt[g + 1] << 32);
     for (unsigned i = 0; i < a->nslot_total; i++) *p++ = a->slot[i];
-    for (unsigned i = 0; i < a->nslot_total; i++) *p++ = a->next[i];
     return need;
 }

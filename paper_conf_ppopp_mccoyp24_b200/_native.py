@@ -26,15 +26,18 @@ class GallatinError(RuntimeError):
 
 
 class Config(ctypes.Structure):
-    _fields_ = [("heap_bytes", ctypes.c_uint64), ("slot_base", ctypes.c_uint32), ("slot_min", ctypes.c_uint32),
-                ("theta", ctypes.c_uint32), ("fence_free", ctypes.c_uint32), ("reserved", ctypes.c_uint32 * 4)]
+    _fields_ = [("heap_bytes", ctypes.c_uint64), ("run_bytes", ctypes.c_uint64), ("slot_base", ctypes.c_uint32),
+                ("slot_min", ctypes.c_uint32), ("run_max", ctypes.c_uint32), ("format_ahead", ctypes.c_uint32),
+                ("fence_free", ctypes.c_uint32), ("reserved", ctypes.c_uint32 * 3)]
 
 
 class Stats(ctypes.Structure):
     _fields_ = [("heap_base", ctypes.c_uint64), ("heap_bytes", ctypes.c_uint64), ("num_segments", ctypes.c_uint64),
                 ("free_segments", ctypes.c_uint64), ("tree_segments", ctypes.c_uint64 * 9),
-                ("large_segments", ctypes.c_uint64), ("errors", ctypes.c_uint64), ("nslot", ctypes.c_uint32 * 9),
-                ("theta", ctypes.c_uint32), ("fence_free", ctypes.c_uint32)]
+                ("large_segments", ctypes.c_uint64), ("errors", ctypes.c_uint64), ("run_bytes", ctypes.c_uint64),
+                ("nslot", ctypes.c_uint32 * 9), ("run_cap", ctypes.c_uint32 * 9), ("slot_base", ctypes.c_uint32),
+                ("slot_min", ctypes.c_uint32), ("run_max", ctypes.c_uint32), ("format_ahead", ctypes.c_uint32),
+                ("fence_free", ctypes.c_uint32)]
 
 
 def declared_functions() -> list[str]:
@@ -139,8 +142,11 @@ def _empty64(n: int):
 
 
 # ------------------------------------------------------------- allocator ---
-def gallatin_init(heap_bytes: int, slot_base: int = 0, slot_min: int = 0, theta: int = 0, fence_free: int = 0) -> None:
-    cfg = Config(heap_bytes=heap_bytes, slot_base=slot_base, slot_min=slot_min, theta=theta, fence_free=fence_free)
+def gallatin_init(heap_bytes: int, slot_base: int = 0, slot_min: int = 0, run_max: int = 0, run_bytes: int = 0,
+                  format_ahead: int = 0, fence_free: int = 0) -> None:
+    """0 = library default for every knob (include/gallatin.h gallatin_config_t)."""
+    cfg = Config(heap_bytes=heap_bytes, run_bytes=run_bytes, slot_base=slot_base, slot_min=slot_min,
+                 run_max=run_max, format_ahead=format_ahead, fence_free=fence_free)
     check(lib().gallatin_init_ex(ctypes.byref(cfg)), "gallatin_init")
 
 
@@ -199,7 +205,15 @@ def gallatin_stats() -> dict:
     return {"heap_base": s.heap_base, "heap_bytes": s.heap_bytes, "num_segments": s.num_segments,
             "free_segments": s.free_segments, "tree_segments": list(s.tree_segments),
             "large_segments": s.large_segments, "errors": s.errors, "nslot": list(s.nslot),
-            "theta": s.theta, "fence_free": s.fence_free}
+            "run_cap": list(s.run_cap), "run_bytes": s.run_bytes, "slot_base": s.slot_base, "slot_min": s.slot_min,
+            "run_max": s.run_max, "format_ahead": s.format_ahead, "fence_free": s.fence_free}
+
+
+def oracle_params() -> dict:
+    """The effective policy knobs, as keyword arguments of oracle.Allocator (tests)."""
+    st = gallatin_stats()
+    return {"slot_base": st["slot_base"], "slot_min": st["slot_min"], "run_max": st["run_max"],
+            "run_bytes": st["run_bytes"], "format_ahead": 1 if st["format_ahead"] == 1 else 0}
 
 
 def gallatin_snapshot() -> np.ndarray:

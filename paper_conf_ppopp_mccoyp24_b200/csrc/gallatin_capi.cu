@@ -20,6 +20,8 @@ using core::View;
 namespace {
 
 constexpr int kThreads = 256;
+// ITEMS=4 per thread once the grid would still fill every SM several times
+constexpr int kItemsMin = 148 * 1024 * 4;
 
 struct State {
     bool init = false;
@@ -86,24 +88,123 @@ __global__ void k_reset(View v) {
         if (i < nseg * 128) reinterpret_cast<uint64_t *>(v.block_free)[i] = 0;
         if (i < S * 16) {
             const uint64_t w = i % 16;
-            v.slots[i] = w == 0 ? core::kSlotEmpty : (w == 1 ? (uint64_t)core::kGidNone : 0);
+            v.slots[i] = w == 0 ? core::kSlotEmpty : 0;
         }
         if (i < 9 * 32) v.fmt_token[i] = 0;
         if (i == 0) *v.err = 0;
     }
 }
 
+// Bulk malloc, ITEMS requests per thread: all slice requests first issue their
+// team RMW (one per team per item, back to back: memory-level parallelism),
+// then take their slice; refills, waits, blocks and large requests follow on
+// the per-request device path.  Lane l of warp w handles w*32*ITEMS + k*32 + l.
+template <int ITEMS>
 __global__ void __launch_bounds__(kThreads) k_bulk_malloc(View v, const uint64_t *__restrict__ sizes,
                                                           void **__restrict__ ptrs, uint64_t n) {
-    const uint64_t i = blockIdx.x * (uint64_t)kThreads + threadIdx.x;
-    if (i >= n) return;
-    ptrs[i] = core::malloc_impl(v, sizes[i], ptx::smid());
+    const uint32_t lane = threadIdx.x & 31;
+    const uint64_t base = ((blockIdx.x * (uint64_t)kThreads + threadIdx.x) >> 5) * (32 * ITEMS) + lane;
+    const uint32_t key = ptx::smid();
+    uint64_t sz[ITEMS], old[ITEMS];
+    uint32_t si[ITEMS];
+    unsigned peers[ITEMS];
+#pragma unroll
+    for (int k = 0; k < ITEMS; k++) {
+        const uint64_t i = base + 32ull * k;
+        sz[k] = i < n ? __ldcs(reinterpret_cast<const unsigned long long *>(sizes) + i) : 0;
+    }
+#pragma unroll
+    for (int k = 0; k < ITEMS; k++) {
+        const bool slice = sz[k] - 1 < core::kMaxSlice;               // 1 .. 4096
+        const uint32_t c = core::slice_class(sz[k]);
+        si[k] = slice ? v.slot_off[c] + key % v.nslot[c] : 0xFFFFFFFFu;
+        peers[k] = __match_any_sync(0xFFFFFFFFu, si[k]);
+        old[k] = 0;
+        if (slice && lane == (uint32_t)__ffs((int)peers[k]) - 1)
+            old[k] = ptx::atom_add(core::slot_word(v, si[k]), (uint64_t)__popc(peers[k]) << 32);
+    }
+#pragma unroll
+    for (int k = 0; k < ITEMS; k++) old[k] = __shfl_sync(0xFFFFFFFFu, old[k], __ffs((int)peers[k]) - 1);
+    const uint32_t lt = ptx::lanemask_lt();
+#pragma unroll
+    for (int k = 0; k < ITEMS; k++) {
+        const uint64_t i = base + 32ull * k;
+        void *p = nullptr;
+        if (si[k] != 0xFFFFFFFFu) {
+            const uint32_t c = core::slice_class(sz[k]);
+            const uint32_t idx = (uint32_t)(old[k] >> 32) + (uint32_t)__popc(peers[k] & lt);
+            if (idx < ((((uint32_t)(old[k] >> 24)) & 0xFF) << core::kSliceLog2))
+                p = core::slice_ptr(v, c, old[k] & core::kRunNone, idx);
+            else if (core::slot_exhausted(v, si[k], c, old[k], idx))
+                p = core::malloc_slice(v, c, key);
+        } else if (sz[k] != 0) {
+            p = core::malloc_impl(v, sz[k], key);
+        }
+        if (i < n) __stcs(reinterpret_cast<unsigned long long *>(ptrs) + i, reinterpret_cast<unsigned long long>(p));
+    }
 }
 
+__device__ __noinline__ void free_slow(const View &v, uint64_t p) {
+    const uint64_t off = p - v.heap;
+    if (off >= (v.nseg << core::kSegLog2)) { atomicAdd(v.err, 1ull); return; }
+    const uint64_t s = off >> core::kSegLog2;
+    const uint32_t t = core::sw_tree(ptx::ld_relaxed(v.seg_word + s));
+    if (t == core::kTreeFree || t == core::kTreeCont || t < core::kTrees) { atomicAdd(v.err, 1ull); return; }
+    core::free_large(v, s, t);
+}
+
+// Bulk free, ITEMS pointers per thread: load pointers, then their segments'
+// table words, team the lanes freeing one block, one release fence
+// per leading lane, then the team counter RMWs back to back.
+template <int ITEMS>
 __global__ void __launch_bounds__(kThreads) k_bulk_free(View v, void *const *__restrict__ ptrs, uint64_t n) {
-    const uint64_t i = blockIdx.x * (uint64_t)kThreads + threadIdx.x;
-    if (i >= n) return;
-    core::free_impl(v, ptrs[i]);
+    const uint32_t lane = threadIdx.x & 31;
+    const uint64_t base = ((blockIdx.x * (uint64_t)kThreads + threadIdx.x) >> 5) * (32 * ITEMS) + lane;
+    const uint64_t heap_bytes = v.nseg << core::kSegLog2;
+    uint64_t p[ITEMS], w[ITEMS];
+    uint32_t gid[ITEMS], oldc[ITEMS];
+    unsigned peers[ITEMS];
+#pragma unroll
+    for (int k = 0; k < ITEMS; k++) {
+        const uint64_t i = base + 32ull * k;
+        p[k] = i < n ? __ldcs(reinterpret_cast<const unsigned long long *>(ptrs) + i) : 0;
+    }
+#pragma unroll
+    for (int k = 0; k < ITEMS; k++) {
+        const uint64_t off = p[k] - v.heap;
+        w[k] = (p[k] && off < heap_bytes) ? ptx::ld_relaxed(v.seg_word + (off >> core::kSegLog2)) : ~0ull;
+    }
+    bool lead_any = false;
+#pragma unroll
+    for (int k = 0; k < ITEMS; k++) {
+        const uint64_t off = p[k] - v.heap;
+        const uint32_t t = core::sw_tree(w[k]);
+        const bool blk = p[k] && t < core::kTrees;                  // slice or whole block
+        gid[k] = blk ? (uint32_t)((off >> core::kSegLog2) * core::kMaxBlocks + ((off & (core::kSegBytes - 1)) >> (16 + t)))
+                     : (0x80000000u | (uint32_t)(k << 5) | lane);
+        peers[k] = __match_any_sync(0xFFFFFFFFu, gid[k]);
+        if (!blk) peers[k] = 0;
+        lead_any |= blk && lane == (uint32_t)__ffs((int)peers[k]) - 1;
+    }
+    if (v.fence_free != 2) {
+        __syncwarp();
+        if (lead_any) ptx::fence_acq_rel();                        // release the team's writes
+    }
+#pragma unroll
+    for (int k = 0; k < ITEMS; k++) {
+        oldc[k] = 0;
+        if (peers[k] && lane == (uint32_t)__ffs((int)peers[k]) - 1)
+            oldc[k] = atomicAdd(v.block_free + gid[k], (uint32_t)__popc(peers[k]));
+    }
+#pragma unroll
+    for (int k = 0; k < ITEMS; k++) {
+        if (peers[k] && lane == (uint32_t)__ffs((int)peers[k]) - 1 && oldc[k] + __popc(peers[k]) == core::kSlices) {
+            atomicExch(v.block_free + gid[k], 0u);                   // the 4096th free
+            ptx::fence_acq_rel();
+            core::return_block(v, gid[k]);
+        }
+        if (p[k] && !peers[k]) free_slow(v, p[k]);
+    }
 }
 
 __global__ void k_replay(View v, const uint8_t *kinds, const uint64_t *args, const uint64_t *keys, uint64_t n,
@@ -119,12 +220,18 @@ __global__ void k_replay(View v, const uint8_t *kinds, const uint64_t *args, con
             out[i] = 0;
         } else {
             core::drain_slots(v);
+            for (uint64_t s = 0; s < v.nseg; s++) core::retire_idle(v, s);
             out[i] = 0;
         }
     }
 }
 
-__global__ void k_drain(View v) { core::drain_slots(v); }
+__global__ void k_drain_slots(View v) { core::drain_slots(v); }
+
+__global__ void k_retire_idle(View v) {
+    const uint64_t s = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
+    if (s < v.nseg) core::retire_idle(v, s);
+}
 
 // -- correctness harness ("checks the correctness of allocated memory")
 __global__ void k_stamp(void *const *ptrs, const uint64_t *sizes, uint64_t n) {
@@ -202,7 +309,7 @@ __global__ void k_usable(View v, void *const *ptrs, const uint64_t *sizes, uint6
 
 // ------------------------------------------------------- host helpers ----
 uint64_t image_words(const View &v) {
-    return 8 + 10ull * v.tree_words + v.nseg * (1 + 65 + 128) + 2ull * v.nslot_total;
+    return 8 + 10ull * v.tree_words + v.nseg * (1 + 65 + 128) + (uint64_t)v.nslot_total;
 }
 
 struct HostCopy {
@@ -276,7 +383,14 @@ int gallatin_init_ex(const gallatin_config_t *cfg_in) {
     if (!cfg.slot_base) cfg.slot_base = (uint32_t)sms;      // one slot per SM
     if (!cfg.slot_min) cfg.slot_min = 4;                     // "capped at four"
     if (!cfg.fence_free) cfg.fence_free = 1;
-    if (cfg.theta >= core::kSlices) return GALLATIN_ERR_INVALID;
+    if (!cfg.format_ahead) cfg.format_ahead = 1;
+    if (!cfg.run_max) cfg.run_max = 16;
+    if (!cfg.run_bytes) {
+        cfg.run_bytes = (nseg << core::kSegLog2) / 64;
+        if (cfg.run_bytes > (64ull << 20)) cfg.run_bytes = 64ull << 20;
+    }
+    if (cfg.run_max > core::kMaxRun || cfg.fence_free > 2 || cfg.format_ahead > 2) return GALLATIN_ERR_INVALID;
+    if (nseg > (1ull << 16)) return GALLATIN_ERR_INVALID;        // 24-bit run index at 64 KB blocks
 
     View v{};
     v.nseg = nseg;
@@ -294,7 +408,12 @@ int gallatin_init_ex(const gallatin_config_t *cfg_in) {
         off += n;
     }
     v.nslot_total = off;
-    v.theta = cfg.theta;
+    for (uint32_t c = 0; c < core::kTrees; c++) {
+        uint64_t m = cfg.run_bytes >> (16 + c);
+        if (m > cfg.run_max) m = cfg.run_max;
+        v.run_cap[c] = m < 1 ? 1u : (uint32_t)m;
+    }
+    v.format_ahead = cfg.format_ahead == 1 ? 1u : 0u;
     v.fence_free = cfg.fence_free;
 
     // metadata: one allocation, 256 B aligned sections
@@ -362,7 +481,10 @@ int gallatin_malloc(const uint64_t *d_sizes, void **d_ptrs, uint64_t n, void *st
     if (!g.init) return GALLATIN_ERR_STATE;
     if (n == 0) return GALLATIN_OK;
     if (!d_sizes || !d_ptrs || n > (1ull << 40)) return GALLATIN_ERR_INVALID;
-    k_bulk_malloc<<<grid_for(n), kThreads, 0, S(stream)>>>(g.v, d_sizes, d_ptrs, n);
+    if (n >= (uint64_t)kItemsMin)
+        k_bulk_malloc<4><<<grid_for((n + 3) / 4), kThreads, 0, S(stream)>>>(g.v, d_sizes, d_ptrs, n);
+    else
+        k_bulk_malloc<1><<<grid_for(n), kThreads, 0, S(stream)>>>(g.v, d_sizes, d_ptrs, n);
     return launch_status();
 }
 
@@ -370,7 +492,10 @@ int gallatin_free(void *const *d_ptrs, uint64_t n, void *stream) {
     if (!g.init) return GALLATIN_ERR_STATE;
     if (n == 0) return GALLATIN_OK;
     if (!d_ptrs || n > (1ull << 40)) return GALLATIN_ERR_INVALID;
-    k_bulk_free<<<grid_for(n), kThreads, 0, S(stream)>>>(g.v, d_ptrs, n);
+    if (n >= (uint64_t)kItemsMin)
+        k_bulk_free<4><<<grid_for((n + 3) / 4), kThreads, 0, S(stream)>>>(g.v, d_ptrs, n);
+    else
+        k_bulk_free<1><<<grid_for(n), kThreads, 0, S(stream)>>>(g.v, d_ptrs, n);
     return launch_status();
 }
 
@@ -416,7 +541,10 @@ int gallatin_free_host(const uint64_t *h_ptrs, uint64_t n, void *stream) {
 
 int gallatin_drain(void *stream) {
     if (!g.init) return GALLATIN_ERR_STATE;
-    k_drain<<<1, 1, 0, S(stream)>>>(g.v);
+    k_drain_slots<<<1, 1, 0, S(stream)>>>(g.v);
+    int rc = launch_status();
+    if (rc) return rc;
+    k_retire_idle<<<grid_for(g.v.nseg), kThreads, 0, S(stream)>>>(g.v);
     return launch_status();
 }
 
@@ -475,7 +603,6 @@ int gallatin_snapshot(uint64_t *out, uint64_t cap, uint64_t *len) {
     memcpy(p, h.block_free.data(), v.nseg * 1024);
     p += v.nseg * 128;
     for (uint32_t i = 0; i < v.nslot_total; i++) *p++ = h.slots[(uint64_t)i * 16];
-    for (uint32_t i = 0; i < v.nslot_total; i++) *p++ = (uint32_t)h.slots[(uint64_t)i * 16 + 1];
     return GALLATIN_OK;
 }
 
@@ -498,7 +625,12 @@ int gallatin_stats(gallatin_stats_t *out) {
     }
     out->errors = h.err;
     for (int c = 0; c < 9; c++) out->nslot[c] = v.nslot[c];
-    out->theta = v.theta;
+    for (int c = 0; c < 9; c++) out->run_cap[c] = v.run_cap[c];
+    out->run_bytes = g.cfg.run_bytes;
+    out->slot_base = g.cfg.slot_base;
+    out->slot_min = g.cfg.slot_min;
+    out->run_max = g.cfg.run_max;
+    out->format_ahead = g.cfg.format_ahead;
     out->fence_free = v.fence_free;
     return GALLATIN_OK;
 }

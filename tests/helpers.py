@@ -5,9 +5,10 @@ import os
 
 import numpy as np
 
-from oracle import GID_NONE, TREE_FREE
+from oracle import TREE_FREE
 
 SEG = 1 << 24
+SLOT_EMPTY = 0xFFFFFF            # issued 0, run length 0, no block (include/gallatin.h)
 GOLDEN = os.path.join(os.path.dirname(__file__), "golden", "paper_geometry.txt")
 
 
@@ -48,7 +49,6 @@ def image_sections(img: np.ndarray) -> dict:
     d["qentries"] = q[:, 1:].copy().view(np.uint16).reshape(nseg, 256)
     d["block_free"] = img[p:p + nseg * 128].copy().view(np.uint32); p += nseg * 128
     d["slots"] = img[p:p + S]; p += S
-    d["next"] = img[p:p + S]; p += S
     assert p == len(img)
     return d
 
@@ -80,8 +80,7 @@ def pristine_image(nseg: int, nslots: int) -> np.ndarray:
     q[:, 1:] = 0xFFFFFFFFFFFFFFFF
     out.append(q.reshape(-1))
     out.append(np.zeros(nseg * 128, dtype=np.uint64))
-    out.append(np.full(nslots, (4096 << 32) | GID_NONE, dtype=np.uint64))
-    out.append(np.full(nslots, GID_NONE, dtype=np.uint64))
+    out.append(np.full(nslots, SLOT_EMPTY, dtype=np.uint64))
     return np.concatenate(out)
 
 
@@ -106,7 +105,7 @@ def diff_images(got: np.ndarray, want: np.ndarray) -> str:
         return f"image lengths differ: {len(got)} vs {len(want)}"
     a, b = image_sections(got), image_sections(want)
     for k in ["magic", "nseg", "levels", "W", "nslots", "err", "segtree", "btrees", "segword", "qcount",
-              "qentries", "block_free", "slots", "next"]:
+              "qentries", "block_free", "slots"]:
         x, y = a[k], b[k]
         if isinstance(x, int):
             if x != y:

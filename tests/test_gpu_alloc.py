@@ -37,10 +37,11 @@ def G():
         G.gallatin_destroy()
 
 
-def _replay_case(G, nseg, theta, kinds, args, keys, slot_base=16, slot_min=2):
-    G.gallatin_init(nseg * SEG, slot_base=slot_base, slot_min=slot_min, theta=theta)
+def _replay_case(G, nseg, run_max, fa, kinds, args, keys, slot_base=16, slot_min=2, run_bytes=32 << 20):
+    G.gallatin_init(nseg * SEG, slot_base=slot_base, slot_min=slot_min, run_max=run_max, run_bytes=run_bytes,
+                    format_ahead=1 if fa else 2)
     out = _u64(G.gallatin_replay(_dev(kinds, np.uint8), _dev(args), _dev(keys)))
-    o2 = oracle.Allocator(nseg, slot_base=slot_base, slot_min=slot_min, theta=theta)
+    o2 = oracle.Allocator(nseg, **G.oracle_params())
     want = o2.replay(kinds, args, keys)
     bad = np.nonzero(out != want)[0]
     assert len(bad) == 0, f"{len(bad)} ops differ; first op {bad[0]} kind {kinds[bad[0]]} size {args[bad[0]]}: " \
@@ -51,27 +52,28 @@ def _replay_case(G, nseg, theta, kinds, args, keys, slot_base=16, slot_min=2):
     return out
 
 
-@pytest.mark.parametrize("seed,nseg,theta", [(1, 4, 0), (2, 8, 0), (3, 6, 2048), (4, 64, 0), (5, 5, 100),
-                                             (6, 16, 0), (7, 3, 4095)])
-def test_serialized_replay_matches_oracle(cuda_ok, G, seed, nseg, theta):
+@pytest.mark.parametrize("seed,nseg,run_max,fa", [(1, 4, 1, 0), (2, 8, 1, 0), (3, 6, 16, 1), (4, 64, 8, 1),
+                                                  (5, 5, 128, 0), (6, 16, 4, 1), (7, 3, 2, 1), (8, 32, 1, 1)])
+def test_serialized_replay_matches_oracle(cuda_ok, G, seed, nseg, run_max, fa):
     """Mixed slices / blocks / multi-segment allocations, interleaved frees,
-    drains and OOM on 3-64 segment heaps (SURVEY 8(c) "Scope of serialized replay")."""
+    drains and OOM on 3-64 segment heaps (SURVEY 8(c) "Scope of serialized
+    replay"); run_max=1, fa=0 is the paper's policy."""
     kinds, args, keys = wg.replay_ops(6000, seed + 100, p_free=0.45, p_drain=0.003, nkeys=64)
-    _replay_case(G, nseg, theta, kinds, args, keys)
+    _replay_case(G, nseg, run_max, fa, kinds, args, keys)
 
 
 def test_serialized_replay_block_boundaries(cuda_ok, G):
-    """Exactly-full blocks, exhausted slots, refill and prefetch edges with a
-    single slot per class (every request hits the same slot)."""
-    n = 3 * 4096 + 7
+    """Exactly-full blocks and runs, exhausted slots and refills with a single
+    slot per class (every request hits the same slot)."""
+    n = 7 * 4096 + 7
     kinds = np.zeros(n, dtype=np.uint8)
     args = np.full(n, 16, dtype=np.uint64)
     keys = np.zeros(n, dtype=np.uint64)
     kinds2 = np.concatenate([kinds, np.ones(4096, dtype=np.uint8), np.array([2], dtype=np.uint8)])
     args2 = np.concatenate([args, np.arange(4096, dtype=np.uint64), np.array([0], dtype=np.uint64)])
     keys2 = np.concatenate([keys, np.zeros(4097, dtype=np.uint64)])
-    for theta in (0, 1, 4095):
-        _replay_case(G, 2, theta, kinds2, args2, keys2, slot_base=1, slot_min=1)
+    for run_max, fa in ((1, 0), (4, 1), (128, 1)):
+        _replay_case(G, 2, run_max, fa, kinds2, args2, keys2, slot_base=1, slot_min=1)
 
 
 def _bulk_round(G, nseg, sizes, check_accounting=True):
@@ -118,7 +120,7 @@ def test_config1_concurrent(cuda_ok, G):
     assert _bulk_round(G, nseg, sizes) == 0
     _assert_pristine(G, nseg)
     # accounting equals O2's on the same sizes
-    o2 = oracle.Allocator(nseg)
+    o2 = oracle.Allocator(nseg, **G.oracle_params())
     o2.malloc_batch(sizes)
     assert o2.usable_live == (1 << 16) * 16
 
