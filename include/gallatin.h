@@ -67,7 +67,8 @@ typedef struct gallatin_config {
     uint32_t run_max;
     uint32_t format_ahead;
     uint32_t fence_free;
-    uint32_t reserved[3];
+    uint32_t bulk_items;   /* requests per thread in the bulk kernels: 0 = auto, 1 or 4 */
+    uint32_t reserved[2];
 } gallatin_config_t;
 
 int gallatin_init(uint64_t heap_bytes);                 /* defaults for the rest */

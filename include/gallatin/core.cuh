@@ -154,7 +154,7 @@ __device__ __noinline__ void return_block(const View &v, uint32_t gid) {
     const uint64_t s = gid / kMaxBlocks;
     const uint32_t pos = atomicAdd(v.q_tail + s, 1u) & (kMaxBlocks - 1);
     uint16_t *slotp = v.q_entries + s * kMaxBlocks + pos;
-    ptx::Backoff wb;
+    ptx::Backoff wb(3, (s << 32) | pos);
     while (ptx::ld_relaxed(slotp) != kRingEmpty) wb.pause();   // previous lap's dequeue in flight
     ptx::st_relaxed(slotp, (uint16_t)(gid % kMaxBlocks));
     ptx::fence_acq_rel();
@@ -196,7 +196,7 @@ __device__ __noinline__ void format_ahead(const View &v, uint32_t t) {
 __device__ __noinline__ uint32_t get_run(const View &v, uint32_t t, uint32_t want, uint32_t *first) {
     const BitTree bt = block_tree(v, t);
     const uint32_t nb = nb_of(t);
-    ptx::Backoff bo;
+    ptx::Backoff bo(4, t);
     uint64_t from = 0;
     for (;;) {
         const uint64_t s = bt_successor<false>(bt, from);    // findSegment
@@ -224,7 +224,7 @@ __device__ __noinline__ uint32_t get_run(const View &v, uint32_t t, uint32_t wan
                 for (uint32_t q = 0; q < got; q++) {
                     uint16_t *ep = ring + ((pos + q) & (kMaxBlocks - 1));
                     uint16_t j;
-                    ptx::Backoff wb;
+                    ptx::Backoff wb(2, (s << 32) | ((pos + q) & 0xFFFFFFFFu));
                     while ((j = ptx::ld_relaxed(ep)) == kRingEmpty) wb.pause();   // enqueue in flight
                     ptx::st_relaxed(ep, kRingEmpty);
                     e[q] = j;
@@ -321,10 +321,11 @@ __device__ __forceinline__ uint32_t block_class(uint64_t size) {
 __device__ __noinline__ bool slot_exhausted(const View &v, uint32_t si, uint32_t c, uint64_t old, uint32_t idx) {
     const uint32_t m = (uint32_t)(old >> 24) & 0xFF;
     if (idx == (m << kSliceLog2)) return refill_slot(v, si, c, m);
-    ptx::Backoff bo;
+    ptx::Backoff bo(1, si);
     for (;;) {
         const uint64_t w = ptx::ld_relaxed(slot_word(v, si));
         if ((uint32_t)(w >> 32) <= ((((uint32_t)(w >> 24)) & 0xFF) << kSliceLog2)) return true;
+        bo.note(w);
         bo.pause();
     }
 }
@@ -369,7 +370,7 @@ __device__ __noinline__ void *malloc_block(const View &v, uint32_t t) {
 __device__ __noinline__ void *malloc_large(const View &v, uint64_t k) {
     if (k > v.nseg) return nullptr;
     const BitTree st = seg_tree(v);
-    ptx::Backoff bo;
+    ptx::Backoff bo(5, k);
     uint64_t i;
     int misses = 0;
     for (;;) {

@@ -74,13 +74,41 @@ __device__ __forceinline__ uint32_t lanemask_lt() {
     return r;
 }
 
+#ifdef GALLATIN_DEBUG_SPIN
+// Debug builds only: a spin loop that exceeds GALLATIN_DEBUG_SPIN pauses writes
+// one record {site, smid, lane, value} per (SM, lane) into host-mapped memory
+// the host can read while the kernel is still spinning.
+__device__ uint64_t *g_spin_log = nullptr;
+#endif
+
 // Bounded exponential backoff for spin loops (waiting on another thread's
 // in-flight refill / ring slot): keeps the spinners off the L2 atomic unit.
 struct Backoff {
     uint32_t ns = 32;
+#ifdef GALLATIN_DEBUG_SPIN
+    uint32_t n = 0, site = 0;
+    uint64_t val = 0;
+    __device__ __forceinline__ Backoff() {}
+    __device__ __forceinline__ Backoff(uint32_t s, uint64_t v) : site(s), val(v) {}
+    __device__ __forceinline__ void note(uint64_t v) { val = v; }
+#else
+    __device__ __forceinline__ Backoff() {}
+    __device__ __forceinline__ Backoff(uint32_t, uint64_t) {}
+    __device__ __forceinline__ void note(uint64_t) {}
+#endif
     __device__ __forceinline__ void pause() {
         __nanosleep(ns);
         if (ns < 1024) ns <<= 1;
+#ifdef GALLATIN_DEBUG_SPIN
+        if (++n == GALLATIN_DEBUG_SPIN && g_spin_log) {
+            uint32_t sm, ln;
+            asm volatile("mov.u32 %0, %%smid;" : "=r"(sm));
+            asm volatile("mov.u32 %0, %%laneid;" : "=r"(ln));
+            volatile uint64_t *r = g_spin_log + 2 * ((uint64_t)sm * 32 + ln);
+            r[1] = val;
+            r[0] = ((uint64_t)site << 48) | ((uint64_t)sm << 8) | ln | (1ull << 63);
+        }
+#endif
     }
 };
 

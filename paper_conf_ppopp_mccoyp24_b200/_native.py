@@ -13,7 +13,7 @@ import re
 import numpy as np
 
 _PKG = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_PKG, "libgallatin.so")
+LIB_PATH = os.environ.get("GALLATIN_LIB") or os.path.join(_PKG, "libgallatin.so")
 HEADER = os.path.join(os.path.dirname(_PKG), "include", "gallatin.h")
 
 OK, ERR_INVALID, ERR_CUDA, ERR_STATE, ERR_NOMEM = 0, -1, -2, -3, -4
@@ -28,7 +28,7 @@ class GallatinError(RuntimeError):
 class Config(ctypes.Structure):
     _fields_ = [("heap_bytes", ctypes.c_uint64), ("run_bytes", ctypes.c_uint64), ("slot_base", ctypes.c_uint32),
                 ("slot_min", ctypes.c_uint32), ("run_max", ctypes.c_uint32), ("format_ahead", ctypes.c_uint32),
-                ("fence_free", ctypes.c_uint32), ("reserved", ctypes.c_uint32 * 3)]
+                ("fence_free", ctypes.c_uint32), ("bulk_items", ctypes.c_uint32), ("reserved", ctypes.c_uint32 * 2)]
 
 
 class Stats(ctypes.Structure):
@@ -143,10 +143,10 @@ def _empty64(n: int):
 
 # ------------------------------------------------------------- allocator ---
 def gallatin_init(heap_bytes: int, slot_base: int = 0, slot_min: int = 0, run_max: int = 0, run_bytes: int = 0,
-                  format_ahead: int = 0, fence_free: int = 0) -> None:
+                  format_ahead: int = 0, fence_free: int = 0, bulk_items: int = 0) -> None:
     """0 = library default for every knob (include/gallatin.h gallatin_config_t)."""
     cfg = Config(heap_bytes=heap_bytes, run_bytes=run_bytes, slot_base=slot_base, slot_min=slot_min,
-                 run_max=run_max, format_ahead=format_ahead, fence_free=fence_free)
+                 run_max=run_max, format_ahead=format_ahead, fence_free=fence_free, bulk_items=bulk_items)
     check(lib().gallatin_init_ex(ctypes.byref(cfg)), "gallatin_init")
 
 

@@ -125,22 +125,45 @@ __global__ void __launch_bounds__(kThreads) k_bulk_malloc(View v, const uint64_t
     }
 #pragma unroll
     for (int k = 0; k < ITEMS; k++) old[k] = __shfl_sync(0xFFFFFFFFu, old[k], __ffs((int)peers[k]) - 1);
+    // Pass 1: valid slices, and every refill DUTY this lane drew (index == run
+    // end) -- discharged before this lane waits on anything, because a
+    // later item's duty may be exactly the refill an earlier item would
+    // otherwise wait for (pre-issued RMWs).
     const uint32_t lt = ptx::lanemask_lt();
+    void *p[ITEMS];
+    bool done[ITEMS];
 #pragma unroll
     for (int k = 0; k < ITEMS; k++) {
-        const uint64_t i = base + 32ull * k;
-        void *p = nullptr;
+        p[k] = nullptr;
+        done[k] = sz[k] == 0;
         if (si[k] != 0xFFFFFFFFu) {
             const uint32_t c = core::slice_class(sz[k]);
+            const uint32_t m = ((uint32_t)(old[k] >> 24)) & 0xFF;
             const uint32_t idx = (uint32_t)(old[k] >> 32) + (uint32_t)__popc(peers[k] & lt);
-            if (idx < ((((uint32_t)(old[k] >> 24)) & 0xFF) << core::kSliceLog2))
-                p = core::slice_ptr(v, c, old[k] & core::kRunNone, idx);
-            else if (core::slot_exhausted(v, si[k], c, old[k], idx))
-                p = core::malloc_slice(v, c, key);
-        } else if (sz[k] != 0) {
-            p = core::malloc_impl(v, sz[k], key);
+            if (idx < (m << core::kSliceLog2)) {
+                p[k] = core::slice_ptr(v, c, old[k] & core::kRunNone, idx);
+                done[k] = true;
+            } else if (idx == (m << core::kSliceLog2)) {
+                done[k] = !core::refill_slot(v, si[k], c, m);     // exhausted heap: NULL
+            }
         }
-        if (i < n) __stcs(reinterpret_cast<unsigned long long *>(ptrs) + i, reinterpret_cast<unsigned long long>(p));
+    }
+    // Pass 2: wait-and-retry slices, whole blocks and segment runs.
+#pragma unroll
+    for (int k = 0; k < ITEMS; k++) {
+        if (!done[k]) {
+            if (si[k] != 0xFFFFFFFFu) {
+                const uint32_t c = core::slice_class(sz[k]);
+                const uint32_t idx = (uint32_t)(old[k] >> 32) + (uint32_t)__popc(peers[k] & lt);
+                if (idx > ((((uint32_t)(old[k] >> 24)) & 0xFF) << core::kSliceLog2))
+                    core::slot_exhausted(v, si[k], c, old[k], idx);        // wait for the refill
+                p[k] = core::malloc_slice(v, c, key);
+            } else {
+                p[k] = core::malloc_impl(v, sz[k], key);
+            }
+        }
+        const uint64_t i = base + 32ull * k;
+        if (i < n) __stcs(reinterpret_cast<unsigned long long *>(ptrs) + i, reinterpret_cast<unsigned long long>(p[k]));
     }
 }
 
@@ -390,6 +413,7 @@ int gallatin_init_ex(const gallatin_config_t *cfg_in) {
         if (cfg.run_bytes > (64ull << 20)) cfg.run_bytes = 64ull << 20;
     }
     if (cfg.run_max > core::kMaxRun || cfg.fence_free > 2 || cfg.format_ahead > 2) return GALLATIN_ERR_INVALID;
+    if (cfg.bulk_items != 0 && cfg.bulk_items != 1 && cfg.bulk_items != 4) return GALLATIN_ERR_INVALID;
     if (nseg > (1ull << 16)) return GALLATIN_ERR_INVALID;        // 24-bit run index at 64 KB blocks
 
     View v{};
@@ -481,7 +505,7 @@ int gallatin_malloc(const uint64_t *d_sizes, void **d_ptrs, uint64_t n, void *st
     if (!g.init) return GALLATIN_ERR_STATE;
     if (n == 0) return GALLATIN_OK;
     if (!d_sizes || !d_ptrs || n > (1ull << 40)) return GALLATIN_ERR_INVALID;
-    if (n >= (uint64_t)kItemsMin)
+    if (g.cfg.bulk_items == 4 || (g.cfg.bulk_items == 0 && n >= (uint64_t)kItemsMin))
         k_bulk_malloc<4><<<grid_for((n + 3) / 4), kThreads, 0, S(stream)>>>(g.v, d_sizes, d_ptrs, n);
     else
         k_bulk_malloc<1><<<grid_for(n), kThreads, 0, S(stream)>>>(g.v, d_sizes, d_ptrs, n);
@@ -492,7 +516,7 @@ int gallatin_free(void *const *d_ptrs, uint64_t n, void *stream) {
     if (!g.init) return GALLATIN_ERR_STATE;
     if (n == 0) return GALLATIN_OK;
     if (!d_ptrs || n > (1ull << 40)) return GALLATIN_ERR_INVALID;
-    if (n >= (uint64_t)kItemsMin)
+    if (g.cfg.bulk_items == 4 || (g.cfg.bulk_items == 0 && n >= (uint64_t)kItemsMin))
         k_bulk_free<4><<<grid_for((n + 3) / 4), kThreads, 0, S(stream)>>>(g.v, d_ptrs, n);
     else
         k_bulk_free<1><<<grid_for(n), kThreads, 0, S(stream)>>>(g.v, d_ptrs, n);
@@ -673,3 +697,13 @@ int gallatin_usable(void *const *d_ptrs, const uint64_t *d_sizes, uint64_t n, ui
 }
 
 }  // extern "C"
+
+#ifdef GALLATIN_DEBUG_SPIN
+// Debug builds only (not part of include/gallatin.h): point the spin-loop
+// watchdog records at host-mapped (pinned) memory of 148*32*2 words.
+extern "C" int gallatin_debug_spin_log(void *host_mapped) {
+    if (cudaMemcpyToSymbol(gallatin::ptx::g_spin_log, &host_mapped, sizeof(void *)) != cudaSuccess)
+        return GALLATIN_ERR_CUDA;
+    return GALLATIN_OK;
+}
+#endif

@@ -191,3 +191,19 @@ def test_reset_restores_pristine(cuda_ok, G):
     G.gallatin_reset()
     img = G.gallatin_snapshot()
     assert not diff_images(img, pristine_image(nseg, int(img[4])))
+
+
+@pytest.mark.parametrize("size", wg.SLICE_SIZES)
+def test_config2_full_size_bench_launch(cuda_ok, G, size):
+    """BASELINE configs[1] at its full size, in the launch configuration
+    bench.py times (default knobs, ITEMS=4 bulk kernels): two warm rounds and
+    one after a reset, each stamp-verified, accounted, overlap-checked, and
+    drained back to the pristine image."""
+    nseg = 1024
+    G.gallatin_init(nseg * SEG)
+    n = min(1 << 24, (8 << 30) // size)
+    for rep in range(3):
+        if rep == 2:
+            G.gallatin_reset()
+        assert _bulk_round(G, nseg, wg.single_sizes(size, n)) == 0
+        _assert_pristine(G, nseg)
