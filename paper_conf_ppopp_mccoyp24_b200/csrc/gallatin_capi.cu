@@ -36,6 +36,11 @@ struct State {
 };
 State g;
 
+// The allocator's device view lives in constant memory (set once by init):
+// kernels and the slow paths they call read it through the constant cache
+// instead of materializing a ~300 B kernel-parameter copy per thread.
+__constant__ View c_view;
+
 #define CUDA_TRY(x)                                                                 \
     do {                                                                            \
         cudaError_t e_ = (x);                                                       \
@@ -59,7 +64,8 @@ int launch_status() {
 }
 
 // ------------------------------------------------------------ kernels ----
-__global__ void k_reset(View v) {
+__global__ void k_reset() {
+    const View &v = c_view;
     const uint64_t W = v.tree_words, nseg = v.nseg;
     const uint64_t S = v.nslot_total;
     const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
@@ -95,13 +101,51 @@ __global__ void k_reset(View v) {
     }
 }
 
+// Slow items of one lane of the bulk malloc kernel.  Refill DUTIES (this lane
+// drew exactly the end of a run) are discharged first, before this lane waits
+// on anything: with pre-issued RMWs a later item's duty may be exactly the
+// refill an earlier item would otherwise wait for.
+// Then waits-and-retries, whole blocks and segment runs.
+__device__ __noinline__ void bulk_malloc_slow(const uint64_t *sizes, void **ptrs, uint64_t n, uint64_t base,
+                                              uint32_t key, uint32_t slow, uint64_t info, int items) {
+    const View &v = c_view;
+    // pass 0: refill duties only (never waits on another slot's refill)
+    for (int k = 0; k < items; k++) {
+        const uint32_t code = (uint32_t)(info >> (16 * k)) & 0xFFFF;
+        if (!((slow >> k) & 1) || !(code & 0x100u)) continue;
+        const uint64_t i = base + 32ull * k;
+        const uint32_t c = core::slice_class(sizes[i]);
+        if (!core::refill_slot(v, v.slot_off[c] + key % v.nslot[c], c, code & 0xFF)) {
+            __stcs(reinterpret_cast<unsigned long long *>(ptrs) + i, 0ull);   // heap exhausted: NULL
+            slow &= ~(1u << k);
+        }
+    }
+    // pass 1: retries after a refill, waits, whole blocks and segment runs
+    for (int k = 0; k < items; k++) {
+        if (!((slow >> k) & 1)) continue;
+        const uint32_t code = (uint32_t)(info >> (16 * k)) & 0xFFFF;
+        const uint64_t i = base + 32ull * k;
+        const uint64_t sz = sizes[i];
+        void *p;
+        if (code & 0x200u) {
+            p = core::malloc_impl(v, sz, key);
+        } else {
+            const uint32_t c = core::slice_class(sz);
+            if (code & 0x400u) core::slot_exhausted(v, v.slot_off[c] + key % v.nslot[c], c, 0, ~0u);  // wait
+            p = core::malloc_slice(v, c, key);
+        }
+        __stcs(reinterpret_cast<unsigned long long *>(ptrs) + i, reinterpret_cast<unsigned long long>(p));
+    }
+}
+
 // Bulk malloc, ITEMS requests per thread: all slice requests first issue their
 // team RMW (one per team per item, back to back: memory-level parallelism),
 // then take their slice; refills, waits, blocks and large requests follow on
 // the per-request device path.  Lane l of warp w handles w*32*ITEMS + k*32 + l.
 template <int ITEMS>
-__global__ void __launch_bounds__(kThreads) k_bulk_malloc(View v, const uint64_t *__restrict__ sizes,
-                                                          void **__restrict__ ptrs, uint64_t n) {
+__global__ void __launch_bounds__(kThreads) k_bulk_malloc(const uint64_t *__restrict__ sizes, void **__restrict__ ptrs,
+                                                          uint64_t n) {
+    const View &v = c_view;
     const uint32_t lane = threadIdx.x & 31;
     const uint64_t base = ((blockIdx.x * (uint64_t)kThreads + threadIdx.x) >> 5) * (32 * ITEMS) + lane;
     const uint32_t key = ptx::smid();
@@ -125,46 +169,35 @@ __global__ void __launch_bounds__(kThreads) k_bulk_malloc(View v, const uint64_t
     }
 #pragma unroll
     for (int k = 0; k < ITEMS; k++) old[k] = __shfl_sync(0xFFFFFFFFu, old[k], __ffs((int)peers[k]) - 1);
-    // Pass 1: valid slices, and every refill DUTY this lane drew (index == run
-    // end) -- discharged before this lane waits on anything, because a
-    // later item's duty may be exactly the refill an earlier item would
-    // otherwise wait for (pre-issued RMWs).
+    // Fast path: every valid slice is computed and stored here; what a slow
+    // item needs later is packed into one byte per item (bit 7..0: run length
+    // of a refill duty, 0x100 duty flag, 0x200 not-a-slice, 0x400 wait), so no
+    // fast-path state is live across the slow path's calls.
     const uint32_t lt = ptx::lanemask_lt();
-    void *p[ITEMS];
-    bool done[ITEMS];
+    uint32_t slow = 0;
+    uint64_t info = 0;
 #pragma unroll
     for (int k = 0; k < ITEMS; k++) {
-        p[k] = nullptr;
-        done[k] = sz[k] == 0;
+        const uint64_t i = base + 32ull * k;
+        void *p = nullptr;
+        uint32_t code = 0;
         if (si[k] != 0xFFFFFFFFu) {
             const uint32_t c = core::slice_class(sz[k]);
             const uint32_t m = ((uint32_t)(old[k] >> 24)) & 0xFF;
             const uint32_t idx = (uint32_t)(old[k] >> 32) + (uint32_t)__popc(peers[k] & lt);
-            if (idx < (m << core::kSliceLog2)) {
-                p[k] = core::slice_ptr(v, c, old[k] & core::kRunNone, idx);
-                done[k] = true;
-            } else if (idx == (m << core::kSliceLog2)) {
-                done[k] = !core::refill_slot(v, si[k], c, m);     // exhausted heap: NULL
-            }
+            if (idx < (m << core::kSliceLog2)) p = core::slice_ptr(v, c, old[k] & core::kRunNone, idx);
+            else code = idx == (m << core::kSliceLog2) ? (0x100u | m) : 0x400u;
+        } else if (sz[k] != 0) {
+            code = 0x200u;
+        }
+        if (code) {
+            slow |= 1u << k;
+            info |= (uint64_t)code << (16 * k);
+        } else if (i < n) {
+            __stcs(reinterpret_cast<unsigned long long *>(ptrs) + i, reinterpret_cast<unsigned long long>(p));
         }
     }
-    // Pass 2: wait-and-retry slices, whole blocks and segment runs.
-#pragma unroll
-    for (int k = 0; k < ITEMS; k++) {
-        if (!done[k]) {
-            if (si[k] != 0xFFFFFFFFu) {
-                const uint32_t c = core::slice_class(sz[k]);
-                const uint32_t idx = (uint32_t)(old[k] >> 32) + (uint32_t)__popc(peers[k] & lt);
-                if (idx > ((((uint32_t)(old[k] >> 24)) & 0xFF) << core::kSliceLog2))
-                    core::slot_exhausted(v, si[k], c, old[k], idx);        // wait for the refill
-                p[k] = core::malloc_slice(v, c, key);
-            } else {
-                p[k] = core::malloc_impl(v, sz[k], key);
-            }
-        }
-        const uint64_t i = base + 32ull * k;
-        if (i < n) __stcs(reinterpret_cast<unsigned long long *>(ptrs) + i, reinterpret_cast<unsigned long long>(p[k]));
-    }
+    if (slow) bulk_malloc_slow(sizes, ptrs, n, base, key, slow, info, ITEMS);
 }
 
 __device__ __noinline__ void free_slow(const View &v, uint64_t p) {
@@ -176,11 +209,33 @@ __device__ __noinline__ void free_slow(const View &v, uint64_t p) {
     core::free_large(v, s, t);
 }
 
+// Rare items of one lane of the bulk free kernel: block returns (this team's
+// free completed 4096) and frees that are not slices/blocks.  The block id is
+// re-derived from the pointer: a segment's tree id cannot change while one of
+// its blocks is out.
+__device__ __noinline__ void bulk_free_slow(void *const *ptrs, uint64_t base, uint32_t done, uint32_t slow, int items) {
+    const View &v = c_view;
+    for (int k = 0; k < items; k++) {
+        const uint64_t p = reinterpret_cast<uint64_t>(ptrs[base + 32ull * k]);
+        if ((done >> k) & 1) {
+            const uint64_t off = p - v.heap;
+            const uint32_t t = core::sw_tree(ptx::ld_relaxed(v.seg_word + (off >> core::kSegLog2)));
+            const uint32_t gid =
+                (uint32_t)((off >> core::kSegLog2) * core::kMaxBlocks + ((off & (core::kSegBytes - 1)) >> (16 + t)));
+            atomicExch(v.block_free + gid, 0u);
+            ptx::fence_acq_rel();
+            core::return_block(v, gid);
+        }
+        if ((slow >> k) & 1) free_slow(v, p);
+    }
+}
+
 // Bulk free, ITEMS pointers per thread: load pointers, then their segments'
 // table words, team the lanes freeing one block, one release fence
 // per leading lane, then the team counter RMWs back to back.
 template <int ITEMS>
-__global__ void __launch_bounds__(kThreads) k_bulk_free(View v, void *const *__restrict__ ptrs, uint64_t n) {
+__global__ void __launch_bounds__(kThreads) k_bulk_free(void *const *__restrict__ ptrs, uint64_t n) {
+    const View &v = c_view;
     const uint32_t lane = threadIdx.x & 31;
     const uint64_t base = ((blockIdx.x * (uint64_t)kThreads + threadIdx.x) >> 5) * (32 * ITEMS) + lane;
     const uint64_t heap_bytes = v.nseg << core::kSegLog2;
@@ -219,19 +274,19 @@ __global__ void __launch_bounds__(kThreads) k_bulk_free(View v, void *const *__r
         if (peers[k] && lane == (uint32_t)__ffs((int)peers[k]) - 1)
             oldc[k] = atomicAdd(v.block_free + gid[k], (uint32_t)__popc(peers[k]));
     }
+    uint32_t done = 0, slow = 0;
 #pragma unroll
     for (int k = 0; k < ITEMS; k++) {
-        if (peers[k] && lane == (uint32_t)__ffs((int)peers[k]) - 1 && oldc[k] + __popc(peers[k]) == core::kSlices) {
-            atomicExch(v.block_free + gid[k], 0u);                   // the 4096th free
-            ptx::fence_acq_rel();
-            core::return_block(v, gid[k]);
-        }
-        if (p[k] && !peers[k]) free_slow(v, p[k]);
+        if (peers[k] && lane == (uint32_t)__ffs((int)peers[k]) - 1 && oldc[k] + __popc(peers[k]) == core::kSlices)
+            done |= 1u << k;                                         // the 4096th free
+        if (p[k] && !peers[k]) slow |= 1u << k;
     }
+    if (done | slow) bulk_free_slow(ptrs, base, done, slow, ITEMS);
 }
 
-__global__ void k_replay(View v, const uint8_t *kinds, const uint64_t *args, const uint64_t *keys, uint64_t n,
+__global__ void k_replay(const uint8_t *kinds, const uint64_t *args, const uint64_t *keys, uint64_t n,
                          uint64_t *out) {
+    const View &v = c_view;
     for (uint64_t i = 0; i < n; i++) {
         const uint8_t k = kinds[i];
         if (k == 0) {
@@ -249,9 +304,10 @@ __global__ void k_replay(View v, const uint8_t *kinds, const uint64_t *args, con
     }
 }
 
-__global__ void k_drain_slots(View v) { core::drain_slots(v); }
+__global__ void k_drain_slots() { core::drain_slots(c_view); }
 
-__global__ void k_retire_idle(View v) {
+__global__ void k_retire_idle() {
+    const View &v = c_view;
     const uint64_t s = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
     if (s < v.nseg) core::retire_idle(v, s);
 }
@@ -295,8 +351,9 @@ __global__ void k_verify(void *const *ptrs, const uint64_t *sizes, uint64_t n, u
     if (lane == 0 && mine) atomicAdd(bad, mine);
 }
 
-__global__ void k_usable(View v, void *const *ptrs, const uint64_t *sizes, uint64_t n, uint64_t *usable,
+__global__ void k_usable(void *const *ptrs, const uint64_t *sizes, uint64_t n, uint64_t *usable,
                          unsigned long long *sum, unsigned long long *bad) {
+    const View &v = c_view;
     const uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
     if (i >= n) return;
     const uint64_t p = reinterpret_cast<uint64_t>(ptrs[i]);
@@ -473,6 +530,7 @@ int gallatin_init_ex(const gallatin_config_t *cfg_in) {
     g.meta = meta;
     g.meta_bytes = total;
     g.v = v;
+    if (cudaMemcpyToSymbol(c_view, &v, sizeof(View)) != cudaSuccess) { free_all(); return GALLATIN_ERR_CUDA; }
     const int rc = gallatin_reset(nullptr);
     if (rc != GALLATIN_OK) { free_all(); return rc; }
     CUDA_TRY(cudaDeviceSynchronize());
@@ -497,7 +555,7 @@ int gallatin_reset(void *stream) {
     if ((uint64_t)g.v.nslot_total * 16 > n) n = (uint64_t)g.v.nslot_total * 16;
     unsigned grid = grid_for(n);
     if (grid > 148 * 16) grid = 148 * 16;
-    k_reset<<<grid, kThreads, 0, S(stream)>>>(g.v);
+    k_reset<<<grid, kThreads, 0, S(stream)>>>();
     return launch_status();
 }
 
@@ -506,9 +564,9 @@ int gallatin_malloc(const uint64_t *d_sizes, void **d_ptrs, uint64_t n, void *st
     if (n == 0) return GALLATIN_OK;
     if (!d_sizes || !d_ptrs || n > (1ull << 40)) return GALLATIN_ERR_INVALID;
     if (g.cfg.bulk_items == 4 || (g.cfg.bulk_items == 0 && n >= (uint64_t)kItemsMin))
-        k_bulk_malloc<4><<<grid_for((n + 3) / 4), kThreads, 0, S(stream)>>>(g.v, d_sizes, d_ptrs, n);
+        k_bulk_malloc<4><<<grid_for((n + 3) / 4), kThreads, 0, S(stream)>>>(d_sizes, d_ptrs, n);
     else
-        k_bulk_malloc<1><<<grid_for(n), kThreads, 0, S(stream)>>>(g.v, d_sizes, d_ptrs, n);
+        k_bulk_malloc<1><<<grid_for(n), kThreads, 0, S(stream)>>>(d_sizes, d_ptrs, n);
     return launch_status();
 }
 
@@ -517,9 +575,9 @@ int gallatin_free(void *const *d_ptrs, uint64_t n, void *stream) {
     if (n == 0) return GALLATIN_OK;
     if (!d_ptrs || n > (1ull << 40)) return GALLATIN_ERR_INVALID;
     if (g.cfg.bulk_items == 4 || (g.cfg.bulk_items == 0 && n >= (uint64_t)kItemsMin))
-        k_bulk_free<4><<<grid_for((n + 3) / 4), kThreads, 0, S(stream)>>>(g.v, d_ptrs, n);
+        k_bulk_free<4><<<grid_for((n + 3) / 4), kThreads, 0, S(stream)>>>(d_ptrs, n);
     else
-        k_bulk_free<1><<<grid_for(n), kThreads, 0, S(stream)>>>(g.v, d_ptrs, n);
+        k_bulk_free<1><<<grid_for(n), kThreads, 0, S(stream)>>>(d_ptrs, n);
     return launch_status();
 }
 
@@ -565,10 +623,10 @@ int gallatin_free_host(const uint64_t *h_ptrs, uint64_t n, void *stream) {
 
 int gallatin_drain(void *stream) {
     if (!g.init) return GALLATIN_ERR_STATE;
-    k_drain_slots<<<1, 1, 0, S(stream)>>>(g.v);
+    k_drain_slots<<<1, 1, 0, S(stream)>>>();
     int rc = launch_status();
     if (rc) return rc;
-    k_retire_idle<<<grid_for(g.v.nseg), kThreads, 0, S(stream)>>>(g.v);
+    k_retire_idle<<<grid_for(g.v.nseg), kThreads, 0, S(stream)>>>();
     return launch_status();
 }
 
@@ -577,7 +635,7 @@ int gallatin_replay(const uint8_t *d_kinds, const uint64_t *d_args, const uint64
     if (!g.init) return GALLATIN_ERR_STATE;
     if (n == 0) return GALLATIN_OK;
     if (!d_kinds || !d_args || !d_keys || !d_out) return GALLATIN_ERR_INVALID;
-    k_replay<<<1, 1, 0, S(stream)>>>(g.v, d_kinds, d_args, d_keys, n, d_out);
+    k_replay<<<1, 1, 0, S(stream)>>>(d_kinds, d_args, d_keys, n, d_out);
     return launch_status();
 }
 
@@ -690,7 +748,7 @@ int gallatin_usable(void *const *d_ptrs, const uint64_t *d_sizes, uint64_t n, ui
     if (!g.init) return GALLATIN_ERR_STATE;
     if (n == 0) return GALLATIN_OK;
     if (!d_ptrs || !d_sizes || !d_sum || !d_bad) return GALLATIN_ERR_INVALID;
-    k_usable<<<grid_for(n), kThreads, 0, S(stream)>>>(g.v, d_ptrs, d_sizes, n, d_usable,
+    k_usable<<<grid_for(n), kThreads, 0, S(stream)>>>(d_ptrs, d_sizes, n, d_usable,
                                                      reinterpret_cast<unsigned long long *>(d_sum),
                                                      reinterpret_cast<unsigned long long *>(d_bad));
     return launch_status();
