@@ -33,7 +33,8 @@ constexpr uint32_t kTreeCont = 0xFFFFFFFEu;
 constexpr uint32_t kGidNone = 0xFFFFFFFFu;
 constexpr uint32_t kAvailBias = 0x80000000u;
 constexpr uint16_t kRingEmpty = 0xFFFF;
-constexpr uint32_t kMaxRun = 128;                   // blocks per slot run (8-bit field)
+constexpr uint32_t kMaxRun = 512;                   // blocks per slot run (10-bit field)
+constexpr uint32_t kRunShift = 22;                  // slot word: issued:32 | run:10 | first:22
 
 __device__ __forceinline__ uint32_t nb_of(uint32_t t) { return kMaxBlocks >> t; }
 
@@ -286,8 +287,9 @@ __device__ __noinline__ uint32_t get_run(const View &v, uint32_t t, uint32_t wan
 // ---- addresses -------------------------------------------------------------
 __device__ __forceinline__ uint64_t *slot_word(const View &v, uint32_t si) { return v.slots + (uint64_t)si * 16; }
 
-constexpr uint32_t kRunNone = 0xFFFFFFu;
+constexpr uint32_t kRunNone = 0x3FFFFFu;
 constexpr uint64_t kSlotEmpty = kRunNone;                 // issued 0, run 0: refill on first use
+__device__ __forceinline__ uint32_t run_len(uint64_t w) { return (uint32_t)(w >> kRunShift) & 0x3FFu; }
 
 // Replace an exhausted run (Alg.3): the run doubles up to the class cap.
 __device__ __noinline__ bool refill_slot(const View &v, uint32_t si, uint32_t c, uint32_t m_prev) {
@@ -299,7 +301,7 @@ __device__ __noinline__ bool refill_slot(const View &v, uint32_t si, uint32_t c,
         ptx::atom_exch(slot_word(v, si), kSlotEmpty);
         return false;
     }
-    ptx::atom_exch(slot_word(v, si), ((uint64_t)got << 24) | first);
+    ptx::atom_exch(slot_word(v, si), ((uint64_t)got << kRunShift) | first);
     return true;
 }
 
@@ -319,12 +321,12 @@ __device__ __forceinline__ uint32_t block_class(uint64_t size) {
 // refill (the lane that drew exactly the end) or wait for the refill.
 // Returns false if the refill found no memory.
 __device__ __noinline__ bool slot_exhausted(const View &v, uint32_t si, uint32_t c, uint64_t old, uint32_t idx) {
-    const uint32_t m = (uint32_t)(old >> 24) & 0xFF;
+    const uint32_t m = run_len(old);
     if (idx == (m << kSliceLog2)) return refill_slot(v, si, c, m);
     ptx::Backoff bo(1, si);
     for (;;) {
         const uint64_t w = ptx::ld_relaxed(slot_word(v, si));
-        if ((uint32_t)(w >> 32) <= ((((uint32_t)(w >> 24)) & 0xFF) << kSliceLog2)) return true;
+        if ((uint32_t)(w >> 32) <= (run_len(w) << kSliceLog2)) return true;
         bo.note(w);
         bo.pause();
     }
@@ -351,7 +353,7 @@ __device__ inline void *malloc_slice(const View &v, uint32_t c, uint32_t key) {
         if (lane == leader) old = ptx::atom_add(sw, (uint64_t)__popc(peers) << 32);
         old = __shfl_sync(peers, old, (int)leader);
         const uint32_t idx = (uint32_t)(old >> 32) + rank;
-        if (idx < ((((uint32_t)(old >> 24)) & 0xFF) << kSliceLog2)) return slice_ptr(v, c, old & kRunNone, idx);
+        if (idx < (run_len(old) << kSliceLog2)) return slice_ptr(v, c, old & kRunNone, idx);
         if (!slot_exhausted(v, si, c, old, idx)) return nullptr;   // nullptr
     }
 }
@@ -440,7 +442,7 @@ __device__ inline void drain_slots(const View &v) {
         for (uint32_t q = 0; q < v.nslot[c]; q++) {
             const uint64_t w = ptx::atom_exch(slot_word(v, v.slot_off[c] + q), kSlotEmpty);
             const uint64_t cnt = w >> 32;
-            const uint32_t m = (uint32_t)(w >> 24) & 0xFF;
+            const uint32_t m = run_len(w);
             const uint64_t first = w & kRunNone;
             for (uint32_t k = 0; k < m; k++) {
                 const uint64_t lo = (uint64_t)k << kSliceLog2;

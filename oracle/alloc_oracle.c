@@ -99,7 +99,7 @@ typedef struct o2 {
     uint32_t *freecnt;            /* per block free counter     */
     oracle_veb *segfree;          /* segment tree               */
     oracle_veb *btree[NUM_BLOCK_TREES];  /* block trees         */
-    uint64_t *slot;               /* cnt << 32 | m << 24 | first block  */
+    uint64_t *slot;               /* cnt << 32 | m << 22 | first block  */
     uint64_t err;                 /* out-of-heap / non-allocated segment frees */
     /* oracle-only bookkeeping for the invariant checks */
     kv_t *live; uint64_t live_cap, live_n;
@@ -153,15 +153,16 @@ static int live_take(o2_t *a, uint64_t k, uint64_t *v) {
 }
 
 /* ---------------------------------------------------------- lifecycle --- */
-#define RUN_NONE 0xFFFFFFu
+#define RUN_NONE 0x3FFFFFu                          /* 22-bit first block */
+#define RUN_SHIFT 22                                /* 10-bit run length  */
 #define SLOT_EMPTY ((uint64_t)RUN_NONE)            /* cnt 0, m 0: refill on first use */
 static uint64_t slot_make(uint64_t cnt, uint32_t m, uint32_t first) {
-    return (cnt << 32) | ((uint64_t)m << 24) | first;
+    return (cnt << 32) | ((uint64_t)m << RUN_SHIFT) | first;
 }
 
 o2_t *o2_create(uint64_t nseg, unsigned slot_base, unsigned slot_min, unsigned run_max,
                 uint64_t run_bytes, unsigned format_ahead) {
-    if (nseg < 1 || nseg > (1ULL << 16) || slot_base < 1 || run_max < 1 || run_max > 128) return NULL;
+    if (nseg < 1 || nseg > (1ULL << 14) || slot_base < 1 || run_max < 1 || run_max > 512) return NULL;
     o2_t *a = (o2_t *)calloc(1, sizeof(o2_t));
     a->nseg = nseg; a->slot_base = slot_base; a->slot_min = slot_min;
     a->run_max = run_max; a->run_bytes = run_bytes; a->format_ahead = format_ahead;
@@ -368,7 +369,7 @@ static uint64_t malloc_slice(o2_t *a, uint32_t c, uint64_t key) {
     unsigned i = a->slot_off[c] + (unsigned)(key % a->nslot[c]);
     for (;;) {
         uint64_t cnt = a->slot[i] >> 32;
-        uint32_t m = (uint32_t)(a->slot[i] >> 24) & 0xFF;
+        uint32_t m = (uint32_t)(a->slot[i] >> RUN_SHIFT) & 0x3FF;
         uint32_t first = (uint32_t)a->slot[i] & RUN_NONE;
         if (cnt < SLICES_PER_BLOCK * m) {                   /* valid = idx < 4096 (per block) */
             a->slot[i] = slot_make(cnt + 1, m, first);
@@ -466,7 +467,7 @@ void o2_drain(o2_t *a) {
         for (unsigned q = 0; q < a->nslot[c]; q++) {
             unsigned i = a->slot_off[c] + q;
             uint64_t cnt = a->slot[i] >> 32;
-            uint32_t m = (uint32_t)(a->slot[i] >> 24) & 0xFF;
+            uint32_t m = (uint32_t)(a->slot[i] >> RUN_SHIFT) & 0x3FF;
             uint32_t first = (uint32_t)a->slot[i] & RUN_NONE;
             a->slot[i] = SLOT_EMPTY;
             for (uint32_t k = 0; k < m; k++) {

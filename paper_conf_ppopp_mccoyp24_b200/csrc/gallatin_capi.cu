@@ -112,10 +112,10 @@ __device__ __noinline__ void bulk_malloc_slow(const uint64_t *sizes, void **ptrs
     // pass 0: refill duties only (never waits on another slot's refill)
     for (int k = 0; k < items; k++) {
         const uint32_t code = (uint32_t)(info >> (16 * k)) & 0xFFFF;
-        if (!((slow >> k) & 1) || !(code & 0x100u)) continue;
+        if (!((slow >> k) & 1) || !(code & 0x400u)) continue;
         const uint64_t i = base + 32ull * k;
         const uint32_t c = core::slice_class(sizes[i]);
-        if (!core::refill_slot(v, v.slot_off[c] + key % v.nslot[c], c, code & 0xFF)) {
+        if (!core::refill_slot(v, v.slot_off[c] + key % v.nslot[c], c, code & 0x3FF)) {
             __stcs(reinterpret_cast<unsigned long long *>(ptrs) + i, 0ull);   // heap exhausted: NULL
             slow &= ~(1u << k);
         }
@@ -127,11 +127,11 @@ __device__ __noinline__ void bulk_malloc_slow(const uint64_t *sizes, void **ptrs
         const uint64_t i = base + 32ull * k;
         const uint64_t sz = sizes[i];
         void *p;
-        if (code & 0x200u) {
+        if (code & 0x800u) {
             p = core::malloc_impl(v, sz, key);
         } else {
             const uint32_t c = core::slice_class(sz);
-            if (code & 0x400u) core::slot_exhausted(v, v.slot_off[c] + key % v.nslot[c], c, 0, ~0u);  // wait
+            if (code & 0x1000u) core::slot_exhausted(v, v.slot_off[c] + key % v.nslot[c], c, 0, ~0u);  // wait
             p = core::malloc_slice(v, c, key);
         }
         __stcs(reinterpret_cast<unsigned long long *>(ptrs) + i, reinterpret_cast<unsigned long long>(p));
@@ -170,9 +170,9 @@ __global__ void __launch_bounds__(kThreads) k_bulk_malloc(const uint64_t *__rest
 #pragma unroll
     for (int k = 0; k < ITEMS; k++) old[k] = __shfl_sync(0xFFFFFFFFu, old[k], __ffs((int)peers[k]) - 1);
     // Fast path: every valid slice is computed and stored here; what a slow
-    // item needs later is packed into one byte per item (bit 7..0: run length
-    // of a refill duty, 0x100 duty flag, 0x200 not-a-slice, 0x400 wait), so no
-    // fast-path state is live across the slow path's calls.
+    // item needs later is packed into 16 bits per item (bits 9..0: run length
+    // of a refill duty, 0x400 duty flag, 0x800 not-a-slice, 0x1000 wait), so
+    // no fast-path state is live across the slow path's calls.
     const uint32_t lt = ptx::lanemask_lt();
     uint32_t slow = 0;
     uint64_t info = 0;
@@ -183,12 +183,12 @@ __global__ void __launch_bounds__(kThreads) k_bulk_malloc(const uint64_t *__rest
         uint32_t code = 0;
         if (si[k] != 0xFFFFFFFFu) {
             const uint32_t c = core::slice_class(sz[k]);
-            const uint32_t m = ((uint32_t)(old[k] >> 24)) & 0xFF;
+            const uint32_t m = core::run_len(old[k]);
             const uint32_t idx = (uint32_t)(old[k] >> 32) + (uint32_t)__popc(peers[k] & lt);
             if (idx < (m << core::kSliceLog2)) p = core::slice_ptr(v, c, old[k] & core::kRunNone, idx);
-            else code = idx == (m << core::kSliceLog2) ? (0x100u | m) : 0x400u;
+            else code = idx == (m << core::kSliceLog2) ? (0x400u | m) : 0x1000u;
         } else if (sz[k] != 0) {
-            code = 0x200u;
+            code = 0x800u;
         }
         if (code) {
             slow |= 1u << k;
@@ -464,14 +464,14 @@ int gallatin_init_ex(const gallatin_config_t *cfg_in) {
     if (!cfg.slot_min) cfg.slot_min = 4;                     // "capped at four"
     if (!cfg.fence_free) cfg.fence_free = 1;
     if (!cfg.format_ahead) cfg.format_ahead = 1;
-    if (!cfg.run_max) cfg.run_max = 16;
+    if (!cfg.run_max) cfg.run_max = 256;
     if (!cfg.run_bytes) {
         cfg.run_bytes = (nseg << core::kSegLog2) / 64;
-        if (cfg.run_bytes > (64ull << 20)) cfg.run_bytes = 64ull << 20;
+        if (cfg.run_bytes > (256ull << 20)) cfg.run_bytes = 256ull << 20;
     }
     if (cfg.run_max > core::kMaxRun || cfg.fence_free > 2 || cfg.format_ahead > 2) return GALLATIN_ERR_INVALID;
     if (cfg.bulk_items != 0 && cfg.bulk_items != 1 && cfg.bulk_items != 4) return GALLATIN_ERR_INVALID;
-    if (nseg > (1ull << 16)) return GALLATIN_ERR_INVALID;        // 24-bit run index at 64 KB blocks
+    if (nseg > (1ull << 14)) return GALLATIN_ERR_INVALID;        // 22-bit run index at 64 KB blocks (256 GiB)
 
     View v{};
     v.nseg = nseg;

@@ -8,7 +8,7 @@ import numpy as np
 from oracle import TREE_FREE
 
 SEG = 1 << 24
-SLOT_EMPTY = 0xFFFFFF            # issued 0, run length 0, no block (include/gallatin.h)
+SLOT_EMPTY = 0x3FFFFF            # issued 0, run length 0, no block (include/gallatin.h)
 GOLDEN = os.path.join(os.path.dirname(__file__), "golden", "paper_geometry.txt")
 
 
