@@ -120,11 +120,16 @@ __device__ __noinline__ void try_free_segment(const View &v, uint64_t s, uint32_
 // ---- Alg. 1 GetSegment(treeId < numBlockTrees) ----------------
 // successor(0) on the segment tree + claimIndex, front first
 // (P:138).  Returns the claimed segment or kNone when every segment is in use.
+// A claimer that loses the race for segment s moves on to successor(s + 1)
+// instead of re-reading from 0, so k concurrent claimers spread over the k
+// lowest free segments in O(k) total RMWs (serially this is successor(0)).
 __device__ __noinline__ uint64_t claim_front(const View &v) {
     const BitTree st = seg_tree(v);
+    uint64_t from = 0;
     for (;;) {
-        uint64_t s = bt_successor<false>(st, 0);
+        uint64_t s = bt_successor<false>(st, from);
         if (s == kNone) {
+            if (from != 0) { from = 0; continue; }
             s = bt_scan_first(st);                         // confirm before failing
             if (s == kNone) return kNone;                  // "All segments in use"
         }
@@ -132,6 +137,7 @@ __device__ __noinline__ uint64_t claim_front(const View &v) {
             ptx::fence_acq_rel();
             return s;
         }
+        from = s + 1;
     }
 }
 
@@ -141,7 +147,14 @@ __device__ __noinline__ uint64_t claim_front(const View &v) {
 __device__ __noinline__ void format_segment(const View &v, uint64_t s, uint32_t t, uint32_t keep) {
     const uint32_t nb = nb_of(t);
     uint16_t *e = v.q_entries + s * kMaxBlocks;
-    for (uint32_t j = keep; j < nb; j++) e[j - keep] = (uint16_t)j;
+    const uint32_t cnt = nb - keep;                       // entries at positions 0 .. cnt-1
+    uint64_t *e4 = reinterpret_cast<uint64_t *>(e);
+    uint32_t q = 0;
+    for (; q + 4 <= cnt; q += 4) {
+        const uint64_t j = keep + q;
+        e4[q / 4] = j | ((j + 1) << 16) | ((j + 2) << 32) | ((j + 3) << 48);
+    }
+    for (; q < cnt; q++) e[q] = (uint16_t)(keep + q);
     ptx::st_relaxed(v.q_head + s, 0u);
     ptx::st_relaxed(v.q_tail + s, nb - keep);
     ptx::fence_acq_rel();
@@ -179,16 +192,28 @@ __device__ __forceinline__ uint32_t gid_of(uint32_t t, uint64_t linear) {
     return (uint32_t)(((linear >> sh) << 8) | (linear & ((1u << sh) - 1)));
 }
 
+// [dev] formatter tokens: at most kFormatters threads format segments for
+// one tree at a time (the paper lets every waiting thread format, P:151-155;
+// one at a time would serialize the bursts in which every slot refills).
+constexpr uint32_t kFormatters = 8;
+__device__ __forceinline__ bool token_try(uint32_t *tok) {
+    if (atomicAdd(tok, 1u) < kFormatters) return true;
+    atomicSub(tok, 1u);
+    return false;
+}
+__device__ __forceinline__ void token_release(uint32_t *tok) {
+    ptx::fence_acq_rel();
+    atomicSub(tok, 1u);
+}
+
 // [dev] format one more segment for tree t when the current one runs low, so
-// that refills rarely wait for a format (one formatter per tree; skipped if
-// the formatter token is busy).
+// that refills rarely wait for a format (skipped if every token is busy).
 __device__ __noinline__ void format_ahead(const View &v, uint32_t t) {
     uint32_t *tok = v.fmt_token + t * 32;
-    if (atomicCAS(tok, 0u, 1u) != 0u) return;
+    if (!token_try(tok)) return;
     const uint64_t s = claim_front(v);
     if (s != kNone) format_segment(v, s, t, 0);
-    ptx::fence_acq_rel();
-    atomicExch(tok, 0u);
+    token_release(tok);
 }
 
 // ---- Alg. 2 GetBlock(treeId), for a RUN of blocks [dev] --------
@@ -222,14 +247,27 @@ __device__ __noinline__ uint32_t get_run(const View &v, uint32_t t, uint32_t wan
                 uint16_t *ring = v.q_entries + s * kMaxBlocks;
                 uint16_t e[kMaxRun];
                 uint32_t p = 1;
-                for (uint32_t q = 0; q < got; q++) {
-                    uint16_t *ep = ring + ((pos + q) & (kMaxBlocks - 1));
-                    uint16_t j;
-                    ptx::Backoff wb(2, (s << 32) | ((pos + q) & 0xFFFFFFFFu));
-                    while ((j = ptx::ld_relaxed(ep)) == kRingEmpty) wb.pause();   // enqueue in flight
-                    ptx::st_relaxed(ep, kRingEmpty);
-                    e[q] = j;
-                    if (q == p && j == e[0] + q) p++;          // consecutive prefix
+                // 16 independent loads in flight per batch (not one round trip per entry)
+                for (uint32_t b = 0; b < got; b += 16) {
+                    uint16_t r[16];
+#pragma unroll
+                    for (int u = 0; u < 16; u++)
+                        if (b + u < got) r[u] = ptx::ld_relaxed(ring + ((pos + b + u) & (kMaxBlocks - 1)));
+#pragma unroll
+                    for (int u = 0; u < 16; u++) {
+                        const uint32_t q = b + u;
+                        if (q >= got) break;
+                        uint16_t *ep = ring + ((pos + q) & (kMaxBlocks - 1));
+                        uint16_t j = r[u];
+                        ptx::Backoff wb(2, (s << 32) | ((pos + q) & 0xFFFFFFFFu));
+                        while (j == kRingEmpty) {                 // enqueue in flight
+                            wb.pause();
+                            j = ptx::ld_relaxed(ep);
+                        }
+                        ptx::st_relaxed(ep, kRingEmpty);
+                        e[q] = j;
+                        if (q == p && j == e[0] + q) p++;      // consecutive prefix
+                    }
                 }
                 ptx::fence_acq_rel();
                 for (uint32_t q = p; q < got; q++) return_block(v, (uint32_t)(s * kMaxBlocks + e[q]));
@@ -262,17 +300,16 @@ __device__ __noinline__ uint32_t get_run(const View &v, uint32_t t, uint32_t wan
             *first = (uint32_t)(s0 * nb);
             return k * nb;
         }
-        // Alg.2: format a segment; [dev] one formatter per tree
+        // Alg.2: format a segment; [dev] bounded formatters per tree
         uint32_t *tok = v.fmt_token + t * 32;
-        if (atomicCAS(tok, 0u, 1u) == 0u) {
+        if (token_try(tok)) {
             if (bt_successor<false>(bt, 0) != kNone) {        // someone published meanwhile
-                atomicExch(tok, 0u);
+                token_release(tok);
                 continue;
             }
             const uint64_t s1 = claim_front(v);
             if (s1 != kNone) format_segment(v, s1, t, want);
-            ptx::fence_acq_rel();
-            atomicExch(tok, 0u);
+            token_release(tok);
             if (s1 == kNone) {
                 if (bt_scan_first(bt) == kNone) return 0;     // "No allocations left"
                 continue;
@@ -280,7 +317,7 @@ __device__ __noinline__ uint32_t get_run(const View &v, uint32_t t, uint32_t wan
             *first = (uint32_t)(s1 * nb);
             return want;
         }
-        while (ptx::ld_relaxed(tok) != 0u && bt_successor<false>(bt, 0) == kNone) bo.pause();
+        while (ptx::ld_relaxed(tok) >= kFormatters && bt_successor<false>(bt, 0) == kNone) bo.pause();
     }
 }
 
@@ -296,7 +333,13 @@ __device__ __noinline__ bool refill_slot(const View &v, uint32_t si, uint32_t c,
     const uint32_t cap = v.run_cap[c];
     const uint32_t want = m_prev == 0 ? 1u : (2 * m_prev < cap ? 2 * m_prev : cap);
     uint32_t first = 0;
+#ifdef GALLATIN_TRACE
+    const uint64_t t0 = ptx::globaltimer();
     const uint32_t got = get_run(v, c, want, &first);
+    ptx::trace(t0, ptx::globaltimer(), ((uint64_t)si << 32) | (c << 24) | (want << 12) | got);
+#else
+    const uint32_t got = get_run(v, c, want, &first);
+#endif
     if (got == 0) {
         ptx::atom_exch(slot_word(v, si), kSlotEmpty);
         return false;
@@ -352,9 +395,23 @@ __device__ inline void *malloc_slice(const View &v, uint32_t c, uint32_t key) {
         uint64_t old = 0;
         if (lane == leader) old = ptx::atom_add(sw, (uint64_t)__popc(peers) << 32);
         old = __shfl_sync(peers, old, (int)leader);
-        const uint32_t idx = (uint32_t)(old >> 32) + rank;
-        if (idx < (run_len(old) << kSliceLog2)) return slice_ptr(v, c, old & kRunNone, idx);
-        if (!slot_exhausted(v, si, c, old, idx)) return nullptr;   // nullptr
+        const uint32_t cnt = (uint32_t)(old >> 32), limit = run_len(old) << kSliceLog2;
+        const uint32_t idx = cnt + rank;
+        if (idx < limit) return slice_ptr(v, c, old & kRunNone, idx);
+        const uint32_t n = (uint32_t)__popc(peers);
+        if (cnt <= limit && limit < cnt + n) {
+            // The refiller is in this team: its team-mates past the end wait at
+            // a warp barrier, not in a sleep loop that would stall the
+            // refiller's own diverged path.
+            unsigned waiters = peers;
+            for (uint32_t k = limit - cnt; k; k--) waiters &= waiters - 1;   // drop the valid lanes
+            bool ok = true;
+            if (idx == limit) ok = refill_slot(v, si, c, run_len(old));
+            ok = __shfl_sync(waiters, ok, __ffs((int)waiters) - 1);
+            if (!ok && idx == limit) return nullptr;                // nullptr
+            continue;
+        }
+        slot_exhausted(v, si, c, old, idx);                           // refill is another warp's
     }
 }
 

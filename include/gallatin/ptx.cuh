@@ -74,6 +74,29 @@ __device__ __forceinline__ uint32_t lanemask_lt() {
     return r;
 }
 
+__device__ __forceinline__ uint64_t globaltimer() {
+    uint64_t t;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+    return t;
+}
+
+#ifdef GALLATIN_TRACE
+// Debug builds only: refill trace records {t0, t1, slot|class|want|got} in a
+// device buffer (gallatin_debug_trace).
+__device__ uint64_t *g_trace = nullptr;
+__device__ unsigned long long g_trace_n = 0;
+__device__ uint64_t g_trace_cap = 0;
+__device__ __forceinline__ void trace(uint64_t t0, uint64_t t1, uint64_t info) {
+    if (!g_trace) return;
+    const unsigned long long i = atomicAdd(&g_trace_n, 1ull);
+    if (i < g_trace_cap) {
+        g_trace[3 * i] = t0;
+        g_trace[3 * i + 1] = t1;
+        g_trace[3 * i + 2] = info;
+    }
+}
+#endif
+
 #ifdef GALLATIN_DEBUG_SPIN
 // Debug builds only: a spin loop that exceeds GALLATIN_DEBUG_SPIN pauses writes
 // one record {site, smid, lane, value} per (SM, lane) into host-mapped memory
@@ -98,7 +121,7 @@ struct Backoff {
 #endif
     __device__ __forceinline__ void pause() {
         __nanosleep(ns);
-        if (ns < 1024) ns <<= 1;
+        if (ns < 256) ns <<= 1;
 #ifdef GALLATIN_DEBUG_SPIN
         if (++n == GALLATIN_DEBUG_SPIN && g_spin_log) {
             uint32_t sm, ln;

@@ -107,7 +107,8 @@ __global__ void k_reset() {
 // refill an earlier item would otherwise wait for.
 // Then waits-and-retries, whole blocks and segment runs.
 __device__ __noinline__ void bulk_malloc_slow(const uint64_t *sizes, void **ptrs, uint64_t n, uint64_t base,
-                                              uint32_t key, uint32_t slow, uint64_t info, int items) {
+                                              uint32_t key, uint32_t slow, uint64_t info, int items,
+                                              unsigned callers) {
     const View &v = c_view;
     // pass 0: refill duties only (never waits on another slot's refill)
     for (int k = 0; k < items; k++) {
@@ -120,6 +121,9 @@ __device__ __noinline__ void bulk_malloc_slow(const uint64_t *sizes, void **ptrs
             slow &= ~(1u << k);
         }
     }
+    // every duty of this warp is discharged before any of its lanes spins
+    // (a sleeping lane stalls its warp-mates' diverged refill path)
+    __syncwarp(callers);
     // pass 1: retries after a refill, waits, whole blocks and segment runs
     for (int k = 0; k < items; k++) {
         if (!((slow >> k) & 1)) continue;
@@ -197,7 +201,8 @@ __global__ void __launch_bounds__(kThreads) k_bulk_malloc(const uint64_t *__rest
             __stcs(reinterpret_cast<unsigned long long *>(ptrs) + i, reinterpret_cast<unsigned long long>(p));
         }
     }
-    if (slow) bulk_malloc_slow(sizes, ptrs, n, base, key, slow, info, ITEMS);
+    const unsigned callers = __ballot_sync(0xFFFFFFFFu, slow != 0);
+    if (slow) bulk_malloc_slow(sizes, ptrs, n, base, key, slow, info, ITEMS, callers);
 }
 
 __device__ __noinline__ void free_slow(const View &v, uint64_t p) {
@@ -762,6 +767,26 @@ int gallatin_usable(void *const *d_ptrs, const uint64_t *d_sizes, uint64_t n, ui
 extern "C" int gallatin_debug_spin_log(void *host_mapped) {
     if (cudaMemcpyToSymbol(gallatin::ptx::g_spin_log, &host_mapped, sizeof(void *)) != cudaSuccess)
         return GALLATIN_ERR_CUDA;
+    return GALLATIN_OK;
+}
+#endif
+
+#ifdef GALLATIN_TRACE
+// Debug builds only: device buffer of cap records (3 words each) for refill
+// traces; returns the number of records written so far through *n.
+extern "C" int gallatin_debug_trace(void *dev_buf, uint64_t cap, uint64_t *n) {
+    if (dev_buf) {
+        unsigned long long z = 0;
+        cudaMemcpyToSymbol(gallatin::ptx::g_trace, &dev_buf, sizeof(void *));
+        cudaMemcpyToSymbol(gallatin::ptx::g_trace_cap, &cap, sizeof(cap));
+        cudaMemcpyToSymbol(gallatin::ptx::g_trace_n, &z, sizeof(z));
+    }
+    if (n) {
+        cudaDeviceSynchronize();
+        unsigned long long v = 0;
+        cudaMemcpyFromSymbol(&v, gallatin::ptx::g_trace_n, sizeof(v));
+        *n = v;
+    }
     return GALLATIN_OK;
 }
 #endif
