@@ -117,6 +117,21 @@ __device__ __noinline__ void try_free_segment(const View &v, uint64_t s, uint32_
     bt_insert(seg_tree(v), s);
 }
 
+// Every formatted segment whose blocks are all home goes back to the segment
+// tree (formatted ahead and never used); returns how many.
+__device__ __noinline__ uint32_t reclaim_idle(const View &v) {
+    uint32_t n = 0;
+    for (uint64_t s = 0; s < v.nseg; s++) {
+        const uint64_t w = ptx::ld_relaxed(v.seg_word + s);
+        const uint32_t t = sw_tree(w);
+        if (t < kTrees && sw_avail(w) == (int32_t)nb_of(t)) {
+            try_free_segment(v, s, t);
+            n++;
+        }
+    }
+    return n;
+}
+
 // ---- Alg. 1 GetSegment(treeId < numBlockTrees) ----------------
 // successor(0) on the segment tree + claimIndex, front first
 // (P:138).  Returns the claimed segment or kNone when every segment is in use.
@@ -131,7 +146,11 @@ __device__ __noinline__ uint64_t claim_front(const View &v) {
         if (s == kNone) {
             if (from != 0) { from = 0; continue; }
             s = bt_scan_first(st);                         // confirm before failing
-            if (s == kNone) return kNone;                  // "All segments in use"
+            if (s == kNone) {
+                // [dev] before failing, return idle formatted segments (all blocks home)
+                if (!reclaim_idle(v)) return kNone;            // "All segments in use"
+                continue;
+            }
         }
         if (bt_delete(st, s)) {
             ptx::fence_acq_rel();
@@ -192,12 +211,11 @@ __device__ __forceinline__ uint32_t gid_of(uint32_t t, uint64_t linear) {
     return (uint32_t)(((linear >> sh) << 8) | (linear & ((1u << sh) - 1)));
 }
 
-// [dev] formatter tokens: at most kFormatters threads format segments for
+// [dev] formatter tokens: at most v.formatters threads format segments for
 // one tree at a time (the paper lets every waiting thread format, P:151-155;
 // one at a time would serialize the bursts in which every slot refills).
-constexpr uint32_t kFormatters = 8;
-__device__ __forceinline__ bool token_try(uint32_t *tok) {
-    if (atomicAdd(tok, 1u) < kFormatters) return true;
+__device__ __forceinline__ bool token_try(uint32_t *tok, uint32_t limit) {
+    if (atomicAdd(tok, 1u) < limit) return true;
     atomicSub(tok, 1u);
     return false;
 }
@@ -210,7 +228,7 @@ __device__ __forceinline__ void token_release(uint32_t *tok) {
 // that refills rarely wait for a format (skipped if every token is busy).
 __device__ __noinline__ void format_ahead(const View &v, uint32_t t) {
     uint32_t *tok = v.fmt_token + t * 32;
-    if (!token_try(tok)) return;
+    if (!token_try(tok, v.formatters)) return;
     const uint64_t s = claim_front(v);
     if (s != kNone) format_segment(v, s, t, 0);
     token_release(tok);
@@ -302,7 +320,7 @@ __device__ __noinline__ uint32_t get_run(const View &v, uint32_t t, uint32_t wan
         }
         // Alg.2: format a segment; [dev] bounded formatters per tree
         uint32_t *tok = v.fmt_token + t * 32;
-        if (token_try(tok)) {
+        if (token_try(tok, v.formatters)) {
             if (bt_successor<false>(bt, 0) != kNone) {        // someone published meanwhile
                 token_release(tok);
                 continue;
@@ -317,7 +335,7 @@ __device__ __noinline__ uint32_t get_run(const View &v, uint32_t t, uint32_t wan
             *first = (uint32_t)(s1 * nb);
             return want;
         }
-        while (ptx::ld_relaxed(tok) >= kFormatters && bt_successor<false>(bt, 0) == kNone) bo.pause();
+        while (ptx::ld_relaxed(tok) >= v.formatters && bt_successor<false>(bt, 0) == kNone) bo.pause();
     }
 }
 

@@ -228,8 +228,29 @@ static void ring_push(ring_t *r, uint16_t j) {
 /* --------------------------------------------- Alg.1 getSegment (front) --- */
 /* successor(0) on the segment tree and claimIndex; front-first
  * invariant: every segment below the claimed one is in use. */
+/* A formatted segment whose blocks are all home goes back to the segment
+ * tree, in segment order (used by drain, and before reporting that every
+ * segment is in use). Returns how many were retired. */
+static uint64_t retire_idle_all(o2_t *a) {
+    uint64_t n = 0;
+    for (uint64_t s = 0; s < a->nseg; s++) {
+        uint32_t t = a->tree[s];
+        if (t < NUM_BLOCK_TREES && (uint32_t)a->avail[s] == nb_of(t)) {
+            ring_t *r = &a->ring[s];
+            a->tree[s] = TREE_FREE; a->avail[s] = 0;
+            r->head = 0; r->count = 0;
+            for (int i = 0; i < 256; i++) r->e[i] = 0xFFFF;
+            oracle_veb_delete(a->btree[t], s);
+            oracle_veb_insert(a->segfree, s);
+            n++;
+        }
+    }
+    return n;
+}
+
 static uint64_t claim_front(o2_t *a) {
     uint64_t s = oracle_veb_successor(a->segfree, 0);
+    if (s == NONE64 && retire_idle_all(a)) s = oracle_veb_successor(a->segfree, 0);
     if (s == NONE64 || s >= a->nseg) return NONE64;        /* "All segments in use" */
     for (uint64_t i = 0; i < s; i++) if (a->tree[i] == TREE_FREE) a->violations |= V_FRONT_FIRST;
     oracle_veb_delete(a->segfree, s);
@@ -478,17 +499,7 @@ void o2_drain(o2_t *a) {
             }
         }
     }
-    for (uint64_t s = 0; s < a->nseg; s++) {
-        uint32_t t = a->tree[s];
-        if (t < NUM_BLOCK_TREES && (uint32_t)a->avail[s] == nb_of(t)) {
-            ring_t *r = &a->ring[s];
-            a->tree[s] = TREE_FREE; a->avail[s] = 0;
-            r->head = 0; r->count = 0;
-            for (int i = 0; i < 256; i++) r->e[i] = 0xFFFF;
-            oracle_veb_delete(a->btree[t], s);
-            oracle_veb_insert(a->segfree, s);
-        }
-    }
+    retire_idle_all(a);
 }
 
 /* Replay: kinds[i] 0 = malloc(args[i]) with slot key keys[i], out[i] = offset

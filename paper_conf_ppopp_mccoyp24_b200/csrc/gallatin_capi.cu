@@ -500,6 +500,7 @@ int gallatin_init_ex(const gallatin_config_t *cfg_in) {
         v.run_cap[c] = m < 1 ? 1u : (uint32_t)m;
     }
     v.format_ahead = cfg.format_ahead == 1 ? 1u : 0u;
+    v.formatters = (uint32_t)(nseg / 128 < 1 ? 1 : (nseg / 128 > 8 ? 8 : nseg / 128));
     v.fence_free = cfg.fence_free;
 
     // metadata: one allocation, 256 B aligned sections
