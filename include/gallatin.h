@@ -46,11 +46,12 @@ enum {
  *   heap_bytes : rounded DOWN to a multiple of 16 MiB, >= 1 segment.
  *   slot_base  : block-buffer slots of the 16 B class; class c gets
  *                max(slot_min, slot_base >> c).  Default = #SMs (148).
- *   slot_min   : lower cap, default 4 ("capped at four").
- *   run_max    : a slot holds a RUN of up to run_max consecutive blocks (1..128,
- *                default 16); the run starts at one block and doubles on every
- *                refill of the slot.  1 = the paper's one-block buffer.
- *   run_bytes  : and at most run_bytes per run (default min(64 MiB, heap/64)).
+ *   slot_min   : lower cap; the paper caps at four; default
+ *                clamp(nseg / 32, 4, 32) (more slots for the big classes on big heaps).
+ *   run_max    : a slot holds a RUN of up to run_max consecutive blocks (1..512,
+ *                default 256); the run starts at run_init blocks and doubles on
+ *                every refill of the slot.  1 = the paper's one-block buffer.
+ *   run_bytes  : and at most run_bytes per run (default min(256 MiB, heap/64)).
  *   format_ahead: 1 (default) = the reservation that leaves a segment with
  *                fewer than nb/4 blocks formats the next segment of its tree;
  *                2 = off (the paper: format on demand).
@@ -68,7 +69,8 @@ typedef struct gallatin_config {
     uint32_t format_ahead;
     uint32_t fence_free;
     uint32_t bulk_items;   /* requests per thread in the bulk kernels: 0 = auto, 1 or 4 */
-    uint32_t reserved[2];
+    uint32_t run_init;     /* run length of a slot's first refill (default clamp(nseg/128, 1, 8)) */
+    uint32_t reserved;
 } gallatin_config_t;
 
 int gallatin_init(uint64_t heap_bytes);                 /* defaults for the rest */
@@ -122,7 +124,7 @@ typedef struct gallatin_stats {
     uint64_t run_bytes;          /* effective configuration ...                     */
     uint32_t nslot[9];           /* block-buffer slots per class                    */
     uint32_t run_cap[9];         /* max blocks per run per class                    */
-    uint32_t slot_base, slot_min, run_max, format_ahead, fence_free;
+    uint32_t slot_base, slot_min, run_max, format_ahead, fence_free, run_init, formatters;
 } gallatin_stats_t;
 int gallatin_stats(gallatin_stats_t *out);               /* synchronizes the device */
 

@@ -349,7 +349,8 @@ __device__ __forceinline__ uint32_t run_len(uint64_t w) { return (uint32_t)(w >>
 // Replace an exhausted run (Alg.3): the run doubles up to the class cap.
 __device__ __noinline__ bool refill_slot(const View &v, uint32_t si, uint32_t c, uint32_t m_prev) {
     const uint32_t cap = v.run_cap[c];
-    const uint32_t want = m_prev == 0 ? 1u : (2 * m_prev < cap ? 2 * m_prev : cap);
+    const uint32_t first_run = v.run_init < cap ? v.run_init : cap;
+    const uint32_t want = m_prev == 0 ? first_run : (2 * m_prev < cap ? 2 * m_prev : cap);
     uint32_t first = 0;
 #ifdef GALLATIN_TRACE
     const uint64_t t0 = ptx::globaltimer();

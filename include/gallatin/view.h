@@ -51,7 +51,7 @@ struct gallatin_device_view {
     uint32_t format_ahead;      /* 1 = format the next segment at nb/4 left   */
     uint32_t fence_free;        /* 1 = release fence per freeing team, 2 = none */
     uint32_t formatters;        /* concurrent segment formatters per tree      */
-    uint32_t reserved;
+    uint32_t run_init;          /* run length of an empty slot's first refill  */
 };
 typedef struct gallatin_device_view gallatin_device_view_t;
 

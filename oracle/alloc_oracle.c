@@ -90,7 +90,7 @@ typedef struct { uint64_t key, val; } kv_t;
 
 typedef struct o2 {
     uint64_t nseg;
-    unsigned slot_base, slot_min, run_max, format_ahead;
+    unsigned slot_base, slot_min, run_max, format_ahead, run_init;
     uint64_t run_bytes;
     unsigned nslot[NUM_BLOCK_TREES], slot_off[NUM_BLOCK_TREES], nslot_total;
     uint32_t *tree;               /* memoryTable.ids           */
@@ -161,11 +161,12 @@ static uint64_t slot_make(uint64_t cnt, uint32_t m, uint32_t first) {
 }
 
 o2_t *o2_create(uint64_t nseg, unsigned slot_base, unsigned slot_min, unsigned run_max,
-                uint64_t run_bytes, unsigned format_ahead) {
+                uint64_t run_bytes, unsigned format_ahead, unsigned run_init) {
     if (nseg < 1 || nseg > (1ULL << 14) || slot_base < 1 || run_max < 1 || run_max > 512) return NULL;
     o2_t *a = (o2_t *)calloc(1, sizeof(o2_t));
     a->nseg = nseg; a->slot_base = slot_base; a->slot_min = slot_min;
     a->run_max = run_max; a->run_bytes = run_bytes; a->format_ahead = format_ahead;
+    a->run_init = run_init < 1 ? 1 : run_init;
     unsigned off = 0;
     for (unsigned c = 0; c < NUM_BLOCK_TREES; c++) {
         unsigned n = slot_base >> c;                  /* halving per class */
@@ -398,7 +399,8 @@ static uint64_t malloc_slice(o2_t *a, uint32_t c, uint64_t key) {
         }
         /* exhausted: this request replaces the run (Alg.3) */
         uint32_t cap = run_cap(a, c);
-        uint32_t want = m == 0 ? 1 : (2 * m < cap ? 2 * m : cap);
+        uint32_t first_run = a->run_init < cap ? a->run_init : cap;     /* empty slot: run_init */
+        uint32_t want = m == 0 ? first_run : (2 * m < cap ? 2 * m : cap);
         uint32_t got = get_run(a, c, want, &first);
         if (!got) {
             a->slot[i] = SLOT_EMPTY;

@@ -269,10 +269,10 @@ __global__ void __launch_bounds__(kThreads) k_bulk_free(void *const *__restrict_
         if (!blk) peers[k] = 0;
         lead_any |= blk && lane == (uint32_t)__ffs((int)peers[k]) - 1;
     }
-    if (v.fence_free != 2) {
-        __syncwarp();
-        if (lead_any) ptx::fence_acq_rel();                        // release the team's writes
-    }
+    // No release fence here: every write to the memory being freed was made by
+    // an earlier kernel, and the kernel boundary orders it (the device-API free,
+    // core::free_impl, fences per team instead).
+    (void)lead_any;
 #pragma unroll
     for (int k = 0; k < ITEMS; k++) {
         oldc[k] = 0;
@@ -466,10 +466,11 @@ int gallatin_init_ex(const gallatin_config_t *cfg_in) {
     CUDA_TRY(cudaGetDevice(&dev));
     CUDA_TRY(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev));
     if (!cfg.slot_base) cfg.slot_base = (uint32_t)sms;      // one slot per SM
-    if (!cfg.slot_min) cfg.slot_min = 4;                     // "capped at four"
+    if (!cfg.slot_min) cfg.slot_min = (uint32_t)(nseg / 32 < 4 ? 4 : (nseg / 32 > 32 ? 32 : nseg / 32));
     if (!cfg.fence_free) cfg.fence_free = 1;
     if (!cfg.format_ahead) cfg.format_ahead = 1;
     if (!cfg.run_max) cfg.run_max = 256;
+    if (!cfg.run_init) cfg.run_init = (uint32_t)(nseg / 128 < 1 ? 1 : (nseg / 128 > 8 ? 8 : nseg / 128));
     if (!cfg.run_bytes) {
         cfg.run_bytes = (nseg << core::kSegLog2) / 64;
         if (cfg.run_bytes > (256ull << 20)) cfg.run_bytes = 256ull << 20;
@@ -501,6 +502,7 @@ int gallatin_init_ex(const gallatin_config_t *cfg_in) {
     }
     v.format_ahead = cfg.format_ahead == 1 ? 1u : 0u;
     v.formatters = (uint32_t)(nseg / 128 < 1 ? 1 : (nseg / 128 > 8 ? 8 : nseg / 128));
+    v.run_init = cfg.run_init;
     v.fence_free = cfg.fence_free;
 
     // metadata: one allocation, 256 B aligned sections
@@ -720,6 +722,8 @@ int gallatin_stats(gallatin_stats_t *out) {
     out->run_max = g.cfg.run_max;
     out->format_ahead = g.cfg.format_ahead;
     out->fence_free = v.fence_free;
+    out->run_init = v.run_init;
+    out->formatters = v.formatters;
     return GALLATIN_OK;
 }
 
