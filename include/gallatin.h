@@ -130,7 +130,8 @@ int gallatin_stats(gallatin_stats_t *out);               /* synchronizes the dev
 
 /* Snapshot image (synchronizes the device).  A flat array of uint64 words:
  *   [0] magic 0x47414C4C494D4731  [1] nseg  [2] tree levels L  [3] W = words
- *   per tree  [4] S = total slots  [5] error counter  [6],[7] 0
+ *   per tree  [4] S = total slots  [5] error counter  [6] number of segments
+ *   whose read-mostly tree-id copy disagrees with the table (always 0)  [7] 0
  *   then: segment tree (W words: level 0 first; bit = segment free)
  *         9 block trees (9*W; bit s of tree t = segment s formatted for t
  *           with blocks available)

@@ -105,6 +105,7 @@ __device__ __forceinline__ void seg_after_rmw(const View &v, uint64_t s, uint64_
 __device__ __noinline__ void try_free_segment(const View &v, uint64_t s, uint32_t t) {
     const uint64_t full = sw_make(t, (int32_t)nb_of(t));
     if (ptx::atom_cas(v.seg_word + s, full, sw_make(kTreeFree, 0)) != full) return;
+    ptx::st_relaxed(v.seg_tid + s, kTreeFree);
     // No block of s is out or in flight: reset its ring.
     ptx::st_relaxed(v.q_head + s, 0u);
     ptx::st_relaxed(v.q_tail + s, 0u);
@@ -176,6 +177,7 @@ __device__ __noinline__ void format_segment(const View &v, uint64_t s, uint32_t 
     for (; q < cnt; q++) e[q] = (uint16_t)(keep + q);
     ptx::st_relaxed(v.q_head + s, 0u);
     ptx::st_relaxed(v.q_tail + s, nb - keep);
+    ptx::st_relaxed(v.seg_tid + s, t);
     ptx::fence_acq_rel();
     const uint64_t delta = sw_retree(kTreeFree, t) + (nb - keep);
     const uint64_t old = ptx::atom_add(v.seg_word + s, delta);
@@ -312,6 +314,7 @@ __device__ __noinline__ uint32_t get_run(const View &v, uint32_t t, uint32_t wan
             const BitTree st = seg_tree(v);
             uint32_t k = 1;
             while (k < want / nb && s0 + k < v.nseg && bt_delete(st, s0 + k)) k++;
+            for (uint32_t q = 0; q < k; q++) ptx::st_relaxed(v.seg_tid + s0 + q, t);
             ptx::fence_acq_rel();
             for (uint32_t q = 0; q < k; q++) ptx::atom_add(v.seg_word + s0 + q, sw_retree(kTreeFree, t));
             ptx::fence_acq_rel();
@@ -462,6 +465,8 @@ __device__ __noinline__ void *malloc_large(const View &v, uint64_t k) {
         bo.pause();
     }
     ptx::fence_acq_rel();
+    ptx::st_relaxed(v.seg_tid + i, kTrees + (uint32_t)k);
+    for (uint64_t m = 1; m < k; m++) ptx::st_relaxed(v.seg_tid + i + m, kTreeCont);
     ptx::atom_add(v.seg_word + i, sw_retree(kTreeFree, kTrees + (uint32_t)k));
     for (uint64_t m = 1; m < k; m++) ptx::atom_add(v.seg_word + i + m, sw_retree(kTreeFree, kTreeCont));
     ptx::fence_acq_rel();
@@ -483,6 +488,7 @@ __device__ __noinline__ void free_large(const View &v, uint64_t s, uint32_t t) {
     ptx::fence_acq_rel();
     ptx::atom_add(v.seg_word + s, sw_retree(t, kTreeFree));
     for (uint64_t m = 1; m < k; m++) ptx::atom_add(v.seg_word + s + m, sw_retree(kTreeCont, kTreeFree));
+    for (uint64_t m = 0; m < k; m++) ptx::st_relaxed(v.seg_tid + s + m, kTreeFree);
     ptx::fence_acq_rel();
     bt_insert_range(seg_tree(v), s, k);
 }

@@ -11,6 +11,8 @@
  *   seg_word    nseg x u64 {tree id:32 | available blocks + 2^31:32}: the
  *               memory table's ids fused with the ring's
  *               reservation count
+ *   seg_tid     nseg x u32: a copy of each table word's tree id, written only
+ *               when a segment changes owner, so frees can read it through L1
  *   q_head/tail nseg x u32 ring counters; q_entries nseg x 256 x u16 block ids
  *               (the per-segment ring queue)
  *   block_free  nseg x 256 x u32 free counters
@@ -34,6 +36,7 @@ struct gallatin_device_view {
     uint64_t *seg_tree;
     uint64_t *block_trees;
     uint64_t *seg_word;
+    uint32_t *seg_tid;          /* tree id of each segment (read-mostly copy) */
     uint32_t *q_head;
     uint32_t *q_tail;
     uint16_t *q_entries;

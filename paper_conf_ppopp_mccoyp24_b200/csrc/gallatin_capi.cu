@@ -87,6 +87,7 @@ __global__ void k_reset() {
         if (i < 9 * W) v.block_trees[i] = 0;
         if (i < nseg) {
             v.seg_word[i] = core::sw_make(core::kTreeFree, 0);
+            v.seg_tid[i] = core::kTreeFree;
             v.q_head[i] = 0;
             v.q_tail[i] = 0;
         }
@@ -255,7 +256,9 @@ __global__ void __launch_bounds__(kThreads) k_bulk_free(void *const *__restrict_
 #pragma unroll
     for (int k = 0; k < ITEMS; k++) {
         const uint64_t off = p[k] - v.heap;
-        w[k] = (p[k] && off < heap_bytes) ? ptx::ld_relaxed(v.seg_word + (off >> core::kSegLog2)) : ~0ull;
+        // tree id of a segment holding a live block cannot change while the
+        // block is out, and L1 is invalidated at launch: a cached read is exact
+        w[k] = (p[k] && off < heap_bytes) ? ((uint64_t)__ldca(v.seg_tid + (off >> core::kSegLog2)) << 32) : ~0ull;
     }
     bool lead_any = false;
 #pragma unroll
@@ -399,7 +402,7 @@ uint64_t image_words(const View &v) {
 
 struct HostCopy {
     std::vector<uint64_t> seg_tree, block_trees, seg_word, slots;
-    std::vector<uint32_t> q_head, q_tail, block_free;
+    std::vector<uint32_t> q_head, q_tail, block_free, seg_tid;
     std::vector<uint16_t> q_entries;
     unsigned long long err = 0;
 };
@@ -423,6 +426,8 @@ int copy_state(HostCopy &h) {
     CUDA_TRY(cudaMemcpy(h.q_tail.data(), v.q_tail, nseg * 4, cudaMemcpyDeviceToHost));
     CUDA_TRY(cudaMemcpy(h.q_entries.data(), v.q_entries, nseg * 512, cudaMemcpyDeviceToHost));
     CUDA_TRY(cudaMemcpy(h.block_free.data(), v.block_free, nseg * 1024, cudaMemcpyDeviceToHost));
+    h.seg_tid.resize(nseg);
+    CUDA_TRY(cudaMemcpy(h.seg_tid.data(), v.seg_tid, nseg * 4, cudaMemcpyDeviceToHost));
     CUDA_TRY(cudaMemcpy(h.slots.data(), v.slots, h.slots.size() * 8, cudaMemcpyDeviceToHost));
     CUDA_TRY(cudaMemcpy(&h.err, v.err, 8, cudaMemcpyDeviceToHost));
     return GALLATIN_OK;
@@ -507,9 +512,9 @@ int gallatin_init_ex(const gallatin_config_t *cfg_in) {
 
     // metadata: one allocation, 256 B aligned sections
     uint64_t sz[11] = {W * 8, 9 * W * 8, nseg * 8, nseg * 4, nseg * 4, nseg * 512, nseg * 1024,
-                       (uint64_t)off * 128, 9 * 128, 128, 0};
+                       (uint64_t)off * 128, 9 * 128, 128, nseg * 4};
     uint64_t total = 0, offs[11];
-    for (int i = 0; i < 10; i++) { offs[i] = total; total += align_up(sz[i], 256); }
+    for (int i = 0; i < 11; i++) { offs[i] = total; total += align_up(sz[i], 256); }
     void *meta = nullptr;
     if (cudaMalloc(&meta, total) != cudaSuccess) { cudaGetLastError(); return GALLATIN_ERR_NOMEM; }
     void *heap = nullptr;
@@ -529,6 +534,7 @@ int gallatin_init_ex(const gallatin_config_t *cfg_in) {
     v.slots = reinterpret_cast<uint64_t *>(m + offs[7]);
     v.fmt_token = reinterpret_cast<uint32_t *>(m + offs[8]);
     v.err = reinterpret_cast<unsigned long long *>(m + offs[9]);
+    v.seg_tid = reinterpret_cast<uint32_t *>(m + offs[10]);
     v.heap = align_up(reinterpret_cast<uint64_t>(heap), core::kSegBytes);   // 16 MiB aligned base
 
     g.init = true;
@@ -670,7 +676,10 @@ int gallatin_snapshot(uint64_t *out, uint64_t cap, uint64_t *len) {
     p[3] = v.tree_words;
     p[4] = v.nslot_total;
     p[5] = h.err;
-    p[6] = 0;
+    // [6]: segments whose read-mostly tree-id copy disagrees with the table (must be 0)
+    uint64_t mism = 0;
+    for (uint64_t s = 0; s < v.nseg; s++) mism += h.seg_tid[s] != (uint32_t)(h.seg_word[s] >> 32);
+    p[6] = mism;
     p[7] = 0;
     p += 8;
     memcpy(p, h.seg_tree.data(), v.tree_words * 8ull);
