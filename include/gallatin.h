@@ -70,7 +70,7 @@ typedef struct gallatin_config {
     uint32_t fence_free;
     uint32_t bulk_items;   /* requests per thread in the bulk kernels: 0 = auto, 1 or 4 */
     uint32_t run_init;     /* run length of a slot's first refill (default clamp(nseg/128, 1, 8)) */
-    uint32_t reserved;
+    uint32_t prefetch;     /* 1 (default) = fetch the next run at the middle of the current one; 2 = off */
 } gallatin_config_t;
 
 int gallatin_init(uint64_t heap_bytes);                 /* defaults for the rest */
@@ -124,7 +124,7 @@ typedef struct gallatin_stats {
     uint64_t run_bytes;          /* effective configuration ...                     */
     uint32_t nslot[9];           /* block-buffer slots per class                    */
     uint32_t run_cap[9];         /* max blocks per run per class                    */
-    uint32_t slot_base, slot_min, run_max, format_ahead, fence_free, run_init, formatters;
+    uint32_t slot_base, slot_min, run_max, format_ahead, fence_free, run_init, formatters, prefetch;
 } gallatin_stats_t;
 int gallatin_stats(gallatin_stats_t *out);               /* synchronizes the device */
 
@@ -142,8 +142,9 @@ int gallatin_stats(gallatin_stats_t *out);               /* synchronizes the dev
  *           FIFO order, 0xFFFF padded, 4 per word little-endian)
  *         block free counters (nseg*256 uint32, 2 per word)
  *         block-buffer slots (S words, class-major: issued count << 32 |
- *           run length << 24 | first block of the run as a linear index in
- *           units of the class's block size; empty = 0x0000000000FFFFFF)
+ *           run length << 22 | first block of the run as a linear index in
+ *           units of the class's block size; empty = 0x00000000003FFFFF)
+ *         prefetched next run per slot (S words, same layout, count 0)
  * gallatin_snapshot_words() gives the length. */
 int gallatin_snapshot_words(uint64_t *words);
 int gallatin_snapshot(uint64_t *h_out, uint64_t cap_words, uint64_t *len_words);

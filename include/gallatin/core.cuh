@@ -351,6 +351,13 @@ __device__ __forceinline__ uint32_t run_len(uint64_t w) { return (uint32_t)(w >>
 
 // Replace an exhausted run (Alg.3): the run doubles up to the class cap.
 __device__ __noinline__ bool refill_slot(const View &v, uint32_t si, uint32_t c, uint32_t m_prev) {
+    if (v.prefetch) {                                         // [dev] the prefetched run, if any
+        const uint64_t nx = ptx::atom_exch(slot_word(v, si) + 1, kSlotEmpty);
+        if (run_len(nx) != 0) {
+            ptx::atom_exch(slot_word(v, si), nx);               // {issued 0, run, first}
+            return true;
+        }
+    }
     const uint32_t cap = v.run_cap[c];
     const uint32_t first_run = v.run_init < cap ? v.run_init : cap;
     const uint32_t want = m_prev == 0 ? first_run : (2 * m_prev < cap ? 2 * m_prev : cap);
@@ -368,6 +375,20 @@ __device__ __noinline__ bool refill_slot(const View &v, uint32_t si, uint32_t c,
     }
     ptx::atom_exch(slot_word(v, si), ((uint64_t)got << kRunShift) | first);
     return true;
+}
+
+// [dev] the request that draws the middle of a run fetches the next run
+// (twice as long, up to the cap) into the slot's second word, so that the
+// refill at the end of the run is one exchange.
+__device__ __noinline__ void prefetch_slot(const View &v, uint32_t si, uint32_t c, uint32_t m) {
+    const uint32_t cap = v.run_cap[c];
+    const uint32_t want = 2 * m < cap ? 2 * m : cap;
+    uint32_t first = 0;
+    const uint32_t got = get_run(v, c, want, &first);
+    if (got == 0) return;
+    const uint64_t run = ((uint64_t)got << kRunShift) | first;
+    if (ptx::atom_cas(slot_word(v, si) + 1, kSlotEmpty, run) != kSlotEmpty)
+        for (uint32_t k = 0; k < got; k++) block_freed(v, gid_of(c, (uint64_t)first + k), kSlices);   // raced: give back
 }
 
 __device__ __forceinline__ void *slice_ptr(const View &v, uint32_t c, uint64_t first, uint64_t idx) {
@@ -419,7 +440,10 @@ __device__ inline void *malloc_slice(const View &v, uint32_t c, uint32_t key) {
         old = __shfl_sync(peers, old, (int)leader);
         const uint32_t cnt = (uint32_t)(old >> 32), limit = run_len(old) << kSliceLog2;
         const uint32_t idx = cnt + rank;
-        if (idx < limit) return slice_ptr(v, c, old & kRunNone, idx);
+        if (idx < limit) {
+            if (v.prefetch && idx == (limit >> 1)) prefetch_slot(v, si, c, run_len(old));
+            return slice_ptr(v, c, old & kRunNone, idx);
+        }
         const uint32_t n = (uint32_t)__popc(peers);
         if (cnt <= limit && limit < cnt + n) {
             // The refiller is in this team: its team-mates past the end wait at
@@ -531,6 +555,9 @@ __device__ inline void drain_slots(const View &v) {
                 const uint64_t issued = cnt <= lo ? 0 : (cnt - lo > kSlices ? kSlices : cnt - lo);
                 if (issued < kSlices) block_freed(v, gid_of(c, first + k), (uint32_t)(kSlices - issued));
             }
+            // a prefetched run was never issued from: all of it comes back
+            const uint64_t nx = ptx::atom_exch(slot_word(v, v.slot_off[c] + q) + 1, kSlotEmpty);
+            for (uint32_t k = 0; k < run_len(nx); k++) block_freed(v, gid_of(c, (nx & kRunNone) + k), kSlices);
         }
     }
 }

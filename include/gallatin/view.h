@@ -16,10 +16,10 @@
  *   q_head/tail nseg x u32 ring counters; q_entries nseg x 256 x u16 block ids
  *               (the per-segment ring queue)
  *   block_free  nseg x 256 x u32 free counters
- *   slots       S x 128 B lines: word 0 = {issued count:32 | run length:8 |
- *               first block:24} (block buffer; a run = consecutive
+ *   slots       S x 128 B lines: word 0 = {issued count:32 | run length:10 |
+ *               first block:22} (block buffer; a run = consecutive
  *               blocks, first block as a linear index in units of the class's
- *               block size)
+ *               block size), word 1 = the prefetched next run (same layout)
  *   fmt_token   9 x 128 B lines: one formatter per block tree
  *   err         u64 error counter (bad frees)
  */
@@ -55,6 +55,8 @@ struct gallatin_device_view {
     uint32_t fence_free;        /* 1 = release fence per freeing team, 2 = none */
     uint32_t formatters;        /* concurrent segment formatters per tree      */
     uint32_t run_init;          /* run length of an empty slot's first refill  */
+    uint32_t prefetch;          /* 1 = fetch the next run at the run's middle  */
+    uint32_t pad;
 };
 typedef struct gallatin_device_view gallatin_device_view_t;
 

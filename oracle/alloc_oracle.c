@@ -100,6 +100,8 @@ typedef struct o2 {
     oracle_veb *segfree;          /* segment tree               */
     oracle_veb *btree[NUM_BLOCK_TREES];  /* block trees         */
     uint64_t *slot;               /* cnt << 32 | m << 22 | first block  */
+    uint64_t *next;               /* prefetched run (m << 22 | first) or empty */
+    unsigned prefetch;
     uint64_t err;                 /* out-of-heap / non-allocated segment frees */
     /* oracle-only bookkeeping for the invariant checks */
     kv_t *live; uint64_t live_cap, live_n;
@@ -161,12 +163,13 @@ static uint64_t slot_make(uint64_t cnt, uint32_t m, uint32_t first) {
 }
 
 o2_t *o2_create(uint64_t nseg, unsigned slot_base, unsigned slot_min, unsigned run_max,
-                uint64_t run_bytes, unsigned format_ahead, unsigned run_init) {
+                uint64_t run_bytes, unsigned format_ahead, unsigned run_init, unsigned prefetch) {
     if (nseg < 1 || nseg > (1ULL << 14) || slot_base < 1 || run_max < 1 || run_max > 512) return NULL;
     o2_t *a = (o2_t *)calloc(1, sizeof(o2_t));
     a->nseg = nseg; a->slot_base = slot_base; a->slot_min = slot_min;
     a->run_max = run_max; a->run_bytes = run_bytes; a->format_ahead = format_ahead;
     a->run_init = run_init < 1 ? 1 : run_init;
+    a->prefetch = prefetch;
     unsigned off = 0;
     for (unsigned c = 0; c < NUM_BLOCK_TREES; c++) {
         unsigned n = slot_base >> c;                  /* halving per class */
@@ -187,7 +190,8 @@ o2_t *o2_create(uint64_t nseg, unsigned slot_base, unsigned slot_min, unsigned r
         for (int i = 0; i < 256; i++) a->ring[s].e[i] = 0xFFFF;
     }
     a->slot = (uint64_t *)malloc(a->nslot_total * sizeof(uint64_t));
-    for (unsigned i = 0; i < a->nslot_total; i++) a->slot[i] = SLOT_EMPTY;
+    a->next = (uint64_t *)malloc(a->nslot_total * sizeof(uint64_t));
+    for (unsigned i = 0; i < a->nslot_total; i++) a->slot[i] = a->next[i] = SLOT_EMPTY;
     return a;
 }
 
@@ -196,7 +200,7 @@ void o2_destroy(o2_t *a) {
     free(a->tree); free(a->avail); free(a->ring); free(a->freecnt);
     oracle_veb_destroy(a->segfree);
     for (unsigned t = 0; t < NUM_BLOCK_TREES; t++) oracle_veb_destroy(a->btree[t]);
-    free(a->slot); free(a->live);
+    free(a->slot); free(a->next); free(a->live);
     free(a);
 }
 
@@ -393,14 +397,26 @@ static uint64_t malloc_slice(o2_t *a, uint32_t c, uint64_t key) {
         uint64_t cnt = a->slot[i] >> 32;
         uint32_t m = (uint32_t)(a->slot[i] >> RUN_SHIFT) & 0x3FF;
         uint32_t first = (uint32_t)a->slot[i] & RUN_NONE;
+        uint32_t cap = run_cap(a, c);
+        uint32_t grow = 2 * m < cap ? 2 * m : cap;
         if (cnt < SLICES_PER_BLOCK * m) {                   /* valid = idx < 4096 (per block) */
             a->slot[i] = slot_make(cnt + 1, m, first);
-            return slice_addr(first, c, cnt);
+            uint64_t off = slice_addr(first, c, cnt);
+            if (a->prefetch && cnt == SLICES_PER_BLOCK * m / 2 && a->next[i] == SLOT_EMPTY) {
+                uint32_t nf;                                  /* [ours] prefetch the next run */
+                uint32_t ng = get_run(a, c, grow, &nf);
+                if (ng) a->next[i] = slot_make(0, ng, nf);
+            }
+            return off;
         }
         /* exhausted: this request replaces the run (Alg.3) */
-        uint32_t cap = run_cap(a, c);
+        if (a->next[i] != SLOT_EMPTY) {                       /* the prefetched run */
+            a->slot[i] = a->next[i];
+            a->next[i] = SLOT_EMPTY;
+            continue;
+        }
         uint32_t first_run = a->run_init < cap ? a->run_init : cap;     /* empty slot: run_init */
-        uint32_t want = m == 0 ? first_run : (2 * m < cap ? 2 * m : cap);
+        uint32_t want = m == 0 ? first_run : grow;
         uint32_t got = get_run(a, c, want, &first);
         if (!got) {
             a->slot[i] = SLOT_EMPTY;
@@ -499,6 +515,11 @@ void o2_drain(o2_t *a) {
                 if (issued < SLICES_PER_BLOCK)
                     block_freed(a, gid_of(c, (uint64_t)first + k), (uint32_t)(SLICES_PER_BLOCK - issued));
             }
+            /* a prefetched run was never issued from: all of it comes back */
+            uint32_t nm = (uint32_t)(a->next[i] >> RUN_SHIFT) & 0x3FF;
+            uint32_t nf = (uint32_t)a->next[i] & RUN_NONE;
+            a->next[i] = SLOT_EMPTY;
+            for (uint32_t k = 0; k < nm; k++) block_freed(a, gid_of(c, (uint64_t)nf + k), (uint32_t)SLICES_PER_BLOCK);
         }
     }
     retire_idle_all(a);
@@ -595,7 +616,7 @@ static void tree_image(const oracle_veb *t, uint64_t nbits, uint64_t *out) {
 uint64_t o2_image_words(const o2_t *a) {
     uint64_t wpl[16]; unsigned L;
     uint64_t W = tree_words(a->nseg, wpl, &L);
-    return 8 + 10 * W + a->nseg * (1 + 65 + 128) + (uint64_t)a->nslot_total;
+    return 8 + 10 * W + a->nseg * (1 + 65 + 128) + 2ULL * a->nslot_total;
 }
 
 /* Canonical image; layout documented in include/gallatin.h. */
@@ -623,5 +644,6 @@ uint64_t o2_image(const o2_t *a, uint64_t *out, uint64_t cap) {
     for (uint64_t g = 0; g < a->nseg * MAX_BLOCKS_PER_SEGMENT; g += 2)
         *p++ = (uint64_t)a->freecnt[g] | ((uint64_t)a->freecnt[g + 1] << 32);
     for (unsigned i = 0; i < a->nslot_total; i++) *p++ = a->slot[i];
+    for (unsigned i = 0; i < a->nslot_total; i++) *p++ = a->next[i];
     return need;
 }

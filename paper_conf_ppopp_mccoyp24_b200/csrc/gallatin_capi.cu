@@ -95,7 +95,7 @@ __global__ void k_reset() {
         if (i < nseg * 128) reinterpret_cast<uint64_t *>(v.block_free)[i] = 0;
         if (i < S * 16) {
             const uint64_t w = i % 16;
-            v.slots[i] = w == 0 ? core::kSlotEmpty : 0;
+            v.slots[i] = w <= 1 ? core::kSlotEmpty : 0;
         }
         if (i < 9 * 32) v.fmt_token[i] = 0;
         if (i == 0) *v.err = 0;
@@ -111,9 +111,15 @@ __device__ __noinline__ void bulk_malloc_slow(const uint64_t *sizes, void **ptrs
                                               uint32_t key, uint32_t slow, uint64_t info, int items,
                                               unsigned callers) {
     const View &v = c_view;
-    // pass 0: refill duties only (never waits on another slot's refill)
+    // pass 0: refill and prefetch duties only (never waits on another slot's refill)
     for (int k = 0; k < items; k++) {
         const uint32_t code = (uint32_t)(info >> (16 * k)) & 0xFFFF;
+        if (((slow >> k) & 1) && (code & 0x2000u)) {
+            const uint32_t c = core::slice_class(sizes[base + 32ull * k]);
+            core::prefetch_slot(v, v.slot_off[c] + key % v.nslot[c], c, code & 0x3FF);
+            slow &= ~(1u << k);                                     // its slice was stored already
+            continue;
+        }
         if (!((slow >> k) & 1) || !(code & 0x400u)) continue;
         const uint64_t i = base + 32ull * k;
         const uint32_t c = core::slice_class(sizes[i]);
@@ -190,17 +196,21 @@ __global__ void __launch_bounds__(kThreads) k_bulk_malloc(const uint64_t *__rest
             const uint32_t c = core::slice_class(sz[k]);
             const uint32_t m = core::run_len(old[k]);
             const uint32_t idx = (uint32_t)(old[k] >> 32) + (uint32_t)__popc(peers[k] & lt);
-            if (idx < (m << core::kSliceLog2)) p = core::slice_ptr(v, c, old[k] & core::kRunNone, idx);
-            else code = idx == (m << core::kSliceLog2) ? (0x400u | m) : 0x1000u;
+            if (idx < (m << core::kSliceLog2)) {
+                p = core::slice_ptr(v, c, old[k] & core::kRunNone, idx);
+                if (v.prefetch && idx == (m << (core::kSliceLog2 - 1))) code = 0x2000u | m;   // prefetch duty
+            } else {
+                code = idx == (m << core::kSliceLog2) ? (0x400u | m) : 0x1000u;
+            }
         } else if (sz[k] != 0) {
             code = 0x800u;
         }
         if (code) {
             slow |= 1u << k;
             info |= (uint64_t)code << (16 * k);
-        } else if (i < n) {
-            __stcs(reinterpret_cast<unsigned long long *>(ptrs) + i, reinterpret_cast<unsigned long long>(p));
         }
+        if (!(code & 0x1C00u) && i < n)                           // valid (maybe with a prefetch duty)
+            __stcs(reinterpret_cast<unsigned long long *>(ptrs) + i, reinterpret_cast<unsigned long long>(p));
     }
     const unsigned callers = __ballot_sync(0xFFFFFFFFu, slow != 0);
     if (slow) bulk_malloc_slow(sizes, ptrs, n, base, key, slow, info, ITEMS, callers);
@@ -397,7 +407,7 @@ __global__ void k_usable(void *const *ptrs, const uint64_t *sizes, uint64_t n, u
 
 // ------------------------------------------------------- host helpers ----
 uint64_t image_words(const View &v) {
-    return 8 + 10ull * v.tree_words + v.nseg * (1 + 65 + 128) + (uint64_t)v.nslot_total;
+    return 8 + 10ull * v.tree_words + v.nseg * (1 + 65 + 128) + 2ull * v.nslot_total;
 }
 
 struct HostCopy {
@@ -482,6 +492,7 @@ int gallatin_init_ex(const gallatin_config_t *cfg_in) {
     }
     if (cfg.run_max > core::kMaxRun || cfg.fence_free > 2 || cfg.format_ahead > 2) return GALLATIN_ERR_INVALID;
     if (cfg.bulk_items != 0 && cfg.bulk_items != 1 && cfg.bulk_items != 4) return GALLATIN_ERR_INVALID;
+    if (cfg.prefetch > 2) return GALLATIN_ERR_INVALID;
     if (nseg > (1ull << 14)) return GALLATIN_ERR_INVALID;        // 22-bit run index at 64 KB blocks (256 GiB)
 
     View v{};
@@ -508,6 +519,7 @@ int gallatin_init_ex(const gallatin_config_t *cfg_in) {
     v.format_ahead = cfg.format_ahead == 1 ? 1u : 0u;
     v.formatters = (uint32_t)(nseg / 128 < 1 ? 1 : (nseg / 128 > 8 ? 8 : nseg / 128));
     v.run_init = cfg.run_init;
+    v.prefetch = cfg.prefetch == 2 ? 0u : 1u;
     v.fence_free = cfg.fence_free;
 
     // metadata: one allocation, 256 B aligned sections
@@ -702,6 +714,7 @@ int gallatin_snapshot(uint64_t *out, uint64_t cap, uint64_t *len) {
     memcpy(p, h.block_free.data(), v.nseg * 1024);
     p += v.nseg * 128;
     for (uint32_t i = 0; i < v.nslot_total; i++) *p++ = h.slots[(uint64_t)i * 16];
+    for (uint32_t i = 0; i < v.nslot_total; i++) *p++ = h.slots[(uint64_t)i * 16 + 1];
     return GALLATIN_OK;
 }
 
@@ -733,6 +746,7 @@ int gallatin_stats(gallatin_stats_t *out) {
     out->fence_free = v.fence_free;
     out->run_init = v.run_init;
     out->formatters = v.formatters;
+    out->prefetch = v.prefetch;
     return GALLATIN_OK;
 }
 

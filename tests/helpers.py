@@ -49,6 +49,7 @@ def image_sections(img: np.ndarray) -> dict:
     d["qentries"] = q[:, 1:].copy().view(np.uint16).reshape(nseg, 256)
     d["block_free"] = img[p:p + nseg * 128].copy().view(np.uint32); p += nseg * 128
     d["slots"] = img[p:p + S]; p += S
+    d["next"] = img[p:p + S]; p += S
     assert p == len(img)
     return d
 
@@ -81,6 +82,7 @@ def pristine_image(nseg: int, nslots: int) -> np.ndarray:
     out.append(q.reshape(-1))
     out.append(np.zeros(nseg * 128, dtype=np.uint64))
     out.append(np.full(nslots, SLOT_EMPTY, dtype=np.uint64))
+    out.append(np.full(nslots, SLOT_EMPTY, dtype=np.uint64))
     return np.concatenate(out)
 
 
@@ -105,7 +107,7 @@ def diff_images(got: np.ndarray, want: np.ndarray) -> str:
         return f"image lengths differ: {len(got)} vs {len(want)}"
     a, b = image_sections(got), image_sections(want)
     for k in ["magic", "nseg", "levels", "W", "nslots", "err", "segtree", "btrees", "segword", "qcount",
-              "qentries", "block_free", "slots"]:
+              "qentries", "block_free", "slots", "next"]:
         x, y = a[k], b[k]
         if isinstance(x, int):
             if x != y:

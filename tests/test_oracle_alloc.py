@@ -25,9 +25,9 @@ def test_block_buffer_slots_match_paper_a40():
     assert [b.nslot(c) for c in range(9)] == [148, 74, 37, 18, 9, 4, 4, 4, 4]
 
 
-@pytest.mark.parametrize("run_max,fa", [(1, 0), (16, 1), (128, 0)])
+@pytest.mark.parametrize("run_max,fa,pf", [(1, 0, 0), (16, 1, 1), (128, 0, 1)])
 @pytest.mark.parametrize("size,blocks", [(16, "blocks_per_segment_16B"), (32, "blocks_per_segment_32B")])
-def test_blocks_per_segment_and_in_order_slices(size, blocks, run_max, fa):
+def test_blocks_per_segment_and_in_order_slices(size, blocks, run_max, fa, pf):
     """256 blocks per segment at 16 B, 128 at 32 B; 4096 slices
     per block handed out in order; segments used front first.  With
     one slot, the k-th request lands at k*size exactly until the segment is
@@ -35,7 +35,7 @@ def test_blocks_per_segment_and_in_order_slices(size, blocks, run_max, fa):
     (the paper) and with growing runs of consecutive blocks (ours)."""
     g = golden()
     nb = g[blocks]
-    a = oracle.Allocator(4, slot_base=1, slot_min=1, run_max=run_max, format_ahead=fa)
+    a = oracle.Allocator(4, slot_base=1, slot_min=1, run_max=run_max, format_ahead=fa, prefetch=pf)
     n = nb * g["slices_per_block"]
     offs = a.malloc_batch(np.full(n + 5, size, dtype=np.uint64), keydiv=0)
     assert np.array_equal(offs[:n], np.arange(n, dtype=np.uint64) * np.uint64(size))
@@ -116,14 +116,15 @@ def test_accounting_matches_closed_form_mixed():
     assert np.array_equal(a.image(), pristine_image(256, 302))
 
 
-@pytest.mark.parametrize("seed,nseg,run_max,fa", [(1, 4, 1, 0), (2, 8, 1, 0), (3, 6, 16, 1), (4, 64, 8, 1),
-                                                  (5, 5, 128, 0), (6, 16, 4, 1)])
-def test_random_sequences_tiny_heaps(seed, nseg, run_max, fa):
+@pytest.mark.parametrize("seed,nseg,run_max,fa,pf", [(1, 4, 1, 0, 0), (2, 8, 1, 0, 0), (3, 6, 16, 1, 1), (4, 64, 8, 1, 1),
+                                                     (5, 5, 128, 0, 0), (6, 16, 4, 1, 0), (7, 32, 512, 1, 1)])
+def test_random_sequences_tiny_heaps(seed, nseg, run_max, fa, pf):
     """Random malloc/free/drain sequences on 4-64 segment heaps, including OOM:
     live allocations re-checked in Python, structure checked, and free-all +
     drain restores the analytic pristine image bit-exactly."""
     kinds, args, keys = wg.replay_ops(20_000, seed, p_free=0.45, p_drain=0.002, nkeys=64)
-    a = oracle.Allocator(nseg, slot_base=16, slot_min=2, run_max=run_max, run_bytes=32 << 20, format_ahead=fa)
+    a = oracle.Allocator(nseg, slot_base=16, slot_min=2, run_max=run_max, run_bytes=32 << 20, format_ahead=fa,
+                         prefetch=pf)
     out = a.replay(kinds, args, keys)
     live = {}
     for i, k in enumerate(kinds):
