@@ -70,7 +70,7 @@ typedef struct gallatin_config {
     uint32_t fence_free;
     uint32_t bulk_items;   /* requests per thread in the bulk kernels: 0 = auto, 1 or 4 */
     uint32_t run_init;     /* run length of a slot's first refill (default clamp(nseg/128, 1, 8)) */
-    uint32_t prefetch;     /* 1 (default) = fetch the next run at the middle of the current one; 2 = off */
+    uint32_t prefetch;     /* 1 = fetch the next run at the middle of the current one; 0/2 = off (default) */
 } gallatin_config_t;
 
 int gallatin_init(uint64_t heap_bytes);                 /* defaults for the rest */

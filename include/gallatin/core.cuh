@@ -381,6 +381,7 @@ __device__ __noinline__ bool refill_slot(const View &v, uint32_t si, uint32_t c,
 // (twice as long, up to the cap) into the slot's second word, so that the
 // refill at the end of the run is one exchange.
 __device__ __noinline__ void prefetch_slot(const View &v, uint32_t si, uint32_t c, uint32_t m) {
+    if (ptx::ld_relaxed(slot_word(v, si) + 1) != kSlotEmpty) return;   // a run is already waiting
     const uint32_t cap = v.run_cap[c];
     const uint32_t want = 2 * m < cap ? 2 * m : cap;
     uint32_t first = 0;

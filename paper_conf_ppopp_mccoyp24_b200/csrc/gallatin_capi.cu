@@ -519,7 +519,7 @@ int gallatin_init_ex(const gallatin_config_t *cfg_in) {
     v.format_ahead = cfg.format_ahead == 1 ? 1u : 0u;
     v.formatters = (uint32_t)(nseg / 128 < 1 ? 1 : (nseg / 128 > 8 ? 8 : nseg / 128));
     v.run_init = cfg.run_init;
-    v.prefetch = cfg.prefetch == 2 ? 0u : 1u;
+    v.prefetch = cfg.prefetch == 1 ? 1u : 0u;              // default off (measured: DESIGN.md)
     v.fence_free = cfg.fence_free;
 
     // metadata: one allocation, 256 B aligned sections
