@@ -59,7 +59,7 @@ class ClockSampler:
         try:
             self.proc = subprocess.Popen(
                 ["nvidia-smi", "-i", str(self.index), f"--query-gpu={self.FIELDS}", "--format=csv,noheader,nounits",
-                 "-lms", "100"], stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+                 "-lms", "20"], stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
         except Exception:
             self.proc = None
             return
@@ -228,11 +228,14 @@ def run_ours(args, rank, world, local):
     peak_src = "MEASURED_PEAKS.json hbm_gbs"
     if not hbm_peak:
         hbm_peak, peak_src = 6650.0, "B200_PROFILING.md fallback"
+    # traffic: DRAM bytes per launch of the dominant kernel on a 2^24-thread
+    # cell, from the committed ncu --set full capture (profiles/traffic.json);
+    # compare with the algorithmic bytes of that launch (16 or 8 B x 2^24)
     traffic = None
     tf = os.path.join(ROOT, "profiles", "traffic.json")
     if os.path.exists(tf):
         try:
-            traffic = json.load(open(tf)).get(f"k_bulk_{dominant}")
+            traffic = json.load(open(tf))["per_cell"][f"k_bulk_{dominant}"]["16"]
         except Exception:
             traffic = None
 
@@ -263,6 +266,8 @@ def run_ours(args, rank, world, local):
             "malloc_ops_s": malloc_ops_s, "free_ops_s": free_ops_s, "per_size": per_cell,
             "roofline": {"bound": "hbm", "kernel": f"k_bulk_{dominant}", "achieved": achieved, "peak": hbm_peak,
                          "unit": "GB/s", "frac": achieved / hbm_peak, "traffic": traffic,
+                         "traffic_algorithmic": bytes_per_op * (1 << 24),
+                         "traffic_note": "DRAM bytes of one 2^24-thread launch (16 B cell, profiles/r1_kernels.md)",
                          "algorithmic_bytes_per_op": bytes_per_op, "peak_source": peak_src},
             "clocks": clocks,
             "e2e": e2e,

@@ -154,7 +154,7 @@ __device__ __noinline__ void bulk_malloc_slow(const uint64_t *sizes, void **ptrs
 // then take their slice; refills, waits, blocks and large requests follow on
 // the per-request device path.  Lane l of warp w handles w*32*ITEMS + k*32 + l.
 template <int ITEMS>
-__global__ void __launch_bounds__(kThreads) k_bulk_malloc(const uint64_t *__restrict__ sizes, void **__restrict__ ptrs,
+__global__ void __launch_bounds__(kThreads, 5) k_bulk_malloc(const uint64_t *__restrict__ sizes, void **__restrict__ ptrs,
                                                           uint64_t n) {
     const View &v = c_view;
     const uint32_t lane = threadIdx.x & 31;
@@ -250,7 +250,7 @@ __device__ __noinline__ void bulk_free_slow(void *const *ptrs, uint64_t base, ui
 // table words, team the lanes freeing one block, one release fence
 // per leading lane, then the team counter RMWs back to back.
 template <int ITEMS>
-__global__ void __launch_bounds__(kThreads) k_bulk_free(void *const *__restrict__ ptrs, uint64_t n) {
+__global__ void __launch_bounds__(kThreads, 6) k_bulk_free(void *const *__restrict__ ptrs, uint64_t n) {
     const View &v = c_view;
     const uint32_t lane = threadIdx.x & 31;
     const uint64_t base = ((blockIdx.x * (uint64_t)kThreads + threadIdx.x) >> 5) * (32 * ITEMS) + lane;
