@@ -102,9 +102,13 @@ def dist_setup(ngpus: int):
 
 
 class Dist:
+    """Process-group plumbing for independent per-GPU replicas: a barrier and
+    max/sum of host scalars (no data-path collective exists)."""
+
     def __init__(self, rank, world, backend):
         self.rank, self.world = rank, world
         self.pg = None
+        self.device = "cuda" if backend == "nccl" else "cpu"
         if world > 1:
             import torch.distributed as dist
             dist.init_process_group(backend)
@@ -118,7 +122,7 @@ class Dist:
         if not self.pg:
             return x
         import torch
-        t = torch.tensor([x], dtype=torch.float64, device="cuda" if torch.cuda.is_available() else "cpu")
+        t = torch.tensor([x], dtype=torch.float64, device=self.device)
         self.pg.all_reduce(t, op=self.pg.ReduceOp.MAX)
         return float(t.item())
 
@@ -126,13 +130,21 @@ class Dist:
         if not self.pg:
             return x
         import torch
-        t = torch.tensor([x], dtype=torch.float64, device="cuda" if torch.cuda.is_available() else "cpu")
+        t = torch.tensor([x], dtype=torch.float64, device=self.device)
         self.pg.all_reduce(t, op=self.pg.ReduceOp.SUM)
         return float(t.item())
 
     def close(self):
         if self.pg:
             self.pg.destroy_process_group()
+
+
+def aggregate(d: "Dist", ops_local: float, ms_local: float) -> tuple[float, float, float]:
+    """Whole-job throughput of independent replicas: every rank's ops over the
+    slowest rank's device time.  Returns (value ops/s, max ms, total ops)."""
+    ms = d.max(ms_local)
+    total = d.sum(ops_local)
+    return total / (ms / 1e3), ms, total
 
 
 def peaks_file() -> dict:
@@ -203,9 +215,7 @@ def run_ours(args, rank, world, local):
     clocks = clk.stop()
     d.barrier()
     ms_local = t0.elapsed_time(t1)
-    ms = d.max(ms_local)
-    total_ops = d.sum(ops_per_step * args.steps)
-    value = total_ops / (ms / 1e3)
+    value, ms, total_ops = aggregate(d, ops_per_step * args.steps, ms_local)
 
     # per-kernel times (the roofline's dominant kernel)
     m_ms = [a.elapsed_time(b) for a, b in zip(ev["m0"], ev["m1"])]
@@ -399,6 +409,7 @@ def cpu_sample(scale_div: int):
     return [(s, max(1, n // scale_div)) for s, n in cells_c2()]
 
 
+
 def time_oracle(cells, steps: int):
     import oracle
     import workload_gen as wg
@@ -428,9 +439,9 @@ def cpu_baseline(args):
 
 
 def run_reference(args, rank, world):
-    if rank != 0:
+    if rank != 0:                      # the reference arm runs on rank 0 only
         return
-    div = 8
+    div = 8 * args.scale
     cells = cpu_sample(div)
     steps = max(1, min(args.steps, 3))
     for _ in range(min(args.warmup, 1)):
