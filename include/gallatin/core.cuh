@@ -72,7 +72,7 @@ __device__ __forceinline__ BitTree block_tree(const View &v, uint32_t t) {
 
 // Make block-tree t's bit for segment s equal its predicate (the derived-bit
 // reconcile loop of DESIGN.md "Quiescent exactness").
-__device__ __noinline__ void btree_reconcile(const View &v, uint32_t t, uint64_t s) {
+__device__ inline __noinline__ void btree_reconcile(const View &v, uint32_t t, uint64_t s) {
     const BitTree bt = block_tree(v, t);
     uint64_t *leaf = bt.w + bt.off[0] + (s >> 6);
     const uint64_t bit = 1ull << (s & 63);
@@ -88,7 +88,7 @@ __device__ __noinline__ void btree_reconcile(const View &v, uint32_t t, uint64_t
     if (flipped) bt_reconcile_up(bt, 0, s >> 6);
 }
 
-__device__ void try_free_segment(const View &v, uint64_t s, uint32_t t);
+__device__ inline __noinline__ void try_free_segment(const View &v, uint64_t s, uint32_t t);
 
 // Every thread whose RMW on seg_word[s] changed a block-tree predicate repairs
 // that bit; the RMW that brings a segment back to "all blocks home" retires it.
@@ -102,7 +102,7 @@ __device__ __forceinline__ void seg_after_rmw(const View &v, uint64_t s, uint64_
 
 // "When all blocks are returned, the segment is freed and re-added to the
 // segment tree".
-__device__ __noinline__ void try_free_segment(const View &v, uint64_t s, uint32_t t) {
+__device__ inline __noinline__ void try_free_segment(const View &v, uint64_t s, uint32_t t) {
     const uint64_t full = sw_make(t, (int32_t)nb_of(t));
     if (ptx::atom_cas(v.seg_word + s, full, sw_make(kTreeFree, 0)) != full) return;
     ptx::st_relaxed(v.seg_tid + s, kTreeFree);
@@ -120,7 +120,7 @@ __device__ __noinline__ void try_free_segment(const View &v, uint64_t s, uint32_
 
 // Every formatted segment whose blocks are all home goes back to the segment
 // tree (formatted ahead and never used); returns how many.
-__device__ __noinline__ uint32_t reclaim_idle(const View &v) {
+__device__ inline __noinline__ uint32_t reclaim_idle(const View &v) {
     uint32_t n = 0;
     for (uint64_t s = 0; s < v.nseg; s++) {
         const uint64_t w = ptx::ld_relaxed(v.seg_word + s);
@@ -139,7 +139,7 @@ __device__ __noinline__ uint32_t reclaim_idle(const View &v) {
 // A claimer that loses the race for segment s moves on to successor(s + 1)
 // instead of re-reading from 0, so k concurrent claimers spread over the k
 // lowest free segments in O(k) total RMWs (serially this is successor(0)).
-__device__ __noinline__ uint64_t claim_front(const View &v) {
+__device__ inline __noinline__ uint64_t claim_front(const View &v) {
     const BitTree st = seg_tree(v);
     uint64_t from = 0;
     for (;;) {
@@ -164,7 +164,7 @@ __device__ __noinline__ uint64_t claim_front(const View &v) {
 // initSegment for tree t: blocks [keep, nb) go into the ring in order
 // and the segment joins block tree t ("broadcast availability");
 // blocks [0, keep) belong to the caller.
-__device__ __noinline__ void format_segment(const View &v, uint64_t s, uint32_t t, uint32_t keep) {
+__device__ inline __noinline__ void format_segment(const View &v, uint64_t s, uint32_t t, uint32_t keep) {
     const uint32_t nb = nb_of(t);
     uint16_t *e = v.q_entries + s * kMaxBlocks;
     const uint32_t cnt = nb - keep;                       // entries at positions 0 .. cnt-1
@@ -185,7 +185,7 @@ __device__ __noinline__ void format_segment(const View &v, uint64_t s, uint32_t 
 }
 
 // ---- block return (Alg.4; ring enqueue P:178) --------------------
-__device__ __noinline__ void return_block(const View &v, uint32_t gid) {
+__device__ inline __noinline__ void return_block(const View &v, uint32_t gid) {
     const uint64_t s = gid / kMaxBlocks;
     const uint32_t pos = atomicAdd(v.q_tail + s, 1u) & (kMaxBlocks - 1);
     uint16_t *slotp = v.q_entries + s * kMaxBlocks + pos;
@@ -228,7 +228,7 @@ __device__ __forceinline__ void token_release(uint32_t *tok) {
 
 // [dev] format one more segment for tree t when the current one runs low, so
 // that refills rarely wait for a format (skipped if every token is busy).
-__device__ __noinline__ void format_ahead(const View &v, uint32_t t) {
+__device__ inline __noinline__ void format_ahead(const View &v, uint32_t t) {
     uint32_t *tok = v.fmt_token + t * 32;
     if (!token_try(tok, v.formatters)) return;
     const uint64_t s = claim_front(v);
@@ -239,7 +239,7 @@ __device__ __noinline__ void format_ahead(const View &v, uint32_t t) {
 // ---- Alg. 2 GetBlock(treeId), for a RUN of blocks [dev] --------
 // Returns the number of consecutive blocks obtained (0 = exhausted) and the
 // first one's linear index (segment * nb + block) in *first.
-__device__ __noinline__ uint32_t get_run(const View &v, uint32_t t, uint32_t want, uint32_t *first) {
+__device__ inline __noinline__ uint32_t get_run(const View &v, uint32_t t, uint32_t want, uint32_t *first) {
     const BitTree bt = block_tree(v, t);
     const uint32_t nb = nb_of(t);
     ptx::Backoff bo(4, t);
@@ -350,7 +350,7 @@ constexpr uint64_t kSlotEmpty = kRunNone;                 // issued 0, run 0: re
 __device__ __forceinline__ uint32_t run_len(uint64_t w) { return (uint32_t)(w >> kRunShift) & 0x3FFu; }
 
 // Replace an exhausted run (Alg.3): the run doubles up to the class cap.
-__device__ __noinline__ bool refill_slot(const View &v, uint32_t si, uint32_t c, uint32_t m_prev) {
+__device__ inline __noinline__ bool refill_slot(const View &v, uint32_t si, uint32_t c, uint32_t m_prev) {
     if (v.prefetch) {                                         // [dev] the prefetched run, if any
         const uint64_t nx = ptx::atom_exch(slot_word(v, si) + 1, kSlotEmpty);
         if (run_len(nx) != 0) {
@@ -380,7 +380,7 @@ __device__ __noinline__ bool refill_slot(const View &v, uint32_t si, uint32_t c,
 // [dev] the request that draws the middle of a run fetches the next run
 // (twice as long, up to the cap) into the slot's second word, so that the
 // refill at the end of the run is one exchange.
-__device__ __noinline__ void prefetch_slot(const View &v, uint32_t si, uint32_t c, uint32_t m) {
+__device__ inline __noinline__ void prefetch_slot(const View &v, uint32_t si, uint32_t c, uint32_t m) {
     if (ptx::ld_relaxed(slot_word(v, si) + 1) != kSlotEmpty) return;   // a run is already waiting
     const uint32_t cap = v.run_cap[c];
     const uint32_t want = 2 * m < cap ? 2 * m : cap;
@@ -407,7 +407,7 @@ __device__ __forceinline__ uint32_t block_class(uint64_t size) {
 // After a team RMW returned `old` and this lane drew idx >= the run's end:
 // refill (the lane that drew exactly the end) or wait for the refill.
 // Returns false if the refill found no memory.
-__device__ __noinline__ bool slot_exhausted(const View &v, uint32_t si, uint32_t c, uint64_t old, uint32_t idx) {
+__device__ inline __noinline__ bool slot_exhausted(const View &v, uint32_t si, uint32_t c, uint64_t old, uint32_t idx) {
     const uint32_t m = run_len(old);
     if (idx == (m << kSliceLog2)) return refill_slot(v, si, c, m);
     ptx::Backoff bo(1, si);
@@ -464,7 +464,7 @@ __device__ inline void *malloc_slice(const View &v, uint32_t c, uint32_t key) {
 
 // (4 KB, 16 MB): one whole block of the smallest fitting tree; its counter is
 // preset to 4095 so that Alg.4's rule returns it on its one free (reading A-2).
-__device__ __noinline__ void *malloc_block(const View &v, uint32_t t) {
+__device__ inline __noinline__ void *malloc_block(const View &v, uint32_t t) {
     uint32_t first = 0;
     if (get_run(v, t, 1, &first) == 0) return nullptr;
     atomicExch(v.block_free + gid_of(t, first), kSlices - 1);
@@ -473,7 +473,7 @@ __device__ __noinline__ void *malloc_block(const View &v, uint32_t t) {
 
 // >= 16 MB: Alg.1 with treeId >= numBlockTrees: claimMultiple from the back
 // (P:110-113); tree id = numBlockTrees + numSegments.
-__device__ __noinline__ void *malloc_large(const View &v, uint64_t k) {
+__device__ inline __noinline__ void *malloc_large(const View &v, uint64_t k) {
     if (k > v.nseg) return nullptr;
     const BitTree st = seg_tree(v);
     ptx::Backoff bo(5, k);
@@ -508,7 +508,7 @@ __device__ inline void *malloc_impl(const View &v, uint64_t size, uint32_t key) 
 }
 
 // segment allocation: return the k segments to the segment tree
-__device__ __noinline__ void free_large(const View &v, uint64_t s, uint32_t t) {
+__device__ inline __noinline__ void free_large(const View &v, uint64_t s, uint32_t t) {
     const uint64_t k = t - kTrees;
     ptx::fence_acq_rel();
     ptx::atom_add(v.seg_word + s, sw_retree(t, kTreeFree));

@@ -83,9 +83,9 @@ __device__ __forceinline__ uint64_t globaltimer() {
 #ifdef GALLATIN_TRACE
 // Debug builds only: refill trace records {t0, t1, slot|class|want|got} in a
 // device buffer (gallatin_debug_trace).
-__device__ uint64_t *g_trace = nullptr;
-__device__ unsigned long long g_trace_n = 0;
-__device__ uint64_t g_trace_cap = 0;
+static __device__ uint64_t *g_trace = nullptr;
+static __device__ unsigned long long g_trace_n = 0;
+static __device__ uint64_t g_trace_cap = 0;
 __device__ __forceinline__ void trace(uint64_t t0, uint64_t t1, uint64_t info) {
     if (!g_trace) return;
     const unsigned long long i = atomicAdd(&g_trace_n, 1ull);
@@ -101,7 +101,7 @@ __device__ __forceinline__ void trace(uint64_t t0, uint64_t t1, uint64_t info) {
 // Debug builds only: a spin loop that exceeds GALLATIN_DEBUG_SPIN pauses writes
 // one record {site, smid, lane, value} per (SM, lane) into host-mapped memory
 // the host can read while the kernel is still spinning.
-__device__ uint64_t *g_spin_log = nullptr;
+static __device__ uint64_t *g_spin_log = nullptr;
 #endif
 
 // Bounded exponential backoff for spin loops (waiting on another thread's

@@ -43,10 +43,13 @@ class Stats(ctypes.Structure):
 
 
 def declared_functions() -> list[str]:
-    """Every function include/gallatin.h declares (for the export check)."""
-    text = open(HEADER).read()
-    text = re.sub(r"/\*.*?\*/", "", text, flags=re.S)
-    return sorted(set(re.findall(r"^\s*(?:const\s+)?[\w ]+?\**\s*\b((?:gallatin|veb)_\w+)\s*\(", text, flags=re.M)))
+    """Every function the include/*.h headers declare (for the export check)."""
+    import glob
+    names = set()
+    for h in glob.glob(os.path.join(os.path.dirname(HEADER), "*.h")):
+        text = re.sub(r"/\*.*?\*/", "", open(h).read(), flags=re.S)
+        names |= set(re.findall(r"^\s*(?:const\s+)?[\w ]+?\**\s*\b((?:gallatin|veb)_\w+)\s*\(", text, flags=re.M))
+    return sorted(names)
 
 
 _lib = None
@@ -321,3 +324,85 @@ class Veb:
         got = ctypes.c_uint64()
         check(lib().veb_snapshot(self._h, out.ctypes.data, n.value, ctypes.byref(got)), "veb_snapshot")
         return out
+
+
+# ------------------------------------------------------ streaming graph ----
+GRAPH_HEADER = os.path.join(os.path.dirname(_PKG), "include", "gallatin_graph.h")
+
+
+def _graph_sigs(L):
+    u64, u32, vp, i32 = ctypes.c_uint64, ctypes.c_uint32, ctypes.c_void_p, ctypes.c_int
+    sig = {
+        "gallatin_graph_create": ([u32, ctypes.POINTER(vp)], i32),
+        "gallatin_graph_destroy": ([vp, vp], i32),
+        "gallatin_graph_insert": ([vp, vp, vp, u64, vp], i32),
+        "gallatin_graph_delete": ([vp, vp, vp, u64, vp], i32),
+        "gallatin_graph_expand": ([vp, vp, u64, vp], i32),
+        "gallatin_graph_export": ([vp, vp, vp, vp, vp], i32),
+        "gallatin_graph_gather": ([vp, vp, vp, vp], i32),
+        "gallatin_graph_counters": ([vp, ctypes.POINTER(ctypes.c_uint64)], i32),
+    }
+    for name, (args, res) in sig.items():
+        f = getattr(L, name)
+        f.argtypes = args
+        f.restype = res
+
+
+def _dptr4(t) -> int:
+    import torch
+    if not isinstance(t, torch.Tensor) or not t.is_cuda or not t.is_contiguous() or t.element_size() != 4:
+        raise TypeError("expected a contiguous 4-byte-element CUDA tensor")
+    return t.data_ptr()
+
+
+class Graph:
+    """Streaming graph of per-vertex edge lists kept by the DEVICE-side
+    allocator (include/gallatin_graph.h; BASELINE configs[4])."""
+
+    def __init__(self, num_vertices: int):
+        L = lib()
+        _graph_sigs(L)
+        h = ctypes.c_void_p()
+        check(L.gallatin_graph_create(num_vertices, ctypes.byref(h)), "gallatin_graph_create")
+        self._h = h
+        self.V = num_vertices
+
+    def destroy(self, stream=None):
+        if self._h:
+            check(lib().gallatin_graph_destroy(self._h, _stream(stream)), "gallatin_graph_destroy")
+            self._h = None
+
+    def insert(self, src, dst, stream=None):
+        check(lib().gallatin_graph_insert(self._h, _dptr4(src), _dptr4(dst), src.numel(), _stream(stream)),
+              "gallatin_graph_insert")
+
+    def delete(self, src, dst, stream=None):
+        check(lib().gallatin_graph_delete(self._h, _dptr4(src), _dptr4(dst), src.numel(), _stream(stream)),
+              "gallatin_graph_delete")
+
+    def expand(self, vertices, stream=None):
+        check(lib().gallatin_graph_expand(self._h, _dptr4(vertices), vertices.numel(), _stream(stream)),
+              "gallatin_graph_expand")
+
+    def export(self, stream=None):
+        """(size uint32[V], cap uint32[V], list pointer int64[V]) CUDA tensors."""
+        import torch
+        size = torch.empty(self.V, dtype=torch.int32, device="cuda")
+        cap = torch.empty(self.V, dtype=torch.int32, device="cuda")
+        ptr = torch.empty(self.V, dtype=torch.int64, device="cuda")
+        check(lib().gallatin_graph_export(self._h, size.data_ptr(), cap.data_ptr(), ptr.data_ptr(), _stream(stream)),
+              "gallatin_graph_export")
+        return size, cap, ptr
+
+    def gather(self, offsets, total: int, stream=None):
+        """CSR copy of every list given the exclusive prefix sum of the sizes."""
+        import torch
+        out = torch.empty(max(total, 1), dtype=torch.int32, device="cuda")
+        check(lib().gallatin_graph_gather(self._h, _dptr(offsets), out.data_ptr(), _stream(stream)),
+              "gallatin_graph_gather")
+        return out[:total]
+
+    def counters(self) -> dict:
+        c = (ctypes.c_uint64 * 3)()
+        check(lib().gallatin_graph_counters(self._h, c), "gallatin_graph_counters")
+        return {"mallocs": c[0], "frees": c[1], "failed": c[2]}

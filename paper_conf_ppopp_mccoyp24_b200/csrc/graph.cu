@@ -1,0 +1,454 @@
+// graph.cu -- the streaming-graph workload (BASELINE configs[4]; PAPER.md
+// S6.12) on the DEVICE-side allocator: every per-vertex edge list
+// is malloc'd, grown, shrunk and freed by GPU threads through
+// include/gallatin/device.cuh.  C-ABI: include/gallatin_graph.h.
+#include <cuda_runtime.h>
+#include <stdint.h>
+#include <stdio.h>
+
+#include "gallatin.h"
+#include "gallatin/device.cuh"
+#include "gallatin_graph.h"
+
+using gallatin::gallatin_free;
+using gallatin::gallatin_malloc;
+
+struct gallatin_graph {
+    uint32_t V;
+    uint64_t *list;       // per-vertex uint32_t* (as u64)
+    uint32_t *size, *cap, *cnt;
+    uint64_t *old;        // list being replaced during a grow / shrink
+    uint32_t *work;       // vertices to process (compacted)
+    uint32_t *work2;      // big vertices (CTA-per-vertex deletes)
+    uint32_t *nwork;      // [0] work, [1] work2
+    unsigned long long *ctr;   // [0] mallocs [1] frees [2] failed mallocs
+    uint64_t *hkeys;      // delete-batch hash: (src << 32 | dst) -> remaining count
+    uint32_t *hcnt;
+    uint64_t hcap;
+};
+
+namespace {
+constexpr int kT = 256;
+constexpr uint64_t kEmpty = ~0ull;
+constexpr uint32_t kBig = 2048;        // lists at least this long delete with a whole CTA
+
+inline cudaStream_t S(void *s) { return reinterpret_cast<cudaStream_t>(s); }
+inline unsigned blocks(uint64_t n) { return (unsigned)((n + kT - 1) / kT); }
+int status() {
+    const cudaError_t e = cudaGetLastError();
+    if (e != cudaSuccess) {
+        fprintf(stderr, "gallatin_graph: %s\n", cudaGetErrorString(e));
+        return GALLATIN_ERR_CUDA;
+    }
+    return GALLATIN_OK;
+}
+
+__device__ __forceinline__ uint32_t next_pow2(uint32_t x) { return x <= 1 ? 1u : 1u << (32 - __clz(x - 1)); }
+__device__ __forceinline__ uint32_t list_cap(uint32_t size) { return next_pow2(size < 4 ? 4 : size); }
+__device__ __forceinline__ uint32_t lane() { return threadIdx.x & 31; }
+
+// one atomic per warp for the statistics counters (all lanes present)
+__device__ __forceinline__ void count_warp(unsigned long long *ctr, bool m, bool f, bool fail) {
+    const unsigned a = __ballot_sync(0xFFFFFFFFu, m), b = __ballot_sync(0xFFFFFFFFu, f),
+                   c = __ballot_sync(0xFFFFFFFFu, fail);
+    if (lane() == 0) {
+        if (a) atomicAdd(ctr + 0, (unsigned long long)__popc(a));
+        if (b) atomicAdd(ctr + 1, (unsigned long long)__popc(b));
+        if (c) atomicAdd(ctr + 2, (unsigned long long)__popc(c));
+    }
+}
+
+// cnt[src] += 1 per edge, one atomic per distinct source in a warp
+__global__ void k_count(gallatin_graph g, const uint32_t *src, uint64_t n) {
+    const uint64_t i = blockIdx.x * (uint64_t)kT + threadIdx.x;
+    const uint32_t s = i < n ? src[i] : 0xFFFFFFFFu;
+    const unsigned peers = __match_any_sync(0xFFFFFFFFu, s);
+    if (s != 0xFFFFFFFFu && lane() == (uint32_t)__ffs((int)peers) - 1) atomicAdd(g.cnt + s, (uint32_t)__popc(peers));
+}
+
+// Per vertex with cnt new edges: a batch that overflows the list reallocates
+// it to the next power of two (device malloc); non-empty old lists are queued
+// for the copy + free.
+__global__ void k_grow(gallatin_graph g) {
+    const uint64_t v = blockIdx.x * (uint64_t)kT + threadIdx.x;
+    bool m = false, fail = false;
+    if (v < g.V) {
+        const uint32_t c = g.cnt[v];
+        if (c) {
+            const uint32_t s = g.size[v], need = s + c;
+            if (need > g.cap[v]) {
+                const uint32_t nc = list_cap(need);
+                void *p = gallatin_malloc((uint64_t)nc * 4);
+                if (!p) {
+                    fail = true;
+                } else {
+                    m = true;
+                    if (s > 0) {
+                        g.old[v] = g.list[v];
+                        g.work[atomicAdd(g.nwork, 1u)] = (uint32_t)v;
+                    }
+                    g.list[v] = reinterpret_cast<uint64_t>(p);
+                    g.cap[v] = nc;
+                }
+            }
+        }
+    }
+    count_warp(g.ctr, m, false, fail);
+}
+
+// warp per queued vertex: copy size[v] entries old -> new, free the old list
+__global__ void k_copy(gallatin_graph g) {
+    const uint32_t nw = *g.nwork;
+    const uint64_t warps = (uint64_t)gridDim.x * (kT / 32);
+    unsigned long long frees = 0;
+    for (uint64_t w = (blockIdx.x * (uint64_t)kT + threadIdx.x) >> 5; w < nw; w += warps) {
+        const uint32_t v = g.work[w], s = g.size[v];
+        const uint32_t *src = reinterpret_cast<const uint32_t *>(g.old[v]);
+        uint32_t *dst = reinterpret_cast<uint32_t *>(g.list[v]);
+        for (uint32_t k = lane(); k < s; k += 32) dst[k] = src[k];
+        __syncwarp();
+        if (lane() == 0) {
+            gallatin_free((void *)src);
+            frees++;
+        }
+    }
+    if (lane() == 0 && frees) atomicAdd(g.ctr + 1, frees);
+}
+
+// append: one atomic per distinct source in a warp reserves the positions
+__global__ void k_scatter(gallatin_graph g, const uint32_t *src, const uint32_t *dst, uint64_t n) {
+    const uint64_t i = blockIdx.x * (uint64_t)kT + threadIdx.x;
+    const uint32_t s = i < n ? src[i] : 0xFFFFFFFFu;
+    const unsigned peers = __match_any_sync(0xFFFFFFFFu, s);
+    const uint32_t leader = (uint32_t)__ffs((int)peers) - 1;
+    uint32_t base = 0;
+    if (s != 0xFFFFFFFFu && lane() == leader) base = atomicAdd(g.size + s, (uint32_t)__popc(peers));
+    base = __shfl_sync(peers, base, (int)leader);
+    if (s == 0xFFFFFFFFu) return;
+    const uint32_t pos = base + (uint32_t)__popc(peers & ((1u << lane()) - 1));
+    reinterpret_cast<uint32_t *>(g.list[s])[pos] = dst[i];
+}
+
+// ---- delete batch ------------------------------------------------------------
+__device__ __forceinline__ uint64_t hmix(uint64_t k) {
+    k ^= k >> 33;
+    k *= 0xff51afd7ed558ccdull;
+    k ^= k >> 33;
+    return k;
+}
+
+__global__ void k_hash_insert(gallatin_graph g, const uint32_t *src, const uint32_t *dst, uint64_t n) {
+    const uint64_t i = blockIdx.x * (uint64_t)kT + threadIdx.x;
+    if (i >= n) return;
+    const uint64_t key = ((uint64_t)src[i] << 32) | dst[i], mask = g.hcap - 1;
+    for (uint64_t h = hmix(key) & mask;; h = (h + 1) & mask) {
+        const uint64_t k = atomicCAS(reinterpret_cast<unsigned long long *>(g.hkeys + h), kEmpty, key);
+        if (k == kEmpty || k == key) {
+            atomicAdd(g.hcnt + h, 1u);
+            return;
+        }
+    }
+}
+
+// take one pending deletion of (v, x); true if this instance is deleted
+__device__ __forceinline__ bool hash_take(const gallatin_graph &g, uint32_t v, uint32_t x) {
+    const uint64_t key = ((uint64_t)v << 32) | x, mask = g.hcap - 1;
+    for (uint64_t h = hmix(key) & mask;; h = (h + 1) & mask) {
+        const uint64_t k = g.hkeys[h];
+        if (k == kEmpty) return false;
+        if (k != key) continue;
+        uint32_t c = *(volatile uint32_t *)(g.hcnt + h);
+        while (c > 0) {
+            const uint32_t o = atomicCAS(g.hcnt + h, c, c - 1);
+            if (o == c) return true;
+            c = o;
+        }
+        return false;
+    }
+}
+
+__global__ void k_list_work(gallatin_graph g) {
+    const uint64_t v = blockIdx.x * (uint64_t)kT + threadIdx.x;
+    if (v >= g.V || g.cnt[v] == 0 || g.size[v] == 0) return;
+    if (g.size[v] >= kBig) g.work2[atomicAdd(g.nwork + 1, 1u)] = (uint32_t)v;
+    else g.work[atomicAdd(g.nwork, 1u)] = (uint32_t)v;
+}
+
+// Shrink after a delete (once per batch per vertex): size 0 frees the list,
+// size <= cap/4 reallocates to the next power of two; executed by one warp.
+__device__ void shrink_warp(const gallatin_graph &g, uint32_t v, uint32_t out, bool &m, bool &f, bool &fail) {
+    const uint32_t cap = g.cap[v];
+    uint64_t np = 0;
+    bool act = false;
+    if (lane() == 0) {
+        g.size[v] = out;
+        if (out == 0) {
+            gallatin_free(reinterpret_cast<void *>(g.list[v]));
+            g.list[v] = 0;
+            g.cap[v] = 0;
+            f = true;
+        } else if (out <= cap / 4 && cap > 4) {
+            const uint32_t nc = list_cap(out);
+            void *p = gallatin_malloc((uint64_t)nc * 4);
+            if (p) {
+                np = reinterpret_cast<uint64_t>(p);
+                act = true;
+                m = f = true;
+            } else {
+                fail = true;
+            }
+        }
+    }
+    act = __shfl_sync(0xFFFFFFFFu, act, 0);
+    if (!act) return;
+    np = __shfl_sync(0xFFFFFFFFu, np, 0);
+    const uint32_t *src = reinterpret_cast<const uint32_t *>(g.list[v]);
+    uint32_t *dst = reinterpret_cast<uint32_t *>(np);
+    for (uint32_t k = lane(); k < out; k += 32) dst[k] = src[k];
+    __syncwarp();
+    if (lane() == 0) {
+        gallatin_free((void *)src);
+        g.list[v] = np;
+        g.cap[v] = list_cap(out);
+    }
+}
+
+// warp per vertex: scan, drop the deleted instances, compact in place
+__global__ void k_delete_small(gallatin_graph g) {
+    const uint32_t nw = g.nwork[0];
+    const uint64_t warps = (uint64_t)gridDim.x * (kT / 32);
+    bool m = false, f = false, fail = false;
+    for (uint64_t w = (blockIdx.x * (uint64_t)kT + threadIdx.x) >> 5; w < nw; w += warps) {
+        const uint32_t v = g.work[w], s = g.size[v];
+        uint32_t *L = reinterpret_cast<uint32_t *>(g.list[v]);
+        uint32_t out = 0;
+        for (uint32_t b = 0; b < s; b += 32) {
+            const uint32_t i = b + lane();
+            uint32_t x = 0;
+            bool keep = false;
+            if (i < s) {
+                x = L[i];
+                keep = !hash_take(g, v, x);
+            }
+            const unsigned km = __ballot_sync(0xFFFFFFFFu, keep);
+            if (keep) L[out + __popc(km & ((1u << lane()) - 1))] = x;    // out <= b: never ahead of the reads
+            out += (uint32_t)__popc(km);
+        }
+        __syncwarp();
+        shrink_warp(g, v, out, m, f, fail);
+    }
+    count_warp(g.ctr, m, f, fail);
+}
+
+// CTA per big vertex: same, with a block-wide prefix per 256-entry chunk
+__global__ void k_delete_big(gallatin_graph g) {
+    __shared__ uint32_t wsum[kT / 32];
+    __shared__ uint32_t out_s;
+    const uint32_t nw = g.nwork[1], wid = threadIdx.x >> 5;
+    bool m = false, f = false, fail = false;
+    for (uint32_t w = blockIdx.x; w < nw; w += gridDim.x) {
+        const uint32_t v = g.work2[w], s = g.size[v];
+        uint32_t *L = reinterpret_cast<uint32_t *>(g.list[v]);
+        if (threadIdx.x == 0) out_s = 0;
+        __syncthreads();
+        for (uint32_t b = 0; b < s; b += kT) {
+            const uint32_t i = b + threadIdx.x;
+            uint32_t x = 0;
+            bool keep = false;
+            if (i < s) {
+                x = L[i];
+                keep = !hash_take(g, v, x);
+            }
+            const unsigned km = __ballot_sync(0xFFFFFFFFu, keep);
+            if (lane() == 0) wsum[wid] = (uint32_t)__popc(km);
+            __syncthreads();
+            uint32_t before = out_s, tot = 0;
+            for (uint32_t q = 0; q < kT / 32; q++) {
+                if (q < wid) before += wsum[q];
+                tot += wsum[q];
+            }
+            if (keep) L[before + __popc(km & ((1u << lane()) - 1))] = x;
+            __syncthreads();
+            if (threadIdx.x == 0) out_s += tot;
+            __syncthreads();
+        }
+        if (wid == 0) shrink_warp(g, v, out_s, m, f, fail);
+        __syncthreads();
+    }
+    count_warp(g.ctr, m, f, fail);
+}
+
+// ---- expansion ---------------------------------------------------------------
+__global__ void k_expand_prep(gallatin_graph g, const uint32_t *vs, uint64_t n) {
+    const uint64_t i = blockIdx.x * (uint64_t)kT + threadIdx.x;
+    if (i >= n) return;
+    const uint32_t s = g.size[vs[i]];
+    g.cnt[vs[i]] = s < 4 ? 4 : s;              // each round appends max(size, 4) edges
+}
+
+__global__ void k_expand_fill(gallatin_graph g, const uint32_t *vs, uint64_t n) {
+    const uint64_t warps = (uint64_t)gridDim.x * (kT / 32);
+    for (uint64_t w = (blockIdx.x * (uint64_t)kT + threadIdx.x) >> 5; w < n; w += warps) {
+        const uint32_t v = vs[w], s0 = g.size[v], add = g.cnt[v];
+        uint32_t *L = reinterpret_cast<uint32_t *>(g.list[v]);
+        for (uint32_t j = lane(); j < add; j += 32) L[s0 + j] = (uint32_t)(((uint64_t)v + s0 + j + 1) % g.V);
+        __syncwarp();
+        if (lane() == 0) g.size[v] = s0 + add;
+    }
+}
+
+__global__ void k_free_all(gallatin_graph g) {
+    const uint64_t v = blockIdx.x * (uint64_t)kT + threadIdx.x;
+    bool f = false;
+    if (v < g.V && g.list[v]) {
+        gallatin_free(reinterpret_cast<void *>(g.list[v]));
+        g.list[v] = 0;
+        g.size[v] = 0;
+        g.cap[v] = 0;
+        f = true;
+    }
+    count_warp(g.ctr, false, f, false);
+}
+
+__global__ void k_export(gallatin_graph g, uint32_t *size, uint32_t *cap, uint64_t *list) {
+    const uint64_t v = blockIdx.x * (uint64_t)kT + threadIdx.x;
+    if (v >= g.V) return;
+    if (size) size[v] = g.size[v];
+    if (cap) cap[v] = g.cap[v];
+    if (list) list[v] = g.list[v];
+}
+
+__global__ void k_gather(gallatin_graph g, const uint64_t *off, uint32_t *out) {
+    const uint64_t warps = (uint64_t)gridDim.x * (kT / 32);
+    for (uint64_t v = (blockIdx.x * (uint64_t)kT + threadIdx.x) >> 5; v < g.V; v += warps) {
+        const uint32_t s = g.size[v];
+        const uint32_t *L = reinterpret_cast<const uint32_t *>(g.list[v]);
+        for (uint32_t k = lane(); k < s; k += 32) out[off[v] + k] = L[k];
+    }
+}
+
+int run_grow(gallatin_graph *g, cudaStream_t st) {
+    k_grow<<<blocks(g->V), kT, 0, st>>>(*g);
+    k_copy<<<148 * 8, kT, 0, st>>>(*g);
+    return status();
+}
+}  // namespace
+
+extern "C" {
+
+int gallatin_graph_create(uint32_t V, gallatin_graph_t **out) {
+    if (!out || V == 0) return GALLATIN_ERR_INVALID;
+    if (!gallatin_is_initialized()) return GALLATIN_ERR_STATE;
+    const int rc = gallatin::bind_device();            // the device API's constant view
+    if (rc != GALLATIN_OK) return rc;
+    gallatin_graph *g = new gallatin_graph{};
+    g->V = V;
+    bool ok = cudaMalloc(&g->list, 8ull * V) == cudaSuccess && cudaMalloc(&g->size, 4ull * V) == cudaSuccess &&
+              cudaMalloc(&g->cap, 4ull * V) == cudaSuccess && cudaMalloc(&g->cnt, 4ull * V) == cudaSuccess &&
+              cudaMalloc(&g->old, 8ull * V) == cudaSuccess && cudaMalloc(&g->work, 4ull * V) == cudaSuccess &&
+              cudaMalloc(&g->work2, 4ull * V) == cudaSuccess && cudaMalloc(&g->nwork, 8) == cudaSuccess &&
+              cudaMalloc(&g->ctr, 24) == cudaSuccess;
+    if (!ok) {
+        cudaGetLastError();
+        gallatin_graph_destroy(g, nullptr);
+        return GALLATIN_ERR_NOMEM;
+    }
+    cudaMemset(g->list, 0, 8ull * V);
+    cudaMemset(g->size, 0, 4ull * V);
+    cudaMemset(g->cap, 0, 4ull * V);
+    cudaMemset(g->ctr, 0, 24);
+    *out = g;
+    return status();
+}
+
+int gallatin_graph_destroy(gallatin_graph_t *g, void *stream) {
+    if (!g) return GALLATIN_ERR_INVALID;
+    if (g->list && gallatin_is_initialized()) k_free_all<<<blocks(g->V), kT, 0, S(stream)>>>(*g);
+    cudaStreamSynchronize(S(stream));
+    void *ptrs[] = {g->list, g->size, g->cap, g->cnt, g->old, g->work, g->work2, g->nwork, g->ctr, g->hkeys, g->hcnt};
+    for (void *p : ptrs)
+        if (p) cudaFree(p);
+    delete g;
+    return status();
+}
+
+int gallatin_graph_insert(gallatin_graph_t *g, const uint32_t *src, const uint32_t *dst, uint64_t n, void *stream) {
+    if (!g || (n && (!src || !dst))) return GALLATIN_ERR_INVALID;
+    if (n == 0) return GALLATIN_OK;
+    cudaStream_t st = S(stream);
+    cudaMemsetAsync(g->cnt, 0, 4ull * g->V, st);
+    cudaMemsetAsync(g->nwork, 0, 8, st);
+    k_count<<<blocks(n), kT, 0, st>>>(*g, src, n);
+    int rc = run_grow(g, st);
+    if (rc) return rc;
+    k_scatter<<<blocks(n), kT, 0, st>>>(*g, src, dst, n);
+    return status();
+}
+
+int gallatin_graph_delete(gallatin_graph_t *g, const uint32_t *src, const uint32_t *dst, uint64_t n, void *stream) {
+    if (!g || (n && (!src || !dst))) return GALLATIN_ERR_INVALID;
+    if (n == 0) return GALLATIN_OK;
+    cudaStream_t st = S(stream);
+    uint64_t cap = 1;
+    while (cap < 2 * n) cap <<= 1;
+    if (cap > g->hcap) {
+        if (g->hkeys) cudaFree(g->hkeys);
+        if (g->hcnt) cudaFree(g->hcnt);
+        g->hkeys = nullptr;
+        g->hcnt = nullptr;
+        if (cudaMalloc(&g->hkeys, 8 * cap) != cudaSuccess || cudaMalloc(&g->hcnt, 4 * cap) != cudaSuccess) {
+            cudaGetLastError();
+            g->hcap = 0;
+            return GALLATIN_ERR_NOMEM;
+        }
+        g->hcap = cap;
+    }
+    gallatin_graph gv = *g;
+    gv.hcap = cap;                               // a power of two <= the allocation
+    cudaMemsetAsync(g->hkeys, 0xFF, 8 * cap, st);
+    cudaMemsetAsync(g->hcnt, 0, 4 * cap, st);
+    cudaMemsetAsync(g->cnt, 0, 4ull * g->V, st);
+    cudaMemsetAsync(g->nwork, 0, 8, st);
+    k_hash_insert<<<blocks(n), kT, 0, st>>>(gv, src, dst, n);
+    k_count<<<blocks(n), kT, 0, st>>>(gv, src, n);
+    k_list_work<<<blocks(g->V), kT, 0, st>>>(gv);
+    k_delete_small<<<148 * 8, kT, 0, st>>>(gv);
+    k_delete_big<<<148 * 4, kT, 0, st>>>(gv);
+    return status();
+}
+
+int gallatin_graph_expand(gallatin_graph_t *g, const uint32_t *vs, uint64_t n, void *stream) {
+    if (!g || (n && !vs)) return GALLATIN_ERR_INVALID;
+    if (n == 0) return GALLATIN_OK;
+    cudaStream_t st = S(stream);
+    cudaMemsetAsync(g->cnt, 0, 4ull * g->V, st);
+    cudaMemsetAsync(g->nwork, 0, 8, st);
+    k_expand_prep<<<blocks(n), kT, 0, st>>>(*g, vs, n);
+    int rc = run_grow(g, st);
+    if (rc) return rc;
+    k_expand_fill<<<148 * 8, kT, 0, st>>>(*g, vs, n);
+    return status();
+}
+
+int gallatin_graph_export(const gallatin_graph_t *g, uint32_t *size, uint32_t *cap, uint64_t *list, void *stream) {
+    if (!g) return GALLATIN_ERR_INVALID;
+    k_export<<<blocks(g->V), kT, 0, S(stream)>>>(*g, size, cap, list);
+    return status();
+}
+
+int gallatin_graph_gather(const gallatin_graph_t *g, const uint64_t *off, uint32_t *out, void *stream) {
+    if (!g || !off || !out) return GALLATIN_ERR_INVALID;
+    k_gather<<<148 * 16, kT, 0, S(stream)>>>(*g, off, out);
+    return status();
+}
+
+int gallatin_graph_counters(const gallatin_graph_t *g, uint64_t out[3]) {
+    if (!g || !out) return GALLATIN_ERR_INVALID;
+    if (cudaDeviceSynchronize() != cudaSuccess) return GALLATIN_ERR_CUDA;
+    unsigned long long c[3];
+    if (cudaMemcpy(c, g->ctr, sizeof(c), cudaMemcpyDeviceToHost) != cudaSuccess) return GALLATIN_ERR_CUDA;
+    for (int i = 0; i < 3; i++) out[i] = c[i];
+    return GALLATIN_OK;
+}
+
+}  // extern "C"

@@ -140,3 +140,60 @@ def replay_ops(n_ops: int, seed: int, p_free: float = 0.4, p_drain: float = 0.0,
             args[i] = sizes[rng.choice(len(sizes), p=w)]
             live.append(i)
     return kinds, args, keys
+
+
+# ------------------------------------------------------- streaming graph ---
+def rmat_edges(scale: int, n: int, seed: int, device: str = "cpu", abcd=(0.57, 0.19, 0.19, 0.05),
+               chunk: int = 1 << 24):
+    """n R-MAT edges over 2^scale vertices (Chakrabarti et al.; SURVEY 8(d) C5:
+    (a,b,c,d) = (0.57, 0.19, 0.19, 0.05), multi-edges kept) with a seeded
+    vertex permutation.  Returns int32 torch tensors (src, dst) on `device`."""
+    import torch
+    g = torch.Generator(device=device)
+    g.manual_seed(seed & ((1 << 63) - 1))
+    a, b, c, _ = abcd
+    src = torch.empty(n, dtype=torch.int32, device=device)
+    dst = torch.empty(n, dtype=torch.int32, device=device)
+    for lo in range(0, n, chunk):
+        m = min(chunk, n - lo)
+        s = torch.zeros(m, dtype=torch.int64, device=device)
+        d = torch.zeros(m, dtype=torch.int64, device=device)
+        for _ in range(scale):
+            r = torch.rand(m, generator=g, device=device)
+            s = s * 2 + (r >= a + b).to(torch.int64)
+            d = d * 2 + (((r >= a) & (r < a + b)) | (r >= a + b + c)).to(torch.int64)
+        src[lo:lo + m] = s.to(torch.int32)
+        dst[lo:lo + m] = d.to(torch.int32)
+    perm = torch.randperm(1 << scale, generator=g, device=device).to(torch.int32)
+    return perm[src.long()], perm[dst.long()]
+
+
+def graph_workload(scale: int, n_edges: int, seed: int | None = None, device: str = "cpu", batches: int = 8,
+                   n_expand: int = 1 << 16, rounds: int = 8) -> dict:
+    """BASELINE configs[4] phases:
+      init    : the first n/2 edges,
+      insert  : the other n/2 in `batches` batches,
+      delete  : `batches` batches of n/16 edges sampled without replacement
+                from the inserted multiset,
+      expand  : min(n_expand, V/4) distinct seeded vertices, `rounds` rounds."""
+    import torch
+    seed = cell_seed(5, scale) if seed is None else seed
+    V = 1 << scale
+    src, dst = rmat_edges(scale, n_edges, seed, device)
+    half = n_edges // 2
+    g = torch.Generator(device=device)
+    g.manual_seed((seed ^ 0x5DEECE66D) & ((1 << 63) - 1))
+    per = torch.randperm(n_edges, generator=g, device=device)
+    db = n_edges // (2 * batches)
+    ins_b = (n_edges - half) // batches
+    nexp = min(n_expand, V // 4)
+    exp_v = torch.randperm(V, generator=g, device=device)[:nexp].to(torch.int32)
+    return {
+        "V": V,
+        "init": (src[:half], dst[:half]),
+        "insert": [(src[half + k * ins_b: half + (k + 1) * ins_b], dst[half + k * ins_b: half + (k + 1) * ins_b])
+                   for k in range(batches)],
+        "delete": [(src[per[k * db:(k + 1) * db]], dst[per[k * db:(k + 1) * db]]) for k in range(batches)],
+        "expand": exp_v,
+        "rounds": rounds,
+    }
