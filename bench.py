@@ -371,7 +371,56 @@ def run_extras(args, G, torch, stream):
     ms, ops = G.gallatin_probe(6, 1 << 24, 1 << 30)
     pk["hbm_copy_gbs"] = ops / ms / 1e6
     out["probes"] = pk
+    out["graph"] = run_graph(args, G, torch, stream)
     return out
+
+
+def run_graph(args, G, torch, stream):
+    """BASELINE configs[4]: R-MAT 2^24 vertices / 2^28 edges on a 16 GiB heap;
+    adjacency lists kept by DEVICE-side malloc/free (include/gallatin_graph.h).
+    Edges/s per phase and the allocator calls the kernels issued."""
+    import workload_gen as wg
+    scale = 24 - max(0, int(np.log2(args.scale)))
+    n = 1 << (scale + 4)
+    G.gallatin_destroy()
+    G.gallatin_init(HEAP_C2)
+    w = wg.graph_workload(scale, n, device="cuda", n_expand=1 << 16)
+    torch.cuda.synchronize()
+    g = G.Graph(w["V"])
+    ev = lambda: torch.cuda.Event(enable_timing=True)  # noqa: E731
+    res = {}
+
+    def timed(name, fn, edges):
+        a, b = ev(), ev()
+        a.record(stream)
+        fn()
+        b.record(stream)
+        torch.cuda.synchronize()
+        ms = a.elapsed_time(b)
+        res[name] = {"ms": ms, "edges": edges, "edges_per_s": edges / ms * 1e3}
+
+    s0, d0 = w["init"]
+    timed("init", lambda: g.insert(s0, d0), s0.numel())
+    timed("bulk_insert", lambda: [g.insert(s, d) for s, d in w["insert"]], sum(s.numel() for s, _ in w["insert"]))
+    timed("bulk_delete", lambda: [g.delete(s, d) for s, d in w["delete"]], sum(s.numel() for s, _ in w["delete"]))
+    size, _, _ = g.export()
+    before = int(size.sum())
+    timed("expansion", lambda: [g.expand(w["expand"]) for _ in range(w["rounds"])], 0)
+    size, cap, _ = g.export()
+    res["expansion"]["edges"] = int(size.sum()) - before
+    res["expansion"]["edges_per_s"] = res["expansion"]["edges"] / res["expansion"]["ms"] * 1e3
+    ctr = g.counters()
+    total_ms = sum(v["ms"] for v in res.values())
+    g.destroy()
+    G.gallatin_drain()
+    st = G.gallatin_stats()
+    G.gallatin_destroy()
+    G.gallatin_init(HEAP_C2)
+    return {"workload": f"BASELINE configs[4]: R-MAT 2^{scale} vertices / 2^{scale + 4} edges, (a,b,c,d)="
+                        "(0.57,0.19,0.19,0.05), 8 insert + 8 delete batches, 2^16-vertex x 8-round expansion, 16 GiB heap",
+            "phases": res, "device_mallocs": ctr["mallocs"], "device_frees": ctr["frees"],
+            "failed_mallocs": ctr["failed"], "allocator_ops_per_s": (ctr["mallocs"] + ctr["frees"]) / total_ms * 1e3,
+            "pristine_after_teardown": st["free_segments"] == st["num_segments"]}
 
 
 def run_e2e(args, G, torch, cells):
