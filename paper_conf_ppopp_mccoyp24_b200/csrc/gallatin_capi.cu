@@ -109,19 +109,19 @@ __global__ void k_reset() {
 // Then waits-and-retries, whole blocks and segment runs.
 __device__ __noinline__ void bulk_malloc_slow(const uint64_t *sizes, void **ptrs, uint64_t n, uint64_t base,
                                               uint32_t key, uint32_t slow, uint64_t info, int items,
-                                              unsigned callers) {
+                                              unsigned callers, uint32_t stride = 32) {
     const View &v = c_view;
     // pass 0: refill and prefetch duties only (never waits on another slot's refill)
     for (int k = 0; k < items; k++) {
         const uint32_t code = (uint32_t)(info >> (16 * k)) & 0xFFFF;
         if (((slow >> k) & 1) && (code & 0x2000u)) {
-            const uint32_t c = core::slice_class(sizes[base + 32ull * k]);
+            const uint32_t c = core::slice_class(sizes[base + (uint64_t)stride * k]);
             core::prefetch_slot(v, v.slot_off[c] + key % v.nslot[c], c, code & 0x3FF);
             slow &= ~(1u << k);                                     // its slice was stored already
             continue;
         }
         if (!((slow >> k) & 1) || !(code & 0x400u)) continue;
-        const uint64_t i = base + 32ull * k;
+        const uint64_t i = base + (uint64_t)stride * k;
         const uint32_t c = core::slice_class(sizes[i]);
         if (!core::refill_slot(v, v.slot_off[c] + key % v.nslot[c], c, code & 0x3FF)) {
             __stcs(reinterpret_cast<unsigned long long *>(ptrs) + i, 0ull);   // heap exhausted: NULL
@@ -135,7 +135,7 @@ __device__ __noinline__ void bulk_malloc_slow(const uint64_t *sizes, void **ptrs
     for (int k = 0; k < items; k++) {
         if (!((slow >> k) & 1)) continue;
         const uint32_t code = (uint32_t)(info >> (16 * k)) & 0xFFFF;
-        const uint64_t i = base + 32ull * k;
+        const uint64_t i = base + (uint64_t)stride * k;
         const uint64_t sz = sizes[i];
         void *p;
         if (code & 0x800u) {
@@ -214,6 +214,77 @@ __global__ void __launch_bounds__(kThreads, 5) k_bulk_malloc(const uint64_t *__r
     }
     const unsigned callers = __ballot_sync(0xFFFFFFFFu, slow != 0);
     if (slow) bulk_malloc_slow(sizes, ptrs, n, base, key, slow, info, ITEMS, callers);
+}
+
+// Bulk malloc with CTA-level aggregation: every warp of a CTA runs on one SM,
+// hence uses one block-buffer slot per class; the CTA's requests of a class
+// are counted in shared memory (one shared atomic per warp team) and ONE
+// global RMW per class per CTA takes their slices (1024 requests at
+// ITEMS=4), so the hot slot words see 32x fewer RMWs than with warp teams.
+// Item k of thread t is request blockIdx*256*ITEMS + k*256 + t.
+template <int ITEMS>
+__global__ void __launch_bounds__(kThreads, 5) k_bulk_malloc_cta(const uint64_t *__restrict__ sizes,
+                                                                  void **__restrict__ ptrs, uint64_t n) {
+    const View &v = c_view;
+    __shared__ uint32_t cnt[core::kTrees];
+    __shared__ uint64_t olds[core::kTrees];
+    const uint32_t lane = threadIdx.x & 31;
+    const uint64_t base = blockIdx.x * (uint64_t)(kThreads * ITEMS) + threadIdx.x;
+    const uint32_t key = ptx::smid();
+    if (threadIdx.x < core::kTrees) cnt[threadIdx.x] = 0;
+    uint64_t sz[ITEMS];
+    uint32_t cls[ITEMS], rank[ITEMS];
+#pragma unroll
+    for (int k = 0; k < ITEMS; k++) {
+        const uint64_t i = base + (uint64_t)kThreads * k;
+        sz[k] = i < n ? __ldcs(reinterpret_cast<const unsigned long long *>(sizes) + i) : 0;
+        cls[k] = sz[k] - 1 < core::kMaxSlice ? core::slice_class(sz[k]) : 0xFFu;
+    }
+    __syncthreads();
+    const uint32_t lt = ptx::lanemask_lt();
+#pragma unroll
+    for (int k = 0; k < ITEMS; k++) {
+        const unsigned peers = __match_any_sync(0xFFFFFFFFu, cls[k]);
+        const uint32_t leader = (uint32_t)__ffs((int)peers) - 1;
+        uint32_t b = 0;
+        if (cls[k] != 0xFFu && lane == leader) b = atomicAdd(&cnt[cls[k]], (uint32_t)__popc(peers));
+        rank[k] = __shfl_sync(0xFFFFFFFFu, b, (int)leader) + (uint32_t)__popc(peers & lt);
+    }
+    __syncthreads();
+    if (threadIdx.x < core::kTrees && cnt[threadIdx.x]) {
+        const uint32_t c = threadIdx.x;
+        olds[c] = ptx::atom_add(core::slot_word(v, v.slot_off[c] + key % v.nslot[c]), (uint64_t)cnt[c] << 32);
+    }
+    __syncthreads();
+    uint32_t slow = 0;
+    uint64_t info = 0;
+#pragma unroll
+    for (int k = 0; k < ITEMS; k++) {
+        const uint64_t i = base + (uint64_t)kThreads * k;
+        void *p = nullptr;
+        uint32_t code = 0;
+        if (cls[k] != 0xFFu) {
+            const uint64_t old = olds[cls[k]];
+            const uint32_t m = core::run_len(old);
+            const uint32_t idx = (uint32_t)(old >> 32) + rank[k];
+            if (idx < (m << core::kSliceLog2)) {
+                p = core::slice_ptr(v, cls[k], old & core::kRunNone, idx);
+                if (v.prefetch && idx == (m << (core::kSliceLog2 - 1))) code = 0x2000u | m;   // prefetch duty
+            } else {
+                code = idx == (m << core::kSliceLog2) ? (0x400u | m) : 0x1000u;
+            }
+        } else if (sz[k] != 0) {
+            code = 0x800u;
+        }
+        if (code) {
+            slow |= 1u << k;
+            info |= (uint64_t)code << (16 * k);
+        }
+        if (!(code & 0x1C00u) && i < n)
+            __stcs(reinterpret_cast<unsigned long long *>(ptrs) + i, reinterpret_cast<unsigned long long>(p));
+    }
+    const unsigned callers = __ballot_sync(0xFFFFFFFFu, slow != 0);
+    if (slow) bulk_malloc_slow(sizes, ptrs, n, base, key, slow, info, ITEMS, callers, kThreads);
 }
 
 __device__ __noinline__ void free_slow(const View &v, uint64_t p) {
@@ -590,7 +661,7 @@ int gallatin_malloc(const uint64_t *d_sizes, void **d_ptrs, uint64_t n, void *st
     if (n == 0) return GALLATIN_OK;
     if (!d_sizes || !d_ptrs || n > (1ull << 40)) return GALLATIN_ERR_INVALID;
     if (g.cfg.bulk_items == 4 || (g.cfg.bulk_items == 0 && n >= (uint64_t)kItemsMin))
-        k_bulk_malloc<4><<<grid_for((n + 3) / 4), kThreads, 0, S(stream)>>>(d_sizes, d_ptrs, n);
+        k_bulk_malloc_cta<4><<<grid_for((n + 3) / 4), kThreads, 0, S(stream)>>>(d_sizes, d_ptrs, n);
     else
         k_bulk_malloc<1><<<grid_for(n), kThreads, 0, S(stream)>>>(d_sizes, d_ptrs, n);
     return launch_status();
