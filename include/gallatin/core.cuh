@@ -161,6 +161,46 @@ __device__ inline __noinline__ uint64_t claim_front(const View &v) {
     }
 }
 
+// [dev] claim a run of up to kmax consecutive free segments starting at the
+// lowest free one, with one atomicAnd on the leaf word: the window
+// [s, s+kmax) within that word is taken at once, the consecutive prefix from
+// s is kept and the rest given back.  Concurrent claimers then get disjoint
+// windows instead of interleaving single segments.  *k = segments claimed
+// (serially: s = successor(0) and the free segments that follow it).
+__device__ inline __noinline__ uint64_t claim_front_run(const View &v, uint32_t kmax, uint32_t *k) {
+    const BitTree st = seg_tree(v);
+    uint64_t from = 0;
+    for (;;) {
+        uint64_t s = bt_successor<false>(st, from);
+        if (s == kNone) {
+            if (from != 0) { from = 0; continue; }
+            s = bt_scan_first(st);
+            if (s == kNone) {
+                if (!reclaim_idle(v)) return kNone;
+                continue;
+            }
+        }
+        const uint64_t wi = s >> 6;
+        const uint32_t lo = (uint32_t)(s & 63);
+        uint64_t hi = lo + (uint64_t)kmax;
+        if (hi > 64) hi = 64;
+        if ((wi << 6) + hi > v.nseg) hi = v.nseg - (wi << 6);
+        const uint64_t mask = bit_range(lo, (uint32_t)hi);
+        uint64_t *leaf = st.w + st.off[0] + wi;
+        const uint64_t old = ptx::atom_and(leaf, ~mask);
+        const uint64_t got = old & mask;
+        const uint32_t run = (uint32_t)__ffsll((long long)~(got >> lo)) - 1;   // 0 if s was lost
+        const uint64_t extra = got & ~bit_range(lo, lo + run);
+        bool flip = old != 0 && (old & ~mask) == 0;
+        if (extra) flip |= ptx::atom_or(leaf, extra) == 0;
+        if (flip) bt_reconcile_up(st, 0, wi);
+        if (run == 0) { from = s + 1; continue; }
+        ptx::fence_acq_rel();
+        *k = run;
+        return s;
+    }
+}
+
 // initSegment for tree t: blocks [keep, nb) go into the ring in order
 // and the segment joins block tree t ("broadcast availability");
 // blocks [0, keep) belong to the caller.
@@ -309,11 +349,32 @@ __device__ inline __noinline__ uint32_t get_run(const View &v, uint32_t t, uint3
         }
         if (want >= nb) {
             // the run covers whole segments: take fresh ones privately [dev]
-            const uint64_t s0 = claim_front(v);
+            uint32_t k = 0;
+            const uint32_t kmax = want / nb;
+            const uint64_t s0 = claim_front_run(v, kmax, &k);
             if (s0 == kNone) return 0;                        // "No allocations left"
             const BitTree st = seg_tree(v);
-            uint32_t k = 1;
-            while (k < want / nb && s0 + k < v.nseg && bt_delete(st, s0 + k)) k++;
+            // extend with the following free segments: one atomicAnd per leaf
+            // word claims the whole window, the consecutive prefix is kept and
+            // the rest given back (serially: the next free segments in order)
+            while (k < kmax && s0 + k < v.nseg && ((s0 + k) & 63) == 0) {
+                const uint64_t x = s0 + k, wi = x >> 6;
+                const uint32_t lo = (uint32_t)(x & 63);
+                uint64_t hi = lo + (uint64_t)(kmax - k);
+                if (hi > 64) hi = 64;
+                if ((wi << 6) + hi > v.nseg) hi = v.nseg - (wi << 6);
+                const uint64_t mask = bit_range(lo, (uint32_t)hi);
+                uint64_t *leaf = st.w + st.off[0] + wi;
+                const uint64_t old = ptx::atom_and(leaf, ~mask);
+                const uint64_t got = old & mask;
+                const uint32_t run = (uint32_t)__ffsll((long long)~(got >> lo)) - 1;   // prefix length
+                const uint64_t extra = got & ~bit_range(lo, lo + run);
+                bool flip = old != 0 && (old & ~mask) == 0;
+                if (extra) flip |= ptx::atom_or(leaf, extra) == 0;
+                if (flip) bt_reconcile_up(st, 0, wi);
+                k += run;
+                if (lo + run < hi) break;                         // the free run ended here
+            }
             for (uint32_t q = 0; q < k; q++) ptx::st_relaxed(v.seg_tid + s0 + q, t);
             ptx::fence_acq_rel();
             for (uint32_t q = 0; q < k; q++) ptx::atom_add(v.seg_word + s0 + q, sw_retree(kTreeFree, t));
