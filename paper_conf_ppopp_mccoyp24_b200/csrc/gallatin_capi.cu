@@ -556,7 +556,7 @@ int gallatin_init_ex(const gallatin_config_t *cfg_in) {
     if (!cfg.fence_free) cfg.fence_free = 1;
     if (!cfg.format_ahead) cfg.format_ahead = 1;
     if (!cfg.run_max) cfg.run_max = 256;
-    if (!cfg.run_init) cfg.run_init = (uint32_t)(nseg / 128 < 1 ? 1 : (nseg / 128 > 8 ? 8 : nseg / 128));
+    if (!cfg.run_init) cfg.run_init = (uint32_t)(nseg / 16 < 1 ? 1 : (nseg / 16 > 64 ? 64 : nseg / 16));
     if (!cfg.run_bytes) {
         cfg.run_bytes = (nseg << core::kSegLog2) / 64;
         if (cfg.run_bytes > (256ull << 20)) cfg.run_bytes = 256ull << 20;
@@ -588,7 +588,7 @@ int gallatin_init_ex(const gallatin_config_t *cfg_in) {
         v.run_cap[c] = m < 1 ? 1u : (uint32_t)m;
     }
     v.format_ahead = cfg.format_ahead == 1 ? 1u : 0u;
-    v.formatters = (uint32_t)(nseg / 128 < 1 ? 1 : (nseg / 128 > 8 ? 8 : nseg / 128));
+    v.formatters = (uint32_t)(nseg / 32 < 1 ? 1 : (nseg / 32 > 32 ? 32 : nseg / 32));
     v.run_init = cfg.run_init;
     v.prefetch = cfg.prefetch == 1 ? 1u : 0u;              // default off (measured: DESIGN.md)
     v.fence_free = cfg.fence_free;
