@@ -415,7 +415,8 @@ static uint64_t malloc_slice(o2_t *a, uint32_t c, uint64_t key) {
             a->next[i] = SLOT_EMPTY;
             continue;
         }
-        uint32_t fr = a->run_init >> c; if (fr < 1) fr = 1;         /* empty slot: run_init >> c */
+        uint32_t fl = a->run_init < 8 ? a->run_init : 8;            /* empty slot: max(run_init >> c, min(run_init, 8)) */
+        uint32_t fr = (a->run_init >> c) > fl ? (a->run_init >> c) : fl;
         uint32_t first_run = fr < cap ? fr : cap;
         uint32_t want = m == 0 ? first_run : grow;
         uint32_t got = get_run(a, c, want, &first);
