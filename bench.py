@@ -371,8 +371,38 @@ def run_extras(args, G, torch, stream):
     ms, ops = G.gallatin_probe(6, 1 << 24, 1 << 30)
     pk["hbm_copy_gbs"] = ops / ms / 1e6
     out["probes"] = pk
+    out["scaling"] = run_scaling(args, G, torch, stream)
     out["graph"] = run_graph(args, G, torch, stream)
     return out
+
+
+def run_scaling(args, G, torch, stream):
+    """BASELINE configs[3]: 64 B mallocs then frees at 2^10 .. 2^26 threads on the
+    16 GiB heap (reset before each run); median of 5 runs per point."""
+    pts = {}
+    for lg in range(10, 27, 2):
+        n = (1 << lg) // args.scale if (1 << lg) // args.scale >= 1024 else 1 << lg
+        st = torch.full((n,), 64, dtype=torch.int64, device="cuda")
+        p = torch.empty_like(st)
+        mm, fm = [], []
+        for it in range(7):
+            G.gallatin_reset()
+            a, b, c = (torch.cuda.Event(enable_timing=True) for _ in range(3))
+            a.record(stream)
+            G.gallatin_malloc(st, p)
+            b.record(stream)
+            G.gallatin_free(p)
+            c.record(stream)
+            torch.cuda.synchronize()
+            if it >= 2:
+                mm.append(a.elapsed_time(b))
+                fm.append(b.elapsed_time(c))
+        m, f = statistics.median(mm), statistics.median(fm)
+        pts[str(n)] = {"malloc_ms": round(m, 5), "free_ms": round(f, 5), "malloc_ops_s": n / m * 1e3,
+                       "free_ops_s": n / f * 1e3}
+        del st, p
+    return {"workload": "BASELINE configs[3]: 64 B, 2^10..2^26 threads (every 4th power), 16 GiB heap, "
+                        "independent per-GPU heap under torchrun", "points": pts}
 
 
 def run_graph(args, G, torch, stream):

@@ -219,3 +219,13 @@ def test_config2_full_size_bench_launch(cuda_ok, G, size):
             G.gallatin_reset()
         assert _bulk_round(G, nseg, wg.single_sizes(size, n)) == 0
         _assert_pristine(G, nseg)
+
+
+@pytest.mark.parametrize("n", [1, 31, 33, 255, 1000, 1 << 10, 4097, 1 << 16, 1 << 26])
+def test_config4_thread_scaling_points(cuda_ok, G, n):
+    """BASELINE configs[3]: 64 B at 2^10..2^26 threads, plus ragged counts
+    (one thread, partial warps and CTAs, one slice past a block)."""
+    nseg = 1024
+    G.gallatin_init(nseg * SEG)
+    assert _bulk_round(G, nseg, wg.single_sizes(64, n)) == 0
+    _assert_pristine(G, nseg)
