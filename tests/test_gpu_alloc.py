@@ -229,3 +229,16 @@ def test_config4_thread_scaling_points(cuda_ok, G, n):
     G.gallatin_init(nseg * SEG)
     assert _bulk_round(G, nseg, wg.single_sizes(64, n)) == 0
     _assert_pristine(G, nseg)
+
+
+def test_config3_full_size_bench_launch(cuda_ok, G):
+    """BASELINE configs[2] at its full size (2^22 threads, 64 GB heap), as
+    bench.py runs it: stamp-verified, accounted, overlap-checked, pristine."""
+    nseg = 4096
+    G.gallatin_init(nseg * SEG)
+    sizes = wg.mixed_sizes(1 << 22)
+    for rep in range(2):
+        if rep:
+            G.gallatin_reset()
+        assert _bulk_round(G, nseg, sizes) == 0
+        _assert_pristine(G, nseg)
