@@ -166,7 +166,9 @@ __global__ void __launch_bounds__(kThreads, 5) k_bulk_malloc(const uint64_t *__r
 #pragma unroll
     for (int k = 0; k < ITEMS; k++) {
         const uint64_t i = base + 32ull * k;
-        sz[k] = i < n ? __ldcs(reinterpret_cast<const unsigned long long *>(sizes) + i) : 0;
+        // unconditional load of a clamped index: the ITEMS loads issue back to back
+        const uint64_t x = __ldcs(reinterpret_cast<const unsigned long long *>(sizes) + (i < n ? i : n - 1));
+        sz[k] = i < n ? x : 0;
     }
 #pragma unroll
     for (int k = 0; k < ITEMS; k++) {
@@ -237,7 +239,9 @@ __global__ void __launch_bounds__(kThreads, 5) k_bulk_malloc_cta(const uint64_t 
 #pragma unroll
     for (int k = 0; k < ITEMS; k++) {
         const uint64_t i = base + (uint64_t)kThreads * k;
-        sz[k] = i < n ? __ldcs(reinterpret_cast<const unsigned long long *>(sizes) + i) : 0;
+        // unconditional load of a clamped index: the ITEMS loads issue back to back
+        const uint64_t x = __ldcs(reinterpret_cast<const unsigned long long *>(sizes) + (i < n ? i : n - 1));
+        sz[k] = i < n ? x : 0;
         cls[k] = sz[k] - 1 < core::kMaxSlice ? core::slice_class(sz[k]) : 0xFFu;
     }
     __syncthreads();
@@ -332,7 +336,8 @@ __global__ void __launch_bounds__(kThreads, 6) k_bulk_free(void *const *__restri
 #pragma unroll
     for (int k = 0; k < ITEMS; k++) {
         const uint64_t i = base + 32ull * k;
-        p[k] = i < n ? __ldcs(reinterpret_cast<const unsigned long long *>(ptrs) + i) : 0;
+        const uint64_t x = __ldcs(reinterpret_cast<const unsigned long long *>(ptrs) + (i < n ? i : n - 1));
+        p[k] = i < n ? x : 0;
     }
 #pragma unroll
     for (int k = 0; k < ITEMS; k++) {
