@@ -561,7 +561,7 @@ int gallatin_init_ex(const gallatin_config_t *cfg_in) {
     if (!cfg.fence_free) cfg.fence_free = 1;
     if (!cfg.format_ahead) cfg.format_ahead = 1;
     if (!cfg.run_max) cfg.run_max = 256;
-    if (!cfg.run_init) cfg.run_init = (uint32_t)(nseg / 16 < 1 ? 1 : (nseg / 16 > 64 ? 64 : nseg / 16));
+    if (!cfg.run_init) cfg.run_init = (uint32_t)(nseg / 4 < 1 ? 1 : (nseg / 4 > 256 ? 256 : nseg / 4));
     if (!cfg.run_bytes) {
         cfg.run_bytes = (nseg << core::kSegLog2) / 64;
         if (cfg.run_bytes > (256ull << 20)) cfg.run_bytes = 256ull << 20;
