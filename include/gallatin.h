@@ -69,7 +69,7 @@ typedef struct gallatin_config {
     uint32_t format_ahead;
     uint32_t fence_free;
     uint32_t bulk_items;   /* requests per thread in the bulk kernels: 0 = auto, 1 or 4 */
-    uint32_t run_init;     /* first run of an empty slot of class c: max(run_init >> c, min(run_init, 8)) blocks (default clamp(nseg/4, 1, 256)) */
+    uint32_t run_init;     /* first run of an empty slot of class c: min(max(run_init >> c, min(run_init, 8)), 256 >> c) blocks (default: the largest power of two <= 256 whose first runs over all slots fit in half the heap) */
     uint32_t prefetch;     /* 1 = fetch the next run at the middle of the current one; 0/2 = off (default) */
 } gallatin_config_t;
 

@@ -420,8 +420,10 @@ __device__ inline __noinline__ bool refill_slot(const View &v, uint32_t si, uint
         }
     }
     const uint32_t cap = v.run_cap[c];
-    const uint32_t fl = v.run_init < 8 ? v.run_init : 8u;              // halves per class, floor min(run_init, 8)
-    const uint32_t fr = (v.run_init >> c) > fl ? (v.run_init >> c) : fl;
+    // halves per class, floor min(run_init, 8), at most one segment (nb blocks)
+    const uint32_t fl = v.run_init < 8 ? v.run_init : 8u;
+    const uint32_t fs = (v.run_init >> c) > fl ? (v.run_init >> c) : fl;
+    const uint32_t fr = fs < (256u >> c) ? fs : (256u >> c);
     const uint32_t first_run = fr < cap ? fr : cap;
     const uint32_t want = m_prev == 0 ? first_run : (2 * m_prev < cap ? 2 * m_prev : cap);
     uint32_t first = 0;

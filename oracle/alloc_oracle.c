@@ -415,8 +415,11 @@ static uint64_t malloc_slice(o2_t *a, uint32_t c, uint64_t key) {
             a->next[i] = SLOT_EMPTY;
             continue;
         }
-        uint32_t fl = a->run_init < 8 ? a->run_init : 8;            /* empty slot: max(run_init >> c, min(run_init, 8)) */
+        /* empty slot: max(run_init >> c, min(run_init, 8)) blocks, at most one
+           segment (256 >> c blocks) and the class cap [ours, DESIGN.md Deviations 5] */
+        uint32_t fl = a->run_init < 8 ? a->run_init : 8;
         uint32_t fr = (a->run_init >> c) > fl ? (a->run_init >> c) : fl;
+        if (fr > (256u >> c)) fr = 256u >> c;
         uint32_t first_run = fr < cap ? fr : cap;
         uint32_t want = m == 0 ? first_run : grow;
         uint32_t got = get_run(a, c, want, &first);

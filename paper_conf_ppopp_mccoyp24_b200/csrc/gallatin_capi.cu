@@ -561,7 +561,6 @@ int gallatin_init_ex(const gallatin_config_t *cfg_in) {
     if (!cfg.fence_free) cfg.fence_free = 1;
     if (!cfg.format_ahead) cfg.format_ahead = 1;
     if (!cfg.run_max) cfg.run_max = 256;
-    if (!cfg.run_init) cfg.run_init = (uint32_t)(nseg / 4 < 1 ? 1 : (nseg / 4 > 256 ? 256 : nseg / 4));
     if (!cfg.run_bytes) {
         cfg.run_bytes = (nseg << core::kSegLog2) / 64;
         if (cfg.run_bytes > (256ull << 20)) cfg.run_bytes = 256ull << 20;
@@ -591,6 +590,24 @@ int gallatin_init_ex(const gallatin_config_t *cfg_in) {
         uint64_t m = cfg.run_bytes >> (16 + c);
         if (m > cfg.run_max) m = cfg.run_max;
         v.run_cap[c] = m < 1 ? 1u : (uint32_t)m;
+    }
+    if (!cfg.run_init) {
+        // [dev] the largest first run (power of two <= 256 blocks) whose
+        // worst case -- every slot of every class holding a fresh first run --
+        // stays within half the heap: whole-segment first runs on big heaps,
+        // the paper's one block on small ones (DESIGN.md Deviations 5)
+        uint32_t r = 256;
+        for (; r > 1; r >>= 1) {
+            uint64_t hoard = 0;
+            for (uint32_t c = 0; c < core::kTrees; c++) {
+                const uint32_t fl = r < 8 ? r : 8u, fs = (r >> c) > fl ? (r >> c) : fl;
+                const uint32_t fr = fs < (256u >> c) ? fs : (256u >> c);
+                const uint32_t first = fr < v.run_cap[c] ? fr : v.run_cap[c];
+                hoard += (uint64_t)v.nslot[c] * first * (65536ull << c);
+            }
+            if (hoard <= (nseg << core::kSegLog2) / 2) break;
+        }
+        cfg.run_init = r;
     }
     v.format_ahead = cfg.format_ahead == 1 ? 1u : 0u;
     v.formatters = (uint32_t)(nseg / 32 < 1 ? 1 : (nseg / 32 > 32 ? 32 : nseg / 32));
