@@ -49,8 +49,11 @@ enum {
  *   slot_min   : lower cap; the paper caps at four; default
  *                clamp(nseg / 32, 4, 32) (more slots for the big classes on big heaps).
  *   run_max    : a slot holds a RUN of up to run_max consecutive blocks (1..512,
- *                default 256); the run starts at run_init blocks and doubles on
- *                every refill of the slot.  1 = the paper's one-block buffer.
+ *                default 256); the run starts at run_init blocks and grows
+ *                2^run_grow-fold on every refill of the slot.  1 = the paper's
+ *                one-block buffer.  Before a run request reports "no memory",
+ *                every slot gives back the blocks of its run no request has
+ *                drawn from, and the request is retried once.
  *   run_bytes  : and at most run_bytes per run (default min(256 MiB, heap/64)).
  *   format_ahead: 1 (default) = the reservation that leaves a segment with
  *                fewer than nb/4 blocks formats the next segment of its tree;
@@ -71,6 +74,7 @@ typedef struct gallatin_config {
     uint32_t bulk_items;   /* requests per thread in the bulk kernels: 0 = auto, 1 or 4 */
     uint32_t run_init;     /* first run of an empty slot of class c: min(max(run_init >> c, min(run_init, 8)), 256 >> c) blocks (default: the largest power of two <= 256 whose first runs over all slots fit in half the heap) */
     uint32_t prefetch;     /* 1 = fetch the next run at the middle of the current one; 0/2 = off (default) */
+    uint32_t run_grow;     /* a refilled run is 2^run_grow times the last one, up to the cap: 1..8 (default 3) */
 } gallatin_config_t;
 
 int gallatin_init(uint64_t heap_bytes);                 /* defaults for the rest */
@@ -125,6 +129,7 @@ typedef struct gallatin_stats {
     uint32_t nslot[9];           /* block-buffer slots per class                    */
     uint32_t run_cap[9];         /* max blocks per run per class                    */
     uint32_t slot_base, slot_min, run_max, format_ahead, fence_free, run_init, formatters, prefetch;
+    uint32_t run_grow;
 } gallatin_stats_t;
 int gallatin_stats(gallatin_stats_t *out);               /* synchronizes the device */
 

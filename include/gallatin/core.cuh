@@ -279,7 +279,7 @@ __device__ inline __noinline__ void format_ahead(const View &v, uint32_t t) {
 // ---- Alg. 2 GetBlock(treeId), for a RUN of blocks [dev] --------
 // Returns the number of consecutive blocks obtained (0 = exhausted) and the
 // first one's linear index (segment * nb + block) in *first.
-__device__ inline __noinline__ uint32_t get_run(const View &v, uint32_t t, uint32_t want, uint32_t *first) {
+__device__ inline __noinline__ uint32_t get_run_once(const View &v, uint32_t t, uint32_t want, uint32_t *first) {
     const BitTree bt = block_tree(v, t);
     const uint32_t nb = nb_of(t);
     ptx::Backoff bo(4, t);
@@ -410,6 +410,49 @@ constexpr uint32_t kRunNone = 0x3FFFFFu;
 constexpr uint64_t kSlotEmpty = kRunNone;                 // issued 0, run 0: refill on first use
 __device__ __forceinline__ uint32_t run_len(uint64_t w) { return (uint32_t)(w >> kRunShift) & 0x3FFu; }
 
+// [dev] Before reporting "no memory", every slot gives back the blocks of its
+// run that no request has drawn from (class-major, slot-ascending): one CAS
+// shrinks the run to ceil(issued / 4096) blocks -- issued and run share the
+// word, so a draw racing the CAS makes it fail and retry, and no draw can land
+// in a dropped block afterwards -- and the dropped blocks return whole.  A
+// prefetched next run returns entirely.  Returns the number of blocks given back.
+__device__ inline __noinline__ uint32_t trim_slots(const View &v) {
+    uint32_t back = 0;
+    for (uint32_t c = 0; c < kTrees; c++) {
+        for (uint32_t q = 0; q < v.nslot[c]; q++) {
+            uint64_t *sw = slot_word(v, v.slot_off[c] + q);
+            uint64_t w = ptx::ld_relaxed(sw);
+            for (;;) {
+                const uint64_t cnt = w >> 32;
+                const uint32_t m = run_len(w);
+                if (cnt >= ((uint64_t)m << kSliceLog2)) break;            // exhausted or empty
+                const uint32_t m2 = (uint32_t)((cnt + kSlices - 1) >> kSliceLog2);
+                const uint64_t nw = m2 == 0 ? kSlotEmpty
+                                            : (w & ~(0x3FFull << kRunShift)) | ((uint64_t)m2 << kRunShift);
+                const uint64_t o = ptx::atom_cas(sw, w, nw);
+                if (o != w) { w = o; continue; }
+                for (uint32_t k = m2; k < m; k++) block_freed(v, gid_of(c, (w & kRunNone) + k), kSlices);
+                back += m - m2;
+                break;
+            }
+            if (v.prefetch) {
+                const uint64_t nx = ptx::atom_exch(sw + 1, kSlotEmpty);
+                for (uint32_t k = 0; k < run_len(nx); k++) block_freed(v, gid_of(c, (nx & kRunNone) + k), kSlices);
+                back += run_len(nx);
+            }
+        }
+    }
+    return back;
+}
+
+// A run of up to `want` blocks of tree t (get_run_once); on "no memory" the
+// slots' undrawn blocks are given back and the request retried once.
+__device__ inline uint32_t get_run(const View &v, uint32_t t, uint32_t want, uint32_t *first) {
+    const uint32_t got = get_run_once(v, t, want, first);
+    if (got != 0 || trim_slots(v) == 0) return got;
+    return get_run_once(v, t, want, first);
+}
+
 // Replace an exhausted run (Alg.3): the run doubles up to the class cap.
 __device__ inline __noinline__ bool refill_slot(const View &v, uint32_t si, uint32_t c, uint32_t m_prev) {
     if (v.prefetch) {                                         // [dev] the prefetched run, if any
@@ -425,7 +468,8 @@ __device__ inline __noinline__ bool refill_slot(const View &v, uint32_t si, uint
     const uint32_t fs = (v.run_init >> c) > fl ? (v.run_init >> c) : fl;
     const uint32_t fr = fs < (256u >> c) ? fs : (256u >> c);
     const uint32_t first_run = fr < cap ? fr : cap;
-    const uint32_t want = m_prev == 0 ? first_run : (2 * m_prev < cap ? 2 * m_prev : cap);
+    const uint32_t grow = m_prev << v.run_grow;                   // x 2^run_grow per refill
+    const uint32_t want = m_prev == 0 ? first_run : (grow < cap ? grow : cap);
     uint32_t first = 0;
 #ifdef GALLATIN_TRACE
     const uint64_t t0 = ptx::globaltimer();
@@ -448,9 +492,10 @@ __device__ inline __noinline__ bool refill_slot(const View &v, uint32_t si, uint
 __device__ inline __noinline__ void prefetch_slot(const View &v, uint32_t si, uint32_t c, uint32_t m) {
     if (ptx::ld_relaxed(slot_word(v, si) + 1) != kSlotEmpty) return;   // a run is already waiting
     const uint32_t cap = v.run_cap[c];
-    const uint32_t want = 2 * m < cap ? 2 * m : cap;
+    const uint32_t grow = m << v.run_grow;
+    const uint32_t want = grow < cap ? grow : cap;
     uint32_t first = 0;
-    const uint32_t got = get_run(v, c, want, &first);
+    const uint32_t got = get_run_once(v, c, want, &first);         // never trims other slots
     if (got == 0) return;
     const uint64_t run = ((uint64_t)got << kRunShift) | first;
     if (ptx::atom_cas(slot_word(v, si) + 1, kSlotEmpty, run) != kSlotEmpty)
@@ -544,9 +589,14 @@ __device__ inline __noinline__ void *malloc_large(const View &v, uint64_t k) {
     ptx::Backoff bo(5, k);
     uint64_t i;
     int misses = 0;
+    bool trimmed = false;
     for (;;) {
         i = bt_find_highest_run(st, k);
         if (i == kNone) {
+            if (!trimmed) {                                   // [dev] as get_run: slots give back first
+                trimmed = true;
+                if (trim_slots(v)) continue;
+            }
             if (++misses > 2) return nullptr;
             bo.pause();
             continue;

@@ -56,7 +56,7 @@ struct gallatin_device_view {
     uint32_t formatters;        /* concurrent segment formatters per tree      */
     uint32_t run_init;          /* run length of an empty slot's first refill  */
     uint32_t prefetch;          /* 1 = fetch the next run at the run's middle  */
-    uint32_t pad;
+    uint32_t run_grow;          /* log2 of the run growth factor per refill    */
 };
 typedef struct gallatin_device_view gallatin_device_view_t;
 

@@ -77,7 +77,8 @@ def lib() -> ctypes.CDLL:
             "oracle_veb_batch": ([vp, i32, vp, u64, vp], None),
             "oracle_veb_image": ([vp, vp, u64], u64),
             "oracle_veb_image_levels": ([ctypes.c_uint, vp], ctypes.c_uint),
-            "o2_create": ([u64, ctypes.c_uint, ctypes.c_uint, ctypes.c_uint, u64, ctypes.c_uint, ctypes.c_uint, ctypes.c_uint], vp),
+            "o2_create": ([u64, ctypes.c_uint, ctypes.c_uint, ctypes.c_uint, u64, ctypes.c_uint, ctypes.c_uint, ctypes.c_uint,
+                           ctypes.c_uint], vp),
             "o2_destroy": ([vp], None),
             "o2_nslot": ([vp, ctypes.c_uint], ctypes.c_uint),
             "o2_errors": ([vp], u64),
@@ -179,11 +180,14 @@ class Allocator:
     """
 
     def __init__(self, nseg: int, slot_base: int = 148, slot_min: int = 4, run_max: int = 1,
-                 run_bytes: int = 64 << 20, format_ahead: int = 0, run_init: int = 1, prefetch: int = 0):
-        """run_max=1, run_init=1, format_ahead=0, prefetch=0 is the paper's one-block buffer."""
+                 run_bytes: int = 64 << 20, format_ahead: int = 0, run_init: int = 1, prefetch: int = 0,
+                 run_grow: int = 1):
+        """run_max=1, run_init=1, format_ahead=0, prefetch=0 is the paper's one-block buffer (P:195);
+        run_grow = log2 of the run growth per refill (DESIGN.md Deviations 5)."""
         self._h = None
         self.nseg = nseg
-        self._h = lib().o2_create(nseg, slot_base, slot_min, run_max, run_bytes, format_ahead, run_init, prefetch)
+        self._h = lib().o2_create(nseg, slot_base, slot_min, run_max, run_bytes, format_ahead, run_init, prefetch,
+                                  run_grow)
         if not self._h:
             raise ValueError("bad allocator parameters")
 

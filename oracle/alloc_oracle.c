@@ -102,6 +102,7 @@ typedef struct o2 {
     uint64_t *slot;               /* cnt << 32 | m << 22 | first block  */
     uint64_t *next;               /* prefetched run (m << 22 | first) or empty */
     unsigned prefetch;
+    unsigned run_grow;            /* a refill takes m << run_grow blocks        */
     uint64_t err;                 /* out-of-heap / non-allocated segment frees */
     /* oracle-only bookkeeping for the invariant checks */
     kv_t *live; uint64_t live_cap, live_n;
@@ -163,13 +164,16 @@ static uint64_t slot_make(uint64_t cnt, uint32_t m, uint32_t first) {
 }
 
 o2_t *o2_create(uint64_t nseg, unsigned slot_base, unsigned slot_min, unsigned run_max,
-                uint64_t run_bytes, unsigned format_ahead, unsigned run_init, unsigned prefetch) {
+                uint64_t run_bytes, unsigned format_ahead, unsigned run_init, unsigned prefetch,
+                unsigned run_grow) {
+    if (run_grow < 1 || run_grow > 8) return NULL;
     if (nseg < 1 || nseg > (1ULL << 14) || slot_base < 1 || run_max < 1 || run_max > 512) return NULL;
     o2_t *a = (o2_t *)calloc(1, sizeof(o2_t));
     a->nseg = nseg; a->slot_base = slot_base; a->slot_min = slot_min;
     a->run_max = run_max; a->run_bytes = run_bytes; a->format_ahead = format_ahead;
     a->run_init = run_init < 1 ? 1 : run_init;
     a->prefetch = prefetch;
+    a->run_grow = run_grow;
     unsigned off = 0;
     for (unsigned c = 0; c < NUM_BLOCK_TREES; c++) {
         unsigned n = slot_base >> c;                  /* halving per class */
@@ -301,11 +305,16 @@ static void block_freed(o2_t *a, uint32_t gid, uint32_t count) {
     }
 }
 
+static uint32_t gid_of(uint32_t t, uint64_t linear) {
+    uint32_t nb = nb_of(t);
+    return (uint32_t)((linear / nb) * MAX_BLOCKS_PER_SEGMENT + linear % nb);
+}
+
 /* --------------------------------------------------- Alg.2 getBlock --- */
 /* A run of up to `want` consecutive blocks of tree t.  Returns the number of
  * blocks (0 = no memory) and the first block's linear index in *first
  * (segment * nb + block). */
-static uint32_t get_run(o2_t *a, uint32_t t, uint32_t want, uint32_t *first) {
+static uint32_t get_run_once(o2_t *a, uint32_t t, uint32_t want, uint32_t *first) {
     uint32_t nb = nb_of(t);
     uint64_t s = oracle_veb_successor(a->btree[t], 0);     /* findSegment */
     if (s != NONE64) {
@@ -349,9 +358,44 @@ static uint32_t get_run(o2_t *a, uint32_t t, uint32_t want, uint32_t *first) {
     return want;
 }
 
-static uint32_t gid_of(uint32_t t, uint64_t linear) {
-    uint32_t nb = nb_of(t);
-    return (uint32_t)((linear / nb) * MAX_BLOCKS_PER_SEGMENT + linear % nb);
+
+/* [ours, DESIGN.md Deviations 5] Before "no memory": every slot, class-major
+ * and slot-ascending, keeps only the ceil(issued / 4096) blocks of its run that
+ * requests have drawn from (an undrawn slot becomes empty); the other blocks
+ * come back whole, in block order, then a prefetched next run comes back
+ * whole.  Returns the number of blocks given back. */
+static uint64_t trim_slots(o2_t *a) {
+    uint64_t back = 0;
+    for (unsigned c = 0; c < NUM_BLOCK_TREES; c++) {
+        for (unsigned q = 0; q < a->nslot[c]; q++) {
+            unsigned i = a->slot_off[c] + q;
+            uint64_t cnt = a->slot[i] >> 32;
+            uint32_t m = (uint32_t)(a->slot[i] >> RUN_SHIFT) & 0x3FF;
+            uint32_t first = (uint32_t)a->slot[i] & RUN_NONE;
+            if (cnt < SLICES_PER_BLOCK * (uint64_t)m) {
+                uint32_t m2 = (uint32_t)((cnt + SLICES_PER_BLOCK - 1) / SLICES_PER_BLOCK);
+                a->slot[i] = m2 == 0 ? SLOT_EMPTY : slot_make(cnt, m2, first);
+                for (uint32_t k = m2; k < m; k++) block_freed(a, gid_of(c, (uint64_t)first + k), SLICES_PER_BLOCK);
+                back += m - m2;
+            }
+            if (a->prefetch) {
+                uint32_t nm = (uint32_t)(a->next[i] >> RUN_SHIFT) & 0x3FF;
+                uint32_t nf = (uint32_t)a->next[i] & RUN_NONE;
+                a->next[i] = SLOT_EMPTY;
+                for (uint32_t k = 0; k < nm; k++) block_freed(a, gid_of(c, (uint64_t)nf + k), SLICES_PER_BLOCK);
+                back += nm;
+            }
+        }
+    }
+    return back;
+}
+
+/* A run of up to `want` blocks (get_run_once); on "no memory" the slots give
+ * back their undrawn blocks and the request is retried once. */
+static uint32_t get_run(o2_t *a, uint32_t t, uint32_t want, uint32_t *first) {
+    uint32_t got = get_run_once(a, t, want, first);
+    if (got || !trim_slots(a)) return got;
+    return get_run_once(a, t, want, first);
 }
 
 /* ------------------------------------------ claimMultiple (back) --- */
@@ -398,13 +442,13 @@ static uint64_t malloc_slice(o2_t *a, uint32_t c, uint64_t key) {
         uint32_t m = (uint32_t)(a->slot[i] >> RUN_SHIFT) & 0x3FF;
         uint32_t first = (uint32_t)a->slot[i] & RUN_NONE;
         uint32_t cap = run_cap(a, c);
-        uint32_t grow = 2 * m < cap ? 2 * m : cap;
+        uint32_t grow = (m << a->run_grow) < cap ? (m << a->run_grow) : cap;   /* [ours] x 2^run_grow */
         if (cnt < SLICES_PER_BLOCK * m) {                   /* valid = idx < 4096 (per block) */
             a->slot[i] = slot_make(cnt + 1, m, first);
             uint64_t off = slice_addr(first, c, cnt);
             if (a->prefetch && cnt == SLICES_PER_BLOCK * m / 2 && a->next[i] == SLOT_EMPTY) {
                 uint32_t nf;                                  /* [ours] prefetch the next run */
-                uint32_t ng = get_run(a, c, grow, &nf);
+                uint32_t ng = get_run_once(a, c, grow, &nf);   /* never trims other slots */
                 if (ng) a->next[i] = slot_make(0, ng, nf);
             }
             return off;
@@ -466,6 +510,7 @@ uint64_t o2_malloc(o2_t *a, uint64_t size, uint64_t key) {
         off = (uint64_t)first * block_bytes(cls);
     } else {
         uint64_t i = claim_multiple(a, cls);
+        if (i == NONE64 && trim_slots(a)) i = claim_multiple(a, cls);   /* [ours] as get_run */
         if (i == NONE64) return NONE64;
         off = i * SEGMENT_BYTES;
     }

@@ -29,7 +29,7 @@ class Config(ctypes.Structure):
     _fields_ = [("heap_bytes", ctypes.c_uint64), ("run_bytes", ctypes.c_uint64), ("slot_base", ctypes.c_uint32),
                 ("slot_min", ctypes.c_uint32), ("run_max", ctypes.c_uint32), ("format_ahead", ctypes.c_uint32),
                 ("fence_free", ctypes.c_uint32), ("bulk_items", ctypes.c_uint32), ("run_init", ctypes.c_uint32),
-                ("prefetch", ctypes.c_uint32)]
+                ("prefetch", ctypes.c_uint32), ("run_grow", ctypes.c_uint32)]
 
 
 class Stats(ctypes.Structure):
@@ -39,7 +39,7 @@ class Stats(ctypes.Structure):
                 ("nslot", ctypes.c_uint32 * 9), ("run_cap", ctypes.c_uint32 * 9), ("slot_base", ctypes.c_uint32),
                 ("slot_min", ctypes.c_uint32), ("run_max", ctypes.c_uint32), ("format_ahead", ctypes.c_uint32),
                 ("fence_free", ctypes.c_uint32), ("run_init", ctypes.c_uint32), ("formatters", ctypes.c_uint32),
-                ("prefetch", ctypes.c_uint32)]
+                ("prefetch", ctypes.c_uint32), ("run_grow", ctypes.c_uint32)]
 
 
 def declared_functions() -> list[str]:
@@ -149,11 +149,11 @@ def _empty64(n: int):
 # ------------------------------------------------------------- allocator ---
 def gallatin_init(heap_bytes: int, slot_base: int = 0, slot_min: int = 0, run_max: int = 0, run_bytes: int = 0,
                   format_ahead: int = 0, fence_free: int = 0, bulk_items: int = 0, run_init: int = 0,
-                  prefetch: int = 0) -> None:
+                  prefetch: int = 0, run_grow: int = 0) -> None:
     """0 = library default for every knob (include/gallatin.h gallatin_config_t)."""
     cfg = Config(heap_bytes=heap_bytes, run_bytes=run_bytes, slot_base=slot_base, slot_min=slot_min,
                  run_max=run_max, format_ahead=format_ahead, fence_free=fence_free, bulk_items=bulk_items,
-                 run_init=run_init, prefetch=prefetch)
+                 run_init=run_init, prefetch=prefetch, run_grow=run_grow)
     check(lib().gallatin_init_ex(ctypes.byref(cfg)), "gallatin_init")
 
 
@@ -214,7 +214,7 @@ def gallatin_stats() -> dict:
             "large_segments": s.large_segments, "errors": s.errors, "nslot": list(s.nslot),
             "run_cap": list(s.run_cap), "run_bytes": s.run_bytes, "slot_base": s.slot_base, "slot_min": s.slot_min,
             "run_max": s.run_max, "format_ahead": s.format_ahead, "fence_free": s.fence_free,
-            "run_init": s.run_init, "formatters": s.formatters, "prefetch": s.prefetch}
+            "run_init": s.run_init, "formatters": s.formatters, "prefetch": s.prefetch, "run_grow": s.run_grow}
 
 
 def oracle_params() -> dict:
@@ -222,7 +222,7 @@ def oracle_params() -> dict:
     st = gallatin_stats()
     return {"slot_base": st["slot_base"], "slot_min": st["slot_min"], "run_max": st["run_max"],
             "run_bytes": st["run_bytes"], "format_ahead": 1 if st["format_ahead"] == 1 else 0,
-            "run_init": st["run_init"], "prefetch": st["prefetch"]}
+            "run_init": st["run_init"], "prefetch": st["prefetch"], "run_grow": st["run_grow"]}
 
 
 def gallatin_snapshot() -> np.ndarray:

@@ -568,6 +568,8 @@ int gallatin_init_ex(const gallatin_config_t *cfg_in) {
     if (cfg.run_max > core::kMaxRun || cfg.fence_free > 2 || cfg.format_ahead > 2) return GALLATIN_ERR_INVALID;
     if (cfg.bulk_items != 0 && cfg.bulk_items != 1 && cfg.bulk_items != 4) return GALLATIN_ERR_INVALID;
     if (cfg.prefetch > 2) return GALLATIN_ERR_INVALID;
+    if (!cfg.run_grow) cfg.run_grow = 3;
+    if (cfg.run_grow > 8) return GALLATIN_ERR_INVALID;
     if (nseg > (1ull << 14)) return GALLATIN_ERR_INVALID;        // 22-bit run index at 64 KB blocks (256 GiB)
 
     View v{};
@@ -612,6 +614,7 @@ int gallatin_init_ex(const gallatin_config_t *cfg_in) {
     v.format_ahead = cfg.format_ahead == 1 ? 1u : 0u;
     v.formatters = (uint32_t)(nseg / 32 < 1 ? 1 : (nseg / 32 > 32 ? 32 : nseg / 32));
     v.run_init = cfg.run_init;
+    v.run_grow = cfg.run_grow;
     v.prefetch = cfg.prefetch == 1 ? 1u : 0u;              // default off (measured: DESIGN.md)
     v.fence_free = cfg.fence_free;
 
@@ -838,6 +841,7 @@ int gallatin_stats(gallatin_stats_t *out) {
     out->format_ahead = g.cfg.format_ahead;
     out->fence_free = v.fence_free;
     out->run_init = v.run_init;
+    out->run_grow = v.run_grow;
     out->formatters = v.formatters;
     out->prefetch = v.prefetch;
     return GALLATIN_OK;

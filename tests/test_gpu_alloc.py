@@ -38,11 +38,11 @@ def G():
 
 
 def _replay_case(G, nseg, run_max, fa, kinds, args, keys, slot_base=16, slot_min=2, run_bytes=32 << 20, pf=None,
-                 run_init=1):
+                 run_init=1, run_grow=0):
     if pf is None:
         pf = run_max > 1                    # the paper's policy (run_max=1) has no prefetch
     G.gallatin_init(nseg * SEG, slot_base=slot_base, slot_min=slot_min, run_max=run_max, run_bytes=run_bytes,
-                    format_ahead=1 if fa else 2, prefetch=1 if pf else 2, run_init=run_init)
+                    format_ahead=1 if fa else 2, prefetch=1 if pf else 2, run_init=run_init, run_grow=run_grow)
     out = _u64(G.gallatin_replay(_dev(kinds, np.uint8), _dev(args), _dev(keys)))
     o2 = oracle.Allocator(nseg, **G.oracle_params())
     want = o2.replay(kinds, args, keys)
@@ -75,17 +75,22 @@ def test_serialized_replay_block_boundaries(cuda_ok, G):
     kinds2 = np.concatenate([kinds, np.ones(4096, dtype=np.uint8), np.array([2], dtype=np.uint8)])
     args2 = np.concatenate([args, np.arange(4096, dtype=np.uint64), np.array([0], dtype=np.uint64)])
     keys2 = np.concatenate([keys, np.zeros(4097, dtype=np.uint64)])
-    for run_max, fa, pf, ri in ((1, 0, 0, 1), (4, 1, 0, 1), (128, 1, 1, 1), (512, 1, 1, 8), (16, 0, 1, 4)):
-        _replay_case(G, 2, run_max, fa, kinds2, args2, keys2, slot_base=1, slot_min=1, pf=pf, run_init=ri)
+    for run_max, fa, pf, ri, rg in ((1, 0, 0, 1, 1), (4, 1, 0, 1, 1), (128, 1, 1, 1, 3), (512, 1, 1, 8, 2),
+                                    (16, 0, 1, 4, 8), (256, 1, 0, 256, 3)):
+        _replay_case(G, 2, run_max, fa, kinds2, args2, keys2, slot_base=1, slot_min=1, pf=pf, run_init=ri,
+                     run_grow=rg)
 
 
-@pytest.mark.parametrize("seed,nseg,run_max,fa,pf,ri", [(11, 8, 64, 1, 1, 4), (12, 48, 512, 1, 1, 8),
-                                                        (13, 6, 16, 0, 1, 2), (14, 12, 256, 1, 0, 1)])
-def test_serialized_replay_runs_prefetch_matrix(cuda_ok, G, seed, nseg, run_max, fa, pf, ri):
-    """The run / prefetch / run_init / format-ahead knobs (DESIGN.md Deviations
-    5) against O2 modelling the same policy, with OOM and drains."""
+@pytest.mark.parametrize("seed,nseg,run_max,fa,pf,ri,rg", [(11, 8, 64, 1, 1, 4, 1), (12, 48, 512, 1, 1, 8, 3),
+                                                           (13, 6, 16, 0, 1, 2, 2), (14, 12, 256, 1, 0, 1, 3),
+                                                           (15, 4, 256, 1, 0, 256, 3), (16, 6, 256, 0, 1, 64, 8),
+                                                           (17, 3, 512, 1, 1, 256, 4)])
+def test_serialized_replay_runs_prefetch_matrix(cuda_ok, G, seed, nseg, run_max, fa, pf, ri, rg):
+    """The run / prefetch / run_init / run_grow / format-ahead knobs (DESIGN.md
+    Deviations 5) against O2 modelling the same policy, with OOM and drains;
+    the whole-segment first runs on 3-6 segment heaps force slot trims."""
     kinds, args, keys = wg.replay_ops(6000, seed + 100, p_free=0.45, p_drain=0.003, nkeys=64)
-    _replay_case(G, nseg, run_max, fa, kinds, args, keys, pf=pf, run_init=ri)
+    _replay_case(G, nseg, run_max, fa, kinds, args, keys, pf=pf, run_init=ri, run_grow=rg)
 
 
 def _bulk_round(G, nseg, sizes, check_accounting=True):

@@ -153,3 +153,49 @@ def test_errors_counted_for_foreign_frees():
     a.free(SEG + 16)           # a FREE segment
     a.free(NONE)               # NULL: no-op
     assert a.errors == 2
+
+
+def test_trim_gives_back_undrawn_blocks_before_oom():
+    """DESIGN.md Deviations 5 (runs) + Alg.2's "no allocations left":
+    a slot's whole-segment run must not starve another request.  On a
+    one-segment heap the 16 B slot's first run takes all 256 blocks; a 64 KB
+    block request then finds no segment, the slot keeps the ceil(1/4096) = 1
+    block it has drawn from and gives back blocks 1..255 in order (FIFO ring,
+    P:178), so the request gets block 1 at 64 KB, the next ones blocks 2..255,
+    and only then NULL -- closed forms from the paper's layout."""
+    a = oracle.Allocator(1, slot_base=1, slot_min=1, run_max=256, run_bytes=16 << 20, run_init=256, run_grow=3)
+    assert a.malloc(16, 0) == 0
+    d = image_sections(a.image())
+    assert int(d["segword"][0]) & 0xFFFFFFFF == 0                 # all 256 blocks held by the run
+    blocks = [a.malloc(65536, 0) for _ in range(255)]
+    assert blocks == [j * 65536 for j in range(1, 256)]
+    assert a.malloc(16, 0) == 16                                   # the kept block still serves the slot
+    assert a.malloc(65536, 0) == NONE                              # nothing left to give back
+    d = image_sections(a.image())
+    assert int(d["slots"][0]) >> 32 == 2 and (int(d["slots"][0]) >> 22) & 0x3FF == 1
+    for off in [0, 16] + blocks:
+        a.free(off)
+    a.drain()
+    img = a.image()
+    assert a.check() == 0
+    assert np.array_equal(img, pristine_image(1, int(img[4])))
+
+
+@pytest.mark.parametrize("run_grow", [1, 2, 3, 8])
+def test_run_growth_factor(run_grow):
+    """A refilled run is 2^run_grow times the last (capped): with one 16 B slot
+    and first run 1 block, the k-th run starts right after the (k-1)-th, so the
+    addresses stay consecutive and the slot's run length after
+    r refills is min(2^(run_grow*r), cap) -- the closed form, read from the
+    image's slot word."""
+    cap = 64
+    a = oracle.Allocator(4, slot_base=1, slot_min=1, run_max=cap, run_bytes=64 << 20, run_init=1, run_grow=run_grow)
+    m, total = 1, 0
+    for r in range(4):
+        total += m * 4096
+        offs = a.malloc_batch(np.full(m * 4096 if r else 4096, 16, dtype=np.uint64), keydiv=0)
+        assert offs[-1] == (total - 1) * 16
+        d = image_sections(a.image())
+        assert (int(d["slots"][0]) >> 22) & 0x3FF == m
+        m = min(m << run_grow, cap)
+    assert a.check() == 0
