@@ -71,7 +71,7 @@ typedef struct gallatin_config {
     uint32_t run_max;
     uint32_t format_ahead;
     uint32_t fence_free;
-    uint32_t bulk_items;   /* requests per thread in the bulk kernels: 0 = auto, 1 or 4 */
+    uint32_t bulk_items;   /* requests per thread in the bulk malloc kernel: 0 = auto, 1, 4, 8 or 16 (free: 1 or 4) */
     uint32_t run_init;     /* first run of an empty slot of class c: min(max(run_init >> c, min(run_init, 8)), 256 >> c) blocks (default: the largest power of two <= 256 whose first runs over all slots fit in half the heap) */
     uint32_t prefetch;     /* 1 = fetch the next run at the middle of the current one; 0/2 = off (default) */
     uint32_t run_grow;     /* a refilled run is 2^run_grow times the last one, up to the cap: 1..8 (default 3) */

@@ -133,17 +133,34 @@ __device__ inline __noinline__ uint32_t reclaim_idle(const View &v) {
     return n;
 }
 
+// [dev] A claimer that lost the race for a bit of leaf word `old` retries at a
+// pseudo-random free bit of that same word (seeded by the thread and the
+// attempt) instead of the next one up: k simultaneous claimers -- every slot
+// refilling at a launch's start -- then collide O(1) times each instead of
+// walking the word one loss at a time.  kNone if the word had no free bit.
+__device__ __forceinline__ uint64_t claim_retry_hint(uint64_t wi, uint64_t old, uint32_t attempt) {
+    if (old == 0) return kNone;
+    const uint32_t tid = blockIdx.x * blockDim.x + threadIdx.x;
+    uint32_t h = (tid * 0x9E3779B1u) ^ (attempt * 0x85EBCA6Bu);
+    h ^= h >> 15;
+    uint32_t r = h % (uint32_t)__popcll((long long)old);
+    uint64_t m = old;
+    for (; r; r--) m &= m - 1;                                // drop r lowest free bits
+    return (wi << 6) + (uint64_t)(__ffsll((long long)m) - 1);
+}
+
 // ---- Alg. 1 GetSegment(treeId < numBlockTrees) ----------------
 // successor(0) on the segment tree + claimIndex, front first
 // (P:138).  Returns the claimed segment or kNone when every segment is in use.
-// A claimer that loses the race for segment s moves on to successor(s + 1)
-// instead of re-reading from 0, so k concurrent claimers spread over the k
-// lowest free segments in O(k) total RMWs (serially this is successor(0)).
+// A claimer that loses the race retries elsewhere (claim_retry_hint; serially
+// the first attempt always wins, so this is successor(0)).
 __device__ inline __noinline__ uint64_t claim_front(const View &v) {
     const BitTree st = seg_tree(v);
-    uint64_t from = 0;
+    uint64_t from = 0, hint = kNone;
+    uint32_t attempt = 0;
     for (;;) {
-        uint64_t s = bt_successor<false>(st, from);
+        uint64_t s = hint != kNone ? hint : bt_successor<false>(st, from);
+        hint = kNone;
         if (s == kNone) {
             if (from != 0) { from = 0; continue; }
             s = bt_scan_first(st);                         // confirm before failing
@@ -153,11 +170,16 @@ __device__ inline __noinline__ uint64_t claim_front(const View &v) {
                 continue;
             }
         }
-        if (bt_delete(st, s)) {
+        uint64_t *leaf = st.w + st.off[0] + (s >> 6);
+        const uint64_t bit = 1ull << (s & 63);
+        const uint64_t old = ptx::atom_and(leaf, ~bit);
+        if (old & bit) {
+            if (old == bit) bt_reconcile_up(st, 0, s >> 6);       // the word emptied
             ptx::fence_acq_rel();
             return s;
         }
-        from = s + 1;
+        hint = claim_retry_hint(s >> 6, old, ++attempt);
+        from = ((s >> 6) + 1) << 6;
     }
 }
 
@@ -169,9 +191,11 @@ __device__ inline __noinline__ uint64_t claim_front(const View &v) {
 // (serially: s = successor(0) and the free segments that follow it).
 __device__ inline __noinline__ uint64_t claim_front_run(const View &v, uint32_t kmax, uint32_t *k) {
     const BitTree st = seg_tree(v);
-    uint64_t from = 0;
+    uint64_t from = 0, hint = kNone;
+    uint32_t attempt = 0;
     for (;;) {
-        uint64_t s = bt_successor<false>(st, from);
+        uint64_t s = hint != kNone ? hint : bt_successor<false>(st, from);
+        hint = kNone;
         if (s == kNone) {
             if (from != 0) { from = 0; continue; }
             s = bt_scan_first(st);
@@ -194,7 +218,11 @@ __device__ inline __noinline__ uint64_t claim_front_run(const View &v, uint32_t 
         bool flip = old != 0 && (old & ~mask) == 0;
         if (extra) flip |= ptx::atom_or(leaf, extra) == 0;
         if (flip) bt_reconcile_up(st, 0, wi);
-        if (run == 0) { from = s + 1; continue; }
+        if (run == 0) {
+            hint = claim_retry_hint(wi, old & ~mask, ++attempt);
+            from = (wi + 1) << 6;
+            continue;
+        }
         ptx::fence_acq_rel();
         *k = run;
         return s;
@@ -276,6 +304,45 @@ __device__ inline __noinline__ void format_ahead(const View &v, uint32_t t) {
     token_release(tok);
 }
 
+// [dev] A run covering whole segments takes up to want/nb fresh segments
+// privately (no ring, no block tree): the lowest free one and the free ones
+// that follow it.  Returns the blocks taken (0 if no segment is free).
+__device__ inline __noinline__ uint32_t take_segments(const View &v, uint32_t t, uint32_t want, uint32_t *first) {
+    const uint32_t nb = nb_of(t);
+    uint32_t k = 0;
+    const uint32_t kmax = want / nb;
+    const uint64_t s0 = claim_front_run(v, kmax, &k);
+    if (s0 == kNone) return 0;
+    const BitTree st = seg_tree(v);
+    // extend with the following free segments: one atomicAnd per leaf
+    // word claims the whole window, the consecutive prefix is kept and
+    // the rest given back (serially: the next free segments in order)
+    while (k < kmax && s0 + k < v.nseg && ((s0 + k) & 63) == 0) {
+        const uint64_t x = s0 + k, wi = x >> 6;
+        const uint32_t lo = (uint32_t)(x & 63);
+        uint64_t hi = lo + (uint64_t)(kmax - k);
+        if (hi > 64) hi = 64;
+        if ((wi << 6) + hi > v.nseg) hi = v.nseg - (wi << 6);
+        const uint64_t mask = bit_range(lo, (uint32_t)hi);
+        uint64_t *leaf = st.w + st.off[0] + wi;
+        const uint64_t old = ptx::atom_and(leaf, ~mask);
+        const uint64_t got = old & mask;
+        const uint32_t run = (uint32_t)__ffsll((long long)~(got >> lo)) - 1;   // prefix length
+        const uint64_t extra = got & ~bit_range(lo, lo + run);
+        bool flip = old != 0 && (old & ~mask) == 0;
+        if (extra) flip |= ptx::atom_or(leaf, extra) == 0;
+        if (flip) bt_reconcile_up(st, 0, wi);
+        k += run;
+        if (lo + run < hi) break;                         // the free run ended here
+    }
+    for (uint32_t q = 0; q < k; q++) ptx::st_relaxed(v.seg_tid + s0 + q, t);
+    ptx::fence_acq_rel();
+    for (uint32_t q = 0; q < k; q++) ptx::atom_add(v.seg_word + s0 + q, sw_retree(kTreeFree, t));
+    ptx::fence_acq_rel();
+    *first = (uint32_t)(s0 * nb);
+    return k * nb;
+}
+
 // ---- Alg. 2 GetBlock(treeId), for a RUN of blocks [dev] --------
 // Returns the number of consecutive blocks obtained (0 = exhausted) and the
 // first one's linear index (segment * nb + block) in *first.
@@ -305,8 +372,7 @@ __device__ inline __noinline__ uint32_t get_run_once(const View &v, uint32_t t, 
                 // getBlock from the segment's ring queue
                 const uint32_t pos = atomicAdd(v.q_head + s, got);
                 uint16_t *ring = v.q_entries + s * kMaxBlocks;
-                uint16_t e[kMaxRun];
-                uint32_t p = 1;
+                uint64_t bm[4] = {0, 0, 0, 0};                   // the dequeued blocks (nb <= 256)
                 // 16 independent loads in flight per batch (not one round trip per entry)
                 for (uint32_t b = 0; b < got; b += 16) {
                     uint16_t r[16];
@@ -325,14 +391,38 @@ __device__ inline __noinline__ uint32_t get_run_once(const View &v, uint32_t t, 
                             j = ptx::ld_relaxed(ep);
                         }
                         ptx::st_relaxed(ep, kRingEmpty);
-                        e[q] = j;
-                        if (q == p && j == e[0] + q) p++;      // consecutive prefix
+                        bm[j >> 6] |= 1ull << (j & 63);
                     }
                 }
                 ptx::fence_acq_rel();
-                for (uint32_t q = p; q < got; q++) return_block(v, (uint32_t)(s * kMaxBlocks + e[q]));
-                *first = (uint32_t)(s * nb + e[0]);
-                return p;
+                // [dev] keep the longest run of consecutive blocks among them
+                // (lowest start on ties): blocks come back in free order, so
+                // the FIFO prefix alone would shrink runs to a block or two
+                uint32_t bs = 0, bl = 0;
+                for (uint32_t j = 0, len = 0; j <= nb; j++) {
+                    if (j < nb && ((bm[j >> 6] >> (j & 63)) & 1)) { len++; continue; }
+                    if (len > bl) { bl = len; bs = j - len; }
+                    len = 0;
+                }
+                for (uint32_t j = bs; j < bs + bl; j++) bm[j >> 6] &= ~(1ull << (j & 63));
+                if (bl < got) {                                   // the rest goes back, ascending: one enqueue
+                    const uint32_t r = got - bl;
+                    const uint32_t tp = atomicAdd(v.q_tail + s, r);
+                    uint32_t q = 0;
+                    for (uint32_t wv = 0; wv < 4; wv++) {
+                        for (uint64_t w = bm[wv]; w; w &= w - 1, q++) {
+                            uint16_t *ep = ring + ((tp + q) & (kMaxBlocks - 1));
+                            ptx::Backoff wb(3, (s << 32) | ((tp + q) & 0xFFFFFFFFu));
+                            while (ptx::ld_relaxed(ep) != kRingEmpty) wb.pause();   // previous lap's dequeue
+                            ptx::st_relaxed(ep, (uint16_t)(wv * 64 + __ffsll((long long)w) - 1));
+                        }
+                    }
+                    ptx::fence_acq_rel();
+                    const uint64_t o3 = ptx::atom_add(v.seg_word + s, (uint64_t)r);
+                    seg_after_rmw(v, s, o3, o3 + r);
+                }
+                *first = (uint32_t)(s * nb + bs);
+                return bl;
             }
             // stale hint (P:158-161's failure case): undo, repair, look further
             seg_after_rmw(v, s, old, old + dec);
@@ -347,41 +437,7 @@ __device__ inline __noinline__ uint32_t get_run_once(const View &v, uint32_t t, 
             bo.pause();
             continue;
         }
-        if (want >= nb) {
-            // the run covers whole segments: take fresh ones privately [dev]
-            uint32_t k = 0;
-            const uint32_t kmax = want / nb;
-            const uint64_t s0 = claim_front_run(v, kmax, &k);
-            if (s0 == kNone) return 0;                        // "No allocations left"
-            const BitTree st = seg_tree(v);
-            // extend with the following free segments: one atomicAnd per leaf
-            // word claims the whole window, the consecutive prefix is kept and
-            // the rest given back (serially: the next free segments in order)
-            while (k < kmax && s0 + k < v.nseg && ((s0 + k) & 63) == 0) {
-                const uint64_t x = s0 + k, wi = x >> 6;
-                const uint32_t lo = (uint32_t)(x & 63);
-                uint64_t hi = lo + (uint64_t)(kmax - k);
-                if (hi > 64) hi = 64;
-                if ((wi << 6) + hi > v.nseg) hi = v.nseg - (wi << 6);
-                const uint64_t mask = bit_range(lo, (uint32_t)hi);
-                uint64_t *leaf = st.w + st.off[0] + wi;
-                const uint64_t old = ptx::atom_and(leaf, ~mask);
-                const uint64_t got = old & mask;
-                const uint32_t run = (uint32_t)__ffsll((long long)~(got >> lo)) - 1;   // prefix length
-                const uint64_t extra = got & ~bit_range(lo, lo + run);
-                bool flip = old != 0 && (old & ~mask) == 0;
-                if (extra) flip |= ptx::atom_or(leaf, extra) == 0;
-                if (flip) bt_reconcile_up(st, 0, wi);
-                k += run;
-                if (lo + run < hi) break;                         // the free run ended here
-            }
-            for (uint32_t q = 0; q < k; q++) ptx::st_relaxed(v.seg_tid + s0 + q, t);
-            ptx::fence_acq_rel();
-            for (uint32_t q = 0; q < k; q++) ptx::atom_add(v.seg_word + s0 + q, sw_retree(kTreeFree, t));
-            ptx::fence_acq_rel();
-            *first = (uint32_t)(s0 * nb);
-            return k * nb;
-        }
+        if (want >= nb) return take_segments(v, t, want, first);   // 0: "No allocations left"
         // Alg.2: format a segment; [dev] bounded formatters per tree
         uint32_t *tok = v.fmt_token + t * 32;
         if (token_try(tok, v.formatters)) {

@@ -27,13 +27,15 @@
  *     (Alg.3, reading A-7).
  *   - [ours, DESIGN.md "Deviations"] a slot holds a RUN of m consecutive
  *     blocks (a contiguous address range) handed out slice by slice in order;
- *     m starts at 1 and doubles on each refill of the slot up to a cap.  With
- *     cap 1 and format_ahead off this is exactly the paper's one-block buffer.
- *     A run comes from the lowest segment of the block tree (up to m of its
- *     ring entries, keeping the longest consecutive prefix and re-enqueueing
- *     the rest), else from fresh segments: when m covers whole segments the
- *     run takes them privately (no ring, no block tree), otherwise one segment
- *     is formatted with the run's blocks removed and the rest published.
+ *     m starts at run_init-derived length and grows 2^run_grow-fold on each
+ *     refill of the slot up to a cap.  With cap 1 and format_ahead off this is
+ *     exactly the paper's one-block buffer.  A run comes from the lowest
+ *     segment of the block tree (up to m of its ring entries, keeping the
+ *     longest run of consecutive block indices among them and re-enqueueing
+ *     the rest in ascending order), else from fresh segments (privately when
+ *     m covers whole segments, else one segment is formatted with the run's
+ *     blocks removed and the rest published).  Before "no memory", every slot
+ *     gives back the blocks of its run no request has drawn from.
  *     format_ahead: the reservation that takes a segment below nb/4 available
  *     blocks formats one more segment for the tree.
  *   - requests in (4 KB, 16 MB): one whole block of tree max(0, ceil(log2
@@ -305,6 +307,23 @@ static void block_freed(o2_t *a, uint32_t gid, uint32_t count) {
     }
 }
 
+/* [ours] the run covers whole segments: take up to want/nb consecutive free
+ * segments from the front, privately (no ring, no block tree).  Returns the
+ * blocks taken, 0 if no segment is free. */
+static uint32_t take_segments(o2_t *a, uint32_t t, uint32_t want, uint32_t *first) {
+    uint32_t nb = nb_of(t);
+    uint64_t s0 = claim_front(a);
+    if (s0 == NONE64) return 0;
+    uint32_t k = 1;
+    while (k < want / nb && s0 + k < a->nseg && oracle_veb_member(a->segfree, s0 + k)) {
+        oracle_veb_delete(a->segfree, s0 + k);
+        k++;
+    }
+    for (uint32_t q = 0; q < k; q++) format_segment(a, s0 + q, t, nb);
+    *first = (uint32_t)(s0 * nb);
+    return k * nb;
+}
+
 static uint32_t gid_of(uint32_t t, uint64_t linear) {
     uint32_t nb = nb_of(t);
     return (uint32_t)((linear / nb) * MAX_BLOCKS_PER_SEGMENT + linear % nb);
@@ -329,28 +348,22 @@ static uint32_t get_run_once(o2_t *a, uint32_t t, uint32_t want, uint32_t *first
             uint64_t f = claim_front(a);                      /* format one segment ahead */
             if (f != NONE64) format_segment(a, f, t, 0);
         }
-        uint16_t e[256] = {0};
-        for (uint32_t q = 0; q < got; q++) e[q] = ring_pop(r);      /* getBlock */
-        uint32_t p = 1;
-        while (p < got && e[p] == e[0] + p) p++;                   /* consecutive prefix */
-        for (uint32_t q = p; q < got; q++) return_block(a, s, e[q], t);
-        *first = (uint32_t)(s * nb + e[0]);
-        return p;
-    }
-    if (want >= nb) {
-        /* the run covers whole segments: take up to want/nb consecutive free
-         * segments from the front, privately (no ring, no block tree) */
-        uint64_t s0 = claim_front(a);
-        if (s0 == NONE64) return 0;                           /* "No allocations left" */
-        uint32_t k = 1;
-        while (k < want / nb && s0 + k < a->nseg && oracle_veb_member(a->segfree, s0 + k)) {
-            oracle_veb_delete(a->segfree, s0 + k);
-            k++;
+        uint8_t in[256] = {0};
+        for (uint32_t q = 0; q < got; q++) in[ring_pop(r)] = 1;     /* getBlock */
+        /* [ours] keep the longest run of consecutive block indices among them
+         * (lowest start on ties); the others go back in ascending order */
+        uint32_t bs = 0, bl = 0, len = 0;
+        for (uint32_t j = 0; j <= nb; j++) {
+            if (j < nb && in[j]) { len++; continue; }
+            if (len > bl) { bl = len; bs = j - len; }
+            len = 0;
         }
-        for (uint32_t q = 0; q < k; q++) format_segment(a, s0 + q, t, nb);
-        *first = (uint32_t)(s0 * nb);
-        return k * nb;
+        for (uint32_t j = 0; j < nb; j++)
+            if (in[j] && (j < bs || j >= bs + bl)) return_block(a, s, j, t);
+        *first = (uint32_t)(s * nb + bs);
+        return bl;
     }
+    if (want >= nb) return take_segments(a, t, want, first);  /* 0: "No allocations left" */
     uint64_t s1 = claim_front(a);                             /* Alg.2 -> getSegment */
     if (s1 == NONE64) return 0;
     format_segment(a, s1, t, want);

@@ -108,12 +108,12 @@ __global__ void k_reset() {
 // refill an earlier item would otherwise wait for.
 // Then waits-and-retries, whole blocks and segment runs.
 __device__ __noinline__ void bulk_malloc_slow(const uint64_t *sizes, void **ptrs, uint64_t n, uint64_t base,
-                                              uint32_t key, uint32_t slow, uint64_t info, int items,
+                                              uint32_t key, uint32_t slow, const uint64_t *info, int items,
                                               unsigned callers, uint32_t stride = 32) {
     const View &v = c_view;
     // pass 0: refill and prefetch duties only (never waits on another slot's refill)
     for (int k = 0; k < items; k++) {
-        const uint32_t code = (uint32_t)(info >> (16 * k)) & 0xFFFF;
+        const uint32_t code = (uint32_t)(info[k >> 2] >> (16 * (k & 3))) & 0xFFFF;
         if (((slow >> k) & 1) && (code & 0x2000u)) {
             const uint32_t c = core::slice_class(sizes[base + (uint64_t)stride * k]);
             core::prefetch_slot(v, v.slot_off[c] + key % v.nslot[c], c, code & 0x3FF);
@@ -134,7 +134,7 @@ __device__ __noinline__ void bulk_malloc_slow(const uint64_t *sizes, void **ptrs
     // pass 1: retries after a refill, waits, whole blocks and segment runs
     for (int k = 0; k < items; k++) {
         if (!((slow >> k) & 1)) continue;
-        const uint32_t code = (uint32_t)(info >> (16 * k)) & 0xFFFF;
+        const uint32_t code = (uint32_t)(info[k >> 2] >> (16 * (k & 3))) & 0xFFFF;
         const uint64_t i = base + (uint64_t)stride * k;
         const uint64_t sz = sizes[i];
         void *p;
@@ -215,7 +215,7 @@ __global__ void __launch_bounds__(kThreads, 5) k_bulk_malloc(const uint64_t *__r
             __stcs(reinterpret_cast<unsigned long long *>(ptrs) + i, reinterpret_cast<unsigned long long>(p));
     }
     const unsigned callers = __ballot_sync(0xFFFFFFFFu, slow != 0);
-    if (slow) bulk_malloc_slow(sizes, ptrs, n, base, key, slow, info, ITEMS, callers);
+    if (slow) bulk_malloc_slow(sizes, ptrs, n, base, key, slow, &info, ITEMS, callers);
 }
 
 // Bulk malloc with CTA-level aggregation: every warp of a CTA runs on one SM,
@@ -234,25 +234,33 @@ __global__ void __launch_bounds__(kThreads, 5) k_bulk_malloc_cta(const uint64_t 
     const uint64_t base = blockIdx.x * (uint64_t)(kThreads * ITEMS) + threadIdx.x;
     const uint32_t key = ptx::smid();
     if (threadIdx.x < core::kTrees) cnt[threadIdx.x] = 0;
-    uint64_t sz[ITEMS];
-    uint32_t cls[ITEMS], rank[ITEMS];
+    // per item: class (0..8 slice class, 0xFE nothing to do, 0xFF block or
+    // segment request) | rank << 8; the sizes themselves are not kept
+    uint32_t cr[ITEMS];
+    uint64_t x[ITEMS];
+    // unconditional loads of clamped indices, all issued before any is used
 #pragma unroll
     for (int k = 0; k < ITEMS; k++) {
         const uint64_t i = base + (uint64_t)kThreads * k;
-        // unconditional load of a clamped index: the ITEMS loads issue back to back
-        const uint64_t x = __ldcs(reinterpret_cast<const unsigned long long *>(sizes) + (i < n ? i : n - 1));
-        sz[k] = i < n ? x : 0;
-        cls[k] = sz[k] - 1 < core::kMaxSlice ? core::slice_class(sz[k]) : 0xFFu;
+        x[k] = __ldcs(reinterpret_cast<const unsigned long long *>(sizes) + (i < n ? i : n - 1));
+    }
+#pragma unroll
+    for (int k = 0; k < ITEMS; k++) {
+        const uint64_t s = base + (uint64_t)kThreads * k < n ? x[k] : 0;
+        const uint32_t lg = 64u - (uint32_t)__clzll((long long)(s - 1));      // ceil(log2 s) for s >= 2
+        const uint32_t sc = (lg > core::kMinSliceLog2 ? lg : core::kMinSliceLog2) - core::kMinSliceLog2;
+        cr[k] = s - 1 < core::kMaxSlice ? sc : (s == 0 ? 0xFEu : 0xFFu);   // branch-free slice_class
     }
     __syncthreads();
     const uint32_t lt = ptx::lanemask_lt();
 #pragma unroll
     for (int k = 0; k < ITEMS; k++) {
-        const unsigned peers = __match_any_sync(0xFFFFFFFFu, cls[k]);
+        const uint32_t c = cr[k];
+        const unsigned peers = __match_any_sync(0xFFFFFFFFu, c);
         const uint32_t leader = (uint32_t)__ffs((int)peers) - 1;
         uint32_t b = 0;
-        if (cls[k] != 0xFFu && lane == leader) b = atomicAdd(&cnt[cls[k]], (uint32_t)__popc(peers));
-        rank[k] = __shfl_sync(0xFFFFFFFFu, b, (int)leader) + (uint32_t)__popc(peers & lt);
+        if (c < core::kTrees && lane == leader) b = atomicAdd(&cnt[c], (uint32_t)__popc(peers));
+        cr[k] = c | ((__shfl_sync(0xFFFFFFFFu, b, (int)leader) + (uint32_t)__popc(peers & lt)) << 8);
     }
     __syncthreads();
     if (threadIdx.x < core::kTrees && cnt[threadIdx.x]) {
@@ -261,34 +269,42 @@ __global__ void __launch_bounds__(kThreads, 5) k_bulk_malloc_cta(const uint64_t 
     }
     __syncthreads();
     uint32_t slow = 0;
-    uint64_t info = 0;
+    uint64_t info[(ITEMS + 3) / 4];
+#pragma unroll
+    for (int q = 0; q < (ITEMS + 3) / 4; q++) info[q] = 0;
 #pragma unroll
     for (int k = 0; k < ITEMS; k++) {
         const uint64_t i = base + (uint64_t)kThreads * k;
+        const uint32_t c = cr[k] & 0xFFu;
         void *p = nullptr;
         uint32_t code = 0;
-        if (cls[k] != 0xFFu) {
-            const uint64_t old = olds[cls[k]];
+        if (c < core::kTrees) {
+            const uint64_t old = olds[c];
             const uint32_t m = core::run_len(old);
-            const uint32_t idx = (uint32_t)(old >> 32) + rank[k];
+            const uint32_t idx = (uint32_t)(old >> 32) + (cr[k] >> 8);
             if (idx < (m << core::kSliceLog2)) {
-                p = core::slice_ptr(v, cls[k], old & core::kRunNone, idx);
+                p = core::slice_ptr(v, c, old & core::kRunNone, idx);
                 if (v.prefetch && idx == (m << (core::kSliceLog2 - 1))) code = 0x2000u | m;   // prefetch duty
             } else {
                 code = idx == (m << core::kSliceLog2) ? (0x400u | m) : 0x1000u;
             }
-        } else if (sz[k] != 0) {
+        } else if (c == 0xFFu) {
             code = 0x800u;
         }
         if (code) {
             slow |= 1u << k;
-            info |= (uint64_t)code << (16 * k);
+            info[k >> 2] |= (uint64_t)code << (16 * (k & 3));
         }
         if (!(code & 0x1C00u) && i < n)
             __stcs(reinterpret_cast<unsigned long long *>(ptrs) + i, reinterpret_cast<unsigned long long>(p));
     }
     const unsigned callers = __ballot_sync(0xFFFFFFFFu, slow != 0);
-    if (slow) bulk_malloc_slow(sizes, ptrs, n, base, key, slow, info, ITEMS, callers, kThreads);
+    if (slow) {
+        uint64_t spill[(ITEMS + 3) / 4];                  // addressed copy only on the slow path
+#pragma unroll
+        for (int q = 0; q < (ITEMS + 3) / 4; q++) spill[q] = info[q];
+        bulk_malloc_slow(sizes, ptrs, n, base, key, slow, spill, ITEMS, callers, kThreads);
+    }
 }
 
 __device__ __noinline__ void free_slow(const View &v, uint64_t p) {
@@ -566,7 +582,9 @@ int gallatin_init_ex(const gallatin_config_t *cfg_in) {
         if (cfg.run_bytes > (256ull << 20)) cfg.run_bytes = 256ull << 20;
     }
     if (cfg.run_max > core::kMaxRun || cfg.fence_free > 2 || cfg.format_ahead > 2) return GALLATIN_ERR_INVALID;
-    if (cfg.bulk_items != 0 && cfg.bulk_items != 1 && cfg.bulk_items != 4) return GALLATIN_ERR_INVALID;
+    if (cfg.bulk_items != 0 && cfg.bulk_items != 1 && cfg.bulk_items != 4 && cfg.bulk_items != 8 &&
+        cfg.bulk_items != 16)
+        return GALLATIN_ERR_INVALID;
     if (cfg.prefetch > 2) return GALLATIN_ERR_INVALID;
     if (!cfg.run_grow) cfg.run_grow = 3;
     if (cfg.run_grow > 8) return GALLATIN_ERR_INVALID;
@@ -685,7 +703,12 @@ int gallatin_malloc(const uint64_t *d_sizes, void **d_ptrs, uint64_t n, void *st
     if (!g.init) return GALLATIN_ERR_STATE;
     if (n == 0) return GALLATIN_OK;
     if (!d_sizes || !d_ptrs || n > (1ull << 40)) return GALLATIN_ERR_INVALID;
-    if (g.cfg.bulk_items == 4 || (g.cfg.bulk_items == 0 && n >= (uint64_t)kItemsMin))
+    const uint32_t items = g.cfg.bulk_items ? g.cfg.bulk_items : (n >= (uint64_t)kItemsMin ? 4u : 1u);
+    if (items == 16)
+        k_bulk_malloc_cta<16><<<grid_for((n + 15) / 16), kThreads, 0, S(stream)>>>(d_sizes, d_ptrs, n);
+    else if (items == 8)
+        k_bulk_malloc_cta<8><<<grid_for((n + 7) / 8), kThreads, 0, S(stream)>>>(d_sizes, d_ptrs, n);
+    else if (items == 4)
         k_bulk_malloc_cta<4><<<grid_for((n + 3) / 4), kThreads, 0, S(stream)>>>(d_sizes, d_ptrs, n);
     else
         k_bulk_malloc<1><<<grid_for(n), kThreads, 0, S(stream)>>>(d_sizes, d_ptrs, n);
@@ -696,7 +719,7 @@ int gallatin_free(void *const *d_ptrs, uint64_t n, void *stream) {
     if (!g.init) return GALLATIN_ERR_STATE;
     if (n == 0) return GALLATIN_OK;
     if (!d_ptrs || n > (1ull << 40)) return GALLATIN_ERR_INVALID;
-    if (g.cfg.bulk_items == 4 || (g.cfg.bulk_items == 0 && n >= (uint64_t)kItemsMin))
+    if (g.cfg.bulk_items >= 4 || (g.cfg.bulk_items == 0 && n >= (uint64_t)kItemsMin))
         k_bulk_free<4><<<grid_for((n + 3) / 4), kThreads, 0, S(stream)>>>(d_ptrs, n);
     else
         k_bulk_free<1><<<grid_for(n), kThreads, 0, S(stream)>>>(d_ptrs, n);

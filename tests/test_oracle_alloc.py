@@ -199,3 +199,27 @@ def test_run_growth_factor(run_grow):
         assert (int(d["slots"][0]) >> 22) & 0x3FF == m
         m = min(m << run_grow, cap)
     assert a.check() == 0
+
+
+def test_shared_run_keeps_longest_consecutive_blocks():
+    """DESIGN.md Deviations 5: a run taken from a block-tree segment keeps the
+    longest run of consecutive block indices among the ring entries it
+    dequeues (lowest start on ties), not the FIFO prefix.  One segment, one
+    64 B slot whose first run is the whole segment (64 blocks of 256 KB,
+    P:174); its 64*4096 slices are drawn, then every block except 9 is
+    freed in the order 30..63, 0..8, 10..29 (ring order).  The refill
+    (want = cap = 64) dequeues those 63 entries and keeps 10..63 (54 blocks),
+    re-enqueueing 0..8; the prefix rule would have kept 30..63."""
+    bb = 64 * 4096                                            # 64 B slices: 256 KB blocks
+    a = oracle.Allocator(1, slot_base=1, slot_min=1, run_max=64, run_bytes=16 << 20, run_init=256, run_grow=1)
+    offs = a.malloc_batch(np.full(64 * 4096, 64, dtype=np.uint64), keydiv=0)
+    assert np.array_equal(offs, np.arange(64 * 4096, dtype=np.uint64) * np.uint64(64))
+    for b in list(range(30, 64)) + list(range(0, 9)) + list(range(10, 30)):
+        a.free_batch(offs[b * 4096:(b + 1) * 4096])
+    nxt = a.malloc_batch(np.full(54 * 4096 + 1, 64, dtype=np.uint64), keydiv=0)
+    assert np.array_equal(nxt[:-1], np.uint64(10 * bb) + np.arange(54 * 4096, dtype=np.uint64) * np.uint64(64))
+    assert nxt[-1] == 0                                       # then blocks 0..8: the next longest run
+    d = image_sections(a.image())
+    w = int(d["slots"][2])                                    # one slot per class: class 2's
+    assert (w >> 22) & 0x3FF == 9 and w & 0x3FFFFF == 0 and w >> 32 == 1
+    assert a.check() == 0
