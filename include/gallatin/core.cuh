@@ -350,9 +350,12 @@ __device__ inline __noinline__ uint32_t get_run_once(const View &v, uint32_t t, 
     const BitTree bt = block_tree(v, t);
     const uint32_t nb = nb_of(t);
     ptx::Backoff bo(4, t);
-    uint64_t from = 0;
+    uint64_t from = 0, hint = kNone;
+    uint32_t attempt = 0;
     for (;;) {
-        const uint64_t s = bt_successor<false>(bt, from);    // findSegment
+        // findSegment; after a lost race, a random other candidate
+        const uint64_t s = hint != kNone ? hint : bt_successor<false>(bt, from);
+        hint = kNone;
         if (s != kNone) {
             // reserve up to `want` blocks of s and validate its tree id in one RMW
             const uint64_t dec = (uint64_t)(-(int64_t)want);
@@ -430,6 +433,8 @@ __device__ inline __noinline__ uint32_t get_run_once(const View &v, uint32_t t, 
             seg_after_rmw(v, s, o2, o2 + want);
             btree_reconcile(v, t, s);
             from = s + 1;
+            hint = claim_retry_hint(s >> 6, ptx::ld_relaxed(bt.w + bt.off[0] + (s >> 6)) & ~(1ull << (s & 63)),
+                                    ++attempt);
             continue;
         }
         if (from != 0) {                                      // re-scan from the front once more
@@ -503,7 +508,7 @@ __device__ inline __noinline__ uint32_t trim_slots(const View &v) {
 
 // A run of up to `want` blocks of tree t (get_run_once); on "no memory" the
 // slots' undrawn blocks are given back and the request retried once.
-__device__ inline uint32_t get_run(const View &v, uint32_t t, uint32_t want, uint32_t *first) {
+__device__ inline __noinline__ uint32_t get_run(const View &v, uint32_t t, uint32_t want, uint32_t *first) {
     const uint32_t got = get_run_once(v, t, want, first);
     if (got != 0 || trim_slots(v) == 0) return got;
     return get_run_once(v, t, want, first);

@@ -31,6 +31,11 @@ namespace {
 constexpr int kT = 256;
 constexpr uint64_t kEmpty = ~0ull;
 constexpr uint32_t kBig = 2048;        // lists at least this long delete with a whole CTA
+#ifndef GALLATIN_GRAPH_MINB
+#define GALLATIN_GRAPH_MINB 4
+#endif
+// kernels that call the device allocator: register cap for >= this many CTAs/SM
+constexpr int kGraphMinBlocks = GALLATIN_GRAPH_MINB;
 
 inline cudaStream_t S(void *s) { return reinterpret_cast<cudaStream_t>(s); }
 inline unsigned blocks(uint64_t n) { return (unsigned)((n + kT - 1) / kT); }
@@ -69,7 +74,7 @@ __global__ void k_count(gallatin_graph g, const uint32_t *src, uint64_t n) {
 // Per vertex with cnt new edges: a batch that overflows the list reallocates
 // it to the next power of two (device malloc); non-empty old lists are queued
 // for the copy + free.
-__global__ void k_grow(gallatin_graph g) {
+__global__ void __launch_bounds__(kT, kGraphMinBlocks) k_grow(gallatin_graph g) {
     const uint64_t v = blockIdx.x * (uint64_t)kT + threadIdx.x;
     bool m = false, fail = false;
     if (v < g.V) {
@@ -97,7 +102,7 @@ __global__ void k_grow(gallatin_graph g) {
 }
 
 // warp per queued vertex: copy size[v] entries old -> new, free the old list
-__global__ void k_copy(gallatin_graph g) {
+__global__ void __launch_bounds__(kT, kGraphMinBlocks) k_copy(gallatin_graph g) {
     const uint32_t nw = *g.nwork;
     const uint64_t warps = (uint64_t)gridDim.x * (kT / 32);
     unsigned long long frees = 0;
@@ -214,7 +219,7 @@ __device__ void shrink_warp(const gallatin_graph &g, uint32_t v, uint32_t out, b
 }
 
 // warp per vertex: scan, drop the deleted instances, compact in place
-__global__ void k_delete_small(gallatin_graph g) {
+__global__ void __launch_bounds__(kT, kGraphMinBlocks) k_delete_small(gallatin_graph g) {
     const uint32_t nw = g.nwork[0];
     const uint64_t warps = (uint64_t)gridDim.x * (kT / 32);
     bool m = false, f = false, fail = false;
@@ -241,7 +246,7 @@ __global__ void k_delete_small(gallatin_graph g) {
 }
 
 // CTA per big vertex: same, with a block-wide prefix per 256-entry chunk
-__global__ void k_delete_big(gallatin_graph g) {
+__global__ void __launch_bounds__(kT, kGraphMinBlocks) k_delete_big(gallatin_graph g) {
     __shared__ uint32_t wsum[kT / 32];
     __shared__ uint32_t out_s;
     const uint32_t nw = g.nwork[1], wid = threadIdx.x >> 5;
@@ -286,7 +291,7 @@ __global__ void k_expand_prep(gallatin_graph g, const uint32_t *vs, uint64_t n) 
     g.cnt[vs[i]] = s < 4 ? 4 : s;              // each round appends max(size, 4) edges
 }
 
-__global__ void k_expand_fill(gallatin_graph g, const uint32_t *vs, uint64_t n) {
+__global__ void __launch_bounds__(kT, kGraphMinBlocks) k_expand_fill(gallatin_graph g, const uint32_t *vs, uint64_t n) {
     const uint64_t warps = (uint64_t)gridDim.x * (kT / 32);
     for (uint64_t w = (blockIdx.x * (uint64_t)kT + threadIdx.x) >> 5; w < n; w += warps) {
         const uint32_t v = vs[w], s0 = g.size[v], add = g.cnt[v];
@@ -297,7 +302,7 @@ __global__ void k_expand_fill(gallatin_graph g, const uint32_t *vs, uint64_t n) 
     }
 }
 
-__global__ void k_free_all(gallatin_graph g) {
+__global__ void __launch_bounds__(kT, kGraphMinBlocks) k_free_all(gallatin_graph g) {
     const uint64_t v = blockIdx.x * (uint64_t)kT + threadIdx.x;
     bool f = false;
     if (v < g.V && g.list[v]) {
