@@ -274,7 +274,7 @@ def run_ours(args, rank, world, local):
                        "l2": "no flush: each step reads %.2f GiB of sizes + writes/reads the pointer array (> 126 MB L2)" % (
                            sum(8 * n for _, n in cells) / 2 ** 30)},
             "malloc_ops_s": malloc_ops_s, "free_ops_s": free_ops_s, "per_size": per_cell,
-            "roofline": {"bound": "hbm", "kernel": f"k_bulk_{dominant}", "achieved": achieved, "peak": hbm_peak,
+            "roofline": {"bound": "hbm", "kernel": "k_bulk_malloc_cta<4>" if dominant == "malloc" else "k_bulk_free<4>", "achieved": achieved, "peak": hbm_peak,
                          "unit": "GB/s", "frac": achieved / hbm_peak, "traffic": traffic,
                          "traffic_algorithmic": bytes_per_op * (1 << 24),
                          "traffic_note": "DRAM bytes of one 2^24-thread launch (16 B cell, profiles/r1_kernels.md)",
@@ -373,6 +373,43 @@ def run_extras(args, G, torch, stream):
     out["probes"] = pk
     out["scaling"] = run_scaling(args, G, torch, stream)
     out["graph"] = run_graph(args, G, torch, stream)
+    out["paper_modes"] = run_paper_modes(args, G, torch)
+    return out
+
+
+def run_paper_modes(args, G, torch):
+    """PAPER.md S6's other modes (experiments.py): utilization on a 2 GB heap
+    with batches of 100,000 (E8), fragmentation of 2^20 allocations
+    (E7), warmed-up vs reset rounds at 2 KB (E6), the variance
+    of 50 rounds (E5) and init time (E1)."""
+    from paper_conf_ppopp_mccoyp24_b200 import experiments as X
+    out = {}
+    G.gallatin_destroy()
+    util = {}
+    for size in [4 << i for i in range(12)]:                    # 4 B .. 8 KB (P:350)
+        G.gallatin_init(2 << 30)
+        r = X.utilization(size, batch=100_000 // args.scale)
+        util[str(size)] = {"utilization": round(r["utilization"], 4), "successes": r["successes"],
+                           "batches": r["batches"]}
+        del r
+        G.gallatin_destroy()
+    out["utilization"] = {"heap_bytes": 2 << 30, "batch": 100_000 // args.scale, "per_size": util,
+                          "note": "successes x size / heap; sizes < 16 B round up to 16 B slices, "
+                                  "8 KB takes a 64 KB block (reading A-2)"}
+    G.gallatin_init(HEAP_C2)
+    frag = {}
+    for size in SIZES:
+        G.gallatin_reset()
+        r = X.fragmentation(size, (1 << 20) // args.scale)
+        frag[str(size)] = {"range_bytes": r["range_bytes"], "range_over_requested": round(r["range_over_requested"], 4)}
+        G.gallatin_free(r["ptrs"])
+        del r
+    out["fragmentation"] = {"n": (1 << 20) // args.scale, "per_size": frag}
+    out["warm_vs_cold_2KB"] = X.warm_vs_cold(2048, (1 << 20) // args.scale, rounds=20)
+    out["variance_64B"] = X.variance(64, (1 << 20) // args.scale, rounds=50)
+    G.gallatin_destroy()
+    out["init"] = X.init_time(HEAP_C2, reps=3)
+    G.gallatin_init(HEAP_C2)
     return out
 
 

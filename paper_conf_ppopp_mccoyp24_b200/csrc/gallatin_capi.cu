@@ -22,6 +22,11 @@ namespace {
 constexpr int kThreads = 256;
 // ITEMS=4 per thread once the grid would still fill every SM several times
 constexpr int kItemsMin = 148 * 1024 * 4;
+// host-array calls are cut into at most kMaxChunks pieces of >= kChunkMin
+// requests, so the copy in of piece i+1, the kernel of piece i and the copy
+// out of piece i-1 overlap (PCIe is full duplex)
+constexpr int kMaxChunks = 8;
+constexpr uint64_t kChunkMin = 1ull << 20;
 
 struct State {
     bool init = false;
@@ -33,6 +38,9 @@ struct State {
     View v{};
     void *scratch = nullptr;
     uint64_t scratch_bytes = 0;
+    // host-array calls: copy-in / copy-out streams and per-chunk events
+    cudaStream_t cin = nullptr, cout = nullptr;
+    cudaEvent_t ev_in[kMaxChunks] = {}, ev_k[kMaxChunks] = {};
 };
 State g;
 
@@ -536,6 +544,12 @@ int copy_state(HostCopy &h) {
 }
 
 int free_all() {
+    if (g.cin) cudaStreamDestroy(g.cin);
+    if (g.cout) cudaStreamDestroy(g.cout);
+    for (int i = 0; i < kMaxChunks; i++) {
+        if (g.ev_in[i]) cudaEventDestroy(g.ev_in[i]);
+        if (g.ev_k[i]) cudaEventDestroy(g.ev_k[i]);
+    }
     if (g.heap_raw) cudaFree(g.heap_raw);
     if (g.meta) cudaFree(g.meta);
     if (g.scratch) cudaFree(g.scratch);
@@ -727,6 +741,14 @@ int gallatin_free(void *const *d_ptrs, uint64_t n, void *stream) {
 }
 
 static int ensure_scratch(uint64_t bytes) {
+    if (!g.cin) {
+        CUDA_TRY(cudaStreamCreateWithFlags(&g.cin, cudaStreamNonBlocking));
+        CUDA_TRY(cudaStreamCreateWithFlags(&g.cout, cudaStreamNonBlocking));
+        for (int i = 0; i < kMaxChunks; i++) {
+            CUDA_TRY(cudaEventCreateWithFlags(&g.ev_in[i], cudaEventDisableTiming));
+            CUDA_TRY(cudaEventCreateWithFlags(&g.ev_k[i], cudaEventDisableTiming));
+        }
+    }
     if (g.scratch_bytes >= bytes) return GALLATIN_OK;
     if (g.scratch) cudaFree(g.scratch);
     g.scratch = nullptr;
@@ -736,6 +758,13 @@ static int ensure_scratch(uint64_t bytes) {
     return GALLATIN_OK;
 }
 
+static uint64_t chunk_of(uint64_t n) {
+    uint64_t c = (n + kMaxChunks - 1) / kMaxChunks;
+    return c < kChunkMin ? kChunkMin : c;
+}
+
+// Pipelined over chunks: copy-in stream -> the caller's stream (kernels, in
+// request order) -> copy-out stream; the call returns after everything landed.
 int gallatin_malloc_host(const uint64_t *h_sizes, uint64_t *h_ptrs, uint64_t n, void *stream) {
     if (!g.init) return GALLATIN_ERR_STATE;
     if (n == 0) return GALLATIN_OK;
@@ -743,11 +772,21 @@ int gallatin_malloc_host(const uint64_t *h_sizes, uint64_t *h_ptrs, uint64_t n, 
     int rc = ensure_scratch(16 * n);
     if (rc) return rc;
     uint64_t *d_sizes = static_cast<uint64_t *>(g.scratch);
-    void **d_ptrs = reinterpret_cast<void **>(d_sizes + n);
-    CUDA_TRY(cudaMemcpyAsync(d_sizes, h_sizes, 8 * n, cudaMemcpyHostToDevice, S(stream)));
-    rc = gallatin_malloc(d_sizes, d_ptrs, n, stream);
-    if (rc) return rc;
-    CUDA_TRY(cudaMemcpyAsync(h_ptrs, d_ptrs, 8 * n, cudaMemcpyDeviceToHost, S(stream)));
+    uint64_t *d_ptrs = d_sizes + n;
+    const uint64_t ch = chunk_of(n);
+    int q = 0;
+    for (uint64_t lo = 0; lo < n; lo += ch, q++) {
+        const uint64_t m = n - lo < ch ? n - lo : ch;
+        CUDA_TRY(cudaMemcpyAsync(d_sizes + lo, h_sizes + lo, 8 * m, cudaMemcpyHostToDevice, g.cin));
+        CUDA_TRY(cudaEventRecord(g.ev_in[q], g.cin));
+        CUDA_TRY(cudaStreamWaitEvent(S(stream), g.ev_in[q], 0));
+        rc = gallatin_malloc(d_sizes + lo, reinterpret_cast<void **>(d_ptrs + lo), m, stream);
+        if (rc) return rc;
+        CUDA_TRY(cudaEventRecord(g.ev_k[q], S(stream)));
+        CUDA_TRY(cudaStreamWaitEvent(g.cout, g.ev_k[q], 0));
+        CUDA_TRY(cudaMemcpyAsync(h_ptrs + lo, d_ptrs + lo, 8 * m, cudaMemcpyDeviceToHost, g.cout));
+    }
+    CUDA_TRY(cudaStreamSynchronize(g.cout));
     CUDA_TRY(cudaStreamSynchronize(S(stream)));
     return GALLATIN_OK;
 }
@@ -758,10 +797,17 @@ int gallatin_free_host(const uint64_t *h_ptrs, uint64_t n, void *stream) {
     if (!h_ptrs) return GALLATIN_ERR_INVALID;
     int rc = ensure_scratch(16 * n);
     if (rc) return rc;
-    void **d_ptrs = static_cast<void **>(g.scratch);
-    CUDA_TRY(cudaMemcpyAsync(d_ptrs, h_ptrs, 8 * n, cudaMemcpyHostToDevice, S(stream)));
-    rc = gallatin_free(d_ptrs, n, stream);
-    if (rc) return rc;
+    uint64_t *d_ptrs = static_cast<uint64_t *>(g.scratch);
+    const uint64_t ch = chunk_of(n);
+    int q = 0;
+    for (uint64_t lo = 0; lo < n; lo += ch, q++) {
+        const uint64_t m = n - lo < ch ? n - lo : ch;
+        CUDA_TRY(cudaMemcpyAsync(d_ptrs + lo, h_ptrs + lo, 8 * m, cudaMemcpyHostToDevice, g.cin));
+        CUDA_TRY(cudaEventRecord(g.ev_in[q], g.cin));
+        CUDA_TRY(cudaStreamWaitEvent(S(stream), g.ev_in[q], 0));
+        rc = gallatin_free(reinterpret_cast<void *const *>(d_ptrs + lo), m, stream);
+        if (rc) return rc;
+    }
     CUDA_TRY(cudaStreamSynchronize(S(stream)));
     return GALLATIN_OK;
 }

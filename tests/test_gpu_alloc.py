@@ -201,6 +201,28 @@ def test_host_buffer_api(cuda_ok, G):
     _assert_pristine(G, nseg)
 
 
+def test_host_buffer_api_chunked(cuda_ok, G):
+    """Host-array calls cut into several copy/kernel/copy chunks (a ragged last
+    chunk): every pointer distinct, aligned to its class, in the heap, and the
+    usable bytes equal the closed form; free-all + drain is pristine."""
+    nseg = 64
+    G.gallatin_init(nseg * SEG)
+    n = 3 * (1 << 20) + 12345
+    sizes = wg.mixed_sizes(n, upper=256, p_large=0.0)
+    p = G.gallatin_malloc_host(sizes)
+    assert np.all(p != 0)
+    base = G.gallatin_stats()["heap_base"]
+    offs = p - np.uint64(base)
+    cls = np.array([class_size(int(s)) for s in sizes[:4096]], dtype=np.uint64)
+    assert np.all(offs[:4096] % cls == 0)
+    assert len(np.unique(p)) == n and int(offs.max()) < nseg * SEG
+    usable, bad = G.gallatin_usable(_dev(p), _dev(sizes))
+    u, c = np.unique(sizes, return_counts=True)
+    assert bad == 0 and usable == sum(class_size(int(a)) * int(b) for a, b in zip(u, c))
+    G.gallatin_free_host(p)
+    _assert_pristine(G, nseg)
+
+
 def test_reset_restores_pristine(cuda_ok, G):
     nseg = 8
     G.gallatin_init(nseg * SEG)

@@ -223,3 +223,34 @@ def test_shared_run_keeps_longest_consecutive_blocks():
     w = int(d["slots"][2])                                    # one slot per class: class 2's
     assert (w >> 22) & 0x3FF == 9 and w & 0x3FFFFF == 0 and w >> 32 == 1
     assert a.check() == 0
+
+
+@pytest.mark.parametrize("size", [4, 16, 64, 256, 4096, 8192, 1 << 20, 1 << 24, 3 << 24])
+def test_utilization_closed_form(size):
+    """E8: batches of 100,000 allocations of one size until
+    the first NULL.  Closed forms from the paper's geometry on an empty heap of
+    nseg segments: a slice class has nseg * (256 >> c) * 4096 slices (P:188,
+    P:264) of which at most one partly drawn block per block-buffer slot
+     is left unissued; a whole-block request (reading A-2) gets exactly
+    nseg * (256 >> t) blocks; a k-segment request exactly floor(nseg / k)
+    (P:138)."""
+    nseg = 8
+    a = oracle.Allocator(nseg, slot_base=148, slot_min=4, run_max=256, run_init=64, run_grow=3,
+                         run_bytes=256 << 20, format_ahead=1)
+    succ = 0
+    while True:
+        o = a.malloc_batch(np.full(100_000, size, dtype=np.uint64), keydiv=32)
+        ok = int((o != NONE).sum())
+        succ += ok
+        if ok < len(o):
+            break
+    assert a.check() == 0
+    if size <= 4096:
+        c = max(0, (size - 1).bit_length() - 4)
+        total = nseg * (256 >> c) * 4096
+        assert total - a.nslot(c) * 4096 <= succ <= total
+    elif size < SEG:
+        t = max(0, (size - 1).bit_length() - 16)
+        assert succ == nseg * (256 >> t)
+    else:
+        assert succ == nseg // -(-size // SEG)
