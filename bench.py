@@ -396,15 +396,22 @@ def run_paper_modes(args, G, torch):
     out["utilization"] = {"heap_bytes": 2 << 30, "batch": 100_000 // args.scale, "per_size": util,
                           "note": "successes x size / heap; sizes < 16 B round up to 16 B slices, "
                                   "8 KB takes a 64 KB block (reading A-2)"}
+    # fragmentation with the default knobs (runs of blocks per slot) and with
+    # the paper's one-block buffer (run_max = run_init = 1, no format-ahead)
+    out["fragmentation"] = {"n": (1 << 20) // args.scale}
+    for name, knobs in (("default", {}), ("paper_policy", dict(run_max=1, run_init=1, format_ahead=2, prefetch=2))):
+        G.gallatin_init(HEAP_C2, **knobs)
+        frag = {}
+        for size in SIZES:
+            G.gallatin_reset()
+            r = X.fragmentation(size, (1 << 20) // args.scale)
+            frag[str(size)] = {"range_bytes": r["range_bytes"],
+                               "range_over_requested": round(r["range_over_requested"], 4)}
+            G.gallatin_free(r["ptrs"])
+            del r
+        out["fragmentation"][name] = frag
+        G.gallatin_destroy()
     G.gallatin_init(HEAP_C2)
-    frag = {}
-    for size in SIZES:
-        G.gallatin_reset()
-        r = X.fragmentation(size, (1 << 20) // args.scale)
-        frag[str(size)] = {"range_bytes": r["range_bytes"], "range_over_requested": round(r["range_over_requested"], 4)}
-        G.gallatin_free(r["ptrs"])
-        del r
-    out["fragmentation"] = {"n": (1 << 20) // args.scale, "per_size": frag}
     out["warm_vs_cold_2KB"] = X.warm_vs_cold(2048, (1 << 20) // args.scale, rounds=20)
     out["variance_64B"] = X.variance(64, (1 << 20) // args.scale, rounds=50)
     G.gallatin_destroy()

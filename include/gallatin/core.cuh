@@ -343,6 +343,20 @@ __device__ inline __noinline__ uint32_t take_segments(const View &v, uint32_t t,
     return k * nb;
 }
 
+// [dev] Blocks of tree t that are reserved past their segment's available
+// count (a negative count: a refiller's give-back of its excess is in
+// flight) will be available again in a moment; a refill about to report "no
+// memory" checks for them (one pass over the table, near exhaustion only) and
+// retries instead.
+constexpr uint32_t kFluxRetries = 64;
+__device__ inline __noinline__ bool flux_pending(const View &v, uint32_t t) {
+    for (uint64_t s = 0; s < v.nseg; s++) {
+        const uint64_t w = ptx::ld_relaxed(v.seg_word + s);
+        if (sw_tree(w) == t && sw_avail(w) < 0) return true;
+    }
+    return false;
+}
+
 // ---- Alg. 2 GetBlock(treeId), for a RUN of blocks [dev] --------
 // Returns the number of consecutive blocks obtained (0 = exhausted) and the
 // first one's linear index (segment * nb + block) in *first.
@@ -351,7 +365,8 @@ __device__ inline __noinline__ uint32_t get_run_once(const View &v, uint32_t t, 
     const uint32_t nb = nb_of(t);
     ptx::Backoff bo(4, t);
     uint64_t from = 0, hint = kNone;
-    uint32_t attempt = 0;
+    uint32_t attempt = 0, flux_retries = 0;
+    bool flux = false;            // saw blocks of tree t reserved beyond the available count
     for (;;) {
         // findSegment; after a lost race, a random other candidate
         const uint64_t s = hint != kNone ? hint : bt_successor<false>(bt, from);
@@ -363,10 +378,16 @@ __device__ inline __noinline__ uint32_t get_run_once(const View &v, uint32_t t, 
             const int32_t a = sw_avail(old);
             if (sw_tree(old) == t && a > 0) {
                 const uint32_t got = (uint32_t)a < want ? (uint32_t)a : want;
-                seg_after_rmw(v, s, old, old + dec);
-                if (got < want) {                               // give back the excess
+                if (got < want) {
+                    // give back the excess at once, then repair the block-tree
+                    // bit once for both RMWs: the over-reservation must not
+                    // drop s from the tree while other refillers search it
                     const uint64_t o2 = ptx::atom_add(v.seg_word + s, (uint64_t)(want - got));
-                    seg_after_rmw(v, s, o2, o2 + (want - got));
+                    if (sw_in_tree(old, t) != sw_in_tree(old + dec, t) ||
+                        sw_in_tree(o2, t) != sw_in_tree(o2 + (want - got), t))
+                        btree_reconcile(v, t, s);
+                } else {
+                    seg_after_rmw(v, s, old, old + dec);
                 }
                 const uint32_t low = nb / 4;
                 if (v.format_ahead && (uint32_t)a >= low && (uint32_t)a - got < low &&
@@ -427,7 +448,9 @@ __device__ inline __noinline__ uint32_t get_run_once(const View &v, uint32_t t, 
                 *first = (uint32_t)(s * nb + bs);
                 return bl;
             }
-            // stale hint (P:158-161's failure case): undo, repair, look further
+            // stale hint (P:158-161's failure case): undo, repair, look further;
+            // a negative count means another refiller's give-back is in flight
+            if (sw_tree(old) == t && a < 0) flux = true;
             seg_after_rmw(v, s, old, old + dec);
             const uint64_t o2 = ptx::atom_add(v.seg_word + s, (uint64_t)want);
             seg_after_rmw(v, s, o2, o2 + want);
@@ -442,7 +465,21 @@ __device__ inline __noinline__ uint32_t get_run_once(const View &v, uint32_t t, 
             bo.pause();
             continue;
         }
-        if (want >= nb) return take_segments(v, t, want, first);   // 0: "No allocations left"
+        // [dev] before reporting "no memory", wait out blocks that are only
+        // transiently unavailable (an over-reservation being given back)
+        if (flux && flux_retries < kFluxRetries) {
+            flux = false;
+            flux_retries++;
+            bo.pause();
+            continue;
+        }
+        if (want >= nb) {
+            const uint32_t k = take_segments(v, t, want, first);
+            if (k || !flux_pending(v, t) || flux_retries >= kFluxRetries) return k;   // 0: "No allocations left"
+            flux_retries++;
+            bo.pause();
+            continue;
+        }
         // Alg.2: format a segment; [dev] bounded formatters per tree
         uint32_t *tok = v.fmt_token + t * 32;
         if (token_try(tok, v.formatters)) {
@@ -454,7 +491,11 @@ __device__ inline __noinline__ uint32_t get_run_once(const View &v, uint32_t t, 
             if (s1 != kNone) format_segment(v, s1, t, want);
             token_release(tok);
             if (s1 == kNone) {
-                if (bt_scan_first(bt) == kNone) return 0;     // "No allocations left"
+                if (bt_scan_first(bt) == kNone) {
+                    if (!flux_pending(v, t) || flux_retries >= kFluxRetries) return 0;   // "No allocations left"
+                    flux_retries++;
+                    bo.pause();
+                }
                 continue;
             }
             *first = (uint32_t)(s1 * nb);
@@ -507,11 +548,19 @@ __device__ inline __noinline__ uint32_t trim_slots(const View &v) {
 }
 
 // A run of up to `want` blocks of tree t (get_run_once); on "no memory" the
-// slots' undrawn blocks are given back and the request retried once.
+// slots' undrawn blocks are given back and the request retried for a SINGLE
+// block (memory is scarce: no slot should hoard a run of it).  Under
+// concurrency the retry repeats while trims still find blocks, and once
+// more after an empty trim: a concurrent refiller's trim may just have given
+// the blocks back.  Serially this is one trim and one retry.
 __device__ inline __noinline__ uint32_t get_run(const View &v, uint32_t t, uint32_t want, uint32_t *first) {
-    const uint32_t got = get_run_once(v, t, want, first);
-    if (got != 0 || trim_slots(v) == 0) return got;
-    return get_run_once(v, t, want, first);
+    uint32_t got = get_run_once(v, t, want, first);
+    for (uint32_t r = 0; got == 0 && r < 8; r++) {
+        const uint32_t back = trim_slots(v);
+        got = get_run_once(v, t, 1, first);
+        if (back == 0 && r >= 1) break;
+    }
+    return got;
 }
 
 // Replace an exhausted run (Alg.3): the run doubles up to the class cap.

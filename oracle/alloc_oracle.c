@@ -404,11 +404,13 @@ static uint64_t trim_slots(o2_t *a) {
 }
 
 /* A run of up to `want` blocks (get_run_once); on "no memory" the slots give
- * back their undrawn blocks and the request is retried once. */
+ * back their undrawn blocks and the request is retried once, for a single
+ * block: memory is scarce, so no slot hoards a run of it (DESIGN.md
+ * Deviations 5, "near exhaustion"). */
 static uint32_t get_run(o2_t *a, uint32_t t, uint32_t want, uint32_t *first) {
     uint32_t got = get_run_once(a, t, want, first);
     if (got || !trim_slots(a)) return got;
-    return get_run_once(a, t, want, first);
+    return get_run_once(a, t, 1, first);
 }
 
 /* ------------------------------------------ claimMultiple (back) --- */

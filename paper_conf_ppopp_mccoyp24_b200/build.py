@@ -14,7 +14,7 @@ NVCC_FLAGS = [
     "-O3", "-std=c++17",
     "-gencode", "arch=compute_100a,code=sm_100a",
     "-lineinfo",
-    "-Xcompiler", "-fPIC,-O2",
+    "-Xcompiler", "-fPIC,-O2,-Wno-attributes",
     "-shared",
 ]
 
