@@ -75,6 +75,10 @@ typedef struct gallatin_config {
     uint32_t run_init;     /* first run of an empty slot of class c: min(max(run_init >> c, min(run_init, 8)), 256 >> c) blocks (default: the largest power of two <= 256 whose first runs over all slots fit in half the heap) */
     uint32_t prefetch;     /* 1 = fetch the next run at the middle of the current one; 0/2 = off (default) */
     uint32_t run_grow;     /* a refilled run is 2^run_grow times the last one, up to the cap: 1..8 (default 3) */
+    uint32_t pipeline;     /* bulk kernels at bulk_items = 0: 1 = persistent CTAs that TMA-load the next tile while
+                              this tile's atomics are in flight; 0/2 = one tile per CTA (default, measured faster) */
+    uint32_t free_team;    /* bulk free: 0/2 = one free-counter RMW per warp team (default, measured faster);
+                              1 = one per block per CTA tile (shared-memory aggregation) */
 } gallatin_config_t;
 
 int gallatin_init(uint64_t heap_bytes);                 /* defaults for the rest */

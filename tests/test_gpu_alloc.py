@@ -269,3 +269,37 @@ def test_config3_full_size_bench_launch(cuda_ok, G):
             G.gallatin_reset()
         assert _bulk_round(G, nseg, sizes) == 0
         _assert_pristine(G, nseg)
+
+
+@pytest.mark.parametrize("knobs", [dict(pipeline=1), dict(free_team=1), dict(bulk_items=8), dict(bulk_items=16),
+                                   dict(bulk_items=1), dict(pipeline=2, free_team=1)])
+@pytest.mark.parametrize("n", [(1 << 21) + 77, 1 << 22])
+def test_bulk_kernel_variants(cuda_ok, G, knobs, n):
+    """Every bulk-kernel variant (persistent TMA-pipelined, CTA-aggregated or
+    warp-team frees, 1/4/8/16 requests per thread) on mixed sizes with a
+    ragged tail: stamp-verified, accounted, overlap-checked, pristine after
+    free-all + drain."""
+    nseg = 1024
+    G.gallatin_init(nseg * SEG, **knobs)
+    sizes = wg.mixed_sizes(n, p_large=2.0 ** -14)
+    assert _bulk_round(G, nseg, sizes) == 0
+    _assert_pristine(G, nseg)
+
+
+def test_bulk_kernels_unaligned_arrays(cuda_ok, G):
+    """Size and pointer arrays that start 8 bytes past a 16-byte boundary
+    (the TMA tile loads fall back to plain loads)."""
+    nseg = 256
+    for knobs in (dict(pipeline=1), {}):
+        G.gallatin_init(nseg * SEG, **knobs)
+        n = (1 << 20) + 3
+        sizes = _dev(np.concatenate([[0], wg.mixed_sizes(n, upper=512, p_large=0.0)]))[1:]
+        ptrs = torch.zeros(n + 1, dtype=torch.int64, device="cuda")[1:]
+        assert sizes.data_ptr() % 16 == 8 and ptrs.data_ptr() % 16 == 8
+        G.gallatin_malloc(sizes, ptrs)
+        G.gallatin_stamp(ptrs, sizes)
+        assert G.gallatin_verify(ptrs, sizes) == 0
+        assert int((ptrs == 0).sum()) == 0
+        G.gallatin_free(ptrs)
+        _assert_pristine(G, nseg)
+        G.gallatin_destroy()
