@@ -330,6 +330,33 @@ def run_extras(args, G, torch, stream):
                   "universe": "2^20", "keys": len(w["insert"]),
                   "successor_hbm_gbs": nq * 16 / succ_ms / 1e6}
 
+    # --- successor on larger universes: 2^24 keys, 2^24 uniform queries ---
+    big = {}
+    for k in (24, 28, 32):
+        vb = G.Veb(k)
+        nk = min(1 << 24, (1 << k) >> 2)
+        bk = torch.from_numpy(wg.distinct_below(wg.cell_seed(1, 400 + k), nk, 1 << k).view(np.int64)).cuda()
+        bq = torch.from_numpy(wg.uniform_below(wg.cell_seed(1, 500 + k), nq, 1 << k).view(np.int64)).cuda()
+        br = torch.empty_like(bq)
+        e0.record(stream)
+        vb.insert(bk, want_out=False)
+        e1.record(stream)
+        torch.cuda.synchronize()
+        bins = e0.elapsed_time(e1)
+        for _ in range(3):
+            vb.successor(bq, br)
+        e0.record(stream)
+        for _ in range(reps):
+            vb.successor(bq, br)
+        e1.record(stream)
+        torch.cuda.synchronize()
+        bms = e0.elapsed_time(e1) / reps
+        big[f"2^{k}"] = {"keys": nk, "queries": nq, "insert_ops_s": nk / bins * 1e3, "successor_ops_s": nq / bms * 1e3,
+                         "successor_ms": bms, "leaf_bytes": (1 << k) // 8}
+        vb.close()
+        del bk, bq, br
+    out["veb"]["large_universes"] = big
+
     # --- mixed-size cell (configs[2] shape) on its own 64 GiB heap ---
     G.gallatin_destroy()
     G.gallatin_init(HEAP_C3)
@@ -445,8 +472,35 @@ def run_scaling(args, G, torch, stream):
         pts[str(n)] = {"malloc_ms": round(m, 5), "free_ms": round(f, 5), "malloc_ops_s": n / m * 1e3,
                        "free_ops_s": n / f * 1e3}
         del st, p
+    # the paper's other scaling sizes (16, 512, 8192 B) up to its 2^20 threads
+    paper = {}
+    for size in (16, 512, 8192):
+        pp = {}
+        for lg in range(10, 21, 2):
+            n = max(1024, (1 << lg) // args.scale)
+            st = torch.full((n,), size, dtype=torch.int64, device="cuda")
+            p = torch.empty_like(st)
+            mm, fm = [], []
+            for it in range(7):
+                G.gallatin_reset()
+                a, b, c = (torch.cuda.Event(enable_timing=True) for _ in range(3))
+                a.record(stream)
+                G.gallatin_malloc(st, p)
+                b.record(stream)
+                G.gallatin_free(p)
+                c.record(stream)
+                torch.cuda.synchronize()
+                if it >= 2:
+                    mm.append(a.elapsed_time(b))
+                    fm.append(b.elapsed_time(c))
+            m, f = statistics.median(mm), statistics.median(fm)
+            pp[str(n)] = {"malloc_ms": round(m, 5), "free_ms": round(f, 5), "malloc_ops_s": n / m * 1e3,
+                          "free_ops_s": n / f * 1e3}
+        paper[str(size)] = pp
     return {"workload": "BASELINE configs[3]: 64 B, 2^10..2^26 threads (every 4th power), 16 GiB heap, "
-                        "independent per-GPU heap under torchrun", "points": pts}
+                        "independent per-GPU heap under torchrun", "points": pts,
+            "paper_sizes": {"workload": "P:329 sizes 16/512/8192 B at 2^10..2^20 threads (every 2nd power)",
+                            "points": paper}}
 
 
 def run_graph(args, G, torch, stream):

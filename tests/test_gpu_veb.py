@@ -136,3 +136,67 @@ def test_concurrent_insert_delete_quiescent_exact(cuda_ok):
     o = oracle.Veb(k)
     o.batch(OV_INSERT, odds)
     assert np.array_equal(g.snapshot(), o.image())
+
+
+@pytest.mark.parametrize("k", [16, 24])
+def test_concurrent_mixed_batches_linearizable(cuda_ok, k):
+    """Concurrent mixed-batch mode: successor / predecessor /
+    member queries race with inserts and deletes of VOLATILE keys on other
+    streams.  Linearizability-style invariants, for every query x:
+    succ(x) is NONE only if no STABLE key (present throughout) is >= x;
+    otherwise x <= succ(x) <= the smallest stable key >= x and succ(x) is a
+    stable or volatile key (never a key that was never present); pred
+    mirrors it; member is 1 on stable keys and 0 on never-present keys.  At
+    quiescence the image is exact."""
+    import paper_conf_ppopp_mccoyp24_b200 as G
+    u = 1 << k
+    seed = wg.cell_seed(1, 300 + k)
+    keys = wg.distinct_below(seed, min(u // 4, 1 << 20), u)
+    third = len(keys) // 3
+    stable, vol_in, vol_out = keys[:third], keys[third:2 * third], keys[2 * third:]
+    q = wg.uniform_below(seed ^ 5, 1 << 20, u)
+    g = G.Veb(k)
+    g.insert(_dev(np.concatenate([stable, vol_out])), want_out=False)
+    torch.cuda.synchronize()
+    s1, s2, s3 = torch.cuda.Stream(), torch.cuda.Stream(), torch.cuda.Stream()
+    dq = _dev(q)
+    di, dd = _dev(vol_in), _dev(vol_out)
+    outs = []
+    for rep in range(4):
+        with torch.cuda.stream(s1):
+            (g.insert if rep % 2 == 0 else g.delete)(di, want_out=False, stream=s1.cuda_stream)
+        with torch.cuda.stream(s2):
+            (g.delete if rep % 2 == 0 else g.insert)(dd, want_out=False, stream=s2.cuda_stream)
+        with torch.cuda.stream(s3):
+            su = torch.empty_like(dq)
+            pr = torch.empty_like(dq)
+            g.successor(dq, su, stream=s3.cuda_stream)
+            g.predecessor(dq, pr, stream=s3.cuda_stream)
+            me = g.member(_dev(stable[:4096]), stream=s3.cuda_stream)
+            outs.append((su, pr, me))
+        torch.cuda.synchronize()
+    st = np.sort(stable)
+    allowed = np.sort(keys)
+    NONE64 = np.uint64(NONE)
+    i_ge = np.searchsorted(st, q, side="left")
+    succ_stable = np.where(i_ge < len(st), st[np.minimum(i_ge, len(st) - 1)], NONE64)
+    i_le = np.searchsorted(st, q, side="right") - 1
+    pred_stable = np.where(i_le >= 0, st[np.maximum(i_le, 0)], NONE64)
+    for su, pr, me in outs:
+        s, p = _u64(su), _u64(pr)
+        none_s = s == NONE64
+        assert np.all(succ_stable[none_s] == NONE64)
+        ok = ~none_s
+        assert np.all(s[ok] >= q[ok]) and np.all(s[ok] <= succ_stable[ok])
+        assert np.all(np.isin(s[ok], allowed))
+        none_p = p == NONE64
+        assert np.all(pred_stable[none_p] == NONE64)
+        okp = ~none_p
+        assert np.all(p[okp] <= q[okp]) and np.all((pred_stable[okp] == NONE64) | (p[okp] >= pred_stable[okp]))
+        assert np.all(np.isin(p[okp], allowed))
+        assert np.all(me.cpu().numpy() == 1)
+    # quiescent: after 4 rounds vol_in was inserted then deleted twice, vol_out the reverse
+    o = oracle.Veb(k)
+    o.batch(OV_INSERT, np.concatenate([stable, vol_out]))
+    assert np.array_equal(g.snapshot(), o.image())
+    g.close()
