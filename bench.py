@@ -537,6 +537,12 @@ def run_graph(args, G, torch, stream):
     size, cap, _ = g.export()
     res["expansion"]["edges"] = int(size.sum()) - before
     res["expansion"]["edges_per_s"] = res["expansion"]["edges"] / res["expansion"]["ms"] * 1e3
+    # P:355's non-bulk variants: one thread per edge under a vertex lock, on
+    # 2^22 edges of the stream (re-inserted, then deleted one at a time)
+    ne = min(1 << 22, w["insert"][0][0].numel())
+    es, ed = w["insert"][0][0][:ne].contiguous(), w["insert"][0][1][:ne].contiguous()
+    timed("edge_insert", lambda: g.insert_edges(es, ed), ne)
+    timed("edge_delete", lambda: g.delete_edges(es, ed), ne)
     ctr = g.counters()
     total_ms = sum(v["ms"] for v in res.values())
     g.destroy()
@@ -545,7 +551,8 @@ def run_graph(args, G, torch, stream):
     G.gallatin_destroy()
     G.gallatin_init(HEAP_C2)
     return {"workload": f"BASELINE configs[4]: R-MAT 2^{scale} vertices / 2^{scale + 4} edges, (a,b,c,d)="
-                        "(0.57,0.19,0.19,0.05), 8 insert + 8 delete batches, 2^16-vertex x 8-round expansion, 16 GiB heap",
+                        "(0.57,0.19,0.19,0.05), 8 insert + 8 delete batches, 2^16-vertex x 8-round expansion, "
+                        "2^22 single-edge inserts + deletes, 16 GiB heap",
             "phases": res, "device_mallocs": ctr["mallocs"], "device_frees": ctr["frees"],
             "failed_mallocs": ctr["failed"], "allocator_ops_per_s": (ctr["mallocs"] + ctr["frees"]) / total_ms * 1e3,
             "pristine_after_teardown": st["free_segments"] == st["num_segments"]}

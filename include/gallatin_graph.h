@@ -44,6 +44,20 @@ int gallatin_graph_delete(gallatin_graph_t *g, const uint32_t *d_src, const uint
  * (v + size_before + j + 1) mod num_vertices. */
 int gallatin_graph_expand(gallatin_graph_t *g, const uint32_t *d_v, uint64_t n, void *stream);
 
+/* Single-edge operations ("edge updates" / "edge deletes", as opposed
+ * to the bulk batches above): one GPU thread per edge, each under its source
+ * vertex's lock.  insert_edges appends d_dst[i] to the list of d_src[i]; a
+ * full list (size == cap) is reallocated to 2*cap (4 if empty) at that edge.
+ * delete_edges removes ONE instance of d_dst[i] from the list of d_src[i] if
+ * present (the newest such entry; the last entry fills the hole); after each removal size 0 frees
+ * the list and size <= cap/4 (cap > 4) reallocates it to nextpow2(max(size, 4)).
+ * Final sizes, capacities and adjacency multisets are independent of the
+ * thread order (reading A-29 per edge).  Asynchronous on `stream`. */
+int gallatin_graph_insert_edges(gallatin_graph_t *g, const uint32_t *d_src, const uint32_t *d_dst, uint64_t n,
+                                void *stream);
+int gallatin_graph_delete_edges(gallatin_graph_t *g, const uint32_t *d_src, const uint32_t *d_dst, uint64_t n,
+                                void *stream);
+
 /* Per-vertex size, capacity and list pointer (any may be NULL). */
 int gallatin_graph_export(const gallatin_graph_t *g, uint32_t *d_size, uint32_t *d_cap, uint64_t *d_list, void *stream);
 /* CSR copy: d_out[d_offsets[v] + k] = list_v[k] for k < size_v (caller gives

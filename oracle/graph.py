@@ -10,6 +10,8 @@ per vertex (reading A-29):
                  -> cap = nextpow2(max(size, 4))
   expand round : every listed vertex appends max(size, 4) edges, edge j to
                  (v + size_before + j + 1) mod V; grow as for inserts.
+  single edges : the same rules applied after every edge (insert_edges /
+                 delete_edges; P:355's non-bulk "edge updates" and deletes).
 The adjacency is kept as a multiset of keys src << 32 | dst (numpy).
 """
 from __future__ import annotations
@@ -64,6 +66,44 @@ class GraphOracle:
         small = touched & (self.size > 0) & (self.size <= self.cap // 4) & (self.cap > 4)
         self.cap[small] = list_cap(self.size[small])
 
+    def insert_edges(self, src: np.ndarray, dst: np.ndarray) -> None:
+        """Single-edge inserts: a full list doubles at the edge that finds it
+        full (0 -> 4 -> 8 ...); cap ends at the smallest power of two >= size
+        reachable by doubling, which for caps that are 0 or powers of two >= 4
+        is max(cap, nextpow2(max(size, 4)))."""
+        c = np.bincount(np.asarray(src, dtype=np.int64), minlength=self.V)
+        need = self.size + c
+        grow = (c > 0) & (need > self.cap)
+        cap = np.where(self.cap == 0, 4, self.cap)
+        while True:                                      # doubling, step by step
+            g = grow & (need > cap)
+            if not g.any():
+                break
+            cap = np.where(g, cap * 2, cap)
+        self.cap = np.where(grow, cap, self.cap)
+        self.size = need
+        self.keys = np.concatenate([self.keys, self._key(src, dst)])
+
+    def delete_edges(self, src: np.ndarray, dst: np.ndarray) -> None:
+        """Single-edge deletes: the per-vertex sizes go down one removal at a
+        time; after each, size 0 frees the list (cap 0) and size <= cap/4 with
+        cap > 4 reallocates to nextpow2(max(size, 4)).  Starting from
+        size > cap/4 the shrinks happen when size reaches cap/4, so the final
+        cap follows from the final size alone (iterated below)."""
+        s0 = self.size.copy()
+        cap0 = self.cap.copy()
+        self.delete(src, dst)                            # multiset + sizes (caps recomputed below)
+        s1 = self.size
+        cap = cap0.copy()
+        moved = s1 < s0
+        while True:
+            sh = moved & (cap > 4) & (s1 <= cap // 4)
+            if not sh.any():
+                break
+            cap = np.where(sh, list_cap(cap // 4), cap)
+        cap = np.where(moved & (s1 == 0), 0, cap)
+        self.cap = np.where(moved, cap, cap0)
+
     def expand(self, vertices: np.ndarray) -> None:
         v = np.asarray(vertices, dtype=np.int64)
         s0 = self.size[v]
@@ -114,6 +154,23 @@ class BruteGraph:
             if n == 0:
                 self.cap[s] = 0
             elif n <= self.cap[s] // 4 and self.cap[s] > 4:
+                self.cap[s] = self._cap(n)
+
+    def insert_edges(self, src, dst):
+        for s, d in zip(src.tolist(), dst.tolist()):
+            if len(self.lists[s]) == self.cap[s]:
+                self.cap[s] = 4 if self.cap[s] == 0 else 2 * self.cap[s]
+            self.lists[s].append(d)
+
+    def delete_edges(self, src, dst):
+        for s, d in zip(src.tolist(), dst.tolist()):
+            if d not in self.lists[s]:
+                continue
+            self.lists[s].remove(d)
+            n = len(self.lists[s])
+            if n == 0:
+                self.cap[s] = 0
+            elif self.cap[s] > 4 and n <= self.cap[s] // 4:
                 self.cap[s] = self._cap(n)
 
     def expand(self, vertices):

@@ -337,6 +337,8 @@ def _graph_sigs(L):
         "gallatin_graph_create": ([u32, ctypes.POINTER(vp)], i32),
         "gallatin_graph_destroy": ([vp, vp], i32),
         "gallatin_graph_insert": ([vp, vp, vp, u64, vp], i32),
+        "gallatin_graph_insert_edges": ([vp, vp, vp, u64, vp], i32),
+        "gallatin_graph_delete_edges": ([vp, vp, vp, u64, vp], i32),
         "gallatin_graph_delete": ([vp, vp, vp, u64, vp], i32),
         "gallatin_graph_expand": ([vp, vp, u64, vp], i32),
         "gallatin_graph_export": ([vp, vp, vp, vp, vp], i32),
@@ -380,6 +382,16 @@ class Graph:
     def delete(self, src, dst, stream=None):
         check(lib().gallatin_graph_delete(self._h, _dptr4(src), _dptr4(dst), src.numel(), _stream(stream)),
               "gallatin_graph_delete")
+
+    def insert_edges(self, src, dst, stream=None):
+        """Single-edge inserts (one thread per edge under a vertex lock)."""
+        check(lib().gallatin_graph_insert_edges(self._h, _dptr4(src), _dptr4(dst), src.numel(), _stream(stream)),
+              "gallatin_graph_insert_edges")
+
+    def delete_edges(self, src, dst, stream=None):
+        """Single-edge deletes (one thread per edge under a vertex lock)."""
+        check(lib().gallatin_graph_delete_edges(self._h, _dptr4(src), _dptr4(dst), src.numel(), _stream(stream)),
+              "gallatin_graph_delete_edges")
 
     def expand(self, vertices, stream=None):
         check(lib().gallatin_graph_expand(self._h, _dptr4(vertices), vertices.numel(), _stream(stream)),

@@ -25,6 +25,7 @@ struct gallatin_graph {
     uint64_t *hkeys;      // delete-batch hash: (src << 32 | dst) -> remaining count
     uint32_t *hcnt;
     uint64_t hcap;
+    uint32_t *lock;       // per-vertex lock word of the single-edge operations
 };
 
 namespace {
@@ -332,6 +333,120 @@ __global__ void k_gather(gallatin_graph g, const uint64_t *off, uint32_t *out) {
     }
 }
 
+// ---- single-edge operations ("edge updates" / "edge deletes") ---------
+// One thread per edge, each under its source vertex's lock: the list grows by
+// doubling when an append finds it full (malloc, copy, free: the allocator is
+// called per overflowing edge, not per batch) and shrinks after every delete
+// that leaves size <= cap/4 (reading A-29 applied per edge).
+__device__ __forceinline__ void vlock(uint32_t *l) {
+    uint32_t ns = 32;
+    while (atomicCAS(l, 0u, 1u) != 0u) {
+        __nanosleep(ns);
+        if (ns < 256) ns <<= 1;
+    }
+    __threadfence();                                      // acquire the previous holder's writes
+}
+__device__ __forceinline__ void vunlock(uint32_t *l) {
+    __threadfence();                                      // release this holder's writes
+    atomicExch(l, 0u);
+}
+__device__ __forceinline__ void copy_list(uint32_t *dst, const uint32_t *src, uint32_t n) {
+    // both lists hold a multiple of 4 entries (caps are powers of two >= 4)
+    uint4 *d = reinterpret_cast<uint4 *>(dst);
+    const uint4 *s = reinterpret_cast<const uint4 *>(src);
+    for (uint32_t k = 0; k < (n + 3) / 4; k++) d[k] = s[k];
+}
+
+__global__ void __launch_bounds__(kT, kGraphMinBlocks) k_edge_insert(gallatin_graph g, const uint32_t *src,
+                                                                      const uint32_t *dst, uint64_t n) {
+    const uint64_t i = blockIdx.x * (uint64_t)kT + threadIdx.x;
+    bool m = false, f = false, fail = false;
+    if (i < n) {
+        const uint32_t v = src[i], x = dst[i];
+        vlock(g.lock + v);
+        const uint32_t s = g.size[v], c = g.cap[v];
+        uint32_t *L = reinterpret_cast<uint32_t *>(g.list[v]);
+        bool ok = true;
+        if (s == c) {                                      // full (or no list): double
+            const uint32_t nc = c ? 2 * c : 4;
+            uint32_t *p = static_cast<uint32_t *>(gallatin_malloc((uint64_t)nc * 4));
+            if (!p) {
+                ok = false;
+                fail = true;
+            } else {
+                m = true;
+                if (L) {
+                    copy_list(p, L, s);
+                    gallatin_free(L);
+                    f = true;
+                }
+                g.list[v] = reinterpret_cast<uint64_t>(p);
+                g.cap[v] = nc;
+                L = p;
+            }
+        }
+        if (ok) {
+            L[s] = x;
+            g.size[v] = s + 1;
+        }
+        vunlock(g.lock + v);
+    }
+    count_warp(g.ctr, m, f, fail);
+}
+
+__global__ void __launch_bounds__(kT, kGraphMinBlocks) k_edge_delete(gallatin_graph g, const uint32_t *src,
+                                                                      const uint32_t *dst, uint64_t n) {
+    const uint64_t i = blockIdx.x * (uint64_t)kT + threadIdx.x;
+    bool m = false, f = false, fail = false;
+    if (i < n) {
+        const uint32_t v = src[i], x = dst[i];
+        vlock(g.lock + v);
+        uint32_t s = g.size[v];
+        const uint32_t c = g.cap[v];
+        uint32_t *L = reinterpret_cast<uint32_t *>(g.list[v]);
+        // newest entries first (appends go to the end): remove one instance,
+        // the last entry fills the hole
+        uint32_t j = 0;
+        bool hit = false;
+        if (s) {
+            const uint4 *L4 = reinterpret_cast<const uint4 *>(L);      // 16 B loads (lists are 16 B aligned)
+            for (int64_t q = (int64_t)(s - 1) / 4; q >= 0 && !hit; q--) {
+                const uint4 e = L4[q];
+                const uint32_t b = 4 * (uint32_t)q;
+                if (b + 3 < s && e.w == x) { j = b + 3; hit = true; }
+                else if (b + 2 < s && e.z == x) { j = b + 2; hit = true; }
+                else if (b + 1 < s && e.y == x) { j = b + 1; hit = true; }
+                else if (e.x == x) { j = b; hit = true; }
+            }
+        }
+        if (hit) {
+            L[j] = L[s - 1];
+            s--;
+            g.size[v] = s;
+            if (s == 0) {
+                gallatin_free(L);
+                g.list[v] = 0;
+                g.cap[v] = 0;
+                f = true;
+            } else if (c > 4 && s <= c / 4) {
+                const uint32_t nc = list_cap(s);
+                uint32_t *p = static_cast<uint32_t *>(gallatin_malloc((uint64_t)nc * 4));
+                if (p) {
+                    copy_list(p, L, s);
+                    gallatin_free(L);
+                    g.list[v] = reinterpret_cast<uint64_t>(p);
+                    g.cap[v] = nc;
+                    m = f = true;
+                } else {
+                    fail = true;
+                }
+            }
+        }
+        vunlock(g.lock + v);
+    }
+    count_warp(g.ctr, m, f, fail);
+}
+
 int run_grow(gallatin_graph *g, cudaStream_t st) {
     k_grow<<<blocks(g->V), kT, 0, st>>>(*g);
     k_copy<<<148 * 8, kT, 0, st>>>(*g);
@@ -352,7 +467,7 @@ int gallatin_graph_create(uint32_t V, gallatin_graph_t **out) {
               cudaMalloc(&g->cap, 4ull * V) == cudaSuccess && cudaMalloc(&g->cnt, 4ull * V) == cudaSuccess &&
               cudaMalloc(&g->old, 8ull * V) == cudaSuccess && cudaMalloc(&g->work, 4ull * V) == cudaSuccess &&
               cudaMalloc(&g->work2, 4ull * V) == cudaSuccess && cudaMalloc(&g->nwork, 8) == cudaSuccess &&
-              cudaMalloc(&g->ctr, 24) == cudaSuccess;
+              cudaMalloc(&g->ctr, 24) == cudaSuccess && cudaMalloc(&g->lock, 4ull * V) == cudaSuccess;
     if (!ok) {
         cudaGetLastError();
         gallatin_graph_destroy(g, nullptr);
@@ -362,6 +477,7 @@ int gallatin_graph_create(uint32_t V, gallatin_graph_t **out) {
     cudaMemset(g->size, 0, 4ull * V);
     cudaMemset(g->cap, 0, 4ull * V);
     cudaMemset(g->ctr, 0, 24);
+    cudaMemset(g->lock, 0, 4ull * V);
     *out = g;
     return status();
 }
@@ -370,7 +486,8 @@ int gallatin_graph_destroy(gallatin_graph_t *g, void *stream) {
     if (!g) return GALLATIN_ERR_INVALID;
     if (g->list && gallatin_is_initialized()) k_free_all<<<blocks(g->V), kT, 0, S(stream)>>>(*g);
     cudaStreamSynchronize(S(stream));
-    void *ptrs[] = {g->list, g->size, g->cap, g->cnt, g->old, g->work, g->work2, g->nwork, g->ctr, g->hkeys, g->hcnt};
+    void *ptrs[] = {g->list, g->size, g->cap, g->cnt, g->old, g->work, g->work2, g->nwork, g->ctr, g->hkeys, g->hcnt,
+                    g->lock};
     for (void *p : ptrs)
         if (p) cudaFree(p);
     delete g;
@@ -432,6 +549,22 @@ int gallatin_graph_expand(gallatin_graph_t *g, const uint32_t *vs, uint64_t n, v
     int rc = run_grow(g, st);
     if (rc) return rc;
     k_expand_fill<<<148 * 8, kT, 0, st>>>(*g, vs, n);
+    return status();
+}
+
+int gallatin_graph_insert_edges(gallatin_graph_t *g, const uint32_t *src, const uint32_t *dst, uint64_t n,
+                                void *stream) {
+    if (!g || (n && (!src || !dst))) return GALLATIN_ERR_INVALID;
+    if (n == 0) return GALLATIN_OK;
+    k_edge_insert<<<blocks(n), kT, 0, S(stream)>>>(*g, src, dst, n);
+    return status();
+}
+
+int gallatin_graph_delete_edges(gallatin_graph_t *g, const uint32_t *src, const uint32_t *dst, uint64_t n,
+                                void *stream) {
+    if (!g || (n && (!src || !dst))) return GALLATIN_ERR_INVALID;
+    if (n == 0) return GALLATIN_OK;
+    k_edge_delete<<<blocks(n), kT, 0, S(stream)>>>(*g, src, dst, n);
     return status();
 }
 

@@ -79,3 +79,35 @@ def test_graph_phases_match_o3(cuda_ok, scale, n):
         assert int(img[6]) == 0
     finally:
         G.gallatin_destroy()
+
+
+@pytest.mark.parametrize("scale,n", [(12, 1 << 16), (16, 1 << 20)])
+def test_graph_single_edge_ops_match_o3(cuda_ok, scale, n):
+    """P:355's non-bulk edge updates and deletes (one thread per edge under a
+    vertex lock, the allocator called per overflowing / shrinking edge),
+    interleaved with bulk batches: sizes, capacities, adjacency multisets and
+    list bytes equal O3's per-edge trajectory; the heap is pristine after
+    teardown."""
+    import paper_conf_ppopp_mccoyp24_b200 as G
+    nseg = 512
+    G.gallatin_init(nseg * SEG)
+    try:
+        w = wg.graph_workload(scale, n, device="cuda", seed=scale + 11)
+        V = w["V"]
+        g = G.Graph(V)
+        o = GraphOracle(V)
+        steps = [("insert", w["init"]), ("insert_edges", w["insert"][0]), ("delete_edges", w["delete"][0]),
+                 ("insert", w["insert"][1]), ("delete_edges", w["delete"][1]), ("delete", w["delete"][2]),
+                 ("insert_edges", w["insert"][2]), ("delete_edges", w["delete"][3])]
+        for kind, (s, d) in steps:
+            getattr(g, kind)(s, d)
+            getattr(o, kind)(_np(s), _np(d))
+            _check(G, g, o, V, kind)
+        assert g.counters()["failed"] == 0
+        g.destroy()
+        G.gallatin_drain()
+        img = G.gallatin_snapshot()
+        msg = diff_images(img, pristine_image(nseg, int(img[4])))
+        assert not msg, msg
+    finally:
+        G.gallatin_destroy()
