@@ -108,14 +108,19 @@ __device__ inline uint64_t bt_successor(const BitTree &t, uint64_t x) {
     for (;;) {
         if (x >= t.nbits) return kNone;
         uint64_t idx = x >> 6;
-        uint64_t w = bt_load<NC>(t.w + t.off[0] + idx) & (~0ull << (x & 63));
+        // allocator trees (coherent loads, mostly-empty leaves): the leaf and
+        // the first summary word on the path are independent loads, issued
+        // together (one round trip, not two); bulk queries (NC) load lazily
+        const uint64_t w0 = bt_load<NC>(t.w + t.off[0] + idx);
+        const uint64_t s1 = (!NC && t.levels > 1) ? bt_load<NC>(t.w + t.off[1] + (idx >> 6)) : 0;
+        const uint64_t w = w0 & (~0ull << (x & 63));
         if (w) return (idx << 6) + (uint64_t)(__ffsll((long long)w) - 1);
         uint32_t lvl = 1;
         for (; lvl < t.levels; lvl++) {
             const uint32_t pos = (uint32_t)(idx & 63);
             const uint64_t p = idx >> 6;
             const uint64_t m = pos == 63 ? 0 : (~0ull << (pos + 1));
-            const uint64_t s = m ? (bt_load<NC>(t.w + t.off[lvl] + p) & m) : 0;
+            const uint64_t s = m ? (((!NC && lvl == 1) ? s1 : bt_load<NC>(t.w + t.off[lvl] + p)) & m) : 0;
             idx = p;
             if (s) { idx = (p << 6) + (uint64_t)(__ffsll((long long)s) - 1); break; }
         }

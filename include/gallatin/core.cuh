@@ -311,8 +311,15 @@ __device__ inline __noinline__ uint32_t take_segments(const View &v, uint32_t t,
     const uint32_t nb = nb_of(t);
     uint32_t k = 0;
     const uint32_t kmax = want / nb;
+#ifdef GALLATIN_TRACE
+    const uint64_t tr0 = ptx::globaltimer();
+#endif
     const uint64_t s0 = claim_front_run(v, kmax, &k);
     if (s0 == kNone) return 0;
+#ifdef GALLATIN_TRACE
+    const uint64_t tr1 = ptx::globaltimer();
+    ptx::trace(tr0, tr1, (1ull << 60) | ((uint64_t)t << 24) | k);
+#endif
     const BitTree st = seg_tree(v);
     // extend with the following free segments: one atomicAnd per leaf
     // word claims the whole window, the consecutive prefix is kept and
@@ -335,10 +342,15 @@ __device__ inline __noinline__ uint32_t take_segments(const View &v, uint32_t t,
         k += run;
         if (lo + run < hi) break;                         // the free run ended here
     }
+    // tree ids (table words and the read-mostly copies) for the free path;
+    // both are read only through a pointer this run hands out, so one fence
+    // before the run is published (refill_slot's exchange) orders them all
     for (uint32_t q = 0; q < k; q++) ptx::st_relaxed(v.seg_tid + s0 + q, t);
-    ptx::fence_acq_rel();
     for (uint32_t q = 0; q < k; q++) ptx::atom_add(v.seg_word + s0 + q, sw_retree(kTreeFree, t));
     ptx::fence_acq_rel();
+#ifdef GALLATIN_TRACE
+    ptx::trace(tr1, ptx::globaltimer(), (2ull << 60) | ((uint64_t)t << 24) | k);
+#endif
     *first = (uint32_t)(s0 * nb);
     return k * nb;
 }
@@ -554,7 +566,13 @@ __device__ inline __noinline__ uint32_t trim_slots(const View &v) {
 // more after an empty trim: a concurrent refiller's trim may just have given
 // the blocks back.  Serially this is one trim and one retry.
 __device__ inline __noinline__ uint32_t get_run(const View &v, uint32_t t, uint32_t want, uint32_t *first) {
+#ifdef GALLATIN_TRACE
+    const uint64_t tr0 = ptx::globaltimer();
     uint32_t got = get_run_once(v, t, want, first);
+    ptx::trace(tr0, ptx::globaltimer(), (3ull << 60) | ((uint64_t)t << 24) | (want << 12) | got);
+#else
+    uint32_t got = get_run_once(v, t, want, first);
+#endif
     for (uint32_t r = 0; got == 0 && r < 8; r++) {
         const uint32_t back = trim_slots(v);
         got = get_run_once(v, t, 1, first);

@@ -242,6 +242,12 @@ __global__ void __launch_bounds__(kThreads, 5) k_bulk_malloc_cta(const uint64_t 
     __shared__ uint64_t olds[core::kTrees];
     const uint32_t lane = threadIdx.x & 31;
     const uint64_t base = blockIdx.x * (uint64_t)(kThreads * ITEMS) + threadIdx.x;
+#ifdef GALLATIN_TRACE
+    if (threadIdx.x == 0 && (blockIdx.x == 0 || blockIdx.x == gridDim.x - 1)) {
+        const uint64_t tk = ptx::globaltimer();
+        ptx::trace(tk, tk, (7ull << 60) | blockIdx.x);
+    }
+#endif
     const uint32_t key = ptx::smid();
     if (threadIdx.x < core::kTrees) cnt[threadIdx.x] = 0;
     // per item: class (0..8 slice class, 0xFE nothing to do, 0xFF block or
