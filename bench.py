@@ -478,6 +478,8 @@ def run_scaling(args, G, torch, stream):
         pp = {}
         for lg in range(10, 21, 2):
             n = max(1024, (1 << lg) // args.scale)
+            if size == 8192 and n * 65536 > HEAP_C2 // 2:
+                continue                        # 8 KB takes a 64 KB block (A-2): > half the heap
             st = torch.full((n,), size, dtype=torch.int64, device="cuda")
             p = torch.empty_like(st)
             mm, fm = [], []

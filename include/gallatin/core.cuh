@@ -702,11 +702,33 @@ __device__ inline void *malloc_slice(const View &v, uint32_t c, uint32_t key) {
 
 // (4 KB, 16 MB): one whole block of the smallest fitting tree; its counter is
 // preset to 4095 so that Alg.4's rule returns it on its one free (reading A-2).
+// [dev] The lanes of a warp asking the same block tree form a team (the
+// paper's coalescing, applied to whole blocks): the team's lowest
+// unserved lane asks GetBlock for as many blocks as lanes remain and the run
+// it gets is dealt out in lane order, until every lane has a block or the
+// tree is exhausted.  A lone request is exactly GetBlock(t) (serial replay).
 __device__ inline __noinline__ void *malloc_block(const View &v, uint32_t t) {
-    uint32_t first = 0;
-    if (get_run(v, t, 1, &first) == 0) return nullptr;
-    atomicExch(v.block_free + gid_of(t, first), kSlices - 1);
-    return reinterpret_cast<void *>(v.heap + ((uint64_t)first << (16 + t)));
+    const unsigned peers = __match_any_sync(__activemask(), t);
+    const uint32_t lane = ptx::lane_id();
+    unsigned pending = peers;
+    void *res = nullptr;
+    while (pending) {
+        const uint32_t leader = (uint32_t)__ffs((int)pending) - 1;
+        uint32_t first = 0, got = 0;
+        if (lane == leader) got = get_run(v, t, (uint32_t)__popc(pending), &first);
+        got = __shfl_sync(peers, got, (int)leader);
+        first = __shfl_sync(peers, first, (int)leader);
+        if (got == 0) break;                                   // "No allocations left"
+        const uint32_t r = (uint32_t)__popc(pending & ptx::lanemask_lt());
+        if (((pending >> lane) & 1) && r < got) {
+            atomicExch(v.block_free + gid_of(t, (uint64_t)first + r), kSlices - 1);
+            res = reinterpret_cast<void *>(v.heap + (((uint64_t)first + r) << (16 + t)));
+        }
+        unsigned served = pending;                            // the lowest `got` pending lanes
+        for (uint32_t k = got; k < (uint32_t)__popc(pending); k++) served &= ~(1u << (31 - __clz((int)served)));
+        pending &= ~served;
+    }
+    return res;
 }
 
 // >= 16 MB: Alg.1 with treeId >= numBlockTrees: claimMultiple from the back

@@ -303,3 +303,25 @@ def test_bulk_kernels_unaligned_arrays(cuda_ok, G):
         G.gallatin_free(ptrs)
         _assert_pristine(G, nseg)
         G.gallatin_destroy()
+
+
+@pytest.mark.parametrize("size,n", [(8192, 1 << 16), (65537, 1 << 12), (3 << 20, 1 << 10)])
+def test_block_path_teams(cuda_ok, G, size, n):
+    """Whole-block requests (A-2) from every lane of every warp: the lanes
+    asking one block tree share GetBlock runs (P:190 coalescing applied to
+    blocks).  Stamp-verified, accounted, overlap-checked, pristine after."""
+    nseg = 1024
+    G.gallatin_init(nseg * SEG)
+    assert _bulk_round(G, nseg, wg.single_sizes(size, n)) == 0
+    _assert_pristine(G, nseg)
+
+
+def test_block_path_mixed_tail(cuda_ok, G):
+    """Block sizes mixed with slices in every warp, ragged count."""
+    nseg = 1024
+    G.gallatin_init(nseg * SEG)
+    rng = np.random.Generator(np.random.PCG64(11))
+    n = (1 << 16) + 123
+    sizes = np.where(rng.random(n) < 0.5, rng.integers(4097, 1 << 18, n), rng.integers(1, 4097, n)).astype(np.uint64)
+    assert _bulk_round(G, nseg, sizes) == 0
+    _assert_pristine(G, nseg)
