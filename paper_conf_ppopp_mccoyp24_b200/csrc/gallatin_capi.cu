@@ -234,8 +234,8 @@ __global__ void __launch_bounds__(kThreads, 5) k_bulk_malloc(const uint64_t *__r
 // global RMW per class per CTA takes their slices (1024 requests at
 // ITEMS=4), so the hot slot words see 32x fewer RMWs than with warp teams.
 // Item k of thread t is request blockIdx*256*ITEMS + k*256 + t.
-template <int ITEMS>
-__global__ void __launch_bounds__(kThreads, 5) k_bulk_malloc_cta(const uint64_t *__restrict__ sizes,
+template <int ITEMS, int MINB = 5>
+__global__ void __launch_bounds__(kThreads, MINB) k_bulk_malloc_cta(const uint64_t *__restrict__ sizes,
                                                                   void **__restrict__ ptrs, uint64_t n) {
     const View &v = c_view;
     __shared__ uint32_t cnt[core::kTrees];
@@ -1023,6 +1023,7 @@ int gallatin_malloc(const uint64_t *d_sizes, void **d_ptrs, uint64_t n, void *st
         k_bulk_malloc_cta<8><<<grid_for((n + 7) / 8), kThreads, 0, S(stream)>>>(d_sizes, d_ptrs, n);
     else if (items == 4)
         k_bulk_malloc_cta<4><<<grid_for((n + 3) / 4), kThreads, 0, S(stream)>>>(d_sizes, d_ptrs, n);
+
     else
         k_bulk_malloc<1><<<grid_for(n), kThreads, 0, S(stream)>>>(d_sizes, d_ptrs, n);
     return launch_status();
