@@ -79,6 +79,9 @@ typedef struct gallatin_config {
                               this tile's atomics are in flight; 0/2 = one tile per CTA (default, measured faster) */
     uint32_t free_team;    /* bulk free: 0/2 = one free-counter RMW per warp team (default, measured faster);
                               1 = one per block per CTA tile (shared-memory aggregation) */
+    uint32_t demand_hint;  /* bulk malloc: 0/1 = a refill takes at least the blocks this slot's share of the launch
+                              needs (the CTA's per-class count x CTAs / slots; DESIGN.md Deviations 10), up to the
+                              run cap (default); 2 = off (runs grow 2^run_grow-fold per refill only) */
 } gallatin_config_t;
 
 int gallatin_init(uint64_t heap_bytes);                 /* defaults for the rest */

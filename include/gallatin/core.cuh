@@ -90,6 +90,70 @@ __device__ inline __noinline__ void btree_reconcile(const View &v, uint32_t t, u
 
 __device__ inline __noinline__ void try_free_segment(const View &v, uint64_t s, uint32_t t);
 
+// ---- exhaustion record [dev] (DESIGN.md Deviations 11) ----------------------
+// Without it every request that finds the heap exhausted repeats the whole
+// confirmation (slot trims, table scans) before reporting NULL: a bulk call
+// asking 2x the heap took minutes.  A request whose run search for tree t
+// failed announces itself (searchers + 1), repeats the search to the end and,
+// if that fails too, records "tree t exhausted in epoch e" -- unless an epoch
+// bump happened meanwhile.  Every RMW that makes blocks or segments available
+// (block return, segment free, format, give-backs of reservations and claim
+// windows) is followed by oom_notify: a fence.sc, then -- only if a search is
+// in flight or a record exists -- one epoch bump.  The fence pair (the
+// searcher's after its announce, the notifier's after its RMW) forbids the
+// store-buffer outcome in which neither sees the other, so a record is never
+// left standing for memory that became available after the search began.
+// Later requests of tree t fail in O(1) while the record's epoch is current.
+constexpr uint64_t kOomFlagMask = 0x3FFull;               // bits 0..9: tree t recorded this epoch
+constexpr uint64_t kOomOne = 1ull << 10;                  // searchers: bits 10..31
+constexpr uint64_t kOomEpoch = 1ull << 32;
+
+__device__ __forceinline__ bool oom_known(const View &v, uint32_t t) {
+    const uint64_t r = ptx::ld_relaxed(v.oom);
+    const uint64_t rec = ptx::ld_relaxed(v.oom + 1 + t);
+    return (r & (1ull << t)) && rec == (r >> 32) + 1;
+}
+
+__device__ inline __noinline__ void oom_notify_slow(const View &v, uint64_t w) {
+    while (w & 0xFFFFFFFFull) {                              // a search in flight or a record
+        const uint64_t o = ptx::atom_cas(v.oom, w, (w + kOomEpoch) & ~kOomFlagMask);
+        if (o == w || (o >> 32) != (w >> 32)) return;         // bumped (by us or after our fence)
+        w = o;
+    }
+}
+__device__ __forceinline__ void oom_notify(const View &v) {
+    ptx::fence_sc();
+    const uint64_t w = ptx::ld_relaxed(v.oom);
+    if (w & 0xFFFFFFFFull) oom_notify_slow(v, w);
+}
+
+// announce a confirming search
+__device__ __forceinline__ void oom_enter(const View &v) {
+    ptx::atom_add(v.oom, kOomOne);
+    ptx::fence_sc();
+}
+// the epoch a search step starts in (acquire: it sees every RMW whose notify
+// bumped the epoch up to this value)
+__device__ __forceinline__ uint64_t oom_epoch(const View &v) {
+    const uint64_t e = ptx::ld_relaxed(v.oom) >> 32;
+    ptx::fence_acq_rel();
+    return e;
+}
+// the search of tree t in epoch e failed: record it unless the epoch moved;
+// then leave the searchers
+__device__ inline __noinline__ void oom_leave(const View &v, uint32_t t, uint64_t e, bool failed) {
+    if (failed) {
+        uint64_t w = ptx::ld_relaxed(v.oom);
+        while ((w >> 32) == e && !(w & (1ull << t))) {
+            const uint64_t o = ptx::atom_cas(v.oom, w, w | (1ull << t));
+            if (o == w) { w |= 1ull << t; break; }
+            w = o;
+        }
+        if ((w >> 32) == e) ptx::st_relaxed(v.oom + 1 + t, e + 1);
+    }
+    ptx::atom_add(v.oom, (uint64_t)(-(int64_t)kOomOne));
+}
+
 // Every thread whose RMW on seg_word[s] changed a block-tree predicate repairs
 // that bit; the RMW that brings a segment back to "all blocks home" retires it.
 __device__ __forceinline__ void seg_after_rmw(const View &v, uint64_t s, uint64_t old, uint64_t now) {
@@ -116,6 +180,7 @@ __device__ inline __noinline__ void try_free_segment(const View &v, uint64_t s, 
     ptx::fence_acq_rel();
     btree_reconcile(v, t, s);
     bt_insert(seg_tree(v), s);
+    oom_notify(v);
 }
 
 // Every formatted segment whose blocks are all home goes back to the segment
@@ -218,6 +283,7 @@ __device__ inline __noinline__ uint64_t claim_front_run(const View &v, uint32_t 
         bool flip = old != 0 && (old & ~mask) == 0;
         if (extra) flip |= ptx::atom_or(leaf, extra) == 0;
         if (flip) bt_reconcile_up(st, 0, wi);
+        if (extra) oom_notify(v);
         if (run == 0) {
             hint = claim_retry_hint(wi, old & ~mask, ++attempt);
             from = (wi + 1) << 6;
@@ -250,6 +316,7 @@ __device__ inline __noinline__ void format_segment(const View &v, uint64_t s, ui
     const uint64_t delta = sw_retree(kTreeFree, t) + (nb - keep);
     const uint64_t old = ptx::atom_add(v.seg_word + s, delta);
     seg_after_rmw(v, s, old, old + delta);
+    oom_notify(v);
 }
 
 // ---- block return (Alg.4; ring enqueue P:178) --------------------
@@ -263,6 +330,7 @@ __device__ inline __noinline__ void return_block(const View &v, uint32_t gid) {
     ptx::fence_acq_rel();
     const uint64_t old = ptx::atom_add(v.seg_word + s, 1ull);
     seg_after_rmw(v, s, old, old + 1);
+    oom_notify(v);
 }
 
 // n slices of block gid came back; the team completing 4096 returns it
@@ -339,6 +407,7 @@ __device__ inline __noinline__ uint32_t take_segments(const View &v, uint32_t t,
         bool flip = old != 0 && (old & ~mask) == 0;
         if (extra) flip |= ptx::atom_or(leaf, extra) == 0;
         if (flip) bt_reconcile_up(st, 0, wi);
+        if (extra) oom_notify(v);
         k += run;
         if (lo + run < hi) break;                         // the free run ended here
     }
@@ -398,6 +467,7 @@ __device__ inline __noinline__ uint32_t get_run_once(const View &v, uint32_t t, 
                     if (sw_in_tree(old, t) != sw_in_tree(old + dec, t) ||
                         sw_in_tree(o2, t) != sw_in_tree(o2 + (want - got), t))
                         btree_reconcile(v, t, s);
+                    oom_notify(v);
                 } else {
                     seg_after_rmw(v, s, old, old + dec);
                 }
@@ -456,6 +526,7 @@ __device__ inline __noinline__ uint32_t get_run_once(const View &v, uint32_t t, 
                     ptx::fence_acq_rel();
                     const uint64_t o3 = ptx::atom_add(v.seg_word + s, (uint64_t)r);
                     seg_after_rmw(v, s, o3, o3 + r);
+                    oom_notify(v);
                 }
                 *first = (uint32_t)(s * nb + bs);
                 return bl;
@@ -467,6 +538,7 @@ __device__ inline __noinline__ uint32_t get_run_once(const View &v, uint32_t t, 
             const uint64_t o2 = ptx::atom_add(v.seg_word + s, (uint64_t)want);
             seg_after_rmw(v, s, o2, o2 + want);
             btree_reconcile(v, t, s);
+            oom_notify(v);
             from = s + 1;
             hint = claim_retry_hint(s >> 6, ptx::ld_relaxed(bt.w + bt.off[0] + (s >> 6)) & ~(1ull << (s & 63)),
                                     ++attempt);
@@ -566,6 +638,7 @@ __device__ inline __noinline__ uint32_t trim_slots(const View &v) {
 // more after an empty trim: a concurrent refiller's trim may just have given
 // the blocks back.  Serially this is one trim and one retry.
 __device__ inline __noinline__ uint32_t get_run(const View &v, uint32_t t, uint32_t want, uint32_t *first) {
+    if (oom_known(v, t)) return 0;                            // [dev] exhaustion record
 #ifdef GALLATIN_TRACE
     const uint64_t tr0 = ptx::globaltimer();
     uint32_t got = get_run_once(v, t, want, first);
@@ -573,16 +646,24 @@ __device__ inline __noinline__ uint32_t get_run(const View &v, uint32_t t, uint3
 #else
     uint32_t got = get_run_once(v, t, want, first);
 #endif
+    if (got) return got;
+    oom_enter(v);
+    uint64_t e = 0;
     for (uint32_t r = 0; got == 0 && r < 8; r++) {
-        const uint32_t back = trim_slots(v);
+        const uint32_t back = trim_slots(v);                  // its block returns bump the epoch
+        e = oom_epoch(v);
         got = get_run_once(v, t, 1, first);
         if (back == 0 && r >= 1) break;
     }
+    oom_leave(v, t, e, got == 0);
     return got;
 }
 
 // Replace an exhausted run (Alg.3): the run doubles up to the class cap.
-__device__ inline __noinline__ bool refill_slot(const View &v, uint32_t si, uint32_t c, uint32_t m_prev) {
+// [dev] `hint` (bulk calls only): the blocks this slot's share of the launch
+// needs (DESIGN.md Deviations 10); the run is at least that long, up to the cap.
+__device__ inline __noinline__ bool refill_slot(const View &v, uint32_t si, uint32_t c, uint32_t m_prev,
+                                                uint32_t hint = 0) {
     if (v.prefetch) {                                         // [dev] the prefetched run, if any
         const uint64_t nx = ptx::atom_exch(slot_word(v, si) + 1, kSlotEmpty);
         if (run_len(nx) != 0) {
@@ -597,7 +678,8 @@ __device__ inline __noinline__ bool refill_slot(const View &v, uint32_t si, uint
     const uint32_t fr = fs < (256u >> c) ? fs : (256u >> c);
     const uint32_t first_run = fr < cap ? fr : cap;
     const uint32_t grow = m_prev << v.run_grow;                   // x 2^run_grow per refill
-    const uint32_t want = m_prev == 0 ? first_run : (grow < cap ? grow : cap);
+    uint32_t want = m_prev == 0 ? first_run : (grow < cap ? grow : cap);
+    if (hint > want) want = hint < cap ? hint : cap;
     uint32_t first = 0;
 #ifdef GALLATIN_TRACE
     const uint64_t t0 = ptx::globaltimer();
@@ -652,6 +734,7 @@ __device__ inline __noinline__ bool slot_exhausted(const View &v, uint32_t si, u
     for (;;) {
         const uint64_t w = ptx::ld_relaxed(slot_word(v, si));
         if ((uint32_t)(w >> 32) <= (run_len(w) << kSliceLog2)) return true;
+        if (oom_known(v, c)) return false;                    // the refill cannot succeed
         bo.note(w);
         bo.pause();
     }
@@ -693,9 +776,10 @@ __device__ inline void *malloc_slice(const View &v, uint32_t c, uint32_t key) {
             bool ok = true;
             if (idx == limit) ok = refill_slot(v, si, c, run_len(old));
             ok = __shfl_sync(waiters, ok, __ffs((int)waiters) - 1);
-            if (!ok && idx == limit) return nullptr;                // nullptr
+            if (!ok) return nullptr;            // nullptr: the team's refill found no memory
             continue;
         }
+        if (oom_known(v, c)) return nullptr;                          // [dev] exhaustion record
         slot_exhausted(v, si, c, old, idx);                           // refill is another warp's
     }
 }
@@ -752,6 +836,7 @@ __device__ inline __noinline__ void *malloc_large(const View &v, uint64_t k) {
             continue;
         }
         if (bt_claim_range(st, i, k)) break;
+        oom_notify(v);                                        // the claim's rollback gave segments back
         bo.pause();
     }
     ptx::fence_acq_rel();
@@ -781,6 +866,7 @@ __device__ inline __noinline__ void free_large(const View &v, uint64_t s, uint32
     for (uint64_t m = 0; m < k; m++) ptx::st_relaxed(v.seg_tid + s + m, kTreeFree);
     ptx::fence_acq_rel();
     bt_insert_range(seg_tree(v), s, k);
+    oom_notify(v);
 }
 
 // ---- Alg. 4 FREE -----------------------------------------------

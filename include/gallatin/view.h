@@ -22,6 +22,9 @@
  *               block size), word 1 = the prefetched next run (same layout)
  *   fmt_token   9 x 128 B lines: one formatter per block tree
  *   err         u64 error counter (bad frees)
+ *   oom         one 128 B line: word 0 = {epoch:32 | searchers:22 | flag:10}
+ *               (the exhaustion record, DESIGN.md Deviations 11), word 1 + t =
+ *               epoch + 1 at which block tree t was confirmed exhausted
  */
 #ifndef GALLATIN_VIEW_H_
 #define GALLATIN_VIEW_H_
@@ -44,6 +47,7 @@ struct gallatin_device_view {
     uint64_t *slots;            /* 16 words (128 B) per slot                  */
     uint32_t *fmt_token;        /* 32 words (128 B) per tree                  */
     unsigned long long *err;
+    uint64_t *oom;              /* exhaustion record (1 line)                  */
     uint32_t tree_levels;       /* L                                           */
     uint32_t tree_words;        /* W                                           */
     uint32_t level_off[GALLATIN_MAX_LEVELS];
@@ -57,6 +61,7 @@ struct gallatin_device_view {
     uint32_t run_init;          /* run length of an empty slot's first refill  */
     uint32_t prefetch;          /* 1 = fetch the next run at the run's middle  */
     uint32_t run_grow;          /* log2 of the run growth factor per refill    */
+    uint32_t demand_hint;       /* 1 = bulk refills sized to the launch's demand */
 };
 typedef struct gallatin_device_view gallatin_device_view_t;
 

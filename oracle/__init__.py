@@ -37,7 +37,7 @@ OV_INSERT, OV_DELETE, OV_MEMBER, OV_SUCC, OV_PRED = range(5)
 VIOLATIONS = {
     1: "front-first (P:138)", 2: "back-first large (P:138)", 4: "free of a non-live pointer",
     8: "overlap", 16: "alignment", 32: "outside heap", 64: "accounting", 128: "trees vs table",
-    256: "ring queue",
+    256: "ring queue", 512: "exhaustion record stands while a full search would succeed",
 }
 
 
@@ -83,6 +83,7 @@ def lib() -> ctypes.CDLL:
             "o2_nslot": ([vp, ctypes.c_uint], ctypes.c_uint),
             "o2_errors": ([vp], u64),
             "o2_violations": ([vp], u64),
+            "o2_oom_fast": ([vp], u64),
             "o2_live_count": ([vp], u64),
             "o2_usable_live": ([vp], u64),
             "o2_usable_size": ([u64], u64),
@@ -213,6 +214,11 @@ class Allocator:
     @property
     def errors(self) -> int:
         return lib().o2_errors(self._h)
+
+    @property
+    def oom_fast(self) -> int:
+        """Run requests failed by the exhaustion record (DESIGN.md Deviations 11)."""
+        return lib().o2_oom_fast(self._h)
 
     @property
     def live_count(self) -> int:

@@ -49,6 +49,14 @@
  *     reading A-11), free counter += 1, the free that completes 4096 returns
  *     the block (reading A-14); otherwise the k segments are
  *     re-inserted into the segment tree.
+ *   - [ours, DESIGN.md Deviations 11] exhaustion record: a run request of
+ *     tree t that fails (after the slot trims) records "t exhausted"; later
+ *     run requests of t fail at once while the record stands.  Every step
+ *     that puts blocks or segments back where a search could find them clears
+ *     all records: a block return, a segment freed, a segment formatted into a
+ *     block tree, and the give-backs inside a run request (an over-reservation
+ *     of a segment's blocks, the re-enqueued blocks outside the kept run, the
+ *     free segments of a claim window past its consecutive prefix).
  *   - drain (reading A-15/SURVEY A15, R-1): retire every block-buffer slot,
  *     the unissued remainder of its run counted as freed; then retire the
  *     segments whose blocks are all home.
@@ -106,6 +114,8 @@ typedef struct o2 {
     unsigned prefetch;
     unsigned run_grow;            /* a refill takes m << run_grow blocks        */
     uint64_t err;                 /* out-of-heap / non-allocated segment frees */
+    uint32_t oom_rec;             /* [ours] bit t: tree t recorded exhausted    */
+    uint64_t oom_fast;            /* run requests failed by the record          */
     /* oracle-only bookkeeping for the invariant checks */
     kv_t *live; uint64_t live_cap, live_n;
     uint64_t usable_live;
@@ -113,7 +123,7 @@ typedef struct o2 {
 } o2_t;
 
 enum { V_FRONT_FIRST = 1, V_BACK_FIRST = 2, V_BAD_FREE = 4, V_OVERLAP = 8,
-       V_ALIGN = 16, V_HEAP = 32, V_ACCOUNT = 64, V_TREES = 128, V_RING = 256 };
+       V_ALIGN = 16, V_HEAP = 32, V_ACCOUNT = 64, V_TREES = 128, V_RING = 256, V_OOM_RECORD = 512 };
 
 /* ------------------------------------------------ live-allocation map --- */
 static uint64_t mix(uint64_t x) { x ^= x >> 33; x *= 0xff51afd7ed558ccdULL; x ^= x >> 33; return x; }
@@ -213,6 +223,7 @@ void o2_destroy(o2_t *a) {
 unsigned o2_nslot(const o2_t *a, unsigned c) { return c < NUM_BLOCK_TREES ? a->nslot[c] : 0; }
 uint64_t o2_errors(const o2_t *a) { return a->err; }
 uint64_t o2_violations(const o2_t *a) { return a->violations; }
+uint64_t o2_oom_fast(const o2_t *a) { return a->oom_fast; }
 uint64_t o2_live_count(const o2_t *a) { return a->live_n; }
 uint64_t o2_usable_live(const o2_t *a) { return a->usable_live; }
 
@@ -253,6 +264,7 @@ static uint64_t retire_idle_all(o2_t *a) {
             for (int i = 0; i < 256; i++) r->e[i] = 0xFFFF;
             oracle_veb_delete(a->btree[t], s);
             oracle_veb_insert(a->segfree, s);
+            a->oom_rec = 0;
             n++;
         }
     }
@@ -284,6 +296,7 @@ static void format_segment(o2_t *a, uint64_t s, uint32_t t, uint32_t keep) {
 
 /* ------------------------------------------ block / segment return --- */
 static void return_block(o2_t *a, uint64_t s, uint32_t j, uint32_t t) {
+    a->oom_rec = 0;
     ring_push(&a->ring[s], (uint16_t)j);                   /* ring enqueue       */
     a->avail[s]++;
     if ((uint32_t)a->avail[s] == nb_of(t)) {               /* every block back  */
@@ -315,9 +328,26 @@ static uint32_t take_segments(o2_t *a, uint32_t t, uint32_t want, uint32_t *firs
     uint64_t s0 = claim_front(a);
     if (s0 == NONE64) return 0;
     uint32_t k = 1;
-    while (k < want / nb && s0 + k < a->nseg && oracle_veb_member(a->segfree, s0 + k)) {
+    const uint64_t kmax = want / nb;
+    while (k < kmax && s0 + k < a->nseg && oracle_veb_member(a->segfree, s0 + k)) {
         oracle_veb_delete(a->segfree, s0 + k);
         k++;
+    }
+    /* [ours] the CUDA claim takes every free segment of a window [x, end) --
+     * end = min(x + segments still wanted, x's word end, nseg), words of 64 --
+     * and gives back those past the consecutive prefix; a window that the
+     * prefix fills up to a word end continues in the next word */
+    for (uint64_t x = s0;;) {
+        uint64_t end = x + (kmax - (x - s0)), wend = (x | 63) + 1;
+        if (end > wend) end = wend;
+        if (end > a->nseg) end = a->nseg;
+        if (s0 + k < end) {
+            for (uint64_t y = s0 + k + 1; y < end; y++)
+                if (oracle_veb_member(a->segfree, y)) { a->oom_rec = 0; break; }
+            break;
+        }
+        if (k >= kmax || end >= a->nseg || (end & 63)) break;
+        x = end;
     }
     for (uint32_t q = 0; q < k; q++) format_segment(a, s0 + q, t, nb);
     *first = (uint32_t)(s0 * nb);
@@ -341,12 +371,13 @@ static uint32_t get_run_once(o2_t *a, uint32_t t, uint32_t want, uint32_t *first
         uint32_t av = (uint32_t)a->avail[s];
         uint32_t got = want < av ? want : av;              /* reserve */
         uint32_t low = nb / 4;
+        if (av < want) a->oom_rec = 0;                      /* over-reservation given back */
         a->avail[s] -= (int32_t)got;
         if (a->avail[s] == 0) oracle_veb_delete(a->btree[t], s);   /* no over-subscription */
         if (a->format_ahead && av >= low && av - got < low &&
             oracle_veb_successor(a->btree[t], s + 1) == NONE64) {
             uint64_t f = claim_front(a);                      /* format one segment ahead */
-            if (f != NONE64) format_segment(a, f, t, 0);
+            if (f != NONE64) { format_segment(a, f, t, 0); a->oom_rec = 0; }
         }
         uint8_t in[256] = {0};
         for (uint32_t q = 0; q < got; q++) in[ring_pop(r)] = 1;     /* getBlock */
@@ -359,7 +390,7 @@ static uint32_t get_run_once(o2_t *a, uint32_t t, uint32_t want, uint32_t *first
             len = 0;
         }
         for (uint32_t j = 0; j < nb; j++)
-            if (in[j] && (j < bs || j >= bs + bl)) return_block(a, s, j, t);
+            if (in[j] && (j < bs || j >= bs + bl)) return_block(a, s, j, t);   /* clears the record */
         *first = (uint32_t)(s * nb + bs);
         return bl;
     }
@@ -367,6 +398,7 @@ static uint32_t get_run_once(o2_t *a, uint32_t t, uint32_t want, uint32_t *first
     uint64_t s1 = claim_front(a);                             /* Alg.2 -> getSegment */
     if (s1 == NONE64) return 0;
     format_segment(a, s1, t, want);
+    a->oom_rec = 0;
     *first = (uint32_t)(s1 * nb);
     return want;
 }
@@ -407,10 +439,49 @@ static uint64_t trim_slots(o2_t *a) {
  * back their undrawn blocks and the request is retried once, for a single
  * block: memory is scarce, so no slot hoards a run of it (DESIGN.md
  * Deviations 5, "near exhaustion"). */
+/* Check of the exhaustion record, without changing any state: would the full
+ * search for one block of tree t (get_run_once, then the slot trims and a
+ * retry) succeed?  It succeeds iff tree t holds a segment, a segment is free
+ * or formatted with all blocks home, or the blocks the trims would give back
+ * include one of tree t or complete a segment's blocks. */
+static int search_would_succeed(const o2_t *a, uint32_t t) {
+    if (oracle_veb_successor(a->btree[t], 0) != NONE64) return 1;
+    if (oracle_veb_successor(a->segfree, 0) != NONE64) return 1;
+    for (uint64_t s = 0; s < a->nseg; s++)
+        if (a->tree[s] < NUM_BLOCK_TREES && (uint32_t)a->avail[s] == nb_of(a->tree[s])) return 1;
+    uint32_t *back = (uint32_t *)calloc(a->nseg, sizeof(uint32_t));
+    int ok = 0;
+    for (unsigned c = 0; c < NUM_BLOCK_TREES && !ok; c++) {
+        for (unsigned q = 0; q < a->nslot[c] && !ok; q++) {
+            unsigned i = a->slot_off[c] + q;
+            uint64_t cnt = a->slot[i] >> 32;
+            uint32_t m = (uint32_t)(a->slot[i] >> RUN_SHIFT) & 0x3FF, first = (uint32_t)a->slot[i] & RUN_NONE;
+            uint32_t m2 = cnt < SLICES_PER_BLOCK * (uint64_t)m ? (uint32_t)((cnt + SLICES_PER_BLOCK - 1) / SLICES_PER_BLOCK) : m;
+            uint32_t nm = a->prefetch ? (uint32_t)(a->next[i] >> RUN_SHIFT) & 0x3FF : 0;
+            uint32_t nf = (uint32_t)a->next[i] & RUN_NONE;
+            for (uint32_t k = 0; k < (m - m2) + nm && !ok; k++) {
+                uint32_t gid = k < m - m2 ? gid_of(c, (uint64_t)first + m2 + k) : gid_of(c, (uint64_t)nf + k - (m - m2));
+                uint64_t s = gid / MAX_BLOCKS_PER_SEGMENT;
+                if (a->freecnt[gid] != 0) continue;             /* not whole: the trim does not return it */
+                if (c == t) ok = 1;
+                else if ((uint32_t)a->avail[s] + ++back[s] == nb_of(c)) ok = 1;
+            }
+        }
+    }
+    free(back);
+    return ok;
+}
+
 static uint32_t get_run(o2_t *a, uint32_t t, uint32_t want, uint32_t *first) {
+    if ((a->oom_rec >> t) & 1) {                              /* [ours] exhaustion record */
+        if (search_would_succeed(a, t)) a->violations |= V_OOM_RECORD;
+        a->oom_fast++;
+        return 0;
+    }
     uint32_t got = get_run_once(a, t, want, first);
-    if (got || !trim_slots(a)) return got;
-    return get_run_once(a, t, 1, first);
+    if (!got && trim_slots(a)) got = get_run_once(a, t, 1, first);
+    if (!got) a->oom_rec |= 1u << t;
+    return got;
 }
 
 /* ------------------------------------------ claimMultiple (back) --- */
@@ -553,6 +624,7 @@ void o2_free(o2_t *a, uint64_t off) {
         block_freed(a, (uint32_t)(s * MAX_BLOCKS_PER_SEGMENT + j), 1);
     } else if (t != TREE_FREE && t != TREE_CONT) {
         uint64_t k = t - NUM_BLOCK_TREES;                    /* P:255 */
+        a->oom_rec = 0;
         for (uint64_t m = 0; m < k; m++) {
             a->tree[s + m] = TREE_FREE; a->avail[s + m] = 0;
             oracle_veb_insert(a->segfree, s + m);            /* P:256 */

@@ -109,6 +109,7 @@ __global__ void k_reset() {
         }
         if (i < 9 * 32) v.fmt_token[i] = 0;
         if (i == 0) *v.err = 0;
+        if (i < 16) v.oom[i] = 0;
     }
 }
 
@@ -119,7 +120,8 @@ __global__ void k_reset() {
 // Then waits-and-retries, whole blocks and segment runs.
 __device__ __noinline__ void bulk_malloc_slow(const uint64_t *sizes, void **ptrs, uint64_t n, uint64_t base,
                                               uint32_t key, uint32_t slow, const uint64_t *info, int items,
-                                              unsigned callers, uint32_t stride = 32) {
+                                              unsigned callers, uint32_t stride = 32,
+                                              const uint32_t *demand = nullptr, uint64_t ctas = 0) {
     const View &v = c_view;
     // pass 0: refill and prefetch duties only (never waits on another slot's refill)
     for (int k = 0; k < items; k++) {
@@ -133,7 +135,10 @@ __device__ __noinline__ void bulk_malloc_slow(const uint64_t *sizes, void **ptrs
         if (!((slow >> k) & 1) || !(code & 0x400u)) continue;
         const uint64_t i = base + (uint64_t)stride * k;
         const uint32_t c = core::slice_class(sizes[i]);
-        if (!core::refill_slot(v, v.slot_off[c] + key % v.nslot[c], c, code & 0x3FF)) {
+        // demand hint: this CTA's requests of class c x CTAs / slots of c, in blocks
+        const uint32_t hint =
+            demand ? (uint32_t)(((uint64_t)demand[c] * ctas / v.nslot[c] + core::kSlices - 1) >> core::kSliceLog2) : 0;
+        if (!core::refill_slot(v, v.slot_off[c] + key % v.nslot[c], c, code & 0x3FF, hint)) {
             __stcs(reinterpret_cast<unsigned long long *>(ptrs) + i, 0ull);   // heap exhausted: NULL
             slow &= ~(1u << k);
         }
@@ -319,7 +324,8 @@ __global__ void __launch_bounds__(kThreads, MINB) k_bulk_malloc_cta(const uint64
         uint64_t spill[(ITEMS + 3) / 4];                  // addressed copy only on the slow path
 #pragma unroll
         for (int q = 0; q < (ITEMS + 3) / 4; q++) spill[q] = info[q];
-        bulk_malloc_slow(sizes, ptrs, n, base, key, slow, spill, ITEMS, callers, kThreads);
+        bulk_malloc_slow(sizes, ptrs, n, base, key, slow, spill, ITEMS, callers, kThreads,
+                         v.demand_hint ? cnt : nullptr, gridDim.x);
     }
 }
 
@@ -888,7 +894,7 @@ int gallatin_init_ex(const gallatin_config_t *cfg_in) {
     if (cfg.bulk_items != 0 && cfg.bulk_items != 1 && cfg.bulk_items != 4 && cfg.bulk_items != 8 &&
         cfg.bulk_items != 16)
         return GALLATIN_ERR_INVALID;
-    if (cfg.prefetch > 2 || cfg.pipeline > 2 || cfg.free_team > 2) return GALLATIN_ERR_INVALID;
+    if (cfg.prefetch > 2 || cfg.pipeline > 2 || cfg.free_team > 2 || cfg.demand_hint > 2) return GALLATIN_ERR_INVALID;
     if (!cfg.run_grow) cfg.run_grow = 3;
     if (cfg.run_grow > 8) return GALLATIN_ERR_INVALID;
     if (nseg > (1ull << 14)) return GALLATIN_ERR_INVALID;        // 22-bit run index at 64 KB blocks (256 GiB)
@@ -938,12 +944,13 @@ int gallatin_init_ex(const gallatin_config_t *cfg_in) {
     v.run_grow = cfg.run_grow;
     v.prefetch = cfg.prefetch == 1 ? 1u : 0u;              // default off (measured: DESIGN.md)
     v.fence_free = cfg.fence_free;
+    v.demand_hint = cfg.demand_hint == 2 ? 0u : 1u;
 
     // metadata: one allocation, 256 B aligned sections
-    uint64_t sz[11] = {W * 8, 9 * W * 8, nseg * 8, nseg * 4, nseg * 4, nseg * 512, nseg * 1024,
-                       (uint64_t)off * 128, 9 * 128, 128, nseg * 4};
-    uint64_t total = 0, offs[11];
-    for (int i = 0; i < 11; i++) { offs[i] = total; total += align_up(sz[i], 256); }
+    uint64_t sz[12] = {W * 8, 9 * W * 8, nseg * 8, nseg * 4, nseg * 4, nseg * 512, nseg * 1024,
+                       (uint64_t)off * 128, 9 * 128, 128, nseg * 4, 128};
+    uint64_t total = 0, offs[12];
+    for (int i = 0; i < 12; i++) { offs[i] = total; total += align_up(sz[i], 256); }
     void *meta = nullptr;
     if (cudaMalloc(&meta, total) != cudaSuccess) { cudaGetLastError(); return GALLATIN_ERR_NOMEM; }
     void *heap = nullptr;
@@ -964,6 +971,7 @@ int gallatin_init_ex(const gallatin_config_t *cfg_in) {
     v.fmt_token = reinterpret_cast<uint32_t *>(m + offs[8]);
     v.err = reinterpret_cast<unsigned long long *>(m + offs[9]);
     v.seg_tid = reinterpret_cast<uint32_t *>(m + offs[10]);
+    v.oom = reinterpret_cast<uint64_t *>(m + offs[11]);
     v.heap = align_up(reinterpret_cast<uint64_t>(heap), core::kSegBytes);   // 16 MiB aligned base
 
     int occ_m = 0, occ_f = 0;

@@ -325,3 +325,74 @@ def test_block_path_mixed_tail(cuda_ok, G):
     sizes = np.where(rng.random(n) < 0.5, rng.integers(4097, 1 << 18, n), rng.integers(1, 4097, n)).astype(np.uint64)
     assert _bulk_round(G, nseg, sizes) == 0
     _assert_pristine(G, nseg)
+
+
+@pytest.mark.parametrize("size,n,nseg", [(16, 1 << 24, 8), (1024, 1 << 18, 4), (8192, 1 << 20, 1024),
+                                         (4096, 1 << 20, 64)])
+def test_oom_fails_fast(cuda_ok, G, size, n, nseg):
+    """A bulk call asking 2-4x the heap (DESIGN.md Deviations 11): it ends in
+    well under a second (it took 0.5-112 s before the exhaustion record), it is
+    granted the capacity up to one partly drawn block per slot, the grants are
+    stamp-verified and disjoint, and free-all + drain is pristine."""
+    import time
+    G.gallatin_init(nseg * SEG)
+    st = G.gallatin_stats()
+    d_sizes = _dev(wg.single_sizes(size, n))
+    torch.cuda.synchronize()
+    t0 = time.time()
+    nulls = _bulk_round(G, nseg, wg.single_sizes(size, n), check_accounting=False)
+    assert time.time() - t0 < 10.0, "exhaustion took too long"
+    granted = n - nulls
+    c = class_size(size)
+    if size > 4096:
+        blocks = nseg * SEG // 65536                     # 64 KB blocks (A-2)
+        assert 0.99 * blocks <= granted <= blocks
+    else:
+        cap = nseg * SEG // c
+        slack = st["nslot"][max(0, (c.bit_length() - 1) - 4)] * 4096
+        assert cap - slack <= granted <= cap
+    _assert_pristine(G, nseg)
+    # timed on its own: the malloc kernel alone
+    G.gallatin_reset()
+    p = torch.empty_like(d_sizes)
+    a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    a.record()
+    G.gallatin_malloc(d_sizes, p)
+    b.record()
+    torch.cuda.synchronize()
+    assert a.elapsed_time(b) < 1000.0, f"exhausting malloc took {a.elapsed_time(b):.1f} ms"
+    G.gallatin_free(p)
+    _assert_pristine(G, nseg)
+
+
+def test_oom_record_cleared_by_frees(cuda_ok, G):
+    """After a class was found exhausted, frees that return blocks make its
+    memory allocatable again (the record's epoch moves), for the same class
+    and for another one."""
+    nseg = 4
+    G.gallatin_init(nseg * SEG)
+    cap16 = nseg * SEG // 16
+    slack = G.gallatin_stats()["nslot"][0] * 4096
+    sizes = _dev(wg.single_sizes(16, 2 * cap16))
+    p = G.gallatin_malloc(sizes)
+    torch.cuda.synchronize()
+    got1 = int((p != 0).sum().item())
+    assert cap16 - slack <= got1 <= cap16
+    # free the first half of the array: whole blocks come back
+    half = p[: cap16].clone()
+    G.gallatin_free(half)
+    q = G.gallatin_malloc(_dev(wg.single_sizes(16, cap16)))
+    torch.cuda.synchronize()
+    got2 = int((q != 0).sum().item())
+    freed = int((half != 0).sum().item())
+    assert got2 >= freed - 2 * slack, f"only {got2} of ~{freed} freed slices allocatable again"
+    G.gallatin_free(p[cap16:].clone())
+    G.gallatin_free(q)
+    # exhausted by 16 B, everything freed: 1 KB requests get the heap
+    G.gallatin_drain()
+    r = G.gallatin_malloc(_dev(wg.single_sizes(1024, nseg * SEG // 1024)))
+    torch.cuda.synchronize()
+    got3 = int((r != 0).sum().item())
+    assert got3 >= nseg * SEG // 1024 - G.gallatin_stats()["nslot"][6] * 4096
+    G.gallatin_free(r)
+    _assert_pristine(G, nseg)

@@ -254,3 +254,46 @@ def test_utilization_closed_form(size):
         assert succ == nseg * (256 >> t)
     else:
         assert succ == nseg // -(-size // SEG)
+
+
+@pytest.mark.parametrize("seed,nseg,run_max,fa,pf", [(21, 2, 1, 0, 0), (22, 3, 16, 1, 1), (23, 4, 64, 1, 0),
+                                                     (24, 2, 256, 0, 1), (25, 6, 8, 1, 1)])
+def test_exhaustion_record_is_exact(seed, nseg, run_max, fa, pf):
+    """DESIGN.md Deviations 11: a request failed by the exhaustion record is
+    one the full search (trims + retry) would fail too.  O2 checks every
+    record-failed request against a side-effect-free dry run of that search
+    (violation bit 512); heavy pressure on 2-6 segment heaps makes records
+    fire thousands of times; free-all + drain is still pristine."""
+    kinds, args, keys = wg.replay_ops(30_000, seed, p_free=0.3, p_drain=0.001, nkeys=64)
+    a = oracle.Allocator(nseg, slot_base=16, slot_min=2, run_max=run_max, run_bytes=32 << 20, format_ahead=fa,
+                         prefetch=pf)
+    out = a.replay(kinds, args, keys)
+    assert a.oom_fast > 100, "the record never fired"
+    assert a.check() == 0, oracle.violation_names(a.check())
+    freed = {int(args[i]) for i, k in enumerate(kinds) if k == 1}
+    for i, k in enumerate(kinds):
+        if k == 0 and out[i] != np.uint64(NONE) and i not in freed:
+            a.free(int(out[i]))
+    a.drain()
+    S = sum(a.nslot(c) for c in range(9))
+    assert np.array_equal(a.image(), pristine_image(nseg, S))
+
+
+def test_exhaustion_record_cleared_by_a_block_return():
+    """Closed form on a one-segment heap with one slot per class (P:134,
+    P:188): 2^20 16 B slices fill it; the next 16 B and 64 KB requests fail
+    (the second by the record); freeing 4095 slices of block 0 returns
+    nothing and the record stands; the 4096th free returns block 0,
+    the record is cleared, and the next 16 B request gets it again."""
+    a = oracle.Allocator(1, slot_base=1, slot_min=1, run_max=256, run_bytes=16 << 20, run_init=256, run_grow=3)
+    offs = a.malloc_batch(np.full(1 << 20, 16, dtype=np.uint64))
+    assert np.array_equal(offs, np.arange(1 << 20, dtype=np.uint64) * 16)
+    assert a.malloc(16, 0) == NONE
+    f0 = a.oom_fast
+    assert a.malloc(65536, 0) == NONE and a.oom_fast == f0 + 1
+    for o in offs[:4095]:
+        a.free(int(o))
+    assert a.malloc(16, 0) == NONE and a.oom_fast == f0 + 2
+    a.free(int(offs[4095]))
+    assert a.malloc(16, 0) == 0                    # block 0 again, slice 0
+    assert a.check() == 0
