@@ -76,12 +76,15 @@ typedef struct gallatin_config {
     uint32_t prefetch;     /* 1 = fetch the next run at the middle of the current one; 0/2 = off (default) */
     uint32_t run_grow;     /* a refilled run is 2^run_grow times the last one, up to the cap: 1..8 (default 3) */
     uint32_t pipeline;     /* bulk kernels at bulk_items = 0: 1 = persistent CTAs that TMA-load the next tile while
-                              this tile's atomics are in flight; 0/2 = one tile per CTA (default, measured faster) */
+                              this tile's atomics are in flight; 3 = persistent CTAs (malloc) / warps (free) that
+                              load the next tile into registers before processing this one; 0/2 = one tile per CTA
+                              (default) */
     uint32_t free_team;    /* bulk free: 0/2 = one free-counter RMW per warp team (default, measured faster);
                               1 = one per block per CTA tile (shared-memory aggregation) */
     uint32_t demand_hint;  /* bulk malloc: 0/1 = a refill takes at least the blocks this slot's share of the launch
                               needs (the CTA's per-class count x CTAs / slots; DESIGN.md Deviations 10), up to the
                               run cap (default); 2 = off (runs grow 2^run_grow-fold per refill only) */
+    uint32_t cta_tiles;    /* pipeline = 3: tiles of 1024 requests per CTA, the next one prefetched (0 = 4) */
 } gallatin_config_t;
 
 int gallatin_init(uint64_t heap_bytes);                 /* defaults for the rest */

@@ -108,11 +108,13 @@ constexpr uint64_t kOomFlagMask = 0x3FFull;               // bits 0..9: tree t r
 constexpr uint64_t kOomOne = 1ull << 10;                  // searchers: bits 10..31
 constexpr uint64_t kOomEpoch = 1ull << 32;
 
-__device__ __forceinline__ bool oom_known(const View &v, uint32_t t) {
-    const uint64_t r = ptx::ld_relaxed(v.oom);
-    const uint64_t rec = ptx::ld_relaxed(v.oom + 1 + t);
+__device__ __forceinline__ bool oom_match(uint64_t r, uint64_t rec, uint32_t t) {
     return (r & (1ull << t)) && rec == (r >> 32) + 1;
 }
+__device__ __forceinline__ bool oom_known(const View &v, uint32_t t) {
+    return oom_match(ptx::ld_relaxed(v.oom), ptx::ld_relaxed(v.oom + 1 + t), t);
+}
+constexpr uint32_t kOomFast = 0xFFFFFFFFu;                // *first of a run request failed by the record
 
 __device__ inline __noinline__ void oom_notify_slow(const View &v, uint64_t w) {
     while (w & 0xFFFFFFFFull) {                              // a search in flight or a record
@@ -441,7 +443,12 @@ __device__ inline __noinline__ bool flux_pending(const View &v, uint32_t t) {
 // ---- Alg. 2 GetBlock(treeId), for a RUN of blocks [dev] --------
 // Returns the number of consecutive blocks obtained (0 = exhausted) and the
 // first one's linear index (segment * nb + block) in *first.
-__device__ inline __noinline__ uint32_t get_run_once(const View &v, uint32_t t, uint32_t want, uint32_t *first) {
+// check_oom: fail at once (*first = kOomFast) if tree t is recorded exhausted
+// -- checked only once the block tree came up empty, with the record loaded
+// at entry, so a refill that finds blocks pays no extra round trip.
+__device__ inline __noinline__ uint32_t get_run_once(const View &v, uint32_t t, uint32_t want, uint32_t *first,
+                                                     bool check_oom = false) {
+    const uint64_t oom_r = check_oom ? ptx::ld_relaxed(v.oom) : 0, oom_rec = check_oom ? ptx::ld_relaxed(v.oom + 1 + t) : 0;
     const BitTree bt = block_tree(v, t);
     const uint32_t nb = nb_of(t);
     ptx::Backoff bo(4, t);
@@ -549,6 +556,10 @@ __device__ inline __noinline__ uint32_t get_run_once(const View &v, uint32_t t, 
             bo.pause();
             continue;
         }
+        if (check_oom && oom_match(oom_r, oom_rec, t)) {      // [dev] exhaustion record
+            *first = kOomFast;
+            return 0;
+        }
         // [dev] before reporting "no memory", wait out blocks that are only
         // transiently unavailable (an over-reservation being given back)
         if (flux && flux_retries < kFluxRetries) {
@@ -638,15 +649,14 @@ __device__ inline __noinline__ uint32_t trim_slots(const View &v) {
 // more after an empty trim: a concurrent refiller's trim may just have given
 // the blocks back.  Serially this is one trim and one retry.
 __device__ inline __noinline__ uint32_t get_run(const View &v, uint32_t t, uint32_t want, uint32_t *first) {
-    if (oom_known(v, t)) return 0;                            // [dev] exhaustion record
 #ifdef GALLATIN_TRACE
     const uint64_t tr0 = ptx::globaltimer();
-    uint32_t got = get_run_once(v, t, want, first);
+    uint32_t got = get_run_once(v, t, want, first, true);
     ptx::trace(tr0, ptx::globaltimer(), (3ull << 60) | ((uint64_t)t << 24) | (want << 12) | got);
 #else
-    uint32_t got = get_run_once(v, t, want, first);
+    uint32_t got = get_run_once(v, t, want, first, true);
 #endif
-    if (got) return got;
+    if (got || *first == kOomFast) return got;                // [dev] exhaustion record
     oom_enter(v);
     uint64_t e = 0;
     for (uint32_t r = 0; got == 0 && r < 8; r++) {

@@ -42,7 +42,7 @@ struct State {
     cudaStream_t cin = nullptr, cout = nullptr;
     cudaEvent_t ev_in[kMaxChunks] = {}, ev_k[kMaxChunks] = {};
     // resident CTAs of the persistent bulk kernels (SMs x occupancy)
-    unsigned pipe_malloc_ctas = 0, pipe_free_ctas = 0;
+    unsigned pipe_malloc_ctas = 0, pipe_free_ctas = 0, pers_malloc_ctas = 0, pers_free_ctas = 0;
 };
 State g;
 
@@ -329,6 +329,118 @@ __global__ void __launch_bounds__(kThreads, MINB) k_bulk_malloc_cta(const uint64
     }
 }
 
+// Persistent form of k_bulk_malloc_cta with the NEXT tile's sizes prefetched
+// into registers: a CTA walks tiles tile, tile + gridDim.x, ... and issues
+// the next tile's loads before this tile's shared-memory ranking, slot RMWs
+// and pointer stores, so the HBM latency of tile i+1 overlaps the L2 round
+// trip of tile i (one tile per CTA serializes load -> RMW -> store and pays a
+// CTA launch per tile).  Per tile exactly k_bulk_malloc_cta's protocol; the
+// class counters and slot words are double-buffered by tile parity so a tile
+// needs two CTA barriers.  A refill duty is discharged within its own tile
+// (bulk_malloc_slow), before the CTA issues its next RMW, as in the one-tile
+// kernel.
+template <int ITEMS>
+__global__ void __launch_bounds__(kThreads, 5) k_bulk_malloc_pers(const uint64_t *__restrict__ sizes,
+                                                                  void **__restrict__ ptrs, uint64_t n,
+                                                                  uint64_t ntiles, uint32_t tiles) {
+    constexpr uint32_t kTile = kThreads * ITEMS;
+    const View &v = c_view;
+    __shared__ uint32_t cnt[2][core::kTrees];
+    __shared__ uint64_t olds[2][core::kTrees];
+    const uint32_t lane = threadIdx.x & 31;
+    const uint32_t key = ptx::smid();
+    const uint32_t lt = ptx::lanemask_lt();
+    if (threadIdx.x < 2 * core::kTrees) (&cnt[0][0])[threadIdx.x] = 0;
+    __syncthreads();
+    __shared__ uint64_t buf[2][ITEMS][kThreads];
+    uint64_t tile = (uint64_t)blockIdx.x * tiles;
+    const uint64_t tend = tile + tiles < ntiles ? tile + tiles : ntiles;
+#pragma unroll
+    for (int k = 0; k < ITEMS; k++) {
+        const uint64_t i = tile * kTile + threadIdx.x + (uint64_t)kThreads * k;
+        ptx::cp_async8(&buf[0][k][threadIdx.x], sizes + (i < n ? i : n - 1));
+    }
+    ptx::cp_async_commit();
+    for (uint32_t it = 0; tile < tend; tile++, it++) {
+        const uint32_t par = it & 1;
+        const uint64_t base = tile * kTile + threadIdx.x;
+        // the next tile's sizes are in flight (cp.async, no registers) while this tile runs
+        const uint64_t nt = tile + 1;
+        if (nt < tend) {
+#pragma unroll
+            for (int k = 0; k < ITEMS; k++) {
+                const uint64_t i = nt * kTile + threadIdx.x + (uint64_t)kThreads * k;
+                ptx::cp_async8(&buf[par ^ 1][k][threadIdx.x], sizes + (i < n ? i : n - 1));
+            }
+        }
+        ptx::cp_async_commit();
+        ptx::cp_async_wait<1>();
+        uint32_t cr[ITEMS];
+#pragma unroll
+        for (int k = 0; k < ITEMS; k++) {
+            const uint64_t s = base + (uint64_t)kThreads * k < n ? buf[par][k][threadIdx.x] : 0;
+            const uint32_t lg = 64u - (uint32_t)__clzll((long long)(s - 1));
+            const uint32_t sc = (lg > core::kMinSliceLog2 ? lg : core::kMinSliceLog2) - core::kMinSliceLog2;
+            cr[k] = s - 1 < core::kMaxSlice ? sc : (s == 0 ? 0xFEu : 0xFFu);
+        }
+#pragma unroll
+        for (int k = 0; k < ITEMS; k++) {
+            const uint32_t c = cr[k];
+            const unsigned peers = __match_any_sync(0xFFFFFFFFu, c);
+            const uint32_t leader = (uint32_t)__ffs((int)peers) - 1;
+            uint32_t b = 0;
+            if (c < core::kTrees && lane == leader) b = atomicAdd(&cnt[par][c], (uint32_t)__popc(peers));
+            cr[k] = c | ((__shfl_sync(0xFFFFFFFFu, b, (int)leader) + (uint32_t)__popc(peers & lt)) << 8);
+        }
+        __syncthreads();
+        if (threadIdx.x < core::kTrees) {
+            const uint32_t c = threadIdx.x;
+            const uint32_t m = cnt[par][c];
+            if (m) olds[par][c] = ptx::atom_add(core::slot_word(v, v.slot_off[c] + key % v.nslot[c]), (uint64_t)m << 32);
+            cnt[par ^ 1][c] = 0;                                   // for the next tile
+        }
+        __syncthreads();
+        uint32_t slow = 0;
+        uint64_t info[(ITEMS + 3) / 4];
+#pragma unroll
+        for (int q = 0; q < (ITEMS + 3) / 4; q++) info[q] = 0;
+#pragma unroll
+        for (int k = 0; k < ITEMS; k++) {
+            const uint64_t i = base + (uint64_t)kThreads * k;
+            const uint32_t c = cr[k] & 0xFFu;
+            void *p = nullptr;
+            uint32_t code = 0;
+            if (c < core::kTrees) {
+                const uint64_t old = olds[par][c];
+                const uint32_t m = core::run_len(old);
+                const uint32_t idx = (uint32_t)(old >> 32) + (cr[k] >> 8);
+                if (idx < (m << core::kSliceLog2)) {
+                    p = core::slice_ptr(v, c, old & core::kRunNone, idx);
+                    if (v.prefetch && idx == (m << (core::kSliceLog2 - 1))) code = 0x2000u | m;
+                } else {
+                    code = idx == (m << core::kSliceLog2) ? (0x400u | m) : 0x1000u;
+                }
+            } else if (c == 0xFFu) {
+                code = 0x800u;
+            }
+            if (code) {
+                slow |= 1u << k;
+                info[k >> 2] |= (uint64_t)code << (16 * (k & 3));
+            }
+            if (!(code & 0x1C00u) && i < n)
+                __stcs(reinterpret_cast<unsigned long long *>(ptrs) + i, reinterpret_cast<unsigned long long>(p));
+        }
+        const unsigned callers = __ballot_sync(0xFFFFFFFFu, slow != 0);
+        if (slow) {
+            uint64_t spill[(ITEMS + 3) / 4];
+#pragma unroll
+            for (int q = 0; q < (ITEMS + 3) / 4; q++) spill[q] = info[q];
+            bulk_malloc_slow(sizes, ptrs, n, base, key, slow, spill, ITEMS, callers, kThreads,
+                             v.demand_hint ? cnt[par] : nullptr, ntiles);
+        }
+    }
+}
+
 // Persistent, software-pipelined form of k_bulk_malloc_cta: a CTA walks
 // tiles of kThreads*ITEMS requests (tile, tile + gridDim.x, ...).  One thread
 // issues a 1-D TMA bulk copy of the NEXT tile's sizes into the other half of a
@@ -539,6 +651,90 @@ __global__ void __launch_bounds__(kThreads, ITEMS <= 4 ? 6 : 4) k_bulk_free(void
         if (p[k] && !peers[k]) slow |= 1u << k;
     }
     if (done | slow) bulk_free_slow(ptrs, base, done, slow, ITEMS);
+}
+
+// One warp tile of the bulk free (lane l frees p[k] = ptrs[base + 32k], base
+// = tile * 32 * ITEMS + l): k_bulk_free's protocol on pointers already loaded.
+// The block id is computed in 32 bits from off >> 16 (segments < 2^22).
+template <int ITEMS>
+__device__ __forceinline__ void free_warp_tile(const View &v, void *const *ptrs, const uint64_t (&p)[ITEMS],
+                                               uint64_t base, uint32_t lane, uint64_t heap_bytes) {
+    uint32_t o16[ITEMS], t[ITEMS];
+#pragma unroll
+    for (int k = 0; k < ITEMS; k++) {
+        const uint64_t off = p[k] - v.heap;
+        const bool in = p[k] && off < heap_bytes;
+        o16[k] = (uint32_t)(off >> 16);                            // segment << 8 | 64 KB unit
+        t[k] = in ? __ldca(v.seg_tid + (o16[k] >> 8)) : core::kTreeFree;
+    }
+    uint32_t gid[ITEMS], oldc[ITEMS];
+    unsigned peers[ITEMS];
+#pragma unroll
+    for (int k = 0; k < ITEMS; k++) {
+        const bool blk = t[k] < core::kTrees;                       // slice or whole block
+        gid[k] = blk ? ((o16[k] & ~0xFFu) | ((o16[k] & 0xFFu) >> t[k])) : (0x80000000u | (uint32_t)(k << 5) | lane);
+        peers[k] = __match_any_sync(0xFFFFFFFFu, gid[k]);
+        if (!blk) peers[k] = 0;
+    }
+#pragma unroll
+    for (int k = 0; k < ITEMS; k++) {
+        oldc[k] = 0;
+        if (peers[k] && lane == (uint32_t)__ffs((int)peers[k]) - 1)
+            oldc[k] = atomicAdd(v.block_free + gid[k], (uint32_t)__popc(peers[k]));
+    }
+    uint32_t done = 0, slow = 0;
+#pragma unroll
+    for (int k = 0; k < ITEMS; k++) {
+        if (peers[k] && lane == (uint32_t)__ffs((int)peers[k]) - 1 && oldc[k] + __popc(peers[k]) == core::kSlices)
+            done |= 1u << k;                                         // the 4096th free
+        if (p[k] && !peers[k]) slow |= 1u << k;
+    }
+    if (done | slow) bulk_free_slow(ptrs, base, done, slow, ITEMS);
+}
+
+// Multi-tile bulk free: CTA b takes CTA tiles b*T .. b*T+T-1 (T = tiles, each
+// kThreads*ITEMS pointers; warp w frees its 32*ITEMS slice of each) and
+// issues the NEXT tile's pointer loads -- per-thread cp.async copies into
+// shared memory, so no register is held across the slow path's calls --
+// before processing this one: their HBM latency overlaps this tile's tree-id
+// loads and counter RMWs.  T is small so the hardware still balances CTAs
+// (a fully persistent grid left a tail of warps stuck in block returns).
+template <int ITEMS>
+__global__ void __launch_bounds__(kThreads, 6) k_bulk_free_pers(void *const *__restrict__ ptrs, uint64_t n,
+                                                                uint64_t nwtiles, uint32_t tiles) {
+    const View &v = c_view;
+    __shared__ uint64_t buf[2][ITEMS][kThreads];
+    const uint32_t lane = threadIdx.x & 31;
+    constexpr uint64_t nwarps = kThreads / 32;
+    const uint64_t heap_bytes = v.nseg << core::kSegLog2;
+    const uint64_t *src = reinterpret_cast<const uint64_t *>(ptrs);
+    uint64_t wt = (uint64_t)blockIdx.x * tiles * nwarps + (threadIdx.x >> 5);
+    const uint64_t wend = wt + (uint64_t)tiles * nwarps < nwtiles ? wt + (uint64_t)tiles * nwarps : nwtiles;
+#pragma unroll
+    for (int k = 0; k < ITEMS; k++) {
+        const uint64_t i = wt * (32 * ITEMS) + 32ull * k + lane;
+        ptx::cp_async8(&buf[0][k][threadIdx.x], src + (i < n ? i : n - 1));
+    }
+    ptx::cp_async_commit();
+    for (uint32_t it = 0; wt < wend; wt += nwarps, it++) {
+        const uint32_t par = it & 1;
+        const uint64_t nt = wt + nwarps;
+        if (nt < wend) {
+#pragma unroll
+            for (int k = 0; k < ITEMS; k++) {
+                const uint64_t i = nt * (32 * ITEMS) + 32ull * k + lane;
+                ptx::cp_async8(&buf[par ^ 1][k][threadIdx.x], src + (i < n ? i : n - 1));
+            }
+        }
+        ptx::cp_async_commit();
+        ptx::cp_async_wait<1>();                                   // this tile's copies landed
+        const uint64_t base = wt * (32 * ITEMS) + lane;
+        uint64_t p[ITEMS];
+#pragma unroll
+        for (int k = 0; k < ITEMS; k++) p[k] = base + 32ull * k < n ? buf[par][k][threadIdx.x] : 0;
+        free_warp_tile<ITEMS>(v, ptrs, p, base, lane, heap_bytes);
+    }
+    ptx::cp_async_wait<0>();
 }
 
 // Bulk free with CTA-level aggregation: the frees of one CTA tile that hit the
@@ -894,7 +1090,8 @@ int gallatin_init_ex(const gallatin_config_t *cfg_in) {
     if (cfg.bulk_items != 0 && cfg.bulk_items != 1 && cfg.bulk_items != 4 && cfg.bulk_items != 8 &&
         cfg.bulk_items != 16)
         return GALLATIN_ERR_INVALID;
-    if (cfg.prefetch > 2 || cfg.pipeline > 2 || cfg.free_team > 2 || cfg.demand_hint > 2) return GALLATIN_ERR_INVALID;
+    if (cfg.prefetch > 2 || cfg.pipeline > 3 || cfg.free_team > 2 || cfg.demand_hint > 2 || cfg.cta_tiles > 1024)
+        return GALLATIN_ERR_INVALID;
     if (!cfg.run_grow) cfg.run_grow = 3;
     if (cfg.run_grow > 8) return GALLATIN_ERR_INVALID;
     if (nseg > (1ull << 14)) return GALLATIN_ERR_INVALID;        // 22-bit run index at 64 KB blocks (256 GiB)
@@ -979,6 +1176,10 @@ int gallatin_init_ex(const gallatin_config_t *cfg_in) {
     CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ_f, k_bulk_free_pipe<4>, kThreads, 0));
     g.pipe_malloc_ctas = (unsigned)(sms * (occ_m > 0 ? occ_m : 1));
     g.pipe_free_ctas = (unsigned)(sms * (occ_f > 0 ? occ_f : 1));
+    CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ_m, k_bulk_malloc_pers<4>, kThreads, 0));
+    CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ_f, k_bulk_free_pers<4>, kThreads, 0));
+    g.pers_malloc_ctas = (unsigned)(sms * (occ_m > 0 ? occ_m : 1));
+    g.pers_free_ctas = (unsigned)(sms * (occ_f > 0 ? occ_f : 1));
     g.init = true;
     g.device = dev;
     g.cfg = cfg;
@@ -1025,6 +1226,10 @@ int gallatin_malloc(const uint64_t *d_sizes, void **d_ptrs, uint64_t n, void *st
         const unsigned grid = ntiles < g.pipe_malloc_ctas ? (unsigned)ntiles : g.pipe_malloc_ctas;
         const uint32_t tma = (reinterpret_cast<uintptr_t>(d_sizes) & 15) == 0;
         k_bulk_malloc_pipe<4><<<grid, kThreads, 0, S(stream)>>>(d_sizes, d_ptrs, n, ntiles, tma);
+    } else if (g.cfg.bulk_items == 0 && items == 4 && g.cfg.pipeline == 3) {
+        const uint64_t ntiles = (n + kThreads * 4 - 1) / (kThreads * 4);
+        const uint32_t T = g.cfg.cta_tiles ? g.cfg.cta_tiles : 4;
+        k_bulk_malloc_pers<4><<<(unsigned)((ntiles + T - 1) / T), kThreads, 0, S(stream)>>>(d_sizes, d_ptrs, n, ntiles, T);
     } else if (items == 16)
         k_bulk_malloc_cta<16><<<grid_for((n + 15) / 16), kThreads, 0, S(stream)>>>(d_sizes, d_ptrs, n);
     else if (items == 8)
@@ -1047,6 +1252,11 @@ int gallatin_free(void *const *d_ptrs, uint64_t n, void *stream) {
         const unsigned grid = want < g.pipe_free_ctas ? (unsigned)want : g.pipe_free_ctas;
         const uint32_t tma = (reinterpret_cast<uintptr_t>(d_ptrs) & 15) == 0;
         k_bulk_free_pipe<4><<<grid, kThreads, 0, S(stream)>>>(d_ptrs, n, nwt, tma);
+    } else if (g.cfg.bulk_items == 0 && n >= (uint64_t)kItemsMin && g.cfg.pipeline == 3) {
+        const uint64_t nwt = (n + 32 * 4 - 1) / (32 * 4);
+        const uint64_t nct = (nwt + kThreads / 32 - 1) / (kThreads / 32);     // CTA tiles
+        const uint32_t T = g.cfg.cta_tiles ? g.cfg.cta_tiles : 4;
+        k_bulk_free_pers<4><<<(unsigned)((nct + T - 1) / T), kThreads, 0, S(stream)>>>(d_ptrs, n, nwt, T);
     } else if (g.cfg.bulk_items == 0 && n >= (uint64_t)kItemsMin && g.cfg.free_team == 1) {
         k_bulk_free_cta<4><<<grid_for((n + 3) / 4), kThreads, 0, S(stream)>>>(d_ptrs, n);
     } else if (g.cfg.bulk_items >= 8)

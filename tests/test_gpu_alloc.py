@@ -271,8 +271,9 @@ def test_config3_full_size_bench_launch(cuda_ok, G):
         _assert_pristine(G, nseg)
 
 
-@pytest.mark.parametrize("knobs", [dict(pipeline=1), dict(free_team=1), dict(bulk_items=8), dict(bulk_items=16),
-                                   dict(bulk_items=1), dict(pipeline=2, free_team=1)])
+@pytest.mark.parametrize("knobs", [dict(pipeline=1), dict(pipeline=2), dict(pipeline=3), dict(free_team=1),
+                                   dict(bulk_items=8), dict(bulk_items=16), dict(bulk_items=1),
+                                   dict(pipeline=2, free_team=1)])
 @pytest.mark.parametrize("n", [(1 << 21) + 77, 1 << 22])
 def test_bulk_kernel_variants(cuda_ok, G, knobs, n):
     """Every bulk-kernel variant (persistent TMA-pipelined, CTA-aggregated or
@@ -290,7 +291,7 @@ def test_bulk_kernels_unaligned_arrays(cuda_ok, G):
     """Size and pointer arrays that start 8 bytes past a 16-byte boundary
     (the TMA tile loads fall back to plain loads)."""
     nseg = 256
-    for knobs in (dict(pipeline=1), {}):
+    for knobs in (dict(pipeline=1), dict(pipeline=2), dict(pipeline=3), {}):
         G.gallatin_init(nseg * SEG, **knobs)
         n = (1 << 20) + 3
         sizes = _dev(np.concatenate([[0], wg.mixed_sizes(n, upper=512, p_large=0.0)]))[1:]

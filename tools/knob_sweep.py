@@ -12,6 +12,8 @@ import sys
 
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 sys.path.insert(0, ROOT)
+if os.environ.get("GALLATIN_PKG_ROOT"):
+    sys.path.insert(0, os.environ["GALLATIN_PKG_ROOT"])  # A/B against another build of the package
 SIZES = [16 << i for i in range(9)]
 
 
