@@ -331,8 +331,9 @@ __device__ inline __noinline__ void return_block(const View &v, uint32_t gid) {
     ptx::st_relaxed(slotp, (uint16_t)(gid % kMaxBlocks));
     ptx::fence_acq_rel();
     const uint64_t old = ptx::atom_add(v.seg_word + s, 1ull);
-    seg_after_rmw(v, s, old, old + 1);
-    oom_notify(v);
+    seg_after_rmw(v, s, old, old + 1);                       // all blocks home: try_free_segment notifies
+    // a search can newly find the segment only if it had no block available
+    if (sw_avail(old) == 0) oom_notify(v);
 }
 
 // n slices of block gid came back; the team completing 4096 returns it
@@ -677,6 +678,7 @@ __device__ inline __noinline__ bool refill_slot(const View &v, uint32_t si, uint
     if (v.prefetch) {                                         // [dev] the prefetched run, if any
         const uint64_t nx = ptx::atom_exch(slot_word(v, si) + 1, kSlotEmpty);
         if (run_len(nx) != 0) {
+            ptx::st_relaxed(slot_word(v, si) + 2, 0ull);
             ptx::atom_exch(slot_word(v, si), nx);               // {issued 0, run, first}
             return true;
         }
@@ -699,9 +701,11 @@ __device__ inline __noinline__ bool refill_slot(const View &v, uint32_t si, uint
     const uint32_t got = get_run(v, c, want, &first);
 #endif
     if (got == 0) {
+        ptx::st_relaxed(slot_word(v, si) + 2, 1ull);        // waiters then consult the exhaustion record
         ptx::atom_exch(slot_word(v, si), kSlotEmpty);
         return false;
     }
+    ptx::st_relaxed(slot_word(v, si) + 2, 0ull);
     ptx::atom_exch(slot_word(v, si), ((uint64_t)got << kRunShift) | first);
     return true;
 }
@@ -742,9 +746,13 @@ __device__ inline __noinline__ bool slot_exhausted(const View &v, uint32_t si, u
     if (idx == (m << kSliceLog2)) return refill_slot(v, si, c, m);
     ptx::Backoff bo(1, si);
     for (;;) {
+        // the slot word and its failed-refill flag share a sector (one round trip)
         const uint64_t w = ptx::ld_relaxed(slot_word(v, si));
+        const uint64_t failed = ptx::ld_relaxed(slot_word(v, si) + 2);
         if ((uint32_t)(w >> 32) <= (run_len(w) << kSliceLog2)) return true;
-        if (oom_known(v, c)) return false;                    // the refill cannot succeed
+        // the last refill found no memory: if tree c is still recorded
+        // exhausted, the pending refill cannot succeed either [dev]
+        if (failed && oom_known(v, c)) return false;
         bo.note(w);
         bo.pause();
     }
@@ -789,8 +797,8 @@ __device__ inline void *malloc_slice(const View &v, uint32_t c, uint32_t key) {
             if (!ok) return nullptr;            // nullptr: the team's refill found no memory
             continue;
         }
-        if (oom_known(v, c)) return nullptr;                          // [dev] exhaustion record
-        slot_exhausted(v, si, c, old, idx);                           // refill is another warp's
+        // refill is another warp's; false: tree c is recorded exhausted [dev]
+        if (!slot_exhausted(v, si, c, old, idx)) return nullptr;
     }
 }
 

@@ -19,7 +19,8 @@
  *   slots       S x 128 B lines: word 0 = {issued count:32 | run length:10 |
  *               first block:22} (block buffer; a run = consecutive
  *               blocks, first block as a linear index in units of the class's
- *               block size), word 1 = the prefetched next run (same layout)
+ *               block size), word 1 = the prefetched next run (same layout),
+ *               word 2 = 1 if the slot's last refill found no memory
  *   fmt_token   9 x 128 B lines: one formatter per block tree
  *   err         u64 error counter (bad frees)
  *   oom         one 128 B line: word 0 = {epoch:32 | searchers:22 | flag:10}

@@ -53,7 +53,8 @@
  *     tree t that fails (after the slot trims) records "t exhausted"; later
  *     run requests of t fail at once while the record stands.  Every step
  *     that puts blocks or segments back where a search could find them clears
- *     all records: a block return, a segment freed, a segment formatted into a
+ *     all records: a block return to a segment with no block available (it
+ *     rejoins its block tree), a segment freed, a segment formatted into a
  *     block tree, and the give-backs inside a run request (an over-reservation
  *     of a segment's blocks, the re-enqueued blocks outside the kept run, the
  *     free segments of a claim window past its consecutive prefix).
@@ -296,7 +297,7 @@ static void format_segment(o2_t *a, uint64_t s, uint32_t t, uint32_t keep) {
 
 /* ------------------------------------------ block / segment return --- */
 static void return_block(o2_t *a, uint64_t s, uint32_t j, uint32_t t) {
-    a->oom_rec = 0;
+    if (a->avail[s] == 0) a->oom_rec = 0;                  /* the segment becomes findable */
     ring_push(&a->ring[s], (uint16_t)j);                   /* ring enqueue       */
     a->avail[s]++;
     if ((uint32_t)a->avail[s] == nb_of(t)) {               /* every block back  */
@@ -306,6 +307,7 @@ static void return_block(o2_t *a, uint64_t s, uint32_t j, uint32_t t) {
         for (int i = 0; i < 256; i++) r->e[i] = 0xFFFF;
         oracle_veb_delete(a->btree[t], s);
         oracle_veb_insert(a->segfree, s);                   /* back to segment tree */
+        a->oom_rec = 0;
     } else if (a->avail[s] == 1) {
         oracle_veb_insert(a->btree[t], s);                  /* re-added (A-16)    */
     }
@@ -390,7 +392,8 @@ static uint32_t get_run_once(o2_t *a, uint32_t t, uint32_t want, uint32_t *first
             len = 0;
         }
         for (uint32_t j = 0; j < nb; j++)
-            if (in[j] && (j < bs || j >= bs + bl)) return_block(a, s, j, t);   /* clears the record */
+            if (in[j] && (j < bs || j >= bs + bl)) return_block(a, s, j, t);
+        if (bl < got) a->oom_rec = 0;                       /* re-enqueued: clears the record */
         *first = (uint32_t)(s * nb + bs);
         return bl;
     }
