@@ -32,14 +32,16 @@ for case in cases.split(","):
     G.gallatin_malloc(st, p)
     b.record()
     torch.cuda.synchronize()
+    t_malloc = a.elapsed_time(b)
     nulls = int((p == 0).sum().item())
+    b.record()                                        # the free alone (not the host-side count above)
     G.gallatin_free(p)
     c.record()
     torch.cuda.synchronize()
     G.gallatin_drain()
     img = G.gallatin_snapshot()
     msg = diff_images(img, pristine_image(nseg, int(img[4])))
-    print(json.dumps({"size": size, "n": n, "heap_segments": nseg, "malloc_ms": round(a.elapsed_time(b), 3),
+    print(json.dumps({"size": size, "n": n, "heap_segments": nseg, "malloc_ms": round(t_malloc, 3),
                       "free_ms": round(b.elapsed_time(c), 3), "wall_s": round(time.time() - t0, 2), "nulls": nulls,
                       "granted": n - nulls, "pristine": not msg}), flush=True)
     del st, p
