@@ -79,12 +79,16 @@ typedef struct gallatin_config {
                               this tile's atomics are in flight; 3 = persistent CTAs (malloc) / warps (free) that
                               load the next tile into registers before processing this one; 0/2 = one tile per CTA
                               (default) */
-    uint32_t free_team;    /* bulk free: 0/2 = one free-counter RMW per warp team (default, measured faster);
-                              1 = one per block per CTA tile (shared-memory aggregation) */
+    uint32_t free_team;    /* bulk free: 0/3 = one free-counter RMW per warp team, 32-bit block-id decode (default);
+                              2 = the same teams with 64-bit decode and clamped loads (k_bulk_free, ablation);
+                              1 = one RMW per block per CTA tile (shared-memory aggregation, ablation) */
     uint32_t demand_hint;  /* bulk malloc: 0/1 = a refill takes at least the blocks this slot's share of the launch
                               needs (the CTA's per-class count x CTAs / slots; DESIGN.md Deviations 10), up to the
                               run cap (default); 2 = off (runs grow 2^run_grow-fold per refill only) */
     uint32_t cta_tiles;    /* pipeline = 3: tiles of 1024 requests per CTA, the next one prefetched (0 = 4) */
+    uint32_t cta_threads;  /* bulk malloc CTA kernel: threads per CTA (4 requests each, one slot RMW per class
+                              per CTA): 0/128 = 128 (default, 10 CTAs/SM), 64, 256 */
+    uint32_t free_threads; /* bulk free kernel: 0/128 = 128-thread CTAs (default), 256 */
 } gallatin_config_t;
 
 int gallatin_init(uint64_t heap_bytes);                 /* defaults for the rest */

@@ -217,16 +217,34 @@ __device__ __forceinline__ uint64_t claim_retry_hint(uint64_t wi, uint64_t old, 
 }
 
 // ---- Alg. 1 GetSegment(treeId < numBlockTrees) ----------------
+// [dev] A claimer that has already lost a race (attempt > 0) and moves on to
+// the next word does not aim at its lowest free bit -- every other loser
+// aims there too, and a launch's first burst of refills (one per slot, all
+// at once) then takes one segment per round -- but at a pseudo-random bit at
+// or above it in that word; the RMW tells whether it was free.
+__device__ __forceinline__ uint64_t claim_spread(uint64_t s, uint32_t attempt) {
+    const uint32_t tid = blockIdx.x * blockDim.x + threadIdx.x;
+    uint32_t h = (tid * 0x27D4EB2Fu) ^ (attempt * 0x165667B1u);
+    h ^= h >> 15;
+    const uint32_t lo = (uint32_t)(s & 63);
+    return (s & ~63ull) | (lo + h % (64u - lo));
+}
+
 // successor(0) on the segment tree + claimIndex, front first
 // (P:138).  Returns the claimed segment or kNone when every segment is in use.
-// A claimer that loses the race retries elsewhere (claim_retry_hint; serially
-// the first attempt always wins, so this is successor(0)).
+// A claimer that loses the race retries elsewhere (claim_retry_hint,
+// claim_spread; serially the first attempt always wins, so this is
+// successor(0)).
 __device__ inline __noinline__ uint64_t claim_front(const View &v) {
     const BitTree st = seg_tree(v);
     uint64_t from = 0, hint = kNone;
     uint32_t attempt = 0;
     for (;;) {
         uint64_t s = hint != kNone ? hint : bt_successor<false>(st, from);
+        if (hint == kNone && attempt > 0 && s != kNone) {
+            s = claim_spread(s, attempt);
+            if (s >= v.nseg) s = v.nseg - 1;
+        }
         hint = kNone;
         if (s == kNone) {
             if (from != 0) { from = 0; continue; }
@@ -262,6 +280,10 @@ __device__ inline __noinline__ uint64_t claim_front_run(const View &v, uint32_t 
     uint32_t attempt = 0;
     for (;;) {
         uint64_t s = hint != kNone ? hint : bt_successor<false>(st, from);
+        if (hint == kNone && attempt > 0 && s != kNone) {
+            s = claim_spread(s, attempt);
+            if (s >= v.nseg) s = v.nseg - 1;
+        }
         hint = kNone;
         if (s == kNone) {
             if (from != 0) { from = 0; continue; }

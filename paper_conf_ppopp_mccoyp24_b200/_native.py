@@ -31,7 +31,8 @@ class Config(ctypes.Structure):
                 ("fence_free", ctypes.c_uint32), ("bulk_items", ctypes.c_uint32), ("run_init", ctypes.c_uint32),
                 ("prefetch", ctypes.c_uint32), ("run_grow", ctypes.c_uint32), ("pipeline", ctypes.c_uint32),
                 ("free_team", ctypes.c_uint32), ("demand_hint", ctypes.c_uint32),
-                ("cta_tiles", ctypes.c_uint32)]
+                ("cta_tiles", ctypes.c_uint32), ("cta_threads", ctypes.c_uint32),
+                ("free_threads", ctypes.c_uint32)]
 
 
 class Stats(ctypes.Structure):
@@ -152,12 +153,14 @@ def _empty64(n: int):
 def gallatin_init(heap_bytes: int, slot_base: int = 0, slot_min: int = 0, run_max: int = 0, run_bytes: int = 0,
                   format_ahead: int = 0, fence_free: int = 0, bulk_items: int = 0, run_init: int = 0,
                   prefetch: int = 0, run_grow: int = 0, pipeline: int = 0, free_team: int = 0,
-                  demand_hint: int = 0, cta_tiles: int = 0) -> None:
+                  demand_hint: int = 0, cta_tiles: int = 0, cta_threads: int = 0,
+                  free_threads: int = 0) -> None:
     """0 = library default for every knob (include/gallatin.h gallatin_config_t)."""
     cfg = Config(heap_bytes=heap_bytes, run_bytes=run_bytes, slot_base=slot_base, slot_min=slot_min,
                  run_max=run_max, format_ahead=format_ahead, fence_free=fence_free, bulk_items=bulk_items,
                  run_init=run_init, prefetch=prefetch, run_grow=run_grow, pipeline=pipeline, free_team=free_team,
-                 demand_hint=demand_hint, cta_tiles=cta_tiles)
+                 demand_hint=demand_hint, cta_tiles=cta_tiles, cta_threads=cta_threads,
+                 free_threads=free_threads)
     check(lib().gallatin_init_ex(ctypes.byref(cfg)), "gallatin_init")
 
 

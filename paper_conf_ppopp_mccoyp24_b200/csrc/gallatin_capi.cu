@@ -239,14 +239,13 @@ __global__ void __launch_bounds__(kThreads, 5) k_bulk_malloc(const uint64_t *__r
 // global RMW per class per CTA takes their slices (1024 requests at
 // ITEMS=4), so the hot slot words see 32x fewer RMWs than with warp teams.
 // Item k of thread t is request blockIdx*256*ITEMS + k*256 + t.
-template <int ITEMS, int MINB = 5>
-__global__ void __launch_bounds__(kThreads, MINB) k_bulk_malloc_cta(const uint64_t *__restrict__ sizes,
+template <int ITEMS, int MINB = 5, int NT = kThreads>
+__global__ void __launch_bounds__(NT, MINB) k_bulk_malloc_cta(const uint64_t *__restrict__ sizes,
                                                                   void **__restrict__ ptrs, uint64_t n) {
     const View &v = c_view;
     __shared__ uint32_t cnt[core::kTrees];
-    __shared__ uint64_t olds[core::kTrees];
     const uint32_t lane = threadIdx.x & 31;
-    const uint64_t base = blockIdx.x * (uint64_t)(kThreads * ITEMS) + threadIdx.x;
+    const uint64_t base = blockIdx.x * (uint64_t)(NT * ITEMS) + threadIdx.x;
 #ifdef GALLATIN_TRACE
     if (threadIdx.x == 0 && (blockIdx.x == 0 || blockIdx.x == gridDim.x - 1)) {
         const uint64_t tk = ptx::globaltimer();
@@ -255,19 +254,27 @@ __global__ void __launch_bounds__(kThreads, MINB) k_bulk_malloc_cta(const uint64
 #endif
     const uint32_t key = ptx::smid();
     if (threadIdx.x < core::kTrees) cnt[threadIdx.x] = 0;
+    // a tile entirely inside the array needs no per-item range checks (CTA-uniform)
+    const bool full = (blockIdx.x + 1ull) * (NT * ITEMS) <= n;
     // per item: class (0..8 slice class, 0xFE nothing to do, 0xFF block or
     // segment request) | rank << 8; the sizes themselves are not kept
     uint32_t cr[ITEMS];
     uint64_t x[ITEMS];
-    // unconditional loads of clamped indices, all issued before any is used
+    // all loads issued before any is used (clamped indices in a ragged tile)
+    if (full) {
 #pragma unroll
-    for (int k = 0; k < ITEMS; k++) {
-        const uint64_t i = base + (uint64_t)kThreads * k;
-        x[k] = __ldcs(reinterpret_cast<const unsigned long long *>(sizes) + (i < n ? i : n - 1));
+        for (int k = 0; k < ITEMS; k++) x[k] = __ldcs(reinterpret_cast<const unsigned long long *>(sizes) + base + NT * k);
+    } else {
+#pragma unroll
+        for (int k = 0; k < ITEMS; k++) {
+            const uint64_t i = base + (uint64_t)NT * k;
+            x[k] = __ldcs(reinterpret_cast<const unsigned long long *>(sizes) + (i < n ? i : n - 1));
+            if (i >= n) x[k] = 0;
+        }
     }
 #pragma unroll
     for (int k = 0; k < ITEMS; k++) {
-        const uint64_t s = base + (uint64_t)kThreads * k < n ? x[k] : 0;
+        const uint64_t s = x[k];
         const uint32_t lg = 64u - (uint32_t)__clzll((long long)(s - 1));      // ceil(log2 s) for s >= 2
         const uint32_t sc = (lg > core::kMinSliceLog2 ? lg : core::kMinSliceLog2) - core::kMinSliceLog2;
         cr[k] = s - 1 < core::kMaxSlice ? sc : (s == 0 ? 0xFEu : 0xFFu);   // branch-free slice_class
@@ -284,9 +291,15 @@ __global__ void __launch_bounds__(kThreads, MINB) k_bulk_malloc_cta(const uint64
         cr[k] = c | ((__shfl_sync(0xFFFFFFFFu, b, (int)leader) + (uint32_t)__popc(peers & lt)) << 8);
     }
     __syncthreads();
+    // per class: the slot RMW's {limit : 32 | first index : 32} and the
+    // address of the run's slice 0, so an item's pointer is one shift-add
+    __shared__ uint64_t lim_lo[core::kTrees];
+    __shared__ uint64_t run_base[core::kTrees];
     if (threadIdx.x < core::kTrees && cnt[threadIdx.x]) {
         const uint32_t c = threadIdx.x;
-        olds[c] = ptx::atom_add(core::slot_word(v, v.slot_off[c] + key % v.nslot[c]), (uint64_t)cnt[c] << 32);
+        const uint64_t old = ptx::atom_add(core::slot_word(v, v.slot_off[c] + key % v.nslot[c]), (uint64_t)cnt[c] << 32);
+        lim_lo[c] = ((uint64_t)(core::run_len(old) << core::kSliceLog2) << 32) | (old >> 32);
+        run_base[c] = reinterpret_cast<uint64_t>(core::slice_ptr(v, c, old & core::kRunNone, 0));
     }
     __syncthreads();
     uint32_t slow = 0;
@@ -295,19 +308,19 @@ __global__ void __launch_bounds__(kThreads, MINB) k_bulk_malloc_cta(const uint64
     for (int q = 0; q < (ITEMS + 3) / 4; q++) info[q] = 0;
 #pragma unroll
     for (int k = 0; k < ITEMS; k++) {
-        const uint64_t i = base + (uint64_t)kThreads * k;
+        const uint64_t i = base + (uint64_t)NT * k;
         const uint32_t c = cr[k] & 0xFFu;
-        void *p = nullptr;
+        uint64_t p = 0;
         uint32_t code = 0;
         if (c < core::kTrees) {
-            const uint64_t old = olds[c];
-            const uint32_t m = core::run_len(old);
-            const uint32_t idx = (uint32_t)(old >> 32) + (cr[k] >> 8);
-            if (idx < (m << core::kSliceLog2)) {
-                p = core::slice_ptr(v, c, old & core::kRunNone, idx);
-                if (v.prefetch && idx == (m << (core::kSliceLog2 - 1))) code = 0x2000u | m;   // prefetch duty
+            const uint64_t ll = lim_lo[c];
+            const uint32_t limit = (uint32_t)(ll >> 32);
+            const uint32_t idx = (uint32_t)ll + (cr[k] >> 8);
+            if (idx < limit) {
+                p = run_base[c] + ((uint64_t)idx << (core::kMinSliceLog2 + c));
+                if (v.prefetch && idx == (limit >> 1)) code = 0x2000u | (limit >> core::kSliceLog2);   // prefetch duty
             } else {
-                code = idx == (m << core::kSliceLog2) ? (0x400u | m) : 0x1000u;
+                code = idx == limit ? (0x400u | (limit >> core::kSliceLog2)) : 0x1000u;
             }
         } else if (c == 0xFFu) {
             code = 0x800u;
@@ -316,15 +329,14 @@ __global__ void __launch_bounds__(kThreads, MINB) k_bulk_malloc_cta(const uint64
             slow |= 1u << k;
             info[k >> 2] |= (uint64_t)code << (16 * (k & 3));
         }
-        if (!(code & 0x1C00u) && i < n)
-            __stcs(reinterpret_cast<unsigned long long *>(ptrs) + i, reinterpret_cast<unsigned long long>(p));
+        if (!(code & 0x1C00u) && (full || i < n)) __stcs(reinterpret_cast<unsigned long long *>(ptrs) + i, p);
     }
     const unsigned callers = __ballot_sync(0xFFFFFFFFu, slow != 0);
     if (slow) {
         uint64_t spill[(ITEMS + 3) / 4];                  // addressed copy only on the slow path
 #pragma unroll
         for (int q = 0; q < (ITEMS + 3) / 4; q++) spill[q] = info[q];
-        bulk_malloc_slow(sizes, ptrs, n, base, key, slow, spill, ITEMS, callers, kThreads,
+        bulk_malloc_slow(sizes, ptrs, n, base, key, slow, spill, ITEMS, callers, NT,
                          v.demand_hint ? cnt : nullptr, gridDim.x);
     }
 }
@@ -599,11 +611,11 @@ __device__ __noinline__ void bulk_free_slow(void *const *ptrs, uint64_t base, ui
 // Bulk free, ITEMS pointers per thread: load pointers, then their segments'
 // table words, team the lanes freeing one block, one release fence
 // per leading lane, then the team counter RMWs back to back.
-template <int ITEMS>
-__global__ void __launch_bounds__(kThreads, ITEMS <= 4 ? 6 : 4) k_bulk_free(void *const *__restrict__ ptrs, uint64_t n) {
+template <int ITEMS, int NT = kThreads>
+__global__ void __launch_bounds__(NT, (ITEMS <= 4 ? 6 : 4) * kThreads / NT) k_bulk_free(void *const *__restrict__ ptrs, uint64_t n) {
     const View &v = c_view;
     const uint32_t lane = threadIdx.x & 31;
-    const uint64_t base = ((blockIdx.x * (uint64_t)kThreads + threadIdx.x) >> 5) * (32 * ITEMS) + lane;
+    const uint64_t base = ((blockIdx.x * (uint64_t)NT + threadIdx.x) >> 5) * (32 * ITEMS) + lane;
     const uint64_t heap_bytes = v.nseg << core::kSegLog2;
     uint64_t p[ITEMS], w[ITEMS];
     uint32_t gid[ITEMS], oldc[ITEMS];
@@ -690,6 +702,27 @@ __device__ __forceinline__ void free_warp_tile(const View &v, void *const *ptrs,
         if (p[k] && !peers[k]) slow |= 1u << k;
     }
     if (done | slow) bulk_free_slow(ptrs, base, done, slow, ITEMS);
+}
+
+// k_bulk_free's protocol through free_warp_tile (32-bit block-id math, one
+// range check per item) with the warp's loads unclamped when its whole tile
+// is in range.
+template <int ITEMS, int NT = kThreads>
+__global__ void __launch_bounds__(NT, 6 * kThreads / NT) k_bulk_free_w(void *const *__restrict__ ptrs, uint64_t n) {
+    const View &v = c_view;
+    const uint32_t lane = threadIdx.x & 31;
+    const uint64_t wbase = ((blockIdx.x * (uint64_t)NT + threadIdx.x) >> 5) * (32 * ITEMS);
+    const uint64_t base = wbase + lane;
+    const unsigned long long *src = reinterpret_cast<const unsigned long long *>(ptrs);
+    uint64_t p[ITEMS];
+    if (wbase + 32 * ITEMS <= n) {
+#pragma unroll
+        for (int k = 0; k < ITEMS; k++) p[k] = __ldcs(src + base + 32ull * k);
+    } else {
+#pragma unroll
+        for (int k = 0; k < ITEMS; k++) p[k] = base + 32ull * k < n ? __ldcs(src + base + 32ull * k) : 0;
+    }
+    free_warp_tile<ITEMS>(v, ptrs, p, base, lane, v.nseg << core::kSegLog2);
 }
 
 // Multi-tile bulk free: CTA b takes CTA tiles b*T .. b*T+T-1 (T = tiles, each
@@ -1090,7 +1123,9 @@ int gallatin_init_ex(const gallatin_config_t *cfg_in) {
     if (cfg.bulk_items != 0 && cfg.bulk_items != 1 && cfg.bulk_items != 4 && cfg.bulk_items != 8 &&
         cfg.bulk_items != 16)
         return GALLATIN_ERR_INVALID;
-    if (cfg.prefetch > 2 || cfg.pipeline > 3 || cfg.free_team > 2 || cfg.demand_hint > 2 || cfg.cta_tiles > 1024)
+    if (cfg.prefetch > 2 || cfg.pipeline > 3 || cfg.free_team > 3 || cfg.demand_hint > 2 || cfg.cta_tiles > 1024 ||
+        (cfg.cta_threads != 0 && cfg.cta_threads != 64 && cfg.cta_threads != 128 && cfg.cta_threads != 256) ||
+        (cfg.free_threads != 0 && cfg.free_threads != 128 && cfg.free_threads != 256))
         return GALLATIN_ERR_INVALID;
     if (!cfg.run_grow) cfg.run_grow = 3;
     if (cfg.run_grow > 8) return GALLATIN_ERR_INVALID;
@@ -1235,7 +1270,12 @@ int gallatin_malloc(const uint64_t *d_sizes, void **d_ptrs, uint64_t n, void *st
     else if (items == 8)
         k_bulk_malloc_cta<8><<<grid_for((n + 7) / 8), kThreads, 0, S(stream)>>>(d_sizes, d_ptrs, n);
     else if (items == 4)
-        k_bulk_malloc_cta<4><<<grid_for((n + 3) / 4), kThreads, 0, S(stream)>>>(d_sizes, d_ptrs, n);
+        if (g.cfg.cta_threads == 0 || g.cfg.cta_threads == 128)        // default (measured)
+            k_bulk_malloc_cta<4, 10, 128><<<(unsigned)((n + 511) / 512), 128, 0, S(stream)>>>(d_sizes, d_ptrs, n);
+        else if (g.cfg.cta_threads == 64)
+            k_bulk_malloc_cta<4, 20, 64><<<(unsigned)((n + 255) / 256), 64, 0, S(stream)>>>(d_sizes, d_ptrs, n);
+        else
+            k_bulk_malloc_cta<4><<<grid_for((n + 3) / 4), kThreads, 0, S(stream)>>>(d_sizes, d_ptrs, n);
 
     else
         k_bulk_malloc<1><<<grid_for(n), kThreads, 0, S(stream)>>>(d_sizes, d_ptrs, n);
@@ -1259,8 +1299,16 @@ int gallatin_free(void *const *d_ptrs, uint64_t n, void *stream) {
         k_bulk_free_pers<4><<<(unsigned)((nct + T - 1) / T), kThreads, 0, S(stream)>>>(d_ptrs, n, nwt, T);
     } else if (g.cfg.bulk_items == 0 && n >= (uint64_t)kItemsMin && g.cfg.free_team == 1) {
         k_bulk_free_cta<4><<<grid_for((n + 3) / 4), kThreads, 0, S(stream)>>>(d_ptrs, n);
+    } else if (g.cfg.bulk_items == 0 && n >= (uint64_t)kItemsMin && g.cfg.free_team != 2) {
+        // default: warp teams, 32-bit block ids, 128-thread CTAs
+        if (g.cfg.free_threads == 256)
+            k_bulk_free_w<4><<<grid_for((n + 3) / 4), kThreads, 0, S(stream)>>>(d_ptrs, n);
+        else
+            k_bulk_free_w<4, 128><<<(unsigned)((n + 511) / 512), 128, 0, S(stream)>>>(d_ptrs, n);
     } else if (g.cfg.bulk_items >= 8)
         k_bulk_free<8><<<grid_for((n + 7) / 8), kThreads, 0, S(stream)>>>(d_ptrs, n);
+    else if ((g.cfg.bulk_items >= 4 || (g.cfg.bulk_items == 0 && n >= (uint64_t)kItemsMin)) && g.cfg.free_threads == 128)
+        k_bulk_free<4, 128><<<(unsigned)((n + 511) / 512), 128, 0, S(stream)>>>(d_ptrs, n);
     else if (g.cfg.bulk_items >= 4 || (g.cfg.bulk_items == 0 && n >= (uint64_t)kItemsMin))
         k_bulk_free<4><<<grid_for((n + 3) / 4), kThreads, 0, S(stream)>>>(d_ptrs, n);
     else
