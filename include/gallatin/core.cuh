@@ -230,6 +230,23 @@ __device__ __forceinline__ uint64_t claim_spread(uint64_t s, uint32_t attempt) {
     return (s & ~63ull) | (lo + h % (64u - lo));
 }
 
+// [dev] The FIRST loss of a segment claim means every concurrent claimer
+// aimed at the same lowest free bit (a launch's first burst: one refill per
+// slot at once); the loser then aims at a pseudo-random bit of the next
+// kSpreadWords leaf words, unseen -- the RMW tells whether it was free --
+// instead of queueing on the one word; later losses use the free bits the
+// RMW returned (claim_retry_hint).  Serially no claim loses.
+constexpr uint32_t kSpreadWords = 4;
+__device__ __forceinline__ uint64_t claim_first_loss(const View &v, uint64_t wi) {
+    const uint32_t tid = blockIdx.x * blockDim.x + threadIdx.x;
+    uint32_t h = tid * 0x9E3779B1u;
+    h ^= h >> 13;
+    h *= 0x85EBCA6Bu;
+    h ^= h >> 16;
+    const uint64_t s = ((wi + h % kSpreadWords) << 6) | ((h >> 8) & 63);
+    return s < v.nseg ? s : v.nseg - 1;
+}
+
 // successor(0) on the segment tree + claimIndex, front first
 // (P:138).  Returns the claimed segment or kNone when every segment is in use.
 // A claimer that loses the race retries elsewhere (claim_retry_hint,
@@ -263,7 +280,7 @@ __device__ inline __noinline__ uint64_t claim_front(const View &v) {
             ptx::fence_acq_rel();
             return s;
         }
-        hint = claim_retry_hint(s >> 6, old, ++attempt);
+        hint = ++attempt == 1 ? claim_first_loss(v, s >> 6) : claim_retry_hint(s >> 6, old, attempt);
         from = ((s >> 6) + 1) << 6;
     }
 }
@@ -309,12 +326,12 @@ __device__ inline __noinline__ uint64_t claim_front_run(const View &v, uint32_t 
         if (flip) bt_reconcile_up(st, 0, wi);
         if (extra) oom_notify(v);
         if (run == 0) {
-            hint = claim_retry_hint(wi, old & ~mask, ++attempt);
+            hint = ++attempt == 1 ? claim_first_loss(v, wi) : claim_retry_hint(wi, old & ~mask, attempt);
             from = (wi + 1) << 6;
             continue;
         }
         ptx::fence_acq_rel();
-        *k = run;
+        *k = run | (attempt << 16);                        // attempts: traced builds read them
         return s;
     }
 }
@@ -410,8 +427,12 @@ __device__ inline __noinline__ uint32_t take_segments(const View &v, uint32_t t,
     const uint64_t s0 = claim_front_run(v, kmax, &k);
     if (s0 == kNone) return 0;
 #ifdef GALLATIN_TRACE
+    const uint32_t attempts = k >> 16;
+#endif
+    k &= 0xFFFFu;
+#ifdef GALLATIN_TRACE
     const uint64_t tr1 = ptx::globaltimer();
-    ptx::trace(tr0, tr1, (1ull << 60) | ((uint64_t)t << 24) | k);
+    ptx::trace(tr0, tr1, (1ull << 60) | ((uint64_t)attempts << 32) | ((uint64_t)t << 24) | k);
 #endif
     const BitTree st = seg_tree(v);
     // extend with the following free segments: one atomicAnd per leaf

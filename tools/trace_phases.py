@@ -51,4 +51,9 @@ for sz in sizes:
         out[f"tag{g_}"] = {"n": int(m.sum()), "p50": round(float(np.percentile(lat, 50)), 2),
                            "p90": round(float(np.percentile(lat, 90)), 2), "max": round(float(lat.max()), 2),
                            "first_start_us": round(float(st_.min()), 1), "last_end_us": round(float(((t[m, 1].astype(np.int64) - base) / 1e3).max()), 1)}
+    m1 = tag == 1
+    if m1.any():
+        att = ((t[m1, 2] >> np.uint64(32)) & np.uint64(0xFFFF)).astype(int)
+        out["claim_attempts"] = {"mean": round(float(att.mean()), 2), "max": int(att.max()),
+                                 "hist": np.bincount(att, minlength=1)[:12].tolist()}
     print(json.dumps(out), flush=True)
