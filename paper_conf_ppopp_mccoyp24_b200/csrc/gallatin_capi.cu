@@ -707,8 +707,8 @@ __device__ __forceinline__ void free_warp_tile(const View &v, void *const *ptrs,
 // k_bulk_free's protocol through free_warp_tile (32-bit block-id math, one
 // range check per item) with the warp's loads unclamped when its whole tile
 // is in range.
-template <int ITEMS, int NT = kThreads>
-__global__ void __launch_bounds__(NT, 6 * kThreads / NT) k_bulk_free_w(void *const *__restrict__ ptrs, uint64_t n) {
+template <int ITEMS, int NT = kThreads, int MINB = 6 * kThreads / NT>
+__global__ void __launch_bounds__(NT, MINB) k_bulk_free_w(void *const *__restrict__ ptrs, uint64_t n) {
     const View &v = c_view;
     const uint32_t lane = threadIdx.x & 31;
     const uint64_t wbase = ((blockIdx.x * (uint64_t)NT + threadIdx.x) >> 5) * (32 * ITEMS);
