@@ -22,15 +22,16 @@ struct gallatin_graph {
     uint32_t *work2;      // big vertices (CTA-per-vertex deletes)
     uint32_t *nwork;      // [0] work, [1] work2
     unsigned long long *ctr;   // [0] mallocs [1] frees [2] failed mallocs
-    uint64_t *hkeys;      // delete-batch hash: (src << 32 | dst) -> remaining count
+    uint32_t *hkeys;      // delete-batch hash, one region per source vertex: dst -> remaining count
     uint32_t *hcnt;
-    uint64_t hcap;
+    uint64_t hcap;        // slots allocated (>= 4 x the batch)
+    uint32_t *hoff;       // per vertex: first slot of its region (next_pow2(2 cnt) slots)
+    uint32_t *hbump;      // region allocator
     uint32_t *lock;       // per-vertex lock word of the single-edge operations
 };
 
 namespace {
 constexpr int kT = 256;
-constexpr uint64_t kEmpty = ~0ull;
 constexpr uint32_t kBig = 2048;        // lists at least this long delete with a whole CTA
 #ifndef GALLATIN_GRAPH_MINB
 #define GALLATIN_GRAPH_MINB 4
@@ -102,13 +103,19 @@ __global__ void __launch_bounds__(kT, kGraphMinBlocks) k_grow(gallatin_graph g) 
     count_warp(g.ctr, m, false, fail);
 }
 
-// warp per queued vertex: copy size[v] entries old -> new, free the old list
+// warp per queued vertex: copy size[v] entries old -> new, free the old list;
+// lists of kHuge entries or more are left to the whole grid (k_copy_huge)
+constexpr uint32_t kHuge = 1u << 16;
 __global__ void __launch_bounds__(kT, kGraphMinBlocks) k_copy(gallatin_graph g) {
     const uint32_t nw = *g.nwork;
     const uint64_t warps = (uint64_t)gridDim.x * (kT / 32);
     unsigned long long frees = 0;
     for (uint64_t w = (blockIdx.x * (uint64_t)kT + threadIdx.x) >> 5; w < nw; w += warps) {
         const uint32_t v = g.work[w], s = g.size[v];
+        if (s >= kHuge) {
+            if (lane() == 0) g.work2[atomicAdd(g.nwork + 1, 1u)] = v;
+            continue;
+        }
         const uint32_t *src = reinterpret_cast<const uint32_t *>(g.old[v]);
         uint32_t *dst = reinterpret_cast<uint32_t *>(g.list[v]);
         for (uint32_t k = lane(); k < s; k += 32) dst[k] = src[k];
@@ -119,6 +126,35 @@ __global__ void __launch_bounds__(kT, kGraphMinBlocks) k_copy(gallatin_graph g) 
         }
     }
     if (lane() == 0 && frees) atomicAdd(g.ctr + 1, frees);
+}
+
+// Huge lists (a hub drawn by the expansion reaches hundreds of MB): every CTA
+// takes 16 KB chunks of each in turn, 16-byte vector copies (lists come from
+// the allocator 16-byte aligned); the old lists are freed afterwards.
+constexpr uint32_t kChunk = 4096;                      // entries per CTA chunk
+__global__ void k_copy_huge(gallatin_graph g) {
+    const uint32_t nb = g.nwork[1];
+    for (uint32_t b = 0; b < nb; b++) {
+        const uint32_t v = g.work2[b], s = g.size[v];
+        const uint4 *src = reinterpret_cast<const uint4 *>(g.old[v]);
+        uint4 *dst = reinterpret_cast<uint4 *>(g.list[v]);
+        const uint32_t q = s / 4, chunks = (s + kChunk - 1) / kChunk;
+        for (uint32_t c = blockIdx.x; c < chunks; c += gridDim.x) {
+            const uint32_t lo = c * (kChunk / 4), hi = min(q, lo + kChunk / 4);
+            for (uint32_t k = lo + threadIdx.x; k < hi; k += kT) dst[k] = src[k];
+            if (c == chunks - 1 && threadIdx.x < (s & 3))              // the last 1-3 entries
+                reinterpret_cast<uint32_t *>(dst)[4 * q + threadIdx.x] =
+                    reinterpret_cast<const uint32_t *>(src)[4 * q + threadIdx.x];
+        }
+    }
+}
+__global__ void __launch_bounds__(kT, kGraphMinBlocks) k_free_huge(gallatin_graph g) {
+    unsigned long long frees = 0;
+    for (uint32_t b = blockIdx.x * kT + threadIdx.x; b < g.nwork[1]; b += gridDim.x * kT) {
+        gallatin_free(reinterpret_cast<void *>(g.old[g.work2[b]]));
+        frees++;
+    }
+    if (frees) atomicAdd(g.ctr + 1, frees);
 }
 
 // append: one atomic per distinct source in a warp reserves the positions
@@ -143,29 +179,61 @@ __device__ __forceinline__ uint64_t hmix(uint64_t k) {
     return k;
 }
 
+// The batch's deletions live in one small open-addressing region per source
+// vertex (next_pow2(2 cnt) slots), so the probes of one vertex's list entries
+// stay in a few cache lines instead of a batch-wide table in HBM (one random
+// DRAM sector per list entry).
+constexpr uint32_t kHEmpty = 0xFFFFFFFFu;
+__device__ __forceinline__ uint32_t region_slots(uint32_t c) { return c ? next_pow2(2 * c) : 0u; }
+
+// hoff[v] = a region of region_slots(cnt[v]) slots: one bump per CTA of the
+// CTA's exclusive prefix (region order is irrelevant)
+__global__ void k_hash_regions(gallatin_graph g) {
+    __shared__ uint32_t wsum[kT / 32];
+    __shared__ uint32_t base;
+    const uint64_t v = blockIdx.x * (uint64_t)kT + threadIdx.x;
+    const uint32_t r = v < g.V ? region_slots(g.cnt[v]) : 0u;
+    uint32_t x = r;                                           // inclusive warp scan
+#pragma unroll
+    for (int d = 1; d < 32; d <<= 1) {
+        const uint32_t y = __shfl_up_sync(0xFFFFFFFFu, x, d);
+        if (lane() >= (uint32_t)d) x += y;
+    }
+    if (lane() == 31) wsum[threadIdx.x >> 5] = x;
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        uint32_t t = 0;
+        for (int w = 0; w < kT / 32; w++) { const uint32_t s = wsum[w]; wsum[w] = t; t += s; }
+        base = t ? atomicAdd(g.hbump, t) : 0u;
+    }
+    __syncthreads();
+    if (v < g.V && r) g.hoff[v] = base + wsum[threadIdx.x >> 5] + x - r;
+}
+
 __global__ void k_hash_insert(gallatin_graph g, const uint32_t *src, const uint32_t *dst, uint64_t n) {
     const uint64_t i = blockIdx.x * (uint64_t)kT + threadIdx.x;
     if (i >= n) return;
-    const uint64_t key = ((uint64_t)src[i] << 32) | dst[i], mask = g.hcap - 1;
-    for (uint64_t h = hmix(key) & mask;; h = (h + 1) & mask) {
-        const uint64_t k = atomicCAS(reinterpret_cast<unsigned long long *>(g.hkeys + h), kEmpty, key);
-        if (k == kEmpty || k == key) {
-            atomicAdd(g.hcnt + h, 1u);
+    const uint32_t s = src[i], key = dst[i];
+    uint32_t *keys = g.hkeys + g.hoff[s], *cnts = g.hcnt + g.hoff[s];
+    const uint32_t mask = region_slots(g.cnt[s]) - 1;
+    for (uint32_t h = (uint32_t)hmix(key) & mask;; h = (h + 1) & mask) {
+        const uint32_t k = atomicCAS(keys + h, kHEmpty, key);
+        if (k == kHEmpty || k == key) {
+            atomicAdd(cnts + h, 1u);
             return;
         }
     }
 }
 
-// take one pending deletion of (v, x); true if this instance is deleted
-__device__ __forceinline__ bool hash_take(const gallatin_graph &g, uint32_t v, uint32_t x) {
-    const uint64_t key = ((uint64_t)v << 32) | x, mask = g.hcap - 1;
-    for (uint64_t h = hmix(key) & mask;; h = (h + 1) & mask) {
-        const uint64_t k = g.hkeys[h];
-        if (k == kEmpty) return false;
-        if (k != key) continue;
-        uint32_t c = *(volatile uint32_t *)(g.hcnt + h);
+// take one pending deletion of x from vertex v's region; true if this instance is deleted
+__device__ __forceinline__ bool hash_take(const uint32_t *keys, uint32_t *cnts, uint32_t mask, uint32_t x) {
+    for (uint32_t h = (uint32_t)hmix(x) & mask;; h = (h + 1) & mask) {
+        const uint32_t k = keys[h];
+        if (k == kHEmpty) return false;
+        if (k != x) continue;
+        uint32_t c = *(volatile uint32_t *)(cnts + h);
         while (c > 0) {
-            const uint32_t o = atomicCAS(g.hcnt + h, c, c - 1);
+            const uint32_t o = atomicCAS(cnts + h, c, c - 1);
             if (o == c) return true;
             c = o;
         }
@@ -227,6 +295,9 @@ __global__ void __launch_bounds__(kT, kGraphMinBlocks) k_delete_small(gallatin_g
     for (uint64_t w = (blockIdx.x * (uint64_t)kT + threadIdx.x) >> 5; w < nw; w += warps) {
         const uint32_t v = g.work[w], s = g.size[v];
         uint32_t *L = reinterpret_cast<uint32_t *>(g.list[v]);
+        const uint32_t *hk = g.hkeys + g.hoff[v];
+        uint32_t *hc = g.hcnt + g.hoff[v];
+        const uint32_t hm = region_slots(g.cnt[v]) - 1;
         uint32_t out = 0;
         for (uint32_t b = 0; b < s; b += 32) {
             const uint32_t i = b + lane();
@@ -234,7 +305,7 @@ __global__ void __launch_bounds__(kT, kGraphMinBlocks) k_delete_small(gallatin_g
             bool keep = false;
             if (i < s) {
                 x = L[i];
-                keep = !hash_take(g, v, x);
+                keep = !hash_take(hk, hc, hm, x);
             }
             const unsigned km = __ballot_sync(0xFFFFFFFFu, keep);
             if (keep) L[out + __popc(km & ((1u << lane()) - 1))] = x;    // out <= b: never ahead of the reads
@@ -255,6 +326,9 @@ __global__ void __launch_bounds__(kT, kGraphMinBlocks) k_delete_big(gallatin_gra
     for (uint32_t w = blockIdx.x; w < nw; w += gridDim.x) {
         const uint32_t v = g.work2[w], s = g.size[v];
         uint32_t *L = reinterpret_cast<uint32_t *>(g.list[v]);
+        const uint32_t *hk = g.hkeys + g.hoff[v];
+        uint32_t *hc = g.hcnt + g.hoff[v];
+        const uint32_t hm = region_slots(g.cnt[v]) - 1;
         if (threadIdx.x == 0) out_s = 0;
         __syncthreads();
         for (uint32_t b = 0; b < s; b += kT) {
@@ -263,7 +337,7 @@ __global__ void __launch_bounds__(kT, kGraphMinBlocks) k_delete_big(gallatin_gra
             bool keep = false;
             if (i < s) {
                 x = L[i];
-                keep = !hash_take(g, v, x);
+                keep = !hash_take(hk, hc, hm, x);
             }
             const unsigned km = __ballot_sync(0xFFFFFFFFu, keep);
             if (lane() == 0) wsum[wid] = (uint32_t)__popc(km);
@@ -296,11 +370,28 @@ __global__ void __launch_bounds__(kT, kGraphMinBlocks) k_expand_fill(gallatin_gr
     const uint64_t warps = (uint64_t)gridDim.x * (kT / 32);
     for (uint64_t w = (blockIdx.x * (uint64_t)kT + threadIdx.x) >> 5; w < n; w += warps) {
         const uint32_t v = vs[w], s0 = g.size[v], add = g.cnt[v];
+        if (add >= kHuge) {                                   // the whole grid fills it (k_expand_huge)
+            if (lane() == 0) g.work2[atomicAdd(g.nwork + 1, 1u)] = v;
+            continue;
+        }
         uint32_t *L = reinterpret_cast<uint32_t *>(g.list[v]);
         for (uint32_t j = lane(); j < add; j += 32) L[s0 + j] = (uint32_t)(((uint64_t)v + s0 + j + 1) % g.V);
         __syncwarp();
         if (lane() == 0) g.size[v] = s0 + add;
     }
+}
+__global__ void k_expand_huge(gallatin_graph g) {
+    const uint32_t nb = g.nwork[1];
+    for (uint32_t b = 0; b < nb; b++) {
+        const uint32_t v = g.work2[b], s0 = g.size[v], add = g.cnt[v];
+        uint32_t *L = reinterpret_cast<uint32_t *>(g.list[v]);
+        for (uint64_t j = blockIdx.x * (uint64_t)kT + threadIdx.x; j < add; j += (uint64_t)gridDim.x * kT)
+            L[s0 + j] = (uint32_t)(((uint64_t)v + s0 + j + 1) % g.V);
+    }
+}
+__global__ void k_expand_huge_size(gallatin_graph g) {
+    for (uint32_t b = blockIdx.x * kT + threadIdx.x; b < g.nwork[1]; b += gridDim.x * kT)
+        g.size[g.work2[b]] += g.cnt[g.work2[b]];
 }
 
 __global__ void __launch_bounds__(kT, kGraphMinBlocks) k_free_all(gallatin_graph g) {
@@ -450,6 +541,8 @@ __global__ void __launch_bounds__(kT, kGraphMinBlocks) k_edge_delete(gallatin_gr
 int run_grow(gallatin_graph *g, cudaStream_t st) {
     k_grow<<<blocks(g->V), kT, 0, st>>>(*g);
     k_copy<<<148 * 8, kT, 0, st>>>(*g);
+    k_copy_huge<<<148 * 8, kT, 0, st>>>(*g);
+    k_free_huge<<<148, kT, 0, st>>>(*g);
     return status();
 }
 }  // namespace
@@ -467,7 +560,8 @@ int gallatin_graph_create(uint32_t V, gallatin_graph_t **out) {
               cudaMalloc(&g->cap, 4ull * V) == cudaSuccess && cudaMalloc(&g->cnt, 4ull * V) == cudaSuccess &&
               cudaMalloc(&g->old, 8ull * V) == cudaSuccess && cudaMalloc(&g->work, 4ull * V) == cudaSuccess &&
               cudaMalloc(&g->work2, 4ull * V) == cudaSuccess && cudaMalloc(&g->nwork, 8) == cudaSuccess &&
-              cudaMalloc(&g->ctr, 24) == cudaSuccess && cudaMalloc(&g->lock, 4ull * V) == cudaSuccess;
+              cudaMalloc(&g->ctr, 24) == cudaSuccess && cudaMalloc(&g->lock, 4ull * V) == cudaSuccess &&
+              cudaMalloc(&g->hoff, 4ull * V) == cudaSuccess && cudaMalloc(&g->hbump, 4) == cudaSuccess;
     if (!ok) {
         cudaGetLastError();
         gallatin_graph_destroy(g, nullptr);
@@ -487,7 +581,7 @@ int gallatin_graph_destroy(gallatin_graph_t *g, void *stream) {
     if (g->list && gallatin_is_initialized()) k_free_all<<<blocks(g->V), kT, 0, S(stream)>>>(*g);
     cudaStreamSynchronize(S(stream));
     void *ptrs[] = {g->list, g->size, g->cap, g->cnt, g->old, g->work, g->work2, g->nwork, g->ctr, g->hkeys, g->hcnt,
-                    g->lock};
+                    g->lock, g->hoff, g->hbump};
     for (void *p : ptrs)
         if (p) cudaFree(p);
     delete g;
@@ -511,14 +605,14 @@ int gallatin_graph_delete(gallatin_graph_t *g, const uint32_t *src, const uint32
     if (!g || (n && (!src || !dst))) return GALLATIN_ERR_INVALID;
     if (n == 0) return GALLATIN_OK;
     cudaStream_t st = S(stream);
-    uint64_t cap = 1;
-    while (cap < 2 * n) cap <<= 1;
+    if (n > (1ull << 29)) return GALLATIN_ERR_INVALID;          // region offsets are 32-bit
+    const uint64_t cap = 4 * n;                                 // sum of next_pow2(2 cnt[v]) <= 4 n
     if (cap > g->hcap) {
         if (g->hkeys) cudaFree(g->hkeys);
         if (g->hcnt) cudaFree(g->hcnt);
         g->hkeys = nullptr;
         g->hcnt = nullptr;
-        if (cudaMalloc(&g->hkeys, 8 * cap) != cudaSuccess || cudaMalloc(&g->hcnt, 4 * cap) != cudaSuccess) {
+        if (cudaMalloc(&g->hkeys, 4 * cap) != cudaSuccess || cudaMalloc(&g->hcnt, 4 * cap) != cudaSuccess) {
             cudaGetLastError();
             g->hcap = 0;
             return GALLATIN_ERR_NOMEM;
@@ -526,13 +620,14 @@ int gallatin_graph_delete(gallatin_graph_t *g, const uint32_t *src, const uint32
         g->hcap = cap;
     }
     gallatin_graph gv = *g;
-    gv.hcap = cap;                               // a power of two <= the allocation
-    cudaMemsetAsync(g->hkeys, 0xFF, 8 * cap, st);
+    cudaMemsetAsync(g->hkeys, 0xFF, 4 * cap, st);
     cudaMemsetAsync(g->hcnt, 0, 4 * cap, st);
+    cudaMemsetAsync(g->hbump, 0, 4, st);
     cudaMemsetAsync(g->cnt, 0, 4ull * g->V, st);
     cudaMemsetAsync(g->nwork, 0, 8, st);
-    k_hash_insert<<<blocks(n), kT, 0, st>>>(gv, src, dst, n);
     k_count<<<blocks(n), kT, 0, st>>>(gv, src, n);
+    k_hash_regions<<<blocks(g->V), kT, 0, st>>>(gv);
+    k_hash_insert<<<blocks(n), kT, 0, st>>>(gv, src, dst, n);
     k_list_work<<<blocks(g->V), kT, 0, st>>>(gv);
     k_delete_small<<<148 * 8, kT, 0, st>>>(gv);
     k_delete_big<<<148 * 4, kT, 0, st>>>(gv);
@@ -548,7 +643,10 @@ int gallatin_graph_expand(gallatin_graph_t *g, const uint32_t *vs, uint64_t n, v
     k_expand_prep<<<blocks(n), kT, 0, st>>>(*g, vs, n);
     int rc = run_grow(g, st);
     if (rc) return rc;
+    cudaMemsetAsync(g->nwork + 1, 0, 4, st);                    // huge lists of this round's fill
     k_expand_fill<<<148 * 8, kT, 0, st>>>(*g, vs, n);
+    k_expand_huge<<<148 * 8, kT, 0, st>>>(*g);
+    k_expand_huge_size<<<148, kT, 0, st>>>(*g);
     return status();
 }
 

@@ -111,3 +111,47 @@ def test_graph_single_edge_ops_match_o3(cuda_ok, scale, n):
         assert not msg, msg
     finally:
         G.gallatin_destroy()
+
+
+def test_graph_huge_lists_match_o3(cuda_ok):
+    """Lists of >= 2^16 entries take the whole-grid paths (k_copy_huge when a
+    batch grows them, k_expand_huge when an expansion round appends to them):
+    a star whose hub receives 2^17 edges in two batches, three expansion
+    rounds on the hub and a few small vertices, then a delete batch; sizes,
+    capacities and multisets equal O3's after every phase; pristine after."""
+    import paper_conf_ppopp_mccoyp24_b200 as G
+    nseg = 256
+    G.gallatin_init(nseg * SEG)
+    try:
+        V = 1 << 12
+        rng = np.random.Generator(np.random.PCG64(5))
+        g, o = G.Graph(V), GraphOracle(V)
+
+        def dev(a):
+            return torch.from_numpy(np.ascontiguousarray(a, dtype=np.int32)).cuda()
+
+        for half in range(2):
+            src = np.where(rng.random(1 << 16) < 0.9, 0, rng.integers(1, V, 1 << 16))
+            dst = rng.integers(0, V, 1 << 16)
+            g.insert(dev(src), dev(dst))
+            o.insert(src.astype(np.int64), dst.astype(np.int64))
+            _check(G, g, o, V, f"insert {half}")
+        vs = np.array([0, 1, 2, 3], dtype=np.int64)
+        for r in range(3):
+            g.expand(dev(vs))
+            o.expand(vs)
+            _check(G, g, o, V, f"expansion round {r}")
+        keys = np.sort(o.sorted_keys())
+        pick = keys[rng.choice(len(keys), 1 << 14, replace=False)]
+        ds, dd = (pick >> np.uint64(32)).astype(np.int64), (pick & np.uint64(0xFFFFFFFF)).astype(np.int64)
+        g.delete(dev(ds), dev(dd))
+        o.delete(ds, dd)
+        _check(G, g, o, V, "delete")
+        assert g.counters()["failed"] == 0
+        g.destroy()
+        G.gallatin_drain()
+        img = G.gallatin_snapshot()
+        msg = diff_images(img, pristine_image(nseg, int(img[4])))
+        assert not msg, msg
+    finally:
+        G.gallatin_destroy()
