@@ -429,58 +429,107 @@ __global__ void k_gather(gallatin_graph g, const uint64_t *off, uint32_t *out) {
 // doubling when an append finds it full (malloc, copy, free: the allocator is
 // called per overflowing edge, not per batch) and shrinks after every delete
 // that leaves size <= cap/4 (reading A-29 applied per edge).
-__device__ __forceinline__ void vlock(uint32_t *l) {
-    uint32_t ns = 32;
-    while (atomicCAS(l, 0u, 1u) != 0u) {
-        __nanosleep(ns);
-        if (ns < 256) ns <<= 1;
-    }
-    __threadfence();                                      // acquire the previous holder's writes
-}
-__device__ __forceinline__ void vunlock(uint32_t *l) {
-    __threadfence();                                      // release this holder's writes
-    atomicExch(l, 0u);
-}
-__device__ __forceinline__ void copy_list(uint32_t *dst, const uint32_t *src, uint32_t n) {
-    // both lists hold a multiple of 4 entries (caps are powers of two >= 4)
+// [dev] The lanes of a warp that hold their vertex's lock are served one at a
+// time by the WHOLE warp: the 32 lanes scan (delete) or copy (grow / shrink)
+// the holder's list together; the holder alone updates size, cap and list,
+// calls the allocator and releases the lock.  Same result as one thread per
+// edge (the holder's operation is unchanged); a hub list is scanned 32 (x4
+// in flight) entries per step instead of one.  Lanes whose lock is taken
+// retry after the round.
+__device__ __forceinline__ void warp_copy(uint32_t *dst, const uint32_t *src, uint32_t n) {
+    // lists hold a multiple of 4 entries (caps are powers of two >= 4) and are 16 B aligned
     uint4 *d = reinterpret_cast<uint4 *>(dst);
     const uint4 *s = reinterpret_cast<const uint4 *>(src);
-    for (uint32_t k = 0; k < (n + 3) / 4; k++) d[k] = s[k];
+    for (uint32_t k = lane(); k < (n + 3) / 4; k += 32) d[k] = s[k];
+}
+
+// last index < s of x in L (all lanes get it), or -1
+__device__ __forceinline__ int64_t warp_find_last(const uint32_t *L, uint32_t s, uint32_t x) {
+    for (int64_t top = s; top > 0; top -= 128) {
+        uint32_t e[4];
+        bool in[4];
+#pragma unroll
+        for (int u = 0; u < 4; u++) {                         // 4 loads in flight per lane
+            const int64_t idx = top - 128 + 32 * u + lane();
+            in[u] = idx >= 0;
+            e[u] = in[u] ? L[idx] : 0u;
+        }
+#pragma unroll
+        for (int u = 3; u >= 0; u--) {
+            const unsigned m = __ballot_sync(0xFFFFFFFFu, in[u] && e[u] == x);
+            if (m) return top - 128 + 32 * u + (31 - __clz((int)m));
+        }
+    }
+    return -1;
 }
 
 __global__ void __launch_bounds__(kT, kGraphMinBlocks) k_edge_insert(gallatin_graph g, const uint32_t *src,
                                                                       const uint32_t *dst, uint64_t n) {
     const uint64_t i = blockIdx.x * (uint64_t)kT + threadIdx.x;
     bool m = false, f = false, fail = false;
-    if (i < n) {
-        const uint32_t v = src[i], x = dst[i];
-        vlock(g.lock + v);
-        const uint32_t s = g.size[v], c = g.cap[v];
-        uint32_t *L = reinterpret_cast<uint32_t *>(g.list[v]);
-        bool ok = true;
-        if (s == c) {                                      // full (or no list): double
-            const uint32_t nc = c ? 2 * c : 4;
-            uint32_t *p = static_cast<uint32_t *>(gallatin_malloc((uint64_t)nc * 4));
-            if (!p) {
-                ok = false;
-                fail = true;
+    const bool active = i < n;
+    const uint32_t v = active ? src[i] : 0u, x = active ? dst[i] : 0u;
+    bool done = !active;
+    uint32_t ns = 32;
+    while (__any_sync(0xFFFFFFFFu, !done)) {
+        const bool got = !done && atomicCAS(g.lock + v, 0u, 1u) == 0u;
+        bool grow = false;
+        if (got) {
+            __threadfence();                                   // acquire the previous holder's writes
+            const uint32_t s = g.size[v];
+            if (s < g.cap[v]) {                                // room: the holder appends alone
+                reinterpret_cast<uint32_t *>(g.list[v])[s] = x;
+                g.size[v] = s + 1;
+                __threadfence();
+                atomicExch(g.lock + v, 0u);
+                done = true;
             } else {
-                m = true;
-                if (L) {
-                    copy_list(p, L, s);
-                    gallatin_free(L);
-                    f = true;
-                }
-                g.list[v] = reinterpret_cast<uint64_t>(p);
-                g.cap[v] = nc;
-                L = p;
+                grow = true;
             }
         }
-        if (ok) {
-            L[s] = x;
-            g.size[v] = s + 1;
+        unsigned holders = __ballot_sync(0xFFFFFFFFu, grow);    // the warp doubles these lists together
+        while (holders) {
+            const int l = __ffs((int)holders) - 1;
+            holders &= holders - 1;
+            const uint32_t vv = __shfl_sync(0xFFFFFFFFu, v, l);
+            const uint32_t s = g.size[vv], c = g.cap[vv];
+            uint32_t *L = reinterpret_cast<uint32_t *>(g.list[vv]);
+            if (s == c) {                                      // full (or no list): double
+                uint64_t p = 0;
+                if (lane() == (uint32_t)l) {
+                    p = reinterpret_cast<uint64_t>(gallatin_malloc((uint64_t)(c ? 2 * c : 4) * 4));
+                    if (!p) fail = true;
+                    else m = true;
+                }
+                p = __shfl_sync(0xFFFFFFFFu, p, l);
+                if (p && L) warp_copy(reinterpret_cast<uint32_t *>(p), L, s);
+                __syncwarp();
+                if (lane() == (uint32_t)l && p) {
+                    if (L) {
+                        gallatin_free(L);
+                        f = true;
+                    }
+                    g.list[vv] = p;
+                    g.cap[vv] = c ? 2 * c : 4;
+                    L = reinterpret_cast<uint32_t *>(p);
+                }
+                if (!p) L = nullptr;
+            }
+            if (lane() == (uint32_t)l) {
+                if (L) {
+                    L[s] = x;
+                    g.size[vv] = s + 1;
+                }
+                __threadfence();                               // release this holder's writes
+                atomicExch(g.lock + vv, 0u);
+                done = true;
+            }
+            __syncwarp();
         }
-        vunlock(g.lock + v);
+        if (!done && !got) {
+            __nanosleep(ns);
+            if (ns < 256) ns <<= 1;
+        }
     }
     count_warp(g.ctr, m, f, fail);
 }
@@ -489,51 +538,66 @@ __global__ void __launch_bounds__(kT, kGraphMinBlocks) k_edge_delete(gallatin_gr
                                                                       const uint32_t *dst, uint64_t n) {
     const uint64_t i = blockIdx.x * (uint64_t)kT + threadIdx.x;
     bool m = false, f = false, fail = false;
-    if (i < n) {
-        const uint32_t v = src[i], x = dst[i];
-        vlock(g.lock + v);
-        uint32_t s = g.size[v];
-        const uint32_t c = g.cap[v];
-        uint32_t *L = reinterpret_cast<uint32_t *>(g.list[v]);
-        // newest entries first (appends go to the end): remove one instance,
-        // the last entry fills the hole
-        uint32_t j = 0;
-        bool hit = false;
-        if (s) {
-            const uint4 *L4 = reinterpret_cast<const uint4 *>(L);      // 16 B loads (lists are 16 B aligned)
-            for (int64_t q = (int64_t)(s - 1) / 4; q >= 0 && !hit; q--) {
-                const uint4 e = L4[q];
-                const uint32_t b = 4 * (uint32_t)q;
-                if (b + 3 < s && e.w == x) { j = b + 3; hit = true; }
-                else if (b + 2 < s && e.z == x) { j = b + 2; hit = true; }
-                else if (b + 1 < s && e.y == x) { j = b + 1; hit = true; }
-                else if (e.x == x) { j = b; hit = true; }
-            }
-        }
-        if (hit) {
-            L[j] = L[s - 1];
-            s--;
-            g.size[v] = s;
-            if (s == 0) {
-                gallatin_free(L);
-                g.list[v] = 0;
-                g.cap[v] = 0;
-                f = true;
-            } else if (c > 4 && s <= c / 4) {
-                const uint32_t nc = list_cap(s);
-                uint32_t *p = static_cast<uint32_t *>(gallatin_malloc((uint64_t)nc * 4));
-                if (p) {
-                    copy_list(p, L, s);
+    const bool active = i < n;
+    const uint32_t v = active ? src[i] : 0u, x = active ? dst[i] : 0u;
+    bool done = !active;
+    uint32_t ns = 32;
+    while (__any_sync(0xFFFFFFFFu, !done)) {
+        const bool got = !done && atomicCAS(g.lock + v, 0u, 1u) == 0u;
+        unsigned holders = __ballot_sync(0xFFFFFFFFu, got);
+        if (holders) __threadfence();
+        while (holders) {
+            const int l = __ffs((int)holders) - 1;
+            holders &= holders - 1;
+            const uint32_t vv = __shfl_sync(0xFFFFFFFFu, v, l), xx = __shfl_sync(0xFFFFFFFFu, x, l);
+            uint32_t s = g.size[vv];
+            const uint32_t c = g.cap[vv];
+            uint32_t *L = reinterpret_cast<uint32_t *>(g.list[vv]);
+            // newest entries first (appends go to the end): remove one
+            // instance, the last entry fills the hole (reading R-7)
+            const int64_t j = s ? warp_find_last(L, s, xx) : -1;
+            uint64_t p = 0;
+            bool copy = false;
+            if (lane() == (uint32_t)l && j >= 0) {
+                L[j] = L[s - 1];
+                s--;
+                g.size[vv] = s;
+                if (s == 0) {
                     gallatin_free(L);
-                    g.list[v] = reinterpret_cast<uint64_t>(p);
-                    g.cap[v] = nc;
-                    m = f = true;
-                } else {
-                    fail = true;
+                    g.list[vv] = 0;
+                    g.cap[vv] = 0;
+                    f = true;
+                } else if (c > 4 && s <= c / 4) {
+                    p = reinterpret_cast<uint64_t>(gallatin_malloc((uint64_t)list_cap(s) * 4));
+                    if (p) copy = true;
+                    else fail = true;
                 }
             }
+            copy = __shfl_sync(0xFFFFFFFFu, copy, l);
+            if (copy) {
+                p = __shfl_sync(0xFFFFFFFFu, p, l);
+                s = __shfl_sync(0xFFFFFFFFu, s, l);
+                __syncwarp();                                  // the hole fill precedes the copy
+                warp_copy(reinterpret_cast<uint32_t *>(p), L, s);
+                __syncwarp();
+                if (lane() == (uint32_t)l) {
+                    gallatin_free(L);
+                    g.list[vv] = p;
+                    g.cap[vv] = list_cap(s);
+                    m = f = true;
+                }
+            }
+            if (lane() == (uint32_t)l) {
+                __threadfence();
+                atomicExch(g.lock + vv, 0u);
+                done = true;
+            }
+            __syncwarp();
         }
-        vunlock(g.lock + v);
+        if (!done && !got) {
+            __nanosleep(ns);
+            if (ns < 256) ns <<= 1;
+        }
     }
     count_warp(g.ctr, m, f, fail);
 }
