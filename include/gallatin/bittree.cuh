@@ -240,13 +240,27 @@ __device__ inline bool bt_claim_range(const BitTree &t, uint64_t i, uint64_t k) 
 // Highest start i such that [i, i+k) is all set (first fit from the back,
 // P:138 / reading A-17), by a top-down walk over the leaf words; kNone if no
 // such run is visible.  Leaf reads are relaxed: the claim re-validates.
-__device__ inline uint64_t bt_find_highest_run(const BitTree &t, uint64_t k) {
+// `below`: only runs entirely below this index (kNone: the whole tree).
+// The leaf words are loaded 8 at a time (independent loads in flight) and
+// walked from the top down in registers.
+__device__ inline uint64_t bt_find_highest_run(const BitTree &t, uint64_t k, uint64_t below = kNone) {
     if (k == 0 || k > t.nbits) return kNone;
-    const uint64_t nw = (t.nbits + 63) / 64;
+    const uint64_t lim = below < t.nbits ? below : t.nbits;
+    if (lim < k) return kNone;
+    const uint64_t nw = (lim + 63) / 64;
+    const uint64_t top_mask = (lim & 63) ? ((1ull << (lim & 63)) - 1) : ~0ull;   // bits < lim in the top word
     uint64_t run = 0;   // length of the set run just above the current word
     uint64_t top = 0;   // highest element of that run
+    uint64_t batch[8];
     for (uint64_t wi = nw; wi-- > 0;) {
-        const uint64_t v = ptx::ld_relaxed(t.w + t.off[0] + wi);
+        const uint32_t slot = (uint32_t)((nw - 1 - wi) & 7);
+        if (slot == 0) {                                      // next 8 words down, loads in flight together
+#pragma unroll
+            for (int q = 0; q < 8; q++)
+                batch[q] = wi >= (uint64_t)q ? ptx::ld_relaxed(t.w + t.off[0] + wi - q) : 0ull;
+        }
+        uint64_t v = batch[slot];
+        if (wi == nw - 1) v &= top_mask;
         const uint64_t base = wi << 6;
         if (v == ~0ull) {
             if (run == 0) top = base + 63;

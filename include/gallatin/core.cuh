@@ -885,8 +885,14 @@ __device__ inline __noinline__ void *malloc_large(const View &v, uint64_t k) {
     uint64_t i;
     int misses = 0;
     bool trimmed = false;
+    uint64_t below = kNone;
+    uint32_t lost = 0;
     for (;;) {
-        i = bt_find_highest_run(st, k);
+        i = bt_find_highest_run(st, k, below);
+        if (i == kNone && below != kNone) {                   // nothing lower: search everything again
+            below = kNone;
+            continue;
+        }
         if (i == kNone) {
             if (!trimmed) {                                   // [dev] as get_run: slots give back first
                 trimmed = true;
@@ -898,7 +904,17 @@ __device__ inline __noinline__ void *malloc_large(const View &v, uint64_t k) {
         }
         if (bt_claim_range(st, i, k)) break;
         oom_notify(v);                                        // the claim's rollback gave segments back
-        bo.pause();
+        // [dev] concurrent claimers of one size all found the same run: the
+        // loser looks below it, at a pseudo-random distance (serially no
+        // claim loses: the highest run)
+        {
+            const uint32_t tid = blockIdx.x * blockDim.x + threadIdx.x;
+            uint32_t h = (tid * 0x9E3779B1u) ^ (++lost * 0x85EBCA6Bu);
+            h ^= h >> 15;
+            const uint32_t span = 128u * (uint32_t)k * (lost < 8 ? lost : 8u);   // widens with each loss
+            const uint64_t jit = (uint64_t)(h % span);
+            below = i > jit ? i - jit : 0;
+        }
     }
     ptx::fence_acq_rel();
     ptx::st_relaxed(v.seg_tid + i, kTrees + (uint32_t)k);
