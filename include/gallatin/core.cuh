@@ -88,7 +88,7 @@ __device__ inline __noinline__ void btree_reconcile(const View &v, uint32_t t, u
     if (flipped) bt_reconcile_up(bt, 0, s >> 6);
 }
 
-__device__ inline __noinline__ void try_free_segment(const View &v, uint64_t s, uint32_t t);
+__device__ inline __noinline__ bool try_free_segment(const View &v, uint64_t s, uint32_t t);
 
 // ---- exhaustion record [dev] (DESIGN.md Deviations 11) ----------------------
 // Without it every request that finds the heap exhausted repeats the whole
@@ -157,20 +157,25 @@ __device__ inline __noinline__ void oom_leave(const View &v, uint32_t t, uint64_
 }
 
 // Every thread whose RMW on seg_word[s] changed a block-tree predicate repairs
-// that bit; the RMW that brings a segment back to "all blocks home" retires it.
-__device__ __forceinline__ void seg_after_rmw(const View &v, uint64_t s, uint64_t old, uint64_t now) {
+// that bit; the RMW that brings a segment back to "all blocks home" retires it
+// -- first: if its retiring CAS succeeds no RMW came between, and the retire
+// reconciles the bit itself (one reconcile instead of two on the free path's
+// tail).  Returns whether the segment was retired.
+__device__ __forceinline__ bool seg_after_rmw(const View &v, uint64_t s, uint64_t old, uint64_t now) {
     const uint32_t to = sw_tree(old), tn = sw_tree(now);
+    if (tn < kTrees && tn == to && sw_avail(now) == (int32_t)nb_of(tn) && sw_avail(old) < sw_avail(now) &&
+        try_free_segment(v, s, tn))
+        return true;
     if (to < kTrees && sw_in_tree(old, to) != sw_in_tree(now, to)) btree_reconcile(v, to, s);
     if (tn < kTrees && tn != to && sw_in_tree(old, tn) != sw_in_tree(now, tn)) btree_reconcile(v, tn, s);
-    if (tn < kTrees && tn == to && sw_avail(now) == (int32_t)nb_of(tn) && sw_avail(old) < sw_avail(now))
-        try_free_segment(v, s, tn);
+    return false;
 }
 
 // "When all blocks are returned, the segment is freed and re-added to the
 // segment tree".
-__device__ inline __noinline__ void try_free_segment(const View &v, uint64_t s, uint32_t t) {
+__device__ inline __noinline__ bool try_free_segment(const View &v, uint64_t s, uint32_t t) {
     const uint64_t full = sw_make(t, (int32_t)nb_of(t));
-    if (ptx::atom_cas(v.seg_word + s, full, sw_make(kTreeFree, 0)) != full) return;
+    if (ptx::atom_cas(v.seg_word + s, full, sw_make(kTreeFree, 0)) != full) return false;
     ptx::st_relaxed(v.seg_tid + s, kTreeFree);
     // No block of s is out or in flight: reset its ring.
     ptx::st_relaxed(v.q_head + s, 0u);
@@ -183,6 +188,7 @@ __device__ inline __noinline__ void try_free_segment(const View &v, uint64_t s, 
     btree_reconcile(v, t, s);
     bt_insert(seg_tree(v), s);
     oom_notify(v);
+    return true;
 }
 
 // Every formatted segment whose blocks are all home goes back to the segment
@@ -370,9 +376,9 @@ __device__ inline __noinline__ void return_block(const View &v, uint32_t gid) {
     ptx::st_relaxed(slotp, (uint16_t)(gid % kMaxBlocks));
     ptx::fence_acq_rel();
     const uint64_t old = ptx::atom_add(v.seg_word + s, 1ull);
-    seg_after_rmw(v, s, old, old + 1);                       // all blocks home: try_free_segment notifies
+    const bool retired = seg_after_rmw(v, s, old, old + 1);   // all blocks home: try_free_segment notified
     // a search can newly find the segment only if it had no block available
-    if (sw_avail(old) == 0) oom_notify(v);
+    if (!retired && sw_avail(old) == 0) oom_notify(v);
 }
 
 // n slices of block gid came back; the team completing 4096 returns it
