@@ -228,12 +228,19 @@ __device__ __forceinline__ uint64_t claim_retry_hint(uint64_t wi, uint64_t old, 
 // aims there too, and a launch's first burst of refills (one per slot, all
 // at once) then takes one segment per round -- but at a pseudo-random bit at
 // or above it in that word; the RMW tells whether it was free.
-__device__ __forceinline__ uint64_t claim_spread(uint64_t s, uint32_t attempt) {
+// A window claim of kmax segments aims at a window boundary (kmax rounded up
+// to a power of two, at most a word), so concurrent windows do not overlap.
+__device__ __forceinline__ uint32_t claim_align(uint32_t kmax) {
+    return kmax >= 64 ? 64u : (kmax <= 1 ? 1u : 1u << (32 - __clz(kmax - 1)));
+}
+__device__ __forceinline__ uint64_t claim_spread(uint64_t s, uint32_t attempt, uint32_t kmax = 1) {
     const uint32_t tid = blockIdx.x * blockDim.x + threadIdx.x;
     uint32_t h = (tid * 0x27D4EB2Fu) ^ (attempt * 0x165667B1u);
     h ^= h >> 15;
     const uint32_t lo = (uint32_t)(s & 63);
-    return (s & ~63ull) | (lo + h % (64u - lo));
+    uint32_t b = (lo + h % (64u - lo)) & ~(claim_align(kmax) - 1);
+    if (b < lo) b = lo;
+    return (s & ~63ull) | b;
 }
 
 // [dev] The FIRST loss of a segment claim means every concurrent claimer
@@ -243,13 +250,14 @@ __device__ __forceinline__ uint64_t claim_spread(uint64_t s, uint32_t attempt) {
 // instead of queueing on the one word; later losses use the free bits the
 // RMW returned (claim_retry_hint).  Serially no claim loses.
 constexpr uint32_t kSpreadWords = 4;
-__device__ __forceinline__ uint64_t claim_first_loss(const View &v, uint64_t wi) {
+__device__ __forceinline__ uint64_t claim_first_loss(const View &v, uint64_t wi, uint32_t kmax = 1) {
     const uint32_t tid = blockIdx.x * blockDim.x + threadIdx.x;
     uint32_t h = tid * 0x9E3779B1u;
     h ^= h >> 13;
     h *= 0x85EBCA6Bu;
     h ^= h >> 16;
-    const uint64_t s = ((wi + h % kSpreadWords) << 6) | ((h >> 8) & 63);
+    const uint32_t words = kSpreadWords + kmax / 2;            // room for the windows of every claimer
+    const uint64_t s = ((wi + h % words) << 6) | (((h >> 8) & 63) & ~(claim_align(kmax) - 1));
     return s < v.nseg ? s : v.nseg - 1;
 }
 
@@ -304,7 +312,7 @@ __device__ inline __noinline__ uint64_t claim_front_run(const View &v, uint32_t 
     for (;;) {
         uint64_t s = hint != kNone ? hint : bt_successor<false>(st, from);
         if (hint == kNone && attempt > 0 && s != kNone) {
-            s = claim_spread(s, attempt);
+            s = claim_spread(s, attempt, kmax);
             if (s >= v.nseg) s = v.nseg - 1;
         }
         hint = kNone;
@@ -332,7 +340,7 @@ __device__ inline __noinline__ uint64_t claim_front_run(const View &v, uint32_t 
         if (flip) bt_reconcile_up(st, 0, wi);
         if (extra) oom_notify(v);
         if (run == 0) {
-            hint = ++attempt == 1 ? claim_first_loss(v, wi) : claim_retry_hint(wi, old & ~mask, attempt);
+            hint = ++attempt == 1 ? claim_first_loss(v, wi, kmax) : claim_retry_hint(wi, old & ~mask, attempt);
             from = (wi + 1) << 6;
             continue;
         }
