@@ -919,14 +919,15 @@ __device__ inline __noinline__ void *malloc_large(const View &v, uint64_t k) {
         if (bt_claim_range(st, i, k)) break;
         oom_notify(v);                                        // the claim's rollback gave segments back
         // [dev] concurrent claimers of one size all found the same run: the
-        // loser looks below it, at a pseudo-random distance (serially no
-        // claim loses: the highest run)
+        // loser looks below it, a pseudo-random number of k-runs down (whole
+        // runs, so equal-size claims stay packed from the top: the heap still
+        // holds floor(nseg / k) of them); serially no claim loses: the
+        // highest run
         {
             const uint32_t tid = blockIdx.x * blockDim.x + threadIdx.x;
             uint32_t h = (tid * 0x9E3779B1u) ^ (++lost * 0x85EBCA6Bu);
             h ^= h >> 15;
-            const uint32_t span = 128u * (uint32_t)k * (lost < 8 ? lost : 8u);   // widens with each loss
-            const uint64_t jit = (uint64_t)(h % span);
+            const uint64_t jit = k * (uint64_t)(h % (128u * (lost < 8 ? lost : 8u)));   // widens with each loss
             below = i > jit ? i - jit : 0;
         }
     }
