@@ -748,7 +748,13 @@ __device__ inline __noinline__ bool refill_slot(const View &v, uint32_t si, uint
     const uint32_t first_run = fr < cap ? fr : cap;
     const uint32_t grow = m_prev << v.run_grow;                   // x 2^run_grow per refill
     uint32_t want = m_prev == 0 ? first_run : (grow < cap ? grow : cap);
-    if (hint > want) want = hint < cap ? hint : cap;
+    if (hint > want) {
+        // whole segments once the hint exceeds one (a run of more than nb
+        // blocks is taken in whole segments: 111 blocks would get 64)
+        const uint32_t nb = nb_of(c);
+        const uint32_t h = hint > nb ? (hint + nb - 1) / nb * nb : hint;
+        want = h < cap ? h : cap;
+    }
     uint32_t first = 0;
 #ifdef GALLATIN_TRACE
     const uint64_t t0 = ptx::globaltimer();

@@ -51,6 +51,17 @@ for sz in sizes:
         out[f"tag{g_}"] = {"n": int(m.sum()), "p50": round(float(np.percentile(lat, 50)), 2),
                            "p90": round(float(np.percentile(lat, 90)), 2), "max": round(float(lat.max()), 2),
                            "first_start_us": round(float(st_.min()), 1), "last_end_us": round(float(((t[m, 1].astype(np.int64) - base) / 1e3).max()), 1)}
+    m0 = tag == 0
+    if m0.any():
+        info = t[m0, 2]
+        want = ((info >> np.uint64(12)) & np.uint64(0xFFF)).astype(int)
+        got = (info & np.uint64(0xFFF)).astype(int)
+        slot = ((info >> np.uint64(32)) & np.uint64(0xFFFFFFF)).astype(int)
+        st0 = (t0[m0] - base) / 1e3
+        pairs, cnts = np.unique(np.stack([want, got], 1), axis=0, return_counts=True)
+        out["refill_want_got"] = {f"{a}->{b}": int(c) for (a, b), c in zip(pairs, cnts)}
+        out["refills_per_slot_max"] = int(np.bincount(slot).max())
+        out["late_refills"] = int((st0 > 20).sum())
     m1 = tag == 1
     if m1.any():
         att = ((t[m1, 2] >> np.uint64(32)) & np.uint64(0xFFFF)).astype(int)
