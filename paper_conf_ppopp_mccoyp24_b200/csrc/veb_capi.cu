@@ -41,22 +41,36 @@ __global__ void __launch_bounds__(kThreads) k_delete(BitTree t, const uint64_t *
     const bool r = bt_delete(t, keys[i]);
     if (out) out[i] = r;
 }
-__global__ void __launch_bounds__(kThreads) k_member(BitTree t, const uint64_t *keys, uint8_t *out, uint64_t n) {
-    const uint64_t i = blockIdx.x * (uint64_t)kThreads + threadIdx.x;
-    if (i >= n) return;
-    out[i] = bt_member<true>(t, keys[i]);
+// Read-only queries, ITEMS per thread: the ITEMS query keys are loaded
+// before any is walked (their HBM latency paid once, not ITEMS times); the
+// tree words come through the read-only path (L1-resident at u <= 2^24).
+enum QueryOp { kMember, kSucc, kPred };
+template <QueryOp OP, int ITEMS, typename OUT>
+__global__ void __launch_bounds__(kThreads) k_query(BitTree t, const uint64_t *__restrict__ q, OUT *__restrict__ out,
+                                                    uint64_t n) {
+    const uint64_t base = blockIdx.x * (uint64_t)(kThreads * ITEMS) + threadIdx.x;
+    uint64_t x[ITEMS];
+#pragma unroll
+    for (int k = 0; k < ITEMS; k++) {
+        const uint64_t i = base + (uint64_t)kThreads * k;
+        x[k] = __ldcs(reinterpret_cast<const unsigned long long *>(q) + (i < n ? i : n - 1));
+    }
+#pragma unroll
+    for (int k = 0; k < ITEMS; k++) {
+        const uint64_t i = base + (uint64_t)kThreads * k;
+        if (i >= n) break;
+        if (OP == kMember) out[i] = (OUT)bt_member<true>(t, x[k]);
+        else if (OP == kSucc) out[i] = (OUT)bt_successor<true>(t, x[k]);
+        else out[i] = (OUT)bt_predecessor<true>(t, x[k]);
+    }
 }
-__global__ void __launch_bounds__(kThreads) k_successor(BitTree t, const uint64_t *__restrict__ q,
-                                                        uint64_t *__restrict__ out, uint64_t n) {
-    const uint64_t i = blockIdx.x * (uint64_t)kThreads + threadIdx.x;
-    if (i >= n) return;
-    out[i] = bt_successor<true>(t, q[i]);
-}
-__global__ void __launch_bounds__(kThreads) k_predecessor(BitTree t, const uint64_t *__restrict__ q,
-                                                          uint64_t *__restrict__ out, uint64_t n) {
-    const uint64_t i = blockIdx.x * (uint64_t)kThreads + threadIdx.x;
-    if (i >= n) return;
-    out[i] = bt_predecessor<true>(t, q[i]);
+template <QueryOp OP, typename OUT>
+int launch_query(const BitTree &t, const uint64_t *q, OUT *out, uint64_t n, cudaStream_t st) {
+    if (n >= (1ull << 20))                                    // enough queries to fill every SM 4-deep
+        k_query<OP, 4, OUT><<<(unsigned)((n + 4 * kThreads - 1) / (4 * kThreads)), kThreads, 0, st>>>(t, q, out, n);
+    else
+        k_query<OP, 1, OUT><<<grid_for(n), kThreads, 0, st>>>(t, q, out, n);
+    return launch_status();
 }
 }  // namespace
 
@@ -107,9 +121,18 @@ int veb_clear(veb_t *h, void *stream) {
 
 VEB_BULK(veb_insert, k_insert, uint8_t, false)
 VEB_BULK(veb_delete, k_delete, uint8_t, false)
-VEB_BULK(veb_member, k_member, uint8_t, true)
-VEB_BULK(veb_successor, k_successor, uint64_t, true)
-VEB_BULK(veb_predecessor, k_predecessor, uint64_t, true)
+
+#define VEB_QUERY(name, op, out_t)                                                         \
+    int name(veb_t *h, const uint64_t *d_keys, out_t *d_out, uint64_t n, void *stream) {   \
+        if (!h) return GALLATIN_ERR_INVALID;                                                \
+        if (n == 0) return GALLATIN_OK;                                                     \
+        if (!d_keys || !d_out) return GALLATIN_ERR_INVALID;                                 \
+        return launch_query<op, out_t>(h->t, d_keys, d_out, n, S(stream));                 \
+    }
+
+VEB_QUERY(veb_member, kMember, uint8_t)
+VEB_QUERY(veb_successor, kSucc, uint64_t)
+VEB_QUERY(veb_predecessor, kPred, uint64_t)
 
 int veb_words(const veb_t *h, uint64_t *words) {
     if (!h || !words) return GALLATIN_ERR_INVALID;
