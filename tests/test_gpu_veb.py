@@ -66,6 +66,18 @@ def test_config1_veb_parity(cuda_ok):
     ])
 
 
+def test_bulk_queries_four_per_thread(cuda_ok):
+    """Query batches of >= 2^20 keys run 4 queries per thread (keys loaded
+    first); a ragged count exercises the clamped tail: successor, predecessor
+    and member equal O1's bit-exactly."""
+    k = 20
+    seed = wg.cell_seed(1, 320)
+    ins = wg.distinct_below(seed, 1 << 16, 1 << k)
+    q = np.concatenate([wg.uniform_below(seed ^ 3, (1 << 20) + 1021, 1 << k),
+                        np.array([0, (1 << k) - 1, 1 << k], dtype=np.uint64)])
+    _run_batches(k, [(OV_INSERT, ins), (OV_SUCC, q), (OV_PRED, q), (OV_MEMBER, q)])
+
+
 @pytest.mark.parametrize("k", [1, 3, 6, 7, 12, 13, 18, 19, 24])
 def test_universe_sizes(cuda_ok, k):
     """Every level count (1..5) incl. partial top words; dense and sparse sets."""
