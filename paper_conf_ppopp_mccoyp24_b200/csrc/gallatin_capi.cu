@@ -674,8 +674,8 @@ __device__ __forceinline__ void free_warp_tile(const View &v, void *const *ptrs,
     uint32_t o16[ITEMS], t[ITEMS];
 #pragma unroll
     for (int k = 0; k < ITEMS; k++) {
-        const uint64_t off = p[k] - v.heap;
-        const bool in = p[k] && off < heap_bytes;
+        const uint64_t off = p[k] - v.heap;                        // NULL: 2^64 - heap, out of range
+        const bool in = off < heap_bytes;
         o16[k] = (uint32_t)(off >> 16);                            // segment << 8 | 64 KB unit
         t[k] = in ? __ldca(v.seg_tid + (o16[k] >> 8)) : core::kTreeFree;
     }
