@@ -88,7 +88,7 @@ typedef struct gallatin_config {
     uint32_t cta_tiles;    /* pipeline = 3: tiles of 1024 requests per CTA, the next one prefetched (0 = 4) */
     uint32_t cta_threads;  /* bulk malloc CTA kernel: threads per CTA (4 requests each, one slot RMW per class
                               per CTA): 0/128 = 128 (default, 10 CTAs/SM), 64, 256 */
-    uint32_t free_threads; /* bulk free kernel: 0/128 = 128-thread CTAs (default), 256 */
+    uint32_t free_threads; /* bulk free kernel: 0 = 64-thread CTAs at 32 registers (64 warps/SM) from 2^23 pointers on, else 128 (default); 64, 128, 256 force that CTA size */
 } gallatin_config_t;
 
 int gallatin_init(uint64_t heap_bytes);                 /* defaults for the rest */

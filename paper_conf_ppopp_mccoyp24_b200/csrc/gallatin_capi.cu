@@ -707,6 +707,7 @@ __device__ __forceinline__ void free_warp_tile(const View &v, void *const *ptrs,
 // k_bulk_free's protocol through free_warp_tile (32-bit block-id math, one
 // range check per item) with the warp's loads unclamped when its whole tile
 // is in range.
+constexpr uint64_t kFreeWideMin = 1ull << 23;     // bulk frees from here on take the 64-warp/SM kernel
 template <int ITEMS, int NT = kThreads, int MINB = 6 * kThreads / NT>
 __global__ void __launch_bounds__(NT, MINB) k_bulk_free_w(void *const *__restrict__ ptrs, uint64_t n) {
     const View &v = c_view;
@@ -1125,7 +1126,7 @@ int gallatin_init_ex(const gallatin_config_t *cfg_in) {
         return GALLATIN_ERR_INVALID;
     if (cfg.prefetch > 2 || cfg.pipeline > 3 || cfg.free_team > 3 || cfg.demand_hint > 2 || cfg.cta_tiles > 1024 ||
         (cfg.cta_threads != 0 && cfg.cta_threads != 64 && cfg.cta_threads != 128 && cfg.cta_threads != 256) ||
-        (cfg.free_threads != 0 && cfg.free_threads != 128 && cfg.free_threads != 256))
+        (cfg.free_threads != 0 && cfg.free_threads != 64 && cfg.free_threads != 128 && cfg.free_threads != 256))
         return GALLATIN_ERR_INVALID;
     if (!cfg.run_grow) cfg.run_grow = 3;
     if (cfg.run_grow > 8) return GALLATIN_ERR_INVALID;
@@ -1300,9 +1301,16 @@ int gallatin_free(void *const *d_ptrs, uint64_t n, void *stream) {
     } else if (g.cfg.bulk_items == 0 && n >= (uint64_t)kItemsMin && g.cfg.free_team == 1) {
         k_bulk_free_cta<4><<<grid_for((n + 3) / 4), kThreads, 0, S(stream)>>>(d_ptrs, n);
     } else if (g.cfg.bulk_items == 0 && n >= (uint64_t)kItemsMin && g.cfg.free_team != 2) {
-        // default: warp teams, 32-bit block ids, 128-thread CTAs
+        // default: warp teams, 32-bit block ids; 64-thread CTAs at 32
+        // registers (64 warps per SM) from kFreeWideMin pointers on, where
+        // more frees in flight shorten a throughput-bound launch, else
+        // 128-thread CTAs at 40 registers (48 warps), whose smaller launches
+        // are bound by the block-return tail (DESIGN.md ablations)
+        const bool wide = g.cfg.free_threads == 64 || (g.cfg.free_threads == 0 && n >= kFreeWideMin);
         if (g.cfg.free_threads == 256)
             k_bulk_free_w<4><<<grid_for((n + 3) / 4), kThreads, 0, S(stream)>>>(d_ptrs, n);
+        else if (wide)
+            k_bulk_free_w<4, 64, 32><<<(unsigned)((n + 255) / 256), 64, 0, S(stream)>>>(d_ptrs, n);
         else
             k_bulk_free_w<4, 128><<<(unsigned)((n + 511) / 512), 128, 0, S(stream)>>>(d_ptrs, n);
     } else if (g.cfg.bulk_items >= 8)

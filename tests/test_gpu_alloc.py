@@ -273,7 +273,8 @@ def test_config3_full_size_bench_launch(cuda_ok, G):
 
 @pytest.mark.parametrize("knobs", [dict(pipeline=1), dict(pipeline=2), dict(pipeline=3), dict(free_team=1),
                                    dict(cta_threads=64), dict(cta_threads=256), dict(free_team=2),
-                                   dict(free_threads=256), dict(free_team=2, free_threads=128),
+                                   dict(free_threads=256), dict(free_threads=64), dict(free_threads=128),
+                                   dict(free_team=2, free_threads=128),
                                    dict(bulk_items=8), dict(bulk_items=16), dict(bulk_items=1),
                                    dict(pipeline=2, free_team=1)])
 @pytest.mark.parametrize("n", [(1 << 21) + 77, 1 << 22])
