@@ -172,19 +172,23 @@ def run_ours(args, rank, world, local):
 
     ev = {"m0": [], "m1": [], "f0": [], "f1": []}
 
-    def step(record: bool):
+    def step(record: bool, st_=None):
+        # calls go to the current stream (the capture stream under a graph,
+        # st_); graph-captured timing events are recorded as external nodes
+        cur = torch.cuda.current_stream()
+        ext = st_ is not None
         for (s, n), st in zip(cells, size_t):
             p = ptrs[:n]
             G.gallatin_reset()
             if record:
-                e = torch.cuda.Event(enable_timing=True); e.record(stream); ev["m0"].append(e)
+                e = torch.cuda.Event(enable_timing=True, external=ext); e.record(cur); ev["m0"].append(e)
             G.gallatin_malloc(st, p)
             if record:
-                e = torch.cuda.Event(enable_timing=True); e.record(stream); ev["m1"].append(e)
-                e = torch.cuda.Event(enable_timing=True); e.record(stream); ev["f0"].append(e)
+                e = torch.cuda.Event(enable_timing=True, external=ext); e.record(cur); ev["m1"].append(e)
+                e = torch.cuda.Event(enable_timing=True, external=ext); e.record(cur); ev["f0"].append(e)
             G.gallatin_free(p)
             if record:
-                e = torch.cuda.Event(enable_timing=True); e.record(stream); ev["f1"].append(e)
+                e = torch.cuda.Event(enable_timing=True, external=ext); e.record(cur); ev["f1"].append(e)
 
     # correctness gate on the bench's own launch configuration (untimed): the
     # first cell's pointers stamp/verify clean and the heap drains to pristine
@@ -201,6 +205,18 @@ def run_ours(args, rank, world, local):
     if bad:
         raise SystemExit(f"stamp-verify failed: {bad} words")
 
+    # the K timed steps as one CUDA graph (same launches, no host launch gaps
+    # between the step's 27 kernels), replayed once untimed to upload it
+    graph = None
+    if args.graph:
+        graph = torch.cuda.CUDAGraph()
+        cap = torch.cuda.Stream()
+        cap.wait_stream(stream)
+        with torch.cuda.graph(graph, stream=cap):
+            for _ in range(args.steps):
+                step(True, cap)
+        graph.replay()
+        torch.cuda.synchronize()
     clk = ClockSampler(local)
     d.barrier()
     torch.cuda.synchronize()
@@ -208,8 +224,11 @@ def run_ours(args, rank, world, local):
     t0 = torch.cuda.Event(enable_timing=True)
     t1 = torch.cuda.Event(enable_timing=True)
     t0.record(stream)
-    for _ in range(args.steps):
-        step(True)
+    if graph is not None:
+        graph.replay()
+    else:
+        for _ in range(args.steps):
+            step(True)
     t1.record(stream)
     torch.cuda.synchronize()
     clocks = clk.stop()
@@ -267,7 +286,8 @@ def run_ours(args, rank, world, local):
             "value": value, "unit": "ops/s", "n_gpus": world, "steps": args.steps, "warmup": max(args.warmup, 3),
             "ms_per_step": ms / args.steps, "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
             "dtype": "u64", "data": "synthetic",
-            "config": {"workload": "BASELINE configs[1]: single-size sweep 16 B-4 KB, n_s=min(2^24, 8GiB/s) threads, "
+            "config": {"launch": "one CUDA graph of the K timed steps" if args.graph else "eager",
+                       "workload": "BASELINE configs[1]: single-size sweep 16 B-4 KB, n_s=min(2^24, 8GiB/s) threads, "
                                    "16 GiB heap, reset+malloc+free per size" + (f" (1/{args.scale} scale)" if args.scale > 1 else ""),
                        "heap_bytes": HEAP_C2, "cells": [[s, n] for s, n in cells],
                        "ops_per_step": ops_per_step, "parallelism": f"replicas x{world}",
@@ -658,6 +678,8 @@ def main():
     ap.add_argument("--scale", type=int, default=1, help="divide every thread count (debug only)")
     ap.add_argument("--no-extras", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
+    ap.add_argument("--no-graph", dest="graph", action="store_false",
+                    help="issue the timed steps eagerly instead of as one CUDA graph")
     args = ap.parse_args()
     rank, world, local = dist_setup(args.gpus)
     if args.impl == "reference":
