@@ -71,24 +71,20 @@ typedef struct gallatin_config {
     uint32_t run_max;
     uint32_t format_ahead;
     uint32_t fence_free;
-    uint32_t bulk_items;   /* requests per thread in the bulk malloc kernel: 0 = auto, 1, 4, 8 or 16 (free: 1 or 4) */
+    uint32_t bulk_items;   /* bulk kernels: 0 = auto (4 from 606,208 requests on, else 1); 1 = one request per
+                              thread and one slot RMW per warp team (k_bulk_malloc<1> / k_bulk_free<1>); 4 = four
+                              per thread, one slot RMW per class per 512-request CTA tile (k_bulk_malloc_cta) and
+                              the warp-team free with 32-bit block ids (k_bulk_free_w) */
     uint32_t run_init;     /* first run of an empty slot of class c: min(max(run_init >> c, min(run_init, 8)), 256 >> c) blocks (default: the largest power of two <= 256 whose first runs over all slots fit in half the heap) */
     uint32_t prefetch;     /* 1 = fetch the next run at the middle of the current one; 0/2 = off (default) */
     uint32_t run_grow;     /* a refilled run is 2^run_grow times the last one, up to the cap: 1..8 (default 3) */
-    uint32_t pipeline;     /* bulk kernels at bulk_items = 0: 1 = persistent CTAs that TMA-load the next tile while
-                              this tile's atomics are in flight; 3 = persistent CTAs (malloc) / warps (free) that
-                              load the next tile into registers before processing this one; 0/2 = one tile per CTA
-                              (default) */
-    uint32_t free_team;    /* bulk free: 0/3 = one free-counter RMW per warp team, 32-bit block-id decode (default);
-                              2 = the same teams with 64-bit decode and clamped loads (k_bulk_free, ablation);
-                              1 = one RMW per block per CTA tile (shared-memory aggregation, ablation) */
     uint32_t demand_hint;  /* bulk malloc: 0/1 = a refill takes at least the blocks this slot's share of the launch
                               needs (the CTA's per-class count x CTAs / slots; DESIGN.md Deviations 10), up to the
                               run cap (default); 2 = off (runs grow 2^run_grow-fold per refill only) */
-    uint32_t cta_tiles;    /* pipeline = 3: tiles of 1024 requests per CTA, the next one prefetched (0 = 4) */
-    uint32_t cta_threads;  /* bulk malloc CTA kernel: threads per CTA (4 requests each, one slot RMW per class
-                              per CTA): 0/128 = 128 (default, 10 CTAs/SM), 64, 256 */
-    uint32_t free_threads; /* bulk free kernel: 0 = 64-thread CTAs at 32 registers (64 warps/SM) from 2^23 pointers on, else 128 (default); 64, 128, 256 force that CTA size */
+    uint32_t oom_record;   /* 0/1 = exhaustion record on (default; DESIGN.md Deviations 11): a run request of a
+                              block tree confirmed exhausted fails in O(1) until memory comes back; 2 = off (every
+                              request repeats the full search with slot trims -- the policy oracle/alloc_runs.c
+                              replays exactly) */
 } gallatin_config_t;
 
 int gallatin_init(uint64_t heap_bytes);                 /* defaults for the rest */
@@ -143,7 +139,7 @@ typedef struct gallatin_stats {
     uint32_t nslot[9];           /* block-buffer slots per class                    */
     uint32_t run_cap[9];         /* max blocks per run per class                    */
     uint32_t slot_base, slot_min, run_max, format_ahead, fence_free, run_init, formatters, prefetch;
-    uint32_t run_grow;
+    uint32_t run_grow, demand_hint, oom_record;
 } gallatin_stats_t;
 int gallatin_stats(gallatin_stats_t *out);               /* synchronizes the device */
 

@@ -707,14 +707,15 @@ __device__ inline __noinline__ uint32_t trim_slots(const View &v) {
 // more after an empty trim: a concurrent refiller's trim may just have given
 // the blocks back.  Serially this is one trim and one retry.
 __device__ inline __noinline__ uint32_t get_run(const View &v, uint32_t t, uint32_t want, uint32_t *first) {
+    const bool rec = v.oom_record != 0;
 #ifdef GALLATIN_TRACE
     const uint64_t tr0 = ptx::globaltimer();
-    uint32_t got = get_run_once(v, t, want, first, true);
+    uint32_t got = get_run_once(v, t, want, first, rec);
     ptx::trace(tr0, ptx::globaltimer(), (3ull << 60) | ((uint64_t)t << 24) | (want << 12) | got);
 #else
-    uint32_t got = get_run_once(v, t, want, first, true);
+    uint32_t got = get_run_once(v, t, want, first, rec);
 #endif
-    if (got || *first == kOomFast) return got;                // [dev] exhaustion record
+    if (got || (rec && *first == kOomFast)) return got;       // [dev] exhaustion record
     oom_enter(v);
     uint64_t e = 0;
     for (uint32_t r = 0; got == 0 && r < 8; r++) {
@@ -723,7 +724,7 @@ __device__ inline __noinline__ uint32_t get_run(const View &v, uint32_t t, uint3
         got = get_run_once(v, t, 1, first);
         if (back == 0 && r >= 1) break;
     }
-    oom_leave(v, t, e, got == 0);
+    oom_leave(v, t, e, rec && got == 0);
     return got;
 }
 

@@ -63,6 +63,7 @@ struct gallatin_device_view {
     uint32_t prefetch;          /* 1 = fetch the next run at the run's middle  */
     uint32_t run_grow;          /* log2 of the run growth factor per refill    */
     uint32_t demand_hint;       /* 1 = bulk refills sized to the launch's demand */
+    uint32_t oom_record;        /* 1 = exhaustion record on (DESIGN.md Deviations 11) */
 };
 typedef struct gallatin_device_view gallatin_device_view_t;
 

@@ -16,8 +16,10 @@
  *
  * Requires gallatin_init.  Arrays are caller-owned DEVICE memory; batch calls
  * are asynchronous on `stream`.  Errors: GALLATIN_ERR_* (gallatin.h); an
- * allocation that returned NULL inside a kernel is reported by
- * gallatin_graph_errors.
+ * allocation that returned NULL inside a kernel is counted in
+ * gallatin_graph_counters()[2]; an edge or expansion entry whose source vertex
+ * id is >= num_vertices is ignored (no list is touched) and counted in
+ * gallatin_graph_counters()[3].
  */
 #ifndef GALLATIN_GRAPH_H_
 #define GALLATIN_GRAPH_H_
@@ -63,8 +65,9 @@ int gallatin_graph_export(const gallatin_graph_t *g, uint32_t *d_size, uint32_t 
 /* CSR copy: d_out[d_offsets[v] + k] = list_v[k] for k < size_v (caller gives
  * the exclusive prefix sum of the sizes). */
 int gallatin_graph_gather(const gallatin_graph_t *g, const uint64_t *d_offsets, uint32_t *d_out, void *stream);
-/* Device counters: [0] mallocs, [1] frees, [2] failed mallocs (synchronizes). */
-int gallatin_graph_counters(const gallatin_graph_t *g, uint64_t out[3]);
+/* Device counters: [0] mallocs, [1] frees, [2] failed mallocs, [3] ignored
+ * entries with a vertex id >= num_vertices (synchronizes). */
+int gallatin_graph_counters(const gallatin_graph_t *g, uint64_t out[4]);
 
 #ifdef __cplusplus
 }

@@ -8,8 +8,12 @@ never imports the product path: the two share no code, header or constant.
 * O1 -- ``Veb``: the textbook (CLRS) van Emde Boas tree with min/max, summary
   and sqrt(U) clusters that PAPER.md S3.1 describes; ``succ`` is the
   paper's ">= x" (P:76).  ``veb_oracle.c``.
-* O2 -- ``Allocator``: the sequential allocator following PAPER.md S4-S5
-  (Alg. 1-4) one request at a time.  ``alloc_oracle.c``.
+* O2-P -- ``Allocator``: the sequential allocator following PAPER.md S4-S5
+  (Alg. 1-4, policy POL) one request at a time.
+  ``alloc_paper.c`` (+ ``alloc_state.c``: lifecycle, invariant checks, image).
+* O2-R -- ``RunsAllocator``: the deviation model (DESIGN.md Deviations 5, 8:
+  runs of blocks, format-ahead, prefetch, slot trims), built on O2-P's
+  primitives.  ``alloc_runs.c``.
 * O3 -- graph adjacency oracle (``graph.py``), per-vertex Python/numpy lists.
 
 Parity status of every function is listed in DESIGN.md ("Oracle pins").
@@ -24,7 +28,8 @@ import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
 _LIB_PATH = os.path.join(_HERE, "liboracle.so")
-_SOURCES = ["veb_oracle.c", "alloc_oracle.c"]
+_SOURCES = ["veb_oracle.c", "alloc_state.c", "alloc_paper.c", "alloc_runs.c"]
+_HEADERS = ["alloc_state.h"]
 
 NONE = (1 << 64) - 1
 TREE_FREE = 0xFFFFFFFF
@@ -37,7 +42,7 @@ OV_INSERT, OV_DELETE, OV_MEMBER, OV_SUCC, OV_PRED = range(5)
 VIOLATIONS = {
     1: "front-first (P:138)", 2: "back-first large (P:138)", 4: "free of a non-live pointer",
     8: "overlap", 16: "alignment", 32: "outside heap", 64: "accounting", 128: "trees vs table",
-    256: "ring queue", 512: "exhaustion record stands while a full search would succeed",
+    256: "ring queue",
 }
 
 
@@ -46,7 +51,7 @@ def build(force: bool = False) -> str:
     srcs = [os.path.join(_HERE, s) for s in _SOURCES]
     if not force and os.path.exists(_LIB_PATH):
         lib_m = os.path.getmtime(_LIB_PATH)
-        if all(os.path.getmtime(s) <= lib_m for s in srcs):
+        if all(os.path.getmtime(s) <= lib_m for s in srcs + [os.path.join(_HERE, h) for h in _HEADERS]):
             return _LIB_PATH
     cmd = ["gcc", "-O2", "-std=c11", "-Wall", "-Wextra", "-fPIC", "-shared", "-o", _LIB_PATH] + srcs
     subprocess.check_call(cmd)
@@ -77,13 +82,13 @@ def lib() -> ctypes.CDLL:
             "oracle_veb_batch": ([vp, i32, vp, u64, vp], None),
             "oracle_veb_image": ([vp, vp, u64], u64),
             "oracle_veb_image_levels": ([ctypes.c_uint, vp], ctypes.c_uint),
-            "o2_create": ([u64, ctypes.c_uint, ctypes.c_uint, ctypes.c_uint, u64, ctypes.c_uint, ctypes.c_uint, ctypes.c_uint,
-                           ctypes.c_uint], vp),
+            "o2_create_paper": ([u64, ctypes.c_uint, ctypes.c_uint], vp),
+            "o2_create_runs": ([u64, ctypes.c_uint, ctypes.c_uint, ctypes.c_uint, u64, ctypes.c_uint, ctypes.c_uint,
+                                ctypes.c_uint, ctypes.c_uint], vp),
             "o2_destroy": ([vp], None),
             "o2_nslot": ([vp, ctypes.c_uint], ctypes.c_uint),
             "o2_errors": ([vp], u64),
             "o2_violations": ([vp], u64),
-            "o2_oom_fast": ([vp], u64),
             "o2_live_count": ([vp], u64),
             "o2_usable_live": ([vp], u64),
             "o2_usable_size": ([u64], u64),
@@ -175,22 +180,22 @@ def veb_image_levels(k: int) -> list[int]:
 
 
 class Allocator:
-    """O2: sequential Gallatin allocator (PAPER.md S4-S5, Alg. 1-4).
+    """O2-P: sequential Gallatin allocator, the paper's policy POL (PAPER.md
+    S4-S5, Alg. 1-4; one-block buffer slots).
 
     Offsets are relative to the heap base; NONE (2^64-1) is NULL.
     """
 
-    def __init__(self, nseg: int, slot_base: int = 148, slot_min: int = 4, run_max: int = 1,
-                 run_bytes: int = 64 << 20, format_ahead: int = 0, run_init: int = 1, prefetch: int = 0,
-                 run_grow: int = 1):
-        """run_max=1, run_init=1, format_ahead=0, prefetch=0 is the paper's one-block buffer (P:195);
-        run_grow = log2 of the run growth per refill (DESIGN.md Deviations 5)."""
+    def __init__(self, nseg: int, slot_base: int = 148, slot_min: int = 4):
         self._h = None
         self.nseg = nseg
-        self._h = lib().o2_create(nseg, slot_base, slot_min, run_max, run_bytes, format_ahead, run_init, prefetch,
-                                  run_grow)
+        self._h = self._create(nseg, slot_base, slot_min)
         if not self._h:
             raise ValueError("bad allocator parameters")
+
+    @staticmethod
+    def _create(nseg, slot_base, slot_min):
+        return lib().o2_create_paper(nseg, slot_base, slot_min)
 
     def close(self):
         if self._h:
@@ -214,11 +219,6 @@ class Allocator:
     @property
     def errors(self) -> int:
         return lib().o2_errors(self._h)
-
-    @property
-    def oom_fast(self) -> int:
-        """Run requests failed by the exhaustion record (DESIGN.md Deviations 11)."""
-        return lib().o2_oom_fast(self._h)
 
     @property
     def live_count(self) -> int:
@@ -255,6 +255,39 @@ class Allocator:
         got = lib().o2_image(self._h, _ptr(out), n)
         assert got == n
         return out
+
+
+class RunsAllocator(Allocator):
+    """O2-R: the deviation model (DESIGN.md Deviations 5, 8; alloc_runs.c):
+    runs of consecutive blocks per slot, format-ahead, prefetch, slot trims
+    before "no memory".  run_max=1, run_init=1, format_ahead=0, prefetch=0 is
+    the paper's one-block buffer; run_grow = log2 of the growth per
+    refill."""
+
+    def __init__(self, nseg: int, slot_base: int = 148, slot_min: int = 4, run_max: int = 1,
+                 run_bytes: int = 64 << 20, format_ahead: int = 0, run_init: int = 1, prefetch: int = 0,
+                 run_grow: int = 1):
+        self._h = None
+        self.nseg = nseg
+        self._h = lib().o2_create_runs(nseg, slot_base, slot_min, run_max, run_bytes, format_ahead, run_init,
+                                       prefetch, run_grow)
+        if not self._h:
+            raise ValueError("bad allocator parameters")
+
+
+PAPER_KNOBS = {"run_max": 1, "run_init": 1, "format_ahead": 0, "prefetch": 0}
+
+
+def is_paper_policy(params: dict) -> bool:
+    """True if the knobs are the paper's one-block buffer."""
+    return all(params.get(k, PAPER_KNOBS[k]) == v for k, v in PAPER_KNOBS.items())
+
+
+def model(nseg: int, **params) -> Allocator:
+    """The O2 model for a set of knobs: O2-P for the paper's policy, else O2-R."""
+    if is_paper_policy(params):
+        return Allocator(nseg, params.get("slot_base", 148), params.get("slot_min", 4))
+    return RunsAllocator(nseg, **params)
 
 
 def usable_size(size: int) -> int:

@@ -29,10 +29,8 @@ class Config(ctypes.Structure):
     _fields_ = [("heap_bytes", ctypes.c_uint64), ("run_bytes", ctypes.c_uint64), ("slot_base", ctypes.c_uint32),
                 ("slot_min", ctypes.c_uint32), ("run_max", ctypes.c_uint32), ("format_ahead", ctypes.c_uint32),
                 ("fence_free", ctypes.c_uint32), ("bulk_items", ctypes.c_uint32), ("run_init", ctypes.c_uint32),
-                ("prefetch", ctypes.c_uint32), ("run_grow", ctypes.c_uint32), ("pipeline", ctypes.c_uint32),
-                ("free_team", ctypes.c_uint32), ("demand_hint", ctypes.c_uint32),
-                ("cta_tiles", ctypes.c_uint32), ("cta_threads", ctypes.c_uint32),
-                ("free_threads", ctypes.c_uint32)]
+                ("prefetch", ctypes.c_uint32), ("run_grow", ctypes.c_uint32), ("demand_hint", ctypes.c_uint32),
+                ("oom_record", ctypes.c_uint32)]
 
 
 class Stats(ctypes.Structure):
@@ -42,7 +40,8 @@ class Stats(ctypes.Structure):
                 ("nslot", ctypes.c_uint32 * 9), ("run_cap", ctypes.c_uint32 * 9), ("slot_base", ctypes.c_uint32),
                 ("slot_min", ctypes.c_uint32), ("run_max", ctypes.c_uint32), ("format_ahead", ctypes.c_uint32),
                 ("fence_free", ctypes.c_uint32), ("run_init", ctypes.c_uint32), ("formatters", ctypes.c_uint32),
-                ("prefetch", ctypes.c_uint32), ("run_grow", ctypes.c_uint32)]
+                ("prefetch", ctypes.c_uint32), ("run_grow", ctypes.c_uint32), ("demand_hint", ctypes.c_uint32),
+                ("oom_record", ctypes.c_uint32)]
 
 
 def declared_functions() -> list[str]:
@@ -124,10 +123,18 @@ def _stream(stream) -> int | None:
     return torch.cuda.current_stream().cuda_stream
 
 
+def _on_device(t) -> None:
+    """Tensors must live on the current device (the allocator's, set at init)."""
+    import torch
+    if t.device.index != torch.cuda.current_device():
+        raise ValueError(f"tensor on {t.device}, the library runs on cuda:{torch.cuda.current_device()}")
+
+
 def _dptr(t) -> int:
     import torch
     if not isinstance(t, torch.Tensor) or not t.is_cuda or not t.is_contiguous() or t.element_size() != 8:
         raise TypeError("expected a contiguous 8-byte-element CUDA tensor")
+    _on_device(t)
     return t.data_ptr()
 
 
@@ -135,6 +142,7 @@ def _dptr1(t) -> int:
     import torch
     if not isinstance(t, torch.Tensor) or not t.is_cuda or not t.is_contiguous() or t.element_size() != 1:
         raise TypeError("expected a contiguous 1-byte-element CUDA tensor")
+    _on_device(t)
     return t.data_ptr()
 
 
@@ -142,6 +150,14 @@ def _hptr(a: np.ndarray) -> int:
     if a.dtype.itemsize != 8 or not a.flags.c_contiguous:
         raise TypeError("expected a contiguous 8-byte numpy array")
     return a.ctypes.data
+
+
+def _need(t, n: int, what: str) -> None:
+    """Raise unless tensor / array t holds at least n elements (the kernels
+    index every output and every paired input by the request count)."""
+    m = t.numel() if hasattr(t, "numel") else len(t)
+    if m < n:
+        raise ValueError(f"{what} holds {m} elements, {n} needed")
 
 
 def _empty64(n: int):
@@ -152,15 +168,12 @@ def _empty64(n: int):
 # ------------------------------------------------------------- allocator ---
 def gallatin_init(heap_bytes: int, slot_base: int = 0, slot_min: int = 0, run_max: int = 0, run_bytes: int = 0,
                   format_ahead: int = 0, fence_free: int = 0, bulk_items: int = 0, run_init: int = 0,
-                  prefetch: int = 0, run_grow: int = 0, pipeline: int = 0, free_team: int = 0,
-                  demand_hint: int = 0, cta_tiles: int = 0, cta_threads: int = 0,
-                  free_threads: int = 0) -> None:
+                  prefetch: int = 0, run_grow: int = 0, demand_hint: int = 0, oom_record: int = 0) -> None:
     """0 = library default for every knob (include/gallatin.h gallatin_config_t)."""
     cfg = Config(heap_bytes=heap_bytes, run_bytes=run_bytes, slot_base=slot_base, slot_min=slot_min,
                  run_max=run_max, format_ahead=format_ahead, fence_free=fence_free, bulk_items=bulk_items,
-                 run_init=run_init, prefetch=prefetch, run_grow=run_grow, pipeline=pipeline, free_team=free_team,
-                 demand_hint=demand_hint, cta_tiles=cta_tiles, cta_threads=cta_threads,
-                 free_threads=free_threads)
+                 run_init=run_init, prefetch=prefetch, run_grow=run_grow, demand_hint=demand_hint,
+                 oom_record=oom_record)
     check(lib().gallatin_init_ex(ctypes.byref(cfg)), "gallatin_init")
 
 
@@ -176,6 +189,7 @@ def gallatin_malloc(sizes, ptrs=None, stream=None):
     """ptrs[i] = device malloc(sizes[i]); int64 CUDA tensors holding u64 values."""
     if ptrs is None:
         ptrs = _empty64(sizes.numel())
+    _need(ptrs, sizes.numel(), "ptrs")
     check(lib().gallatin_malloc(_dptr(sizes), _dptr(ptrs), sizes.numel(), _stream(stream)), "gallatin_malloc")
     return ptrs
 
@@ -187,6 +201,7 @@ def gallatin_free(ptrs, stream=None) -> None:
 def gallatin_malloc_host(sizes: np.ndarray, out: np.ndarray | None = None, stream=None) -> np.ndarray:
     if out is None:
         out = np.empty(len(sizes), dtype=np.uint64)
+    _need(out, len(sizes), "out")
     check(lib().gallatin_malloc_host(_hptr(sizes), _hptr(out), len(sizes), _stream(stream)), "gallatin_malloc_host")
     return out
 
@@ -208,6 +223,8 @@ def gallatin_replay(kinds, args, keys, out=None, stream=None):
     n = kinds.numel()
     if out is None:
         out = _empty64(n)
+    for t, what in ((args, "args"), (keys, "keys"), (out, "out")):
+        _need(t, n, what)
     check(lib().gallatin_replay(_dptr1(kinds), _dptr(args), _dptr(keys), n, _dptr(out), _stream(stream)),
           "gallatin_replay")
     return out
@@ -221,11 +238,12 @@ def gallatin_stats() -> dict:
             "large_segments": s.large_segments, "errors": s.errors, "nslot": list(s.nslot),
             "run_cap": list(s.run_cap), "run_bytes": s.run_bytes, "slot_base": s.slot_base, "slot_min": s.slot_min,
             "run_max": s.run_max, "format_ahead": s.format_ahead, "fence_free": s.fence_free,
-            "run_init": s.run_init, "formatters": s.formatters, "prefetch": s.prefetch, "run_grow": s.run_grow}
+            "run_init": s.run_init, "formatters": s.formatters, "prefetch": s.prefetch, "run_grow": s.run_grow,
+            "demand_hint": s.demand_hint, "oom_record": s.oom_record}
 
 
 def oracle_params() -> dict:
-    """The effective policy knobs, as keyword arguments of oracle.Allocator (tests)."""
+    """The effective policy knobs, as keyword arguments of oracle.model() (tests)."""
     st = gallatin_stats()
     return {"slot_base": st["slot_base"], "slot_min": st["slot_min"], "run_max": st["run_max"],
             "run_bytes": st["run_bytes"], "format_ahead": 1 if st["format_ahead"] == 1 else 0,
@@ -242,11 +260,13 @@ def gallatin_snapshot() -> np.ndarray:
 
 
 def gallatin_stamp(ptrs, sizes, stream=None) -> None:
+    _need(sizes, ptrs.numel(), "sizes")
     check(lib().gallatin_stamp(_dptr(ptrs), _dptr(sizes), ptrs.numel(), _stream(stream)), "gallatin_stamp")
 
 
 def gallatin_verify(ptrs, sizes, stream=None) -> int:
     import torch
+    _need(sizes, ptrs.numel(), "sizes")
     bad = torch.zeros(1, dtype=torch.int64, device="cuda")
     check(lib().gallatin_verify(_dptr(ptrs), _dptr(sizes), ptrs.numel(), _dptr(bad), _stream(stream)),
           "gallatin_verify")
@@ -256,6 +276,9 @@ def gallatin_verify(ptrs, sizes, stream=None) -> int:
 def gallatin_usable(ptrs, sizes, usable=None, stream=None) -> tuple[int, int]:
     """(sum of usable bytes read from the memory table, #pointers contradicting their request)."""
     import torch
+    _need(sizes, ptrs.numel(), "sizes")
+    if usable is not None:
+        _need(usable, ptrs.numel(), "usable")
     acc = torch.zeros(2, dtype=torch.int64, device="cuda")
     up = _dptr(usable) if usable is not None else None
     check(lib().gallatin_usable(_dptr(ptrs), _dptr(sizes), ptrs.numel(), up, acc.data_ptr(), acc.data_ptr() + 8,
@@ -316,11 +339,13 @@ class Veb:
 
     def successor(self, q, out=None, stream=None):
         out = _empty64(q.numel()) if out is None else out
+        _need(out, q.numel(), "out")
         check(lib().veb_successor(self._h, _dptr(q), _dptr(out), q.numel(), _stream(stream)), "veb_successor")
         return out
 
     def predecessor(self, q, out=None, stream=None):
         out = _empty64(q.numel()) if out is None else out
+        _need(out, q.numel(), "out")
         check(lib().veb_predecessor(self._h, _dptr(q), _dptr(out), q.numel(), _stream(stream)), "veb_predecessor")
         return out
 
@@ -361,6 +386,7 @@ def _dptr4(t) -> int:
     import torch
     if not isinstance(t, torch.Tensor) or not t.is_cuda or not t.is_contiguous() or t.element_size() != 4:
         raise TypeError("expected a contiguous 4-byte-element CUDA tensor")
+    _on_device(t)
     return t.data_ptr()
 
 
@@ -382,20 +408,24 @@ class Graph:
             self._h = None
 
     def insert(self, src, dst, stream=None):
+        _need(dst, src.numel(), "dst")
         check(lib().gallatin_graph_insert(self._h, _dptr4(src), _dptr4(dst), src.numel(), _stream(stream)),
               "gallatin_graph_insert")
 
     def delete(self, src, dst, stream=None):
+        _need(dst, src.numel(), "dst")
         check(lib().gallatin_graph_delete(self._h, _dptr4(src), _dptr4(dst), src.numel(), _stream(stream)),
               "gallatin_graph_delete")
 
     def insert_edges(self, src, dst, stream=None):
         """Single-edge inserts (one thread per edge under a vertex lock)."""
+        _need(dst, src.numel(), "dst")
         check(lib().gallatin_graph_insert_edges(self._h, _dptr4(src), _dptr4(dst), src.numel(), _stream(stream)),
               "gallatin_graph_insert_edges")
 
     def delete_edges(self, src, dst, stream=None):
         """Single-edge deletes (one thread per edge under a vertex lock)."""
+        _need(dst, src.numel(), "dst")
         check(lib().gallatin_graph_delete_edges(self._h, _dptr4(src), _dptr4(dst), src.numel(), _stream(stream)),
               "gallatin_graph_delete_edges")
 
@@ -422,6 +452,6 @@ class Graph:
         return out[:total]
 
     def counters(self) -> dict:
-        c = (ctypes.c_uint64 * 3)()
+        c = (ctypes.c_uint64 * 4)()
         check(lib().gallatin_graph_counters(self._h, c), "gallatin_graph_counters")
-        return {"mallocs": c[0], "frees": c[1], "failed": c[2]}
+        return {"mallocs": c[0], "frees": c[1], "failed": c[2], "bad_vertex": c[3]}

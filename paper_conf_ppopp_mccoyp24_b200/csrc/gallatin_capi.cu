@@ -41,8 +41,6 @@ struct State {
     // host-array calls: copy-in / copy-out streams and per-chunk events
     cudaStream_t cin = nullptr, cout = nullptr;
     cudaEvent_t ev_in[kMaxChunks] = {}, ev_k[kMaxChunks] = {};
-    // resident CTAs of the persistent bulk kernels (SMs x occupancy)
-    unsigned pipe_malloc_ctas = 0, pipe_free_ctas = 0, pers_malloc_ctas = 0, pers_free_ctas = 0;
 };
 State g;
 
@@ -341,236 +339,6 @@ __global__ void __launch_bounds__(NT, MINB) k_bulk_malloc_cta(const uint64_t *__
     }
 }
 
-// Persistent form of k_bulk_malloc_cta with the NEXT tile's sizes prefetched
-// into registers: a CTA walks tiles tile, tile + gridDim.x, ... and issues
-// the next tile's loads before this tile's shared-memory ranking, slot RMWs
-// and pointer stores, so the HBM latency of tile i+1 overlaps the L2 round
-// trip of tile i (one tile per CTA serializes load -> RMW -> store and pays a
-// CTA launch per tile).  Per tile exactly k_bulk_malloc_cta's protocol; the
-// class counters and slot words are double-buffered by tile parity so a tile
-// needs two CTA barriers.  A refill duty is discharged within its own tile
-// (bulk_malloc_slow), before the CTA issues its next RMW, as in the one-tile
-// kernel.
-template <int ITEMS>
-__global__ void __launch_bounds__(kThreads, 5) k_bulk_malloc_pers(const uint64_t *__restrict__ sizes,
-                                                                  void **__restrict__ ptrs, uint64_t n,
-                                                                  uint64_t ntiles, uint32_t tiles) {
-    constexpr uint32_t kTile = kThreads * ITEMS;
-    const View &v = c_view;
-    __shared__ uint32_t cnt[2][core::kTrees];
-    __shared__ uint64_t olds[2][core::kTrees];
-    const uint32_t lane = threadIdx.x & 31;
-    const uint32_t key = ptx::smid();
-    const uint32_t lt = ptx::lanemask_lt();
-    if (threadIdx.x < 2 * core::kTrees) (&cnt[0][0])[threadIdx.x] = 0;
-    __syncthreads();
-    __shared__ uint64_t buf[2][ITEMS][kThreads];
-    uint64_t tile = (uint64_t)blockIdx.x * tiles;
-    const uint64_t tend = tile + tiles < ntiles ? tile + tiles : ntiles;
-#pragma unroll
-    for (int k = 0; k < ITEMS; k++) {
-        const uint64_t i = tile * kTile + threadIdx.x + (uint64_t)kThreads * k;
-        ptx::cp_async8(&buf[0][k][threadIdx.x], sizes + (i < n ? i : n - 1));
-    }
-    ptx::cp_async_commit();
-    for (uint32_t it = 0; tile < tend; tile++, it++) {
-        const uint32_t par = it & 1;
-        const uint64_t base = tile * kTile + threadIdx.x;
-        // the next tile's sizes are in flight (cp.async, no registers) while this tile runs
-        const uint64_t nt = tile + 1;
-        if (nt < tend) {
-#pragma unroll
-            for (int k = 0; k < ITEMS; k++) {
-                const uint64_t i = nt * kTile + threadIdx.x + (uint64_t)kThreads * k;
-                ptx::cp_async8(&buf[par ^ 1][k][threadIdx.x], sizes + (i < n ? i : n - 1));
-            }
-        }
-        ptx::cp_async_commit();
-        ptx::cp_async_wait<1>();
-        uint32_t cr[ITEMS];
-#pragma unroll
-        for (int k = 0; k < ITEMS; k++) {
-            const uint64_t s = base + (uint64_t)kThreads * k < n ? buf[par][k][threadIdx.x] : 0;
-            const uint32_t lg = 64u - (uint32_t)__clzll((long long)(s - 1));
-            const uint32_t sc = (lg > core::kMinSliceLog2 ? lg : core::kMinSliceLog2) - core::kMinSliceLog2;
-            cr[k] = s - 1 < core::kMaxSlice ? sc : (s == 0 ? 0xFEu : 0xFFu);
-        }
-#pragma unroll
-        for (int k = 0; k < ITEMS; k++) {
-            const uint32_t c = cr[k];
-            const unsigned peers = __match_any_sync(0xFFFFFFFFu, c);
-            const uint32_t leader = (uint32_t)__ffs((int)peers) - 1;
-            uint32_t b = 0;
-            if (c < core::kTrees && lane == leader) b = atomicAdd(&cnt[par][c], (uint32_t)__popc(peers));
-            cr[k] = c | ((__shfl_sync(0xFFFFFFFFu, b, (int)leader) + (uint32_t)__popc(peers & lt)) << 8);
-        }
-        __syncthreads();
-        if (threadIdx.x < core::kTrees) {
-            const uint32_t c = threadIdx.x;
-            const uint32_t m = cnt[par][c];
-            if (m) olds[par][c] = ptx::atom_add(core::slot_word(v, v.slot_off[c] + key % v.nslot[c]), (uint64_t)m << 32);
-            cnt[par ^ 1][c] = 0;                                   // for the next tile
-        }
-        __syncthreads();
-        uint32_t slow = 0;
-        uint64_t info[(ITEMS + 3) / 4];
-#pragma unroll
-        for (int q = 0; q < (ITEMS + 3) / 4; q++) info[q] = 0;
-#pragma unroll
-        for (int k = 0; k < ITEMS; k++) {
-            const uint64_t i = base + (uint64_t)kThreads * k;
-            const uint32_t c = cr[k] & 0xFFu;
-            void *p = nullptr;
-            uint32_t code = 0;
-            if (c < core::kTrees) {
-                const uint64_t old = olds[par][c];
-                const uint32_t m = core::run_len(old);
-                const uint32_t idx = (uint32_t)(old >> 32) + (cr[k] >> 8);
-                if (idx < (m << core::kSliceLog2)) {
-                    p = core::slice_ptr(v, c, old & core::kRunNone, idx);
-                    if (v.prefetch && idx == (m << (core::kSliceLog2 - 1))) code = 0x2000u | m;
-                } else {
-                    code = idx == (m << core::kSliceLog2) ? (0x400u | m) : 0x1000u;
-                }
-            } else if (c == 0xFFu) {
-                code = 0x800u;
-            }
-            if (code) {
-                slow |= 1u << k;
-                info[k >> 2] |= (uint64_t)code << (16 * (k & 3));
-            }
-            if (!(code & 0x1C00u) && i < n)
-                __stcs(reinterpret_cast<unsigned long long *>(ptrs) + i, reinterpret_cast<unsigned long long>(p));
-        }
-        const unsigned callers = __ballot_sync(0xFFFFFFFFu, slow != 0);
-        if (slow) {
-            uint64_t spill[(ITEMS + 3) / 4];
-#pragma unroll
-            for (int q = 0; q < (ITEMS + 3) / 4; q++) spill[q] = info[q];
-            bulk_malloc_slow(sizes, ptrs, n, base, key, slow, spill, ITEMS, callers, kThreads,
-                             v.demand_hint ? cnt[par] : nullptr, ntiles);
-        }
-    }
-}
-
-// Persistent, software-pipelined form of k_bulk_malloc_cta: a CTA walks
-// tiles of kThreads*ITEMS requests (tile, tile + gridDim.x, ...).  One thread
-// issues a 1-D TMA bulk copy of the NEXT tile's sizes into the other half of a
-// double buffer in shared memory (completion on an mbarrier) before this
-// tile's slot RMWs, so the HBM latency of tile i+1 overlaps the L2 round trip
-// of tile i's atomics and its pointer stores, with nothing staged in
-// registers across the slow path's calls.  (One tile per CTA serializes
-// load -> atomic -> store and pays a CTA launch per tile.)  Each tile runs
-// exactly k_bulk_malloc_cta's protocol: one global RMW per class per tile,
-// the same slow path.  A ragged last tile, or a sizes array that is not
-// 16-byte aligned (tma = 0), is loaded directly.
-template <int ITEMS>
-__global__ void __launch_bounds__(kThreads, 4) k_bulk_malloc_pipe(const uint64_t *__restrict__ sizes,
-                                                                  void **__restrict__ ptrs, uint64_t n,
-                                                                  uint64_t ntiles, uint32_t tma) {
-    constexpr uint32_t kTile = kThreads * ITEMS;
-    const View &v = c_view;
-    __shared__ __align__(128) uint64_t buf[2][kTile];
-    __shared__ __align__(8) uint64_t bar[2];
-    __shared__ uint32_t cnt[2][core::kTrees];
-    __shared__ uint64_t olds[2][core::kTrees];
-    const uint32_t lane = threadIdx.x & 31;
-    const uint32_t key = ptx::smid();
-    if (threadIdx.x == 0) {
-        ptx::mbar_init(&bar[0], 1);
-        ptx::mbar_init(&bar[1], 1);
-        ptx::fence_mbar_init();
-    }
-    if (threadIdx.x < 2 * core::kTrees) (&cnt[0][0])[threadIdx.x] = 0;
-    __syncthreads();
-    const uint32_t lt = ptx::lanemask_lt();
-    uint64_t tile = blockIdx.x;
-    if (threadIdx.x == 0 && tma && tile < ntiles && (tile + 1) * kTile <= n)
-        ptx::bulk_load(buf[0], sizes + tile * kTile, kTile * 8, &bar[0]);
-    for (uint32_t it = 0; tile < ntiles; tile += gridDim.x, it++) {
-        const uint32_t par = it & 1;
-        const uint64_t nt = tile + gridDim.x;
-        // buf[par^1] was last read before the previous tile's first barrier
-        if (threadIdx.x == 0 && tma && nt < ntiles && (nt + 1) * kTile <= n)
-            ptx::bulk_load(buf[par ^ 1], sizes + nt * kTile, kTile * 8, &bar[par ^ 1]);
-        const uint64_t base = tile * kTile + threadIdx.x;
-        uint64_t x[ITEMS];
-        if (tma && (tile + 1) * kTile <= n) {
-            ptx::mbar_wait(&bar[par], (it >> 1) & 1);
-#pragma unroll
-            for (int k = 0; k < ITEMS; k++) x[k] = buf[par][k * kThreads + threadIdx.x];
-        } else {
-#pragma unroll
-            for (int k = 0; k < ITEMS; k++) {
-                const uint64_t i = base + (uint64_t)kThreads * k;
-                x[k] = i < n ? __ldcs(reinterpret_cast<const unsigned long long *>(sizes) + i) : 0;
-            }
-        }
-        uint32_t cr[ITEMS];
-#pragma unroll
-        for (int k = 0; k < ITEMS; k++) {
-            const uint64_t s = x[k];
-            const uint32_t lg = 64u - (uint32_t)__clzll((long long)(s - 1));
-            const uint32_t sc = (lg > core::kMinSliceLog2 ? lg : core::kMinSliceLog2) - core::kMinSliceLog2;
-            cr[k] = s - 1 < core::kMaxSlice ? sc : (s == 0 ? 0xFEu : 0xFFu);
-        }
-#pragma unroll
-        for (int k = 0; k < ITEMS; k++) {
-            const uint32_t c = cr[k];
-            const unsigned peers = __match_any_sync(0xFFFFFFFFu, c);
-            const uint32_t leader = (uint32_t)__ffs((int)peers) - 1;
-            uint32_t b = 0;
-            if (c < core::kTrees && lane == leader) b = atomicAdd(&cnt[par][c], (uint32_t)__popc(peers));
-            cr[k] = c | ((__shfl_sync(0xFFFFFFFFu, b, (int)leader) + (uint32_t)__popc(peers & lt)) << 8);
-        }
-        __syncthreads();
-        if (threadIdx.x < core::kTrees) {
-            const uint32_t c = threadIdx.x;
-            const uint32_t m = cnt[par][c];
-            if (m) olds[par][c] = ptx::atom_add(core::slot_word(v, v.slot_off[c] + key % v.nslot[c]), (uint64_t)m << 32);
-            cnt[par ^ 1][c] = 0;                                   // for the next tile
-        }
-        __syncthreads();
-        uint32_t slow = 0;
-        uint64_t info[(ITEMS + 3) / 4];
-#pragma unroll
-        for (int q = 0; q < (ITEMS + 3) / 4; q++) info[q] = 0;
-#pragma unroll
-        for (int k = 0; k < ITEMS; k++) {
-            const uint64_t i = base + (uint64_t)kThreads * k;
-            const uint32_t c = cr[k] & 0xFFu;
-            void *p = nullptr;
-            uint32_t code = 0;
-            if (c < core::kTrees) {
-                const uint64_t old = olds[par][c];
-                const uint32_t m = core::run_len(old);
-                const uint32_t idx = (uint32_t)(old >> 32) + (cr[k] >> 8);
-                if (idx < (m << core::kSliceLog2)) {
-                    p = core::slice_ptr(v, c, old & core::kRunNone, idx);
-                    if (v.prefetch && idx == (m << (core::kSliceLog2 - 1))) code = 0x2000u | m;
-                } else {
-                    code = idx == (m << core::kSliceLog2) ? (0x400u | m) : 0x1000u;
-                }
-            } else if (c == 0xFFu) {
-                code = 0x800u;
-            }
-            if (code) {
-                slow |= 1u << k;
-                info[k >> 2] |= (uint64_t)code << (16 * (k & 3));
-            }
-            if (!(code & 0x1C00u) && i < n)
-                __stcs(reinterpret_cast<unsigned long long *>(ptrs) + i, reinterpret_cast<unsigned long long>(p));
-        }
-        const unsigned callers = __ballot_sync(0xFFFFFFFFu, slow != 0);
-        if (slow) {
-            uint64_t spill[(ITEMS + 3) / 4];
-#pragma unroll
-            for (int q = 0; q < (ITEMS + 3) / 4; q++) spill[q] = info[q];
-            bulk_malloc_slow(sizes, ptrs, n, base, key, slow, spill, ITEMS, callers, kThreads);
-        }
-    }
-}
-
 __device__ __noinline__ void free_slow(const View &v, uint64_t p) {
     const uint64_t off = p - v.heap;
     if (off >= (v.nseg << core::kSegLog2)) { atomicAdd(v.err, 1ull); return; }
@@ -578,13 +346,6 @@ __device__ __noinline__ void free_slow(const View &v, uint64_t p) {
     const uint32_t t = core::sw_tree(ptx::ld_relaxed(v.seg_word + s));
     if (t == core::kTreeFree || t == core::kTreeCont || t < core::kTrees) { atomicAdd(v.err, 1ull); return; }
     core::free_large(v, s, t);
-}
-
-__device__ __noinline__ void bulk_free_return(uint32_t gid) {
-    const View &v = c_view;
-    atomicExch(v.block_free + gid, 0u);
-    ptx::fence_acq_rel();
-    core::return_block(v, gid);
 }
 
 // Rare items of one lane of the bulk free kernel: block returns (this team's
@@ -726,206 +487,6 @@ __global__ void __launch_bounds__(NT, MINB) k_bulk_free_w(void *const *__restric
     free_warp_tile<ITEMS>(v, ptrs, p, base, lane, v.nseg << core::kSegLog2);
 }
 
-// Multi-tile bulk free: CTA b takes CTA tiles b*T .. b*T+T-1 (T = tiles, each
-// kThreads*ITEMS pointers; warp w frees its 32*ITEMS slice of each) and
-// issues the NEXT tile's pointer loads -- per-thread cp.async copies into
-// shared memory, so no register is held across the slow path's calls --
-// before processing this one: their HBM latency overlaps this tile's tree-id
-// loads and counter RMWs.  T is small so the hardware still balances CTAs
-// (a fully persistent grid left a tail of warps stuck in block returns).
-template <int ITEMS>
-__global__ void __launch_bounds__(kThreads, 6) k_bulk_free_pers(void *const *__restrict__ ptrs, uint64_t n,
-                                                                uint64_t nwtiles, uint32_t tiles) {
-    const View &v = c_view;
-    __shared__ uint64_t buf[2][ITEMS][kThreads];
-    const uint32_t lane = threadIdx.x & 31;
-    constexpr uint64_t nwarps = kThreads / 32;
-    const uint64_t heap_bytes = v.nseg << core::kSegLog2;
-    const uint64_t *src = reinterpret_cast<const uint64_t *>(ptrs);
-    uint64_t wt = (uint64_t)blockIdx.x * tiles * nwarps + (threadIdx.x >> 5);
-    const uint64_t wend = wt + (uint64_t)tiles * nwarps < nwtiles ? wt + (uint64_t)tiles * nwarps : nwtiles;
-#pragma unroll
-    for (int k = 0; k < ITEMS; k++) {
-        const uint64_t i = wt * (32 * ITEMS) + 32ull * k + lane;
-        ptx::cp_async8(&buf[0][k][threadIdx.x], src + (i < n ? i : n - 1));
-    }
-    ptx::cp_async_commit();
-    for (uint32_t it = 0; wt < wend; wt += nwarps, it++) {
-        const uint32_t par = it & 1;
-        const uint64_t nt = wt + nwarps;
-        if (nt < wend) {
-#pragma unroll
-            for (int k = 0; k < ITEMS; k++) {
-                const uint64_t i = nt * (32 * ITEMS) + 32ull * k + lane;
-                ptx::cp_async8(&buf[par ^ 1][k][threadIdx.x], src + (i < n ? i : n - 1));
-            }
-        }
-        ptx::cp_async_commit();
-        ptx::cp_async_wait<1>();                                   // this tile's copies landed
-        const uint64_t base = wt * (32 * ITEMS) + lane;
-        uint64_t p[ITEMS];
-#pragma unroll
-        for (int k = 0; k < ITEMS; k++) p[k] = base + 32ull * k < n ? buf[par][k][threadIdx.x] : 0;
-        free_warp_tile<ITEMS>(v, ptrs, p, base, lane, heap_bytes);
-    }
-    ptx::cp_async_wait<0>();
-}
-
-// Bulk free with CTA-level aggregation: the frees of one CTA tile that hit the
-// same block are summed in a shared-memory table (one shared RMW per warp
-// team, P:315's coalescing widened from a warp to a CTA) and ONE global
-// atomicAdd per distinct block per tile updates its free counter; the thread
-// whose RMW completes 4096 returns the block (reading A-14 of P:250).  The
-// hot free counters -- every warp of a region frees into the same few blocks
-// -- then see ~8x fewer RMWs, which serialize per address at L2.  Same
-// per-pointer decode as k_bulk_free; non-slice pointers take free_slow.
-constexpr uint32_t kFreeTable = 1024;               // shared table entries: >= the requests of a tile, never full
-template <int ITEMS>
-__global__ void __launch_bounds__(kThreads, 6) k_bulk_free_cta(void *const *__restrict__ ptrs, uint64_t n) {
-    const View &v = c_view;
-    __shared__ uint32_t keys[kFreeTable];
-    __shared__ uint32_t cnts[kFreeTable];
-    const uint32_t lane = threadIdx.x & 31;
-    const uint64_t base = ((blockIdx.x * (uint64_t)kThreads + threadIdx.x) >> 5) * (32 * ITEMS) + lane;
-    const uint64_t heap_bytes = v.nseg << core::kSegLog2;
-    for (uint32_t i = threadIdx.x; i < kFreeTable; i += kThreads) {
-        keys[i] = 0xFFFFFFFFu;
-        cnts[i] = 0;
-    }
-    uint64_t p[ITEMS], w[ITEMS];
-#pragma unroll
-    for (int k = 0; k < ITEMS; k++) {
-        const uint64_t i = base + 32ull * k;
-        const uint64_t x = __ldcs(reinterpret_cast<const unsigned long long *>(ptrs) + (i < n ? i : n - 1));
-        p[k] = i < n ? x : 0;
-    }
-#pragma unroll
-    for (int k = 0; k < ITEMS; k++) {
-        const uint64_t off = p[k] - v.heap;
-        w[k] = (p[k] && off < heap_bytes) ? ((uint64_t)__ldca(v.seg_tid + (off >> core::kSegLog2)) << 32) : ~0ull;
-    }
-    __syncthreads();                                       // table initialized
-    uint32_t slow = 0;
-#pragma unroll
-    for (int k = 0; k < ITEMS; k++) {
-        const uint64_t off = p[k] - v.heap;
-        const uint32_t t = core::sw_tree(w[k]);
-        const bool blk = p[k] && t < core::kTrees;
-        const uint32_t gid = blk ? (uint32_t)((off >> core::kSegLog2) * core::kMaxBlocks +
-                                              ((off & (core::kSegBytes - 1)) >> (16 + t)))
-                                 : (0x80000000u | (uint32_t)(k << 5) | lane);
-        const unsigned peers = __match_any_sync(0xFFFFFFFFu, gid);
-        if (!blk) {
-            if (p[k]) slow |= 1u << k;
-            continue;
-        }
-        if (lane == (uint32_t)__ffs((int)peers) - 1) {
-            uint32_t h = (gid * 0x9E3779B1u) >> 22;            // 10-bit hash
-#pragma unroll 1
-            for (;;) {                                     // at most ITEMS*kThreads keys: a free entry exists
-                const uint32_t k0 = atomicCAS(&keys[h], 0xFFFFFFFFu, gid);
-                if (k0 == 0xFFFFFFFFu || k0 == gid) break;
-                h = (h + 1) & (kFreeTable - 1);
-            }
-            atomicAdd(&cnts[h], (uint32_t)__popc(peers));
-        }
-    }
-    __syncthreads();                                       // every team counted
-    constexpr int kPer = kFreeTable / kThreads;
-    uint32_t gk[kPer], ck[kPer], ok[kPer];
-#pragma unroll
-    for (int q = 0; q < kPer; q++) {
-        gk[q] = keys[threadIdx.x + kThreads * q];
-        ck[q] = cnts[threadIdx.x + kThreads * q];
-    }
-#pragma unroll
-    for (int q = 0; q < kPer; q++) ok[q] = gk[q] != 0xFFFFFFFFu ? atomicAdd(v.block_free + gk[q], ck[q]) : 0;
-#pragma unroll
-    for (int q = 0; q < kPer; q++)
-        if (gk[q] != 0xFFFFFFFFu && ok[q] + ck[q] == core::kSlices) bulk_free_return(gk[q]);   // the 4096th free
-    if (slow) {
-        for (int k = 0; k < ITEMS; k++)
-            if ((slow >> k) & 1) free_slow(v, reinterpret_cast<uint64_t>(ptrs[base + 32ull * k]));
-    }
-}
-
-// Persistent, software-pipelined bulk free: each warp walks warp tiles of
-// 32*ITEMS pointers; lane 0 issues a 1-D TMA bulk copy of the warp's NEXT
-// tile into its half of a per-warp double buffer (mbarrier completion) before
-// this tile's tree-id loads and counter RMWs.  Per tile, the protocol of
-// k_bulk_free.  Ragged last tiles / unaligned arrays load directly.
-template <int ITEMS>
-__global__ void __launch_bounds__(kThreads, 6) k_bulk_free_pipe(void *const *__restrict__ ptrs, uint64_t n,
-                                                                uint64_t nwtiles, uint32_t tma) {
-    constexpr uint32_t kWT = 32 * ITEMS;
-    constexpr uint32_t kWarps = kThreads / 32;
-    const View &v = c_view;
-    __shared__ __align__(128) uint64_t buf[kWarps][2][kWT];
-    __shared__ __align__(8) uint64_t bar[kWarps][2];
-    const uint32_t lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-    const uint64_t nwarps = (uint64_t)gridDim.x * kWarps;
-    const uint64_t *src = reinterpret_cast<const uint64_t *>(ptrs);
-    uint64_t wt = (blockIdx.x * (uint64_t)kThreads + threadIdx.x) >> 5;
-    const uint64_t heap_bytes = v.nseg << core::kSegLog2;
-    if (lane == 0) {
-        ptx::mbar_init(&bar[warp][0], 1);
-        ptx::mbar_init(&bar[warp][1], 1);
-        ptx::fence_mbar_init();
-        if (tma && wt < nwtiles && (wt + 1) * kWT <= n) ptx::bulk_load(buf[warp][0], src + wt * kWT, kWT * 8, &bar[warp][0]);
-    }
-    for (uint32_t it = 0; wt < nwtiles; wt += nwarps, it++) {
-        const uint32_t par = it & 1;
-        __syncwarp();                                          // buf[par^1]'s last readers are done
-        if (lane == 0 && tma && wt + nwarps < nwtiles && (wt + nwarps + 1) * kWT <= n)
-            ptx::bulk_load(buf[warp][par ^ 1], src + (wt + nwarps) * kWT, kWT * 8, &bar[warp][par ^ 1]);
-        const uint64_t base = wt * kWT + lane;
-        uint64_t p[ITEMS];
-        if (tma && (wt + 1) * kWT <= n) {
-            ptx::mbar_wait(&bar[warp][par], (it >> 1) & 1);
-#pragma unroll
-            for (int k = 0; k < ITEMS; k++) p[k] = buf[warp][par][32 * k + lane];
-        } else {
-#pragma unroll
-            for (int k = 0; k < ITEMS; k++) {
-                const uint64_t i = base + 32ull * k;
-                p[k] = i < n ? __ldcs(reinterpret_cast<const unsigned long long *>(src) + i) : 0;
-            }
-        }
-        uint64_t w[ITEMS];
-#pragma unroll
-        for (int k = 0; k < ITEMS; k++) {
-            const uint64_t off = p[k] - v.heap;
-            w[k] = (p[k] && off < heap_bytes) ? ((uint64_t)__ldca(v.seg_tid + (off >> core::kSegLog2)) << 32) : ~0ull;
-        }
-        uint32_t gid[ITEMS];
-        unsigned peers[ITEMS];
-#pragma unroll
-        for (int k = 0; k < ITEMS; k++) {
-            const uint64_t off = p[k] - v.heap;
-            const uint32_t t = core::sw_tree(w[k]);
-            const bool blk = p[k] && t < core::kTrees;
-            gid[k] = blk ? (uint32_t)((off >> core::kSegLog2) * core::kMaxBlocks + ((off & (core::kSegBytes - 1)) >> (16 + t)))
-                         : (0x80000000u | (uint32_t)(k << 5) | lane);
-            peers[k] = __match_any_sync(0xFFFFFFFFu, gid[k]);
-            if (!blk) peers[k] = 0;
-        }
-        uint32_t oldc[ITEMS];
-#pragma unroll
-        for (int k = 0; k < ITEMS; k++) {
-            oldc[k] = 0;
-            if (peers[k] && lane == (uint32_t)__ffs((int)peers[k]) - 1)
-                oldc[k] = atomicAdd(v.block_free + gid[k], (uint32_t)__popc(peers[k]));
-        }
-        uint32_t done = 0, slow = 0;
-#pragma unroll
-        for (int k = 0; k < ITEMS; k++) {
-            if (p[k] && !peers[k]) slow |= 1u << k;
-            if (peers[k] && lane == (uint32_t)__ffs((int)peers[k]) - 1 && oldc[k] + __popc(peers[k]) == core::kSlices)
-                done |= 1u << k;                                         // the 4096th free
-        }
-        if (done | slow) bulk_free_slow(ptrs, base, done, slow, ITEMS);
-    }
-}
 
 __global__ void k_replay(const uint8_t *kinds, const uint64_t *args, const uint64_t *keys, uint64_t n,
                          uint64_t *out) {
@@ -1121,13 +682,8 @@ int gallatin_init_ex(const gallatin_config_t *cfg_in) {
         if (cfg.run_bytes > (256ull << 20)) cfg.run_bytes = 256ull << 20;
     }
     if (cfg.run_max > core::kMaxRun || cfg.fence_free > 2 || cfg.format_ahead > 2) return GALLATIN_ERR_INVALID;
-    if (cfg.bulk_items != 0 && cfg.bulk_items != 1 && cfg.bulk_items != 4 && cfg.bulk_items != 8 &&
-        cfg.bulk_items != 16)
-        return GALLATIN_ERR_INVALID;
-    if (cfg.prefetch > 2 || cfg.pipeline > 3 || cfg.free_team > 3 || cfg.demand_hint > 2 || cfg.cta_tiles > 1024 ||
-        (cfg.cta_threads != 0 && cfg.cta_threads != 64 && cfg.cta_threads != 128 && cfg.cta_threads != 256) ||
-        (cfg.free_threads != 0 && cfg.free_threads != 64 && cfg.free_threads != 128 && cfg.free_threads != 256))
-        return GALLATIN_ERR_INVALID;
+    if (cfg.bulk_items != 0 && cfg.bulk_items != 1 && cfg.bulk_items != 4) return GALLATIN_ERR_INVALID;
+    if (cfg.prefetch > 2 || cfg.demand_hint > 2 || cfg.oom_record > 2) return GALLATIN_ERR_INVALID;
     if (!cfg.run_grow) cfg.run_grow = 3;
     if (cfg.run_grow > 8) return GALLATIN_ERR_INVALID;
     if (nseg > (1ull << 14)) return GALLATIN_ERR_INVALID;        // 22-bit run index at 64 KB blocks (256 GiB)
@@ -1178,6 +734,7 @@ int gallatin_init_ex(const gallatin_config_t *cfg_in) {
     v.prefetch = cfg.prefetch == 1 ? 1u : 0u;              // default off (measured: DESIGN.md)
     v.fence_free = cfg.fence_free;
     v.demand_hint = cfg.demand_hint == 2 ? 0u : 1u;
+    v.oom_record = cfg.oom_record == 2 ? 0u : 1u;
 
     // metadata: one allocation, 256 B aligned sections
     uint64_t sz[12] = {W * 8, 9 * W * 8, nseg * 8, nseg * 4, nseg * 4, nseg * 512, nseg * 1024,
@@ -1207,15 +764,6 @@ int gallatin_init_ex(const gallatin_config_t *cfg_in) {
     v.oom = reinterpret_cast<uint64_t *>(m + offs[11]);
     v.heap = align_up(reinterpret_cast<uint64_t>(heap), core::kSegBytes);   // 16 MiB aligned base
 
-    int occ_m = 0, occ_f = 0;
-    CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ_m, k_bulk_malloc_pipe<4>, kThreads, 0));
-    CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ_f, k_bulk_free_pipe<4>, kThreads, 0));
-    g.pipe_malloc_ctas = (unsigned)(sms * (occ_m > 0 ? occ_m : 1));
-    g.pipe_free_ctas = (unsigned)(sms * (occ_f > 0 ? occ_f : 1));
-    CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ_m, k_bulk_malloc_pers<4>, kThreads, 0));
-    CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ_f, k_bulk_free_pers<4>, kThreads, 0));
-    g.pers_malloc_ctas = (unsigned)(sms * (occ_m > 0 ? occ_m : 1));
-    g.pers_free_ctas = (unsigned)(sms * (occ_f > 0 ? occ_f : 1));
     g.init = true;
     g.device = dev;
     g.cfg = cfg;
@@ -1257,27 +805,8 @@ int gallatin_malloc(const uint64_t *d_sizes, void **d_ptrs, uint64_t n, void *st
     if (n == 0) return GALLATIN_OK;
     if (!d_sizes || !d_ptrs || n > (1ull << 40)) return GALLATIN_ERR_INVALID;
     const uint32_t items = g.cfg.bulk_items ? g.cfg.bulk_items : (n >= (uint64_t)kItemsMin ? 4u : 1u);
-    if (g.cfg.bulk_items == 0 && items == 4 && g.cfg.pipeline == 1) {
-        const uint64_t ntiles = (n + kThreads * 4 - 1) / (kThreads * 4);
-        const unsigned grid = ntiles < g.pipe_malloc_ctas ? (unsigned)ntiles : g.pipe_malloc_ctas;
-        const uint32_t tma = (reinterpret_cast<uintptr_t>(d_sizes) & 15) == 0;
-        k_bulk_malloc_pipe<4><<<grid, kThreads, 0, S(stream)>>>(d_sizes, d_ptrs, n, ntiles, tma);
-    } else if (g.cfg.bulk_items == 0 && items == 4 && g.cfg.pipeline == 3) {
-        const uint64_t ntiles = (n + kThreads * 4 - 1) / (kThreads * 4);
-        const uint32_t T = g.cfg.cta_tiles ? g.cfg.cta_tiles : 4;
-        k_bulk_malloc_pers<4><<<(unsigned)((ntiles + T - 1) / T), kThreads, 0, S(stream)>>>(d_sizes, d_ptrs, n, ntiles, T);
-    } else if (items == 16)
-        k_bulk_malloc_cta<16><<<grid_for((n + 15) / 16), kThreads, 0, S(stream)>>>(d_sizes, d_ptrs, n);
-    else if (items == 8)
-        k_bulk_malloc_cta<8><<<grid_for((n + 7) / 8), kThreads, 0, S(stream)>>>(d_sizes, d_ptrs, n);
-    else if (items == 4)
-        if (g.cfg.cta_threads == 0 || g.cfg.cta_threads == 128)        // default (measured)
-            k_bulk_malloc_cta<4, 10, 128><<<(unsigned)((n + 511) / 512), 128, 0, S(stream)>>>(d_sizes, d_ptrs, n);
-        else if (g.cfg.cta_threads == 64)
-            k_bulk_malloc_cta<4, 20, 64><<<(unsigned)((n + 255) / 256), 64, 0, S(stream)>>>(d_sizes, d_ptrs, n);
-        else
-            k_bulk_malloc_cta<4><<<grid_for((n + 3) / 4), kThreads, 0, S(stream)>>>(d_sizes, d_ptrs, n);
-
+    if (items == 4)   // 128-thread CTAs, 4 requests per thread, one slot RMW per class per CTA
+        k_bulk_malloc_cta<4, 10, 128><<<(unsigned)((n + 511) / 512), 128, 0, S(stream)>>>(d_sizes, d_ptrs, n);
     else
         k_bulk_malloc<1><<<grid_for(n), kThreads, 0, S(stream)>>>(d_sizes, d_ptrs, n);
     return launch_status();
@@ -1287,38 +816,15 @@ int gallatin_free(void *const *d_ptrs, uint64_t n, void *stream) {
     if (!g.init) return GALLATIN_ERR_STATE;
     if (n == 0) return GALLATIN_OK;
     if (!d_ptrs || n > (1ull << 40)) return GALLATIN_ERR_INVALID;
-    if (g.cfg.bulk_items == 0 && n >= (uint64_t)kItemsMin && g.cfg.pipeline == 1) {
-        const uint64_t nwt = (n + 32 * 4 - 1) / (32 * 4);
-        const uint64_t want = (nwt + kThreads / 32 - 1) / (kThreads / 32);
-        const unsigned grid = want < g.pipe_free_ctas ? (unsigned)want : g.pipe_free_ctas;
-        const uint32_t tma = (reinterpret_cast<uintptr_t>(d_ptrs) & 15) == 0;
-        k_bulk_free_pipe<4><<<grid, kThreads, 0, S(stream)>>>(d_ptrs, n, nwt, tma);
-    } else if (g.cfg.bulk_items == 0 && n >= (uint64_t)kItemsMin && g.cfg.pipeline == 3) {
-        const uint64_t nwt = (n + 32 * 4 - 1) / (32 * 4);
-        const uint64_t nct = (nwt + kThreads / 32 - 1) / (kThreads / 32);     // CTA tiles
-        const uint32_t T = g.cfg.cta_tiles ? g.cfg.cta_tiles : 4;
-        k_bulk_free_pers<4><<<(unsigned)((nct + T - 1) / T), kThreads, 0, S(stream)>>>(d_ptrs, n, nwt, T);
-    } else if (g.cfg.bulk_items == 0 && n >= (uint64_t)kItemsMin && g.cfg.free_team == 1) {
-        k_bulk_free_cta<4><<<grid_for((n + 3) / 4), kThreads, 0, S(stream)>>>(d_ptrs, n);
-    } else if (g.cfg.bulk_items == 0 && n >= (uint64_t)kItemsMin && g.cfg.free_team != 2) {
-        // default: warp teams, 32-bit block ids; 64-thread CTAs at 32
-        // registers (64 warps per SM) from kFreeWideMin pointers on, where
-        // more frees in flight shorten a throughput-bound launch, else
-        // 128-thread CTAs at 40 registers (48 warps), whose smaller launches
-        // are bound by the block-return tail (DESIGN.md ablations)
-        const bool wide = g.cfg.free_threads == 64 || (g.cfg.free_threads == 0 && n >= kFreeWideMin);
-        if (g.cfg.free_threads == 256)
-            k_bulk_free_w<4><<<grid_for((n + 3) / 4), kThreads, 0, S(stream)>>>(d_ptrs, n);
-        else if (wide)
-            k_bulk_free_w<4, 64, 32><<<(unsigned)((n + 255) / 256), 64, 0, S(stream)>>>(d_ptrs, n);
-        else
-            k_bulk_free_w<4, 128><<<(unsigned)((n + 511) / 512), 128, 0, S(stream)>>>(d_ptrs, n);
-    } else if (g.cfg.bulk_items >= 8)
-        k_bulk_free<8><<<grid_for((n + 7) / 8), kThreads, 0, S(stream)>>>(d_ptrs, n);
-    else if ((g.cfg.bulk_items >= 4 || (g.cfg.bulk_items == 0 && n >= (uint64_t)kItemsMin)) && g.cfg.free_threads == 128)
-        k_bulk_free<4, 128><<<(unsigned)((n + 511) / 512), 128, 0, S(stream)>>>(d_ptrs, n);
-    else if (g.cfg.bulk_items >= 4 || (g.cfg.bulk_items == 0 && n >= (uint64_t)kItemsMin))
-        k_bulk_free<4><<<grid_for((n + 3) / 4), kThreads, 0, S(stream)>>>(d_ptrs, n);
+    const uint32_t items = g.cfg.bulk_items ? g.cfg.bulk_items : (n >= (uint64_t)kItemsMin ? 4u : 1u);
+    if (items == 4 && n >= kFreeWideMin)
+        // 64-thread CTAs at 32 registers (64 warps per SM): more frees in
+        // flight shorten a throughput-bound launch
+        k_bulk_free_w<4, 64, 32><<<(unsigned)((n + 255) / 256), 64, 0, S(stream)>>>(d_ptrs, n);
+    else if (items == 4)
+        // 128-thread CTAs at 40 registers (48 warps): smaller launches end on
+        // the block-return tail, which the 32-register kernel lengthens
+        k_bulk_free_w<4, 128><<<(unsigned)((n + 511) / 512), 128, 0, S(stream)>>>(d_ptrs, n);
     else
         k_bulk_free<1><<<grid_for(n), kThreads, 0, S(stream)>>>(d_ptrs, n);
     return launch_status();
@@ -1497,6 +1003,8 @@ int gallatin_stats(gallatin_stats_t *out) {
     out->run_grow = v.run_grow;
     out->formatters = v.formatters;
     out->prefetch = v.prefetch;
+    out->demand_hint = v.demand_hint;
+    out->oom_record = v.oom_record;
     return GALLATIN_OK;
 }
 

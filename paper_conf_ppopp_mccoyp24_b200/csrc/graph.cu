@@ -21,7 +21,7 @@ struct gallatin_graph {
     uint32_t *work;       // vertices to process (compacted)
     uint32_t *work2;      // big vertices (CTA-per-vertex deletes)
     uint32_t *nwork;      // [0] work, [1] work2
-    unsigned long long *ctr;   // [0] mallocs [1] frees [2] failed mallocs
+    unsigned long long *ctr;   // [0] mallocs [1] frees [2] failed mallocs [3] vertex ids >= V (ignored)
     uint32_t *hkeys;      // delete-batch hash, one region per source vertex: dst -> remaining count
     uint32_t *hcnt;
     uint64_t hcap;        // slots allocated (>= 4 x the batch)
@@ -66,9 +66,14 @@ __device__ __forceinline__ void count_warp(unsigned long long *ctr, bool m, bool
 }
 
 // cnt[src] += 1 per edge, one atomic per distinct source in a warp
+// (a source id >= V is ignored by the whole batch and counted in ctr[3])
 __global__ void k_count(gallatin_graph g, const uint32_t *src, uint64_t n) {
     const uint64_t i = blockIdx.x * (uint64_t)kT + threadIdx.x;
-    const uint32_t s = i < n ? src[i] : 0xFFFFFFFFu;
+    uint32_t s = i < n ? src[i] : 0xFFFFFFFFu;
+    if (s != 0xFFFFFFFFu && s >= g.V) {
+        atomicAdd(g.ctr + 3, 1ull);
+        s = 0xFFFFFFFFu;
+    }
     const unsigned peers = __match_any_sync(0xFFFFFFFFu, s);
     if (s != 0xFFFFFFFFu && lane() == (uint32_t)__ffs((int)peers) - 1) atomicAdd(g.cnt + s, (uint32_t)__popc(peers));
 }
@@ -160,7 +165,8 @@ __global__ void __launch_bounds__(kT, kGraphMinBlocks) k_free_huge(gallatin_grap
 // append: one atomic per distinct source in a warp reserves the positions
 __global__ void k_scatter(gallatin_graph g, const uint32_t *src, const uint32_t *dst, uint64_t n) {
     const uint64_t i = blockIdx.x * (uint64_t)kT + threadIdx.x;
-    const uint32_t s = i < n ? src[i] : 0xFFFFFFFFu;
+    uint32_t s = i < n ? src[i] : 0xFFFFFFFFu;
+    if (s >= g.V) s = 0xFFFFFFFFu;                            // counted by k_count
     const unsigned peers = __match_any_sync(0xFFFFFFFFu, s);
     const uint32_t leader = (uint32_t)__ffs((int)peers) - 1;
     uint32_t base = 0;
@@ -214,6 +220,7 @@ __global__ void k_hash_insert(gallatin_graph g, const uint32_t *src, const uint3
     const uint64_t i = blockIdx.x * (uint64_t)kT + threadIdx.x;
     if (i >= n) return;
     const uint32_t s = src[i], key = dst[i];
+    if (s >= g.V) return;                                     // counted by k_count
     uint32_t *keys = g.hkeys + g.hoff[s], *cnts = g.hcnt + g.hoff[s];
     const uint32_t mask = region_slots(g.cnt[s]) - 1;
     for (uint32_t h = (uint32_t)hmix(key) & mask;; h = (h + 1) & mask) {
@@ -362,6 +369,10 @@ __global__ void __launch_bounds__(kT, kGraphMinBlocks) k_delete_big(gallatin_gra
 __global__ void k_expand_prep(gallatin_graph g, const uint32_t *vs, uint64_t n) {
     const uint64_t i = blockIdx.x * (uint64_t)kT + threadIdx.x;
     if (i >= n) return;
+    if (vs[i] >= g.V) {                        // ignored, counted
+        atomicAdd(g.ctr + 3, 1ull);
+        return;
+    }
     const uint32_t s = g.size[vs[i]];
     g.cnt[vs[i]] = s < 4 ? 4 : s;              // each round appends max(size, 4) edges
 }
@@ -369,7 +380,9 @@ __global__ void k_expand_prep(gallatin_graph g, const uint32_t *vs, uint64_t n) 
 __global__ void __launch_bounds__(kT, kGraphMinBlocks) k_expand_fill(gallatin_graph g, const uint32_t *vs, uint64_t n) {
     const uint64_t warps = (uint64_t)gridDim.x * (kT / 32);
     for (uint64_t w = (blockIdx.x * (uint64_t)kT + threadIdx.x) >> 5; w < n; w += warps) {
-        const uint32_t v = vs[w], s0 = g.size[v], add = g.cnt[v];
+        const uint32_t v = vs[w];
+        if (v >= g.V) continue;
+        const uint32_t s0 = g.size[v], add = g.cnt[v];
         if (add >= kHuge) {                                   // the whole grid fills it (k_expand_huge)
             if (lane() == 0) g.work2[atomicAdd(g.nwork + 1, 1u)] = v;
             continue;
@@ -467,7 +480,9 @@ __global__ void __launch_bounds__(kT, kGraphMinBlocks) k_edge_insert(gallatin_gr
                                                                       const uint32_t *dst, uint64_t n) {
     const uint64_t i = blockIdx.x * (uint64_t)kT + threadIdx.x;
     bool m = false, f = false, fail = false;
-    const bool active = i < n;
+    const bool in = i < n && src[i] < g.V;
+    if (i < n && !in) atomicAdd(g.ctr + 3, 1ull);             // vertex id >= V: ignored, counted
+    const bool active = in;
     const uint32_t v = active ? src[i] : 0u, x = active ? dst[i] : 0u;
     bool done = !active;
     uint32_t ns = 32;
@@ -538,7 +553,9 @@ __global__ void __launch_bounds__(kT, kGraphMinBlocks) k_edge_delete(gallatin_gr
                                                                       const uint32_t *dst, uint64_t n) {
     const uint64_t i = blockIdx.x * (uint64_t)kT + threadIdx.x;
     bool m = false, f = false, fail = false;
-    const bool active = i < n;
+    const bool in = i < n && src[i] < g.V;
+    if (i < n && !in) atomicAdd(g.ctr + 3, 1ull);             // vertex id >= V: ignored, counted
+    const bool active = in;
     const uint32_t v = active ? src[i] : 0u, x = active ? dst[i] : 0u;
     bool done = !active;
     uint32_t ns = 32;
@@ -624,7 +641,7 @@ int gallatin_graph_create(uint32_t V, gallatin_graph_t **out) {
               cudaMalloc(&g->cap, 4ull * V) == cudaSuccess && cudaMalloc(&g->cnt, 4ull * V) == cudaSuccess &&
               cudaMalloc(&g->old, 8ull * V) == cudaSuccess && cudaMalloc(&g->work, 4ull * V) == cudaSuccess &&
               cudaMalloc(&g->work2, 4ull * V) == cudaSuccess && cudaMalloc(&g->nwork, 8) == cudaSuccess &&
-              cudaMalloc(&g->ctr, 24) == cudaSuccess && cudaMalloc(&g->lock, 4ull * V) == cudaSuccess &&
+              cudaMalloc(&g->ctr, 32) == cudaSuccess && cudaMalloc(&g->lock, 4ull * V) == cudaSuccess &&
               cudaMalloc(&g->hoff, 4ull * V) == cudaSuccess && cudaMalloc(&g->hbump, 4) == cudaSuccess;
     if (!ok) {
         cudaGetLastError();
@@ -634,7 +651,7 @@ int gallatin_graph_create(uint32_t V, gallatin_graph_t **out) {
     cudaMemset(g->list, 0, 8ull * V);
     cudaMemset(g->size, 0, 4ull * V);
     cudaMemset(g->cap, 0, 4ull * V);
-    cudaMemset(g->ctr, 0, 24);
+    cudaMemset(g->ctr, 0, 32);
     cudaMemset(g->lock, 0, 4ull * V);
     *out = g;
     return status();
@@ -742,12 +759,12 @@ int gallatin_graph_gather(const gallatin_graph_t *g, const uint64_t *off, uint32
     return status();
 }
 
-int gallatin_graph_counters(const gallatin_graph_t *g, uint64_t out[3]) {
+int gallatin_graph_counters(const gallatin_graph_t *g, uint64_t out[4]) {
     if (!g || !out) return GALLATIN_ERR_INVALID;
     if (cudaDeviceSynchronize() != cudaSuccess) return GALLATIN_ERR_CUDA;
-    unsigned long long c[3];
+    unsigned long long c[4];
     if (cudaMemcpy(c, g->ctr, sizeof(c), cudaMemcpyDeviceToHost) != cudaSuccess) return GALLATIN_ERR_CUDA;
-    for (int i = 0; i < 3; i++) out[i] = c[i];
+    for (int i = 0; i < 4; i++) out[i] = c[i];
     return GALLATIN_OK;
 }
 

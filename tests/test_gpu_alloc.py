@@ -14,7 +14,7 @@ import torch
 
 import oracle
 import workload_gen as wg
-from helpers import SEG, class_size, diff_images, pristine_image
+from helpers import SEG, check_live_invariants, class_size, diff_images, pristine_image
 
 pytestmark = pytest.mark.gpu
 NONE = (1 << 64) - 1
@@ -38,13 +38,21 @@ def G():
 
 
 def _replay_case(G, nseg, run_max, fa, kinds, args, keys, slot_base=16, slot_min=2, run_bytes=32 << 20, pf=None,
-                 run_init=1, run_grow=0):
+                 run_init=1, run_grow=0, record=None):
+    """GPU serialized replay vs O2: O2-P at the paper's knobs (with the
+    exhaustion record on, where it is state-neutral), O2-R otherwise (the GPU
+    with the record off: O2-R does not model it)."""
     if pf is None:
         pf = run_max > 1                    # the paper's policy (run_max=1) has no prefetch
+    paper = run_max == 1 and not fa and not pf and run_init == 1
+    if record is None:
+        record = paper
     G.gallatin_init(nseg * SEG, slot_base=slot_base, slot_min=slot_min, run_max=run_max, run_bytes=run_bytes,
-                    format_ahead=1 if fa else 2, prefetch=1 if pf else 2, run_init=run_init, run_grow=run_grow)
+                    format_ahead=1 if fa else 2, prefetch=1 if pf else 2, run_init=run_init, run_grow=run_grow,
+                    oom_record=1 if record else 2)
     out = _u64(G.gallatin_replay(_dev(kinds, np.uint8), _dev(args), _dev(keys)))
-    o2 = oracle.Allocator(nseg, **G.oracle_params())
+    o2 = oracle.model(nseg, **G.oracle_params())
+    assert isinstance(o2, oracle.RunsAllocator) != paper
     want = o2.replay(kinds, args, keys)
     bad = np.nonzero(out != want)[0]
     assert len(bad) == 0, f"{len(bad)} ops differ; first op {bad[0]} kind {kinds[bad[0]]} size {args[bad[0]]}: " \
@@ -93,6 +101,52 @@ def test_serialized_replay_runs_prefetch_matrix(cuda_ok, G, seed, nseg, run_max,
     _replay_case(G, nseg, run_max, fa, kinds, args, keys, pf=pf, run_init=ri, run_grow=rg)
 
 
+def test_serialized_replay_default_knobs(cuda_ok, G):
+    """The production knobs gallatin_init picks for a 64-segment heap (148
+    slots at 16 B, slot_min 4, runs up to 256 blocks / heap/64 bytes, x8
+    growth, the derived first run, format-ahead) with the exhaustion record
+    off, against O2-R; keys span every slot."""
+    nseg = 64
+    kinds, args, keys = wg.replay_ops(8000, 141, p_free=0.45, p_drain=0.002, nkeys=148 * 4)
+    G.gallatin_init(nseg * SEG, oom_record=2)
+    st = G.gallatin_stats()
+    assert st["slot_base"] == 148 and st["run_max"] == 256 and st["format_ahead"] == 1 and st["run_grow"] == 3
+    out = _u64(G.gallatin_replay(_dev(kinds, np.uint8), _dev(args), _dev(keys)))
+    o2 = oracle.model(nseg, **G.oracle_params())
+    want = o2.replay(kinds, args, keys)
+    assert np.array_equal(out, want), f"{int((out != want).sum())} ops differ"
+    msg = diff_images(G.gallatin_snapshot(), o2.image())
+    assert not msg, msg
+
+
+@pytest.mark.parametrize("seed,nseg", [(151, 3), (152, 6), (153, 16)])
+def test_serialized_replay_record_on_invariants(cuda_ok, G, seed, nseg):
+    """Run knobs with the exhaustion record ON (the production setting) under
+    heavy OOM: the record is a concurrency device O2-R does not model, so the
+    replay is checked by the invariants instead -- every pointer in the heap,
+    aligned to its class, live allocations disjoint, the accounting of the
+    live set equal to the closed form, and free-all + drain pristine."""
+    kinds, args, keys = wg.replay_ops(6000, seed, p_free=0.4, p_drain=0.003, nkeys=64)
+    G.gallatin_init(nseg * SEG, slot_base=16, slot_min=2, run_max=64, run_bytes=32 << 20, format_ahead=1,
+                    prefetch=1, run_init=4, run_grow=2)
+    out = _u64(G.gallatin_replay(_dev(kinds, np.uint8), _dev(args), _dev(keys)))
+    live = {}
+    for i, k in enumerate(kinds):
+        if k == 0 and out[i] != np.uint64(NONE):
+            live[i] = (int(out[i]), int(args[i]))
+        elif k == 1:
+            live.pop(int(args[i]), None)
+        elif k == 2:
+            pass
+    assert (out[kinds == 0] == np.uint64(NONE)).sum() > 100          # OOM exercised
+    offs = np.array([v[0] for v in live.values()], dtype=np.uint64)
+    sizes = [v[1] for v in live.values()]
+    check_live_invariants(nseg, offs, sizes)
+    assert G.gallatin_stats()["errors"] == 0
+    G.gallatin_free(_dev(offs + np.uint64(G.gallatin_stats()["heap_base"])))
+    _assert_pristine(G, nseg)
+
+
 def _bulk_round(G, nseg, sizes, check_accounting=True):
     """malloc -> stamp -> verify -> usable/overlap checks -> free; returns #NULL."""
     d_sizes = _dev(sizes)
@@ -137,7 +191,7 @@ def test_config1_concurrent(cuda_ok, G):
     assert _bulk_round(G, nseg, sizes) == 0
     _assert_pristine(G, nseg)
     # accounting equals O2's on the same sizes
-    o2 = oracle.Allocator(nseg, **G.oracle_params())
+    o2 = oracle.model(nseg, **G.oracle_params())
     o2.malloc_batch(sizes)
     assert o2.usable_live == (1 << 16) * 16
 
@@ -271,18 +325,15 @@ def test_config3_full_size_bench_launch(cuda_ok, G):
         _assert_pristine(G, nseg)
 
 
-@pytest.mark.parametrize("knobs", [dict(pipeline=1), dict(pipeline=2), dict(pipeline=3), dict(free_team=1),
-                                   dict(cta_threads=64), dict(cta_threads=256), dict(free_team=2),
-                                   dict(free_threads=256), dict(free_threads=64), dict(free_threads=128),
-                                   dict(free_team=2, free_threads=128),
-                                   dict(bulk_items=8), dict(bulk_items=16), dict(bulk_items=1),
-                                   dict(pipeline=2, free_team=1)])
-@pytest.mark.parametrize("n", [(1 << 21) + 77, 1 << 22])
+@pytest.mark.parametrize("knobs", [dict(bulk_items=1), dict(bulk_items=4), dict(demand_hint=2), dict(oom_record=2),
+                                   dict(prefetch=1), dict(fence_free=2), dict(run_max=1, format_ahead=2, run_init=1)])
+@pytest.mark.parametrize("n", [(1 << 21) + 77, (1 << 23) + 5])
 def test_bulk_kernel_variants(cuda_ok, G, knobs, n):
-    """Every bulk-kernel variant (persistent TMA-pipelined, CTA-aggregated or
-    warp-team frees, 1/4/8/16 requests per thread) on mixed sizes with a
-    ragged tail: stamp-verified, accounted, overlap-checked, pristine after
-    free-all + drain."""
+    """Both bulk-kernel pairs (one request per thread with warp teams; four
+    per thread with one slot RMW per class per CTA tile) at both free CTA
+    shapes (2^21 and 2^23+ pointers), and the policy knobs, on mixed sizes
+    with a ragged tail: stamp-verified, accounted, overlap-checked, pristine
+    after free-all + drain."""
     nseg = 1024
     G.gallatin_init(nseg * SEG, **knobs)
     sizes = wg.mixed_sizes(n, p_large=2.0 ** -14)
@@ -290,11 +341,36 @@ def test_bulk_kernel_variants(cuda_ok, G, knobs, n):
     _assert_pristine(G, nseg)
 
 
+@pytest.mark.parametrize("items", [1, 4])
+def test_malloc_zero_and_nulls(cuda_ok, G, items):
+    """malloc(0) is NULL (reading A-4) in both bulk kernels, next to real
+    requests in the same warps and CTA tiles; freeing the NULLs is a no-op
+    (P:241); non-power-of-two sizes round up to their class."""
+    nseg = 64
+    G.gallatin_init(nseg * SEG, bulk_items=items)
+    n = (1 << 20) + 17
+    rng = np.random.Generator(np.random.PCG64(5))
+    sizes = rng.integers(0, 4097, n).astype(np.uint64)
+    sizes[rng.random(n) < 0.25] = 0
+    d = _dev(sizes)
+    p = G.gallatin_malloc(d)
+    torch.cuda.synchronize()
+    pu = _u64(p)
+    assert np.all((pu == 0) == (sizes == 0)), "malloc(0) must be NULL and every other request granted"
+    G.gallatin_stamp(p, d)
+    assert G.gallatin_verify(p, d) == 0
+    usum, ubad = G.gallatin_usable(p, d)
+    assert ubad == 0 and usum == sum(class_size(int(s)) for s in sizes)
+    G.gallatin_free(p)
+    assert G.gallatin_stats()["errors"] == 0
+    _assert_pristine(G, nseg)
+
+
 def test_bulk_kernels_unaligned_arrays(cuda_ok, G):
-    """Size and pointer arrays that start 8 bytes past a 16-byte boundary
-    (the TMA tile loads fall back to plain loads)."""
+    """Size and pointer arrays that start 8 bytes past a 16-byte boundary,
+    through both bulk-kernel pairs."""
     nseg = 256
-    for knobs in (dict(pipeline=1), dict(pipeline=2), dict(pipeline=3), {}):
+    for knobs in (dict(bulk_items=1), {}):
         G.gallatin_init(nseg * SEG, **knobs)
         n = (1 << 20) + 3
         sizes = _dev(np.concatenate([[0], wg.mixed_sizes(n, upper=512, p_large=0.0)]))[1:]

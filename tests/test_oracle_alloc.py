@@ -1,20 +1,30 @@
-"""Pins for O2, the sequential allocator oracle (oracle/alloc_oracle.c).
+"""Pins for O2, the sequential allocator oracle (oracle/alloc_*.c).
 
-Each test checks O2 against something other than O2: numbers PAPER.md prints
-(tests/golden/paper_geometry.txt), closed forms derived in the test from the
-paper's rules, and invariants recomputed here in Python from the returned
-offsets (in heap, aligned, non-overlapping, byte accounting, pristine image
-after free-all + drain).
+O2-P (``oracle.Allocator``, alloc_paper.c) is the paper's policy POL; O2-R
+(``oracle.RunsAllocator``, alloc_runs.c) is the deviation model (DESIGN.md
+Deviations 5, 8).  Each test checks O2 against something other than O2:
+numbers PAPER.md prints (tests/golden/paper_geometry.txt), closed forms
+derived in the test from the paper's rules, invariants recomputed here in
+Python from the returned offsets, and a naive brute-force simulation written
+from the policy text (tests/pol_sim.py).  DESIGN.md 11 lists which test pins
+which O2 function.
 """
 import numpy as np
 import pytest
 
 import oracle
 import workload_gen as wg
+from helpers import SEG, check_live_invariants, class_size, diff_images, golden, image_sections, pristine_image
 from oracle import NONE, TREE_CONT, TREE_FREE
-from helpers import SEG, check_live_invariants, class_size, golden, image_sections, pristine_image
+from pol_sim import PolSim
 
 
+def runs(nseg, **kw):
+    kw.setdefault("run_bytes", 32 << 20)
+    return oracle.RunsAllocator(nseg, **kw)
+
+
+# ------------------------------------------------------------ O2-P (POL) ---
 def test_block_buffer_slots_match_paper_a40():
     """on the A40 the 16 B buffer holds 128 blocks, halving per class,
     capped below at four."""
@@ -25,17 +35,18 @@ def test_block_buffer_slots_match_paper_a40():
     assert [b.nslot(c) for c in range(9)] == [148, 74, 37, 18, 9, 4, 4, 4, 4]
 
 
-@pytest.mark.parametrize("run_max,fa,pf", [(1, 0, 0), (16, 1, 1), (128, 0, 1)])
+@pytest.mark.parametrize("knobs", [None, dict(run_max=16, format_ahead=1, prefetch=1),
+                                   dict(run_max=128, prefetch=1)])
 @pytest.mark.parametrize("size,blocks", [(16, "blocks_per_segment_16B"), (32, "blocks_per_segment_32B")])
-def test_blocks_per_segment_and_in_order_slices(size, blocks, run_max, fa, pf):
+def test_blocks_per_segment_and_in_order_slices(size, blocks, knobs):
     """256 blocks per segment at 16 B, 128 at 32 B; 4096 slices
     per block handed out in order; segments used front first.  With
     one slot, the k-th request lands at k*size exactly until the segment is
     full, then the next segment starts at 16 MB -- with one-block buffers
-    (the paper) and with growing runs of consecutive blocks (ours)."""
+    (O2-P, the paper) and with growing runs of consecutive blocks (O2-R)."""
     g = golden()
     nb = g[blocks]
-    a = oracle.Allocator(4, slot_base=1, slot_min=1, run_max=run_max, format_ahead=fa, prefetch=pf)
+    a = oracle.Allocator(4, slot_base=1, slot_min=1) if knobs is None else runs(4, slot_base=1, slot_min=1, **knobs)
     n = nb * g["slices_per_block"]
     offs = a.malloc_batch(np.full(n + 5, size, dtype=np.uint64), keydiv=0)
     assert np.array_equal(offs[:n], np.arange(n, dtype=np.uint64) * np.uint64(size))
@@ -88,6 +99,27 @@ def test_large_allocations_come_from_the_back():
     assert a.check() == 0
 
 
+def test_size_classes_rounding_and_zero():
+    """A-1..A-4 closed forms: malloc(0) is NULL; 1 and 16 B share the 16 B
+    class, 17 B takes 32 B, 4095 B the 4 KB class; 4097 B a
+    whole 64 KB block of the tree the 16 B slices use (A-1, A-2); exactly 16 MB one segment (A-3) from the back
+    (P:138), 16 MB + 1 two segments."""
+    a = oracle.Allocator(8, slot_base=1, slot_min=1)
+    assert a.malloc(0, 0) == NONE and a.live_count == 0
+    assert [a.malloc(s, 0) for s in (1, 16, 5)] == [0, 16, 32]               # one 16 B block, in order
+    assert a.malloc(17, 0) == SEG                                             # 32 B class: next segment
+    assert a.malloc(4095, 0) == 2 * SEG and a.malloc(4096, 0) == 2 * SEG + 4096
+    assert a.malloc(4097, 0) == 65536          # a whole 64 KB block of tree 0: block 1 of segment 0 (A-2)
+    assert a.malloc(SEG, 0) == 7 * SEG
+    assert a.malloc(SEG + 1, 0) == 5 * SEG
+    d = image_sections(a.image())
+    assert list(d["segword"][5:8] >> np.uint64(32)) == [9 + 2, TREE_CONT, 9 + 1]
+    assert a.usable_live == 3 * 16 + 32 + 2 * 4096 + 65536 + 3 * SEG
+    assert [oracle.usable_size(s) for s in (0, 1, 17, 4095, 4097, SEG, SEG + 1)] == \
+        [class_size(s) for s in (0, 1, 17, 4095, 4097, SEG, SEG + 1)]
+    assert a.check() == 0
+
+
 def test_capacity_closed_form_single_class():
     """One slot, one class, empty heap: exactly nseg * (256 >> c) * 4096
     slices fit, then NULL."""
@@ -101,9 +133,10 @@ def test_capacity_closed_form_single_class():
         assert a.usable_live == cap * size == nseg * SEG
 
 
-def test_accounting_matches_closed_form_mixed():
+@pytest.mark.parametrize("model", ["paper", "runs"])
+def test_accounting_matches_closed_form_mixed(model):
     sizes = wg.mixed_sizes(50_000, seed=5, p_large=2.0 ** -9)
-    a = oracle.Allocator(256)
+    a = oracle.Allocator(256) if model == "paper" else runs(256, run_max=256, format_ahead=1, run_init=8, run_grow=3)
     offs = a.malloc_batch(sizes, keydiv=32)
     ok = offs != np.uint64(NONE)
     assert ok.all()
@@ -116,15 +149,16 @@ def test_accounting_matches_closed_form_mixed():
     assert np.array_equal(a.image(), pristine_image(256, 302))
 
 
-@pytest.mark.parametrize("seed,nseg,run_max,fa,pf", [(1, 4, 1, 0, 0), (2, 8, 1, 0, 0), (3, 6, 16, 1, 1), (4, 64, 8, 1, 1),
-                                                     (5, 5, 128, 0, 0), (6, 16, 4, 1, 0), (7, 32, 512, 1, 1)])
-def test_random_sequences_tiny_heaps(seed, nseg, run_max, fa, pf):
+@pytest.mark.parametrize("seed,nseg,knobs", [(1, 4, None), (2, 8, None), (3, 6, dict(run_max=16, format_ahead=1, prefetch=1)),
+                                             (4, 64, dict(run_max=8, format_ahead=1, prefetch=1)),
+                                             (5, 5, dict(run_max=128)), (6, 16, dict(run_max=4, format_ahead=1)),
+                                             (7, 32, dict(run_max=512, format_ahead=1, prefetch=1))])
+def test_random_sequences_tiny_heaps(seed, nseg, knobs):
     """Random malloc/free/drain sequences on 4-64 segment heaps, including OOM:
     live allocations re-checked in Python, structure checked, and free-all +
     drain restores the analytic pristine image bit-exactly."""
     kinds, args, keys = wg.replay_ops(20_000, seed, p_free=0.45, p_drain=0.002, nkeys=64)
-    a = oracle.Allocator(nseg, slot_base=16, slot_min=2, run_max=run_max, run_bytes=32 << 20, format_ahead=fa,
-                         prefetch=pf)
+    a = oracle.Allocator(nseg, 16, 2) if knobs is None else runs(nseg, slot_base=16, slot_min=2, **knobs)
     out = a.replay(kinds, args, keys)
     live = {}
     for i, k in enumerate(kinds):
@@ -138,7 +172,7 @@ def test_random_sequences_tiny_heaps(seed, nseg, run_max, fa, pf):
         assert check_live_invariants(nseg, offs, sizes) == a.usable_live
     assert a.check() == 0, oracle.violation_names(a.check())
     assert a.errors == 0
-    nulls = sum(1 for i, k in enumerate(kinds) if k == 0 and out[i] == np.uint64(NONE))
+    nulls = sum(1 for i, k in enumerate(kinds) if k == 0 and out[i] == np.uint64(NONE) and args[i] != 0)
     assert nulls > 0 or nseg >= 64   # the tiny heaps do hit OOM
     for o in offs:
         a.free(o)
@@ -155,15 +189,66 @@ def test_errors_counted_for_foreign_frees():
     assert a.errors == 2
 
 
+# --------------------------------------------- brute-force simulation pin ---
+SIM_CASES = [
+    (11, 3, 16, 2, None), (12, 4, 16, 2, None), (13, 8, 16, 2, None), (14, 6, 4, 1, None), (15, 2, 148, 4, None),
+    (16, 6, 16, 2, dict(run_max=16, format_ahead=1, prefetch=1)),
+    (17, 5, 16, 2, dict(run_max=128)),
+    (18, 16, 16, 2, dict(run_max=4, format_ahead=1)),
+    (19, 3, 16, 2, dict(run_max=512, run_init=256, run_grow=4, format_ahead=1, prefetch=1)),
+    (20, 6, 16, 2, dict(run_max=256, run_init=64, run_grow=8, prefetch=1)),
+    (21, 4, 1, 1, dict(run_max=256, run_init=256, run_grow=3, format_ahead=1)),
+    # production-shaped knobs (gallatin_init defaults at 64 segments): 148 slots at 16 B,
+    # runs up to 256 blocks / 16 MB, format-ahead, x8 growth, first runs of 4 blocks
+    (22, 64, 148, 4, dict(run_max=256, run_bytes=16 << 20, run_init=4, run_grow=3, format_ahead=1)),
+]
+
+
+@pytest.mark.parametrize("seed,nseg,sb,sm,knobs", SIM_CASES)
+def test_o2_matches_brute_force_simulation(seed, nseg, sb, sm, knobs):
+    """Every offset and the whole canonical image after a random op list
+    (slices of every class, non-power-of-two sizes, malloc(0), whole blocks,
+    1 and 2+ segments, frees, drains, OOM) equal a naive simulation written
+    from the policy text (tests/pol_sim.py: set scans instead of vEB trees,
+    deques for rings) -- for O2-P at the paper's knobs and O2-R at run /
+    format-ahead / prefetch / trim settings."""
+    kinds, args, keys = wg.replay_ops(4000 if nseg < 64 else 6000, seed, p_free=0.45, p_drain=0.003, nkeys=64)
+    kw = dict(knobs or {})
+    if knobs is not None:
+        kw.setdefault("run_bytes", 32 << 20)
+    sim = PolSim(nseg, sb, sm, **kw)
+    a = oracle.model(nseg, slot_base=sb, slot_min=sm, **kw)
+    assert isinstance(a, oracle.RunsAllocator) == (knobs is not None)
+    want = sim.replay(kinds, args, keys)
+    got = a.replay(kinds, args, keys)
+    bad = np.nonzero(got != want)[0]
+    assert len(bad) == 0, f"op {bad[0]} (kind {kinds[bad[0]]}, arg {args[bad[0]]}): o2 {got[bad[0]]:#x} sim {want[bad[0]]:#x}"
+    msg = diff_images(a.image(), sim.image())
+    assert not msg, msg
+    assert (got == NONE).sum() > (kinds == 0).sum() // 20 or nseg >= 64     # OOM exercised on the tiny heaps
+
+
+@pytest.mark.parametrize("seed,nseg", [(31, 3), (32, 8), (33, 32)])
+def test_runs_model_at_paper_knobs_equals_paper_core(seed, nseg):
+    """O2-R with run_max = run_init = 1, no format-ahead, no prefetch is the
+    paper's one-block buffer: offsets and images equal O2-P's (its trims
+    give back nothing when every run is one partly drawn block)."""
+    kinds, args, keys = wg.replay_ops(8000, seed, p_free=0.45, p_drain=0.003, nkeys=64)
+    a, b = oracle.Allocator(nseg, 16, 2), runs(nseg, slot_base=16, slot_min=2, run_max=1, run_init=1)
+    assert np.array_equal(a.replay(kinds, args, keys), b.replay(kinds, args, keys))
+    assert np.array_equal(a.image(), b.image())
+
+
+# --------------------------------------------------- O2-R closed forms ---
 def test_trim_gives_back_undrawn_blocks_before_oom():
-    """DESIGN.md Deviations 5 (runs) + Alg.2's "no allocations left":
+    """R5 (DESIGN.md Deviations 8) + Alg.2's "no allocations left":
     a slot's whole-segment run must not starve another request.  On a
     one-segment heap the 16 B slot's first run takes all 256 blocks; a 64 KB
     block request then finds no segment, the slot keeps the ceil(1/4096) = 1
     block it has drawn from and gives back blocks 1..255 in order (FIFO ring,
     P:178), so the request gets block 1 at 64 KB, the next ones blocks 2..255,
     and only then NULL -- closed forms from the paper's layout."""
-    a = oracle.Allocator(1, slot_base=1, slot_min=1, run_max=256, run_bytes=16 << 20, run_init=256, run_grow=3)
+    a = runs(1, slot_base=1, slot_min=1, run_max=256, run_bytes=16 << 20, run_init=256, run_grow=3)
     assert a.malloc(16, 0) == 0
     d = image_sections(a.image())
     assert int(d["segword"][0]) & 0xFFFFFFFF == 0                 # all 256 blocks held by the run
@@ -183,13 +268,13 @@ def test_trim_gives_back_undrawn_blocks_before_oom():
 
 @pytest.mark.parametrize("run_grow", [1, 2, 3, 8])
 def test_run_growth_factor(run_grow):
-    """A refilled run is 2^run_grow times the last (capped): with one 16 B slot
-    and first run 1 block, the k-th run starts right after the (k-1)-th, so the
-    addresses stay consecutive and the slot's run length after
-    r refills is min(2^(run_grow*r), cap) -- the closed form, read from the
-    image's slot word."""
+    """R1: a refilled run is 2^run_grow times the last (capped): with one 16 B
+    slot and first run 1 block, the k-th run starts right after the (k-1)-th,
+    so the addresses stay consecutive and the slot's run length
+    after r refills is min(2^(run_grow*r), cap) -- the closed form, read from
+    the image's slot word."""
     cap = 64
-    a = oracle.Allocator(4, slot_base=1, slot_min=1, run_max=cap, run_bytes=64 << 20, run_init=1, run_grow=run_grow)
+    a = runs(4, slot_base=1, slot_min=1, run_max=cap, run_bytes=64 << 20, run_init=1, run_grow=run_grow)
     m, total = 1, 0
     for r in range(4):
         total += m * 4096
@@ -201,17 +286,28 @@ def test_run_growth_factor(run_grow):
     assert a.check() == 0
 
 
+@pytest.mark.parametrize("run_init,c,want", [(1, 0, 1), (4, 0, 4), (256, 0, 256), (256, 3, 32), (256, 8, 1),
+                                             (64, 5, 8), (64, 4, 8), (2, 7, 2)])
+def test_first_run_length(run_init, c, want):
+    """R1 first run: min(max(run_init >> c, min(run_init, 8)), 256 >> c)
+    blocks -- read from the slot word after one request of class c."""
+    a = runs(8, slot_base=1, slot_min=1, run_max=512, run_bytes=1 << 30, run_init=run_init, run_grow=1)
+    assert a.malloc(16 << c, 0) == 0
+    w = int(image_sections(a.image())["slots"][c])
+    assert (w >> 22) & 0x3FF == want and w >> 32 == 1 and w & 0x3FFFFF == 0
+
+
 def test_shared_run_keeps_longest_consecutive_blocks():
-    """DESIGN.md Deviations 5: a run taken from a block-tree segment keeps the
-    longest run of consecutive block indices among the ring entries it
-    dequeues (lowest start on ties), not the FIFO prefix.  One segment, one
-    64 B slot whose first run is the whole segment (64 blocks of 256 KB,
-    P:174); its 64*4096 slices are drawn, then every block except 9 is
-    freed in the order 30..63, 0..8, 10..29 (ring order).  The refill
-    (want = cap = 64) dequeues those 63 entries and keeps 10..63 (54 blocks),
-    re-enqueueing 0..8; the prefix rule would have kept 30..63."""
+    """R2: a run taken from a block-tree segment keeps the longest run of
+    consecutive block indices among the ring entries it dequeues (lowest
+    start on ties), not the FIFO prefix.  One segment, one 64 B slot whose
+    first run is the whole segment (64 blocks of 256 KB); its
+    64*4096 slices are drawn, then every block except 9 is freed in the order
+    30..63, 0..8, 10..29 (ring order).  The refill (want = cap = 64)
+    dequeues those 63 entries and keeps 10..63 (54 blocks), re-enqueueing
+    0..8; the prefix rule would have kept 30..63."""
     bb = 64 * 4096                                            # 64 B slices: 256 KB blocks
-    a = oracle.Allocator(1, slot_base=1, slot_min=1, run_max=64, run_bytes=16 << 20, run_init=256, run_grow=1)
+    a = runs(1, slot_base=1, slot_min=1, run_max=64, run_bytes=16 << 20, run_init=256, run_grow=1)
     offs = a.malloc_batch(np.full(64 * 4096, 64, dtype=np.uint64), keydiv=0)
     assert np.array_equal(offs, np.arange(64 * 4096, dtype=np.uint64) * np.uint64(64))
     for b in list(range(30, 64)) + list(range(0, 9)) + list(range(10, 30)):
@@ -225,6 +321,68 @@ def test_shared_run_keeps_longest_consecutive_blocks():
     assert a.check() == 0
 
 
+def test_whole_segment_runs_taken_privately():
+    """R2 (>= nb blocks): a run of whole segments takes the lowest free
+    segment and the free ones right after it, with no ring and no block-tree
+    entry.  4 segments; two 16 MB requests take 3 and 2 from the back
+    (P:138); the 16 B slot's first run is segment 0 (256 blocks, 1 MB run
+    cap 512 blocks), its refill wants 512 blocks = 2 segments but only
+    segment 1 is free before the taken ones, so the run is 256 blocks at
+    segment 1 -- and slices stay consecutive across the boundary."""
+    a = runs(4, slot_base=1, slot_min=1, run_max=512, run_bytes=32 << 20, run_init=256, run_grow=1)
+    assert [a.malloc(SEG, 0), a.malloc(SEG, 0)] == [3 * SEG, 2 * SEG]
+    n = (1 << 20) + 3
+    offs = a.malloc_batch(np.full(n, 16, dtype=np.uint64), keydiv=0)
+    assert np.array_equal(offs, np.arange(n, dtype=np.uint64) * np.uint64(16))
+    d = image_sections(a.image())
+    assert list(d["segword"][:2]) == [0, 0]                   # tree 0, no block available, both
+    assert not d["btrees"].any() and int(d["qcount"][:2].sum()) == 0
+    w = int(d["slots"][0])
+    assert (w >> 22) & 0x3FF == 256 and w & 0x3FFFFF == 256 and w >> 32 == 3   # second run: segment 1
+    assert int(d["segtree"][0]) == 0                          # no segment free
+    assert a.malloc(16, 0) == (1 << 20) * 16 + 3 * 16 and a.check() == 0
+
+
+def test_format_ahead_closed_form():
+    """R3: the reservation that takes a segment's available blocks from >= nb/4
+    to < nb/4 formats the next segment of its tree.  One 16 B slot (nb = 256,
+    nb/4 = 64), runs of 1, 2, 4, 8, then 16 blocks (run_max 16): the first
+    comes from a fresh segment (no format-ahead there), the run that takes
+    blocks 191..206 leaves 49 < 64 of 65: the refill at slice 191 * 4096
+    formats segment 1 (tree 0, 256 available, in block tree 0)."""
+    a = runs(4, slot_base=1, slot_min=1, run_max=16, run_bytes=32 << 20, format_ahead=1, run_init=1, run_grow=1)
+    a.malloc_batch(np.full(191 * 4096, 16, dtype=np.uint64), keydiv=0)
+    d = image_sections(a.image())
+    assert int(d["segword"][1]) >> 32 == TREE_FREE and int(d["segword"][0]) & 0xFFFFFFFF == 256 - 191
+    assert a.malloc(16, 0) == 191 * 65536
+    d = image_sections(a.image())
+    assert int(d["segword"][0]) & 0xFFFFFFFF == 256 - 207
+    assert int(d["segword"][1]) == (0 << 32) | 256 and int(d["btrees"][0][0]) == 0b11
+    assert list(d["qentries"][1][:3]) == [0, 1, 2] and int(d["qcount"][1]) == 256
+    assert a.check() == 0
+
+
+def test_prefetch_closed_form():
+    """R4: the request drawing the middle of a run (index 2048 of a one-block
+    run) fetches the next run -- 2^run_grow times as long -- into the slot's
+    second word; the run's end swaps it in and the slices stay consecutive.
+    One 16 B slot, runs of 1, 2, 4 blocks from segment 0's ring."""
+    a = runs(4, slot_base=1, slot_min=1, run_max=16, run_bytes=32 << 20, prefetch=1, run_init=1, run_grow=1)
+    a.malloc_batch(np.full(2048, 16, dtype=np.uint64), keydiv=0)
+    assert int(image_sections(a.image())["next"][0]) == 0x3FFFFF              # not yet
+    a.malloc(16, 0)                                                          # draws index 2048
+    assert int(image_sections(a.image())["next"][0]) == (2 << 22) | 1        # blocks 1..2
+    offs = a.malloc_batch(np.full(2047 + 1, 16, dtype=np.uint64), keydiv=0)  # to the run's end + 1
+    assert offs[-1] == 4096 * 16
+    d = image_sections(a.image())
+    assert int(d["slots"][0]) == (1 << 32) | (2 << 22) | 1                 # one slice of blocks 1..2 drawn
+    assert int(d["next"][0]) == 0x3FFFFF
+    a.malloc_batch(np.full(4095, 16, dtype=np.uint64), keydiv=0)            # index 4096 of the 2-block run next
+    a.malloc(16, 0)
+    assert int(image_sections(a.image())["next"][0]) == (4 << 22) | 3        # blocks 3..6
+    assert a.check() == 0
+
+
 @pytest.mark.parametrize("size", [4, 16, 64, 256, 4096, 8192, 1 << 20, 1 << 24, 3 << 24])
 def test_utilization_closed_form(size):
     """E8: batches of 100,000 allocations of one size until
@@ -235,8 +393,8 @@ def test_utilization_closed_form(size):
     nseg * (256 >> t) blocks; a k-segment request exactly floor(nseg / k)
     (P:138)."""
     nseg = 8
-    a = oracle.Allocator(nseg, slot_base=148, slot_min=4, run_max=256, run_init=64, run_grow=3,
-                         run_bytes=256 << 20, format_ahead=1)
+    a = runs(nseg, slot_base=148, slot_min=4, run_max=256, run_init=64, run_grow=3, run_bytes=256 << 20,
+             format_ahead=1)
     succ = 0
     while True:
         o = a.malloc_batch(np.full(100_000, size, dtype=np.uint64), keydiv=32)
@@ -254,46 +412,3 @@ def test_utilization_closed_form(size):
         assert succ == nseg * (256 >> t)
     else:
         assert succ == nseg // -(-size // SEG)
-
-
-@pytest.mark.parametrize("seed,nseg,run_max,fa,pf", [(21, 2, 1, 0, 0), (22, 3, 16, 1, 1), (23, 4, 64, 1, 0),
-                                                     (24, 2, 256, 0, 1), (25, 6, 8, 1, 1)])
-def test_exhaustion_record_is_exact(seed, nseg, run_max, fa, pf):
-    """DESIGN.md Deviations 11: a request failed by the exhaustion record is
-    one the full search (trims + retry) would fail too.  O2 checks every
-    record-failed request against a side-effect-free dry run of that search
-    (violation bit 512); heavy pressure on 2-6 segment heaps makes records
-    fire thousands of times; free-all + drain is still pristine."""
-    kinds, args, keys = wg.replay_ops(30_000, seed, p_free=0.3, p_drain=0.001, nkeys=64)
-    a = oracle.Allocator(nseg, slot_base=16, slot_min=2, run_max=run_max, run_bytes=32 << 20, format_ahead=fa,
-                         prefetch=pf)
-    out = a.replay(kinds, args, keys)
-    assert a.oom_fast > 100, "the record never fired"
-    assert a.check() == 0, oracle.violation_names(a.check())
-    freed = {int(args[i]) for i, k in enumerate(kinds) if k == 1}
-    for i, k in enumerate(kinds):
-        if k == 0 and out[i] != np.uint64(NONE) and i not in freed:
-            a.free(int(out[i]))
-    a.drain()
-    S = sum(a.nslot(c) for c in range(9))
-    assert np.array_equal(a.image(), pristine_image(nseg, S))
-
-
-def test_exhaustion_record_cleared_by_a_block_return():
-    """Closed form on a one-segment heap with one slot per class (P:134,
-    P:188): 2^20 16 B slices fill it; the next 16 B and 64 KB requests fail
-    (the second by the record); freeing 4095 slices of block 0 returns
-    nothing and the record stands; the 4096th free returns block 0,
-    the record is cleared, and the next 16 B request gets it again."""
-    a = oracle.Allocator(1, slot_base=1, slot_min=1, run_max=256, run_bytes=16 << 20, run_init=256, run_grow=3)
-    offs = a.malloc_batch(np.full(1 << 20, 16, dtype=np.uint64))
-    assert np.array_equal(offs, np.arange(1 << 20, dtype=np.uint64) * 16)
-    assert a.malloc(16, 0) == NONE
-    f0 = a.oom_fast
-    assert a.malloc(65536, 0) == NONE and a.oom_fast == f0 + 1
-    for o in offs[:4095]:
-        a.free(int(o))
-    assert a.malloc(16, 0) == NONE and a.oom_fast == f0 + 2
-    a.free(int(offs[4095]))
-    assert a.malloc(16, 0) == 0                    # block 0 again, slice 0
-    assert a.check() == 0

@@ -119,7 +119,10 @@ def replay_ops(n_ops: int, seed: int, p_free: float = 0.4, p_drain: float = 0.0,
     args[i]) -- each live allocation freed at most once; 2 = drain."""
     rng = np.random.Generator(np.random.PCG64(seed))
     if sizes is None:
-        sizes = SLICE_SIZES + [5000, 70000, 1 << 20, 3 << 20, 16 << 20, 40 << 20]
+        # every slice class, non-power-of-two slices (rounding, A-4), malloc(0)
+        # (NULL), whole blocks, exactly one segment (A-3) and one byte more
+        sizes = SLICE_SIZES + [0, 1, 17, 100, 4095, 5000, 70000, 1 << 20, 3 << 20, 16 << 20, (16 << 20) + 1,
+                               40 << 20]
     sizes = np.asarray(sizes, dtype=np.uint64)
     w = None if size_weights is None else np.asarray(size_weights, dtype=float) / sum(size_weights)
     kinds = np.zeros(n_ops, dtype=np.uint8)
