@@ -244,10 +244,20 @@ def run_ours(args, rank, world, local):
     free_ops_s = nsum / (sum(f_ms) / 1e3)
     per_cell = {}
     for i, (s, n) in enumerate(cells):
-        mm = statistics.median(m_ms[i::len(cells)])
-        fm = statistics.median(f_ms[i::len(cells)])
+        mi, fi = m_ms[i::len(cells)], f_ms[i::len(cells)]
+        mm, fm = statistics.median(mi), statistics.median(fi)
         per_cell[str(s)] = {"n": n, "malloc_ms": round(mm, 4), "free_ms": round(fm, 4),
+                            "malloc_ms_p10_p90": [round(x, 4) for x in pctl(mi)],
+                            "free_ms_p10_p90": [round(x, 4) for x in pctl(fi)],
                             "malloc_ops_s": n / mm * 1e3, "free_ops_s": n / fm * 1e3}
+
+    # the replayed steps left a correct allocator: no bad free was counted,
+    # and draining gives back every segment (the pristine state, by stats)
+    G.gallatin_drain()
+    st = G.gallatin_stats()
+    if st["errors"] or st["free_segments"] != st["num_segments"] or any(st["tree_segments"]) or st["large_segments"]:
+        raise SystemExit(f"allocator state after the timed steps is not pristine: {st}")
+    rmw = count_rmws(G, torch, cells, size_t, ptrs)
     dominant = "malloc" if sum(m_ms) >= sum(f_ms) else "free"
     bytes_per_op = 16 if dominant == "malloc" else 8
     kern_ms = sum(m_ms) if dominant == "malloc" else sum(f_ms)
@@ -293,7 +303,7 @@ def run_ours(args, rank, world, local):
                        "ops_per_step": ops_per_step, "parallelism": f"replicas x{world}",
                        "l2": "no flush: each step reads %.2f GiB of sizes + writes/reads the pointer array (> 126 MB L2)" % (
                            sum(8 * n for _, n in cells) / 2 ** 30)},
-            "malloc_ops_s": malloc_ops_s, "free_ops_s": free_ops_s, "per_size": per_cell,
+            "malloc_ops_s": malloc_ops_s, "free_ops_s": free_ops_s, "per_size": per_cell, "rmw_counts": rmw,
             "roofline": {"bound": "hbm", "kernel": "k_bulk_malloc_cta<4,10,128>" if dominant == "malloc" else "k_bulk_free_w<4,64,32>", "achieved": achieved, "peak": hbm_peak,
                          "unit": "GB/s", "frac": achieved / hbm_peak, "traffic": traffic,
                          "traffic_algorithmic": bytes_per_op * (1 << 24),
@@ -305,8 +315,107 @@ def run_ours(args, rank, world, local):
             "cpu_baseline": cpu,
         }
         line.update(extras)
+        line["fractions"] = fractions(line, hbm_peak)
         print(json.dumps(line))
     d.close()
+
+
+def pctl(xs):
+    """(p10, p90) of a sample."""
+    a = np.sort(np.asarray(xs, dtype=float))
+    return float(np.percentile(a, 10)), float(np.percentile(a, 90))
+
+
+def count_rmws(G, torch, cells, size_t, ptrs) -> dict:
+    """Per cell, the L2 RMWs the bulk kernels issue at minimum (SURVEY 8(d)
+    "Algorithmic work per unit"): malloc = one slot RMW per class per
+    512-request CTA tile (single size: ceil(n / 512)); free = one counter RMW
+    per (warp, block) team, counted from the pointers one malloc returns (lane
+    l of warp w frees ptrs[128 w + 32 k + l]: teams per 32-pointer row)."""
+    base = G.gallatin_stats()["heap_base"]
+    out = {}
+    for (s, n), st in zip(cells, size_t):
+        G.gallatin_reset()
+        p = ptrs[:n]
+        G.gallatin_malloc(st, p)
+        c = max(0, (s - 1).bit_length() - 4)
+        rows = (n + 31) // 32
+        g = torch.full((rows * 32,), -1, dtype=torch.int64, device="cuda")
+        g[:n] = (p - base) >> (16 + c)
+        g = torch.sort(g.view(rows, 32), dim=1).values
+        teams = int(((g[:, 1:] != g[:, :-1]).sum() + rows).item())
+        G.gallatin_free(p)
+        out[str(s)] = {"malloc_slot_rmws": (n + 511) // 512, "free_team_rmws": teams, "nslot": G.gallatin_stats()["nslot"][c]}
+    torch.cuda.synchronize()
+    G.gallatin_reset()
+    return out
+
+
+def fractions(line: dict, hbm_peak: float) -> dict:
+    """Roofline fractions of every config (BASELINE north_star: "give each as
+    absolute ops/s and as a fraction of the atomic/HBM roofline").  Peaks: the
+    same-session probes (PK1-PK7) and MEASURED_PEAKS hbm_gbs."""
+    pk = line.get("probes")
+    fr = {}
+    per = line["per_size"]
+    rmw = line["rmw_counts"]
+    tm = sum(v["malloc_ms"] for v in per.values())
+    tf = sum(v["free_ms"] for v in per.values())
+    n_all = sum(v["n"] for v in per.values())
+    c2 = {"frac_hbm_malloc": n_all * 16 / (tm / 1e3) / 1e9 / hbm_peak,
+          "frac_hbm_free": n_all * 8 / (tf / 1e3) / 1e9 / hbm_peak}
+    if pk:
+        a_dist32 = pk["atom_distinct"]["u32_random"]
+        per_cell = {}
+        for sz, v in per.items():
+            r = rmw[sz]
+            a_hot = pk["atom_hot"].get(str(r["nslot"])) or pk["atom_hot"]["148"]
+            per_cell[sz] = {
+                "frac_atom_malloc": (r["malloc_slot_rmws"] / (v["malloc_ms"] / 1e3)) / a_hot,
+                "frac_atom_free": (r["free_team_rmws"] / (v["free_ms"] / 1e3)) / a_dist32,
+                "frac_bump": v["malloc_ops_s"] / pk["bump_cta_16B"],
+                "frac_hbm_malloc": v["n"] * 16 / (v["malloc_ms"] / 1e3) / 1e9 / hbm_peak,
+                "frac_hbm_free": v["n"] * 8 / (v["free_ms"] / 1e3) / 1e9 / hbm_peak}
+        c2["frac_atom_malloc"] = sum(rmw[k]["malloc_slot_rmws"] for k in per) / (tm / 1e3) / pk["atom_hot"]["148"]
+        c2["frac_atom_free"] = sum(rmw[k]["free_team_rmws"] for k in per) / (tf / 1e3) / a_dist32
+        c2["frac_bump"] = line["malloc_ops_s"] / pk["bump_cta_16B"]
+        c2["per_size"] = per_cell
+        c2["peaks_used"] = {"A_hot(NSLOT)": "probes.atom_hot[NSLOT(c)]", "A_dist": "probes.atom_distinct.u32_random",
+                            "bump": "probes.bump_cta_16B (PK5b: 1 RMW per 512-request tile + 16 B I/O)"}
+    fr["C2"] = c2
+    if "veb" in line and pk:
+        v = line["veb"]
+        fr["C1_veb"] = {
+            "successor_frac_hbm": v["successor_ops_s"] * 16 / 1e9 / hbm_peak,
+            "successor_frac_l2_load": v["successor_ops_s"] / pk["load_random_8B_L2_16MB"],
+            "insert_frac_atom": v["insert_ops_s"] / pk["atom_distinct"]["u64_random"],
+            "delete_frac_atom": v["delete_ops_s"] / pk["atom_distinct"]["u64_random"],
+            "note": "successor: >= 1 dependent 8 B tree load per query (L2 random-load rate, PK6) + 16 B HBM; "
+                    "insert/delete: >= 1 distinct-address RMW per key (PK1 u64)"}
+        big = {}
+        for k, b in v.get("large_universes", {}).items():
+            big[k] = {"successor_frac_hbm": b["successor_ops_s"] * 16 / 1e9 / hbm_peak,
+                      "successor_frac_l2_load": b["successor_ops_s"] / pk["load_random_8B_L2_16MB"],
+                      "successor_frac_hbm_random_load": b["successor_ops_s"] / pk["load_random_8B_HBM_4GB"],
+                      "insert_frac_atom": b["insert_ops_s"] / pk["atom_distinct"]["u64_random"]}
+        fr["C1_veb"]["large_universes"] = big
+    if "mixed" in line:
+        m = line["mixed"]
+        fr["C3"] = {"frac_hbm_malloc": m["malloc_ops_s"] * 16 / 1e9 / hbm_peak,
+                    "frac_hbm_free": m["free_ops_s"] * 8 / 1e9 / hbm_peak}
+        if pk:
+            fr["C3"]["frac_bump"] = m["malloc_ops_s"] / pk["bump_cta_16B"]
+    if "scaling" in line:
+        fr["C4"] = {n: {"frac_hbm_malloc": v["malloc_ops_s"] * 16 / 1e9 / hbm_peak,
+                        "frac_hbm_free": v["free_ops_s"] * 8 / 1e9 / hbm_peak}
+                    for n, v in line["scaling"]["points"].items()}
+    if "graph" in line:
+        bpe = {"init": 12, "bulk_insert": 12, "bulk_delete": 8, "expansion": 4, "edge_insert": 12, "edge_delete": 8}
+        fr["C5"] = {k: {"frac_hbm_min": v["edges_per_s"] * bpe[k] / 1e9 / hbm_peak, "bytes_per_edge_min": bpe[k]}
+                    for k, v in line["graph"]["phases"].items() if k in bpe}
+        fr["C5"]["note"] = "lower-bound bytes per edge (8 B src+dst read, 4 B list write; deletes read 8 B); " \
+                           "list copies on grow/shrink not counted"
+    return fr
 
 
 def run_extras(args, G, torch, stream):
@@ -403,25 +512,110 @@ def run_extras(args, G, torch, stream):
     G.gallatin_destroy()
     G.gallatin_init(HEAP_C2)
 
-    # --- peak probes ---
-    pk = {}
-    nt = 1 << 24
-    ms, ops = G.gallatin_probe(1, nt, 1 << 21)
-    pk["atom_distinct_ops_s"] = ops / ms * 1e3
-    for lines in (4, 37, 148):
-        ms, ops = G.gallatin_probe(2, nt, lines)
-        pk[f"atom_hot{lines}_ops_s"] = ops / ms * 1e3
-    ms, ops = G.gallatin_probe(4, nt, 148)
-    pk["bump_ceiling_ops_s"] = ops / ms * 1e3
-    ms, ops = G.gallatin_probe(5, nt, 1)
-    pk["fence_per_warp_ops_s"] = ops / ms * 1e3
-    ms, ops = G.gallatin_probe(6, 1 << 24, 1 << 30)
-    pk["hbm_copy_gbs"] = ops / ms / 1e6
-    out["probes"] = pk
+    out["probes"] = run_probes(G)
+    out["grid"] = run_grid(args, G, torch, stream)
     out["scaling"] = run_scaling(args, G, torch, stream)
     out["graph"] = run_graph(args, G, torch, stream)
     out["paper_modes"] = run_paper_modes(args, G, torch)
     return out
+
+
+def run_grid(args, G, torch, stream) -> dict:
+    """BASELINE configs[1] as a full grid: every size 16 B..4 KB
+    x n = 2^20..2^24 threads on the 16 GiB heap.  The 39 cells with s*n <= 8 GiB
+    are timed (reset before every repetition, P:283; median and p10/p90 of 5);
+    the 6 others are capacity runs (one call asking more than the heap holds:
+    NULL count and time).  At the headline n of every size, warm rounds (no
+    reset, after one untimed round) are timed beside the cold ones."""
+    ev = lambda: torch.cuda.Event(enable_timing=True)  # noqa: E731
+    reps = 5
+    cells, cap_runs, warm = {}, {}, {}
+    for s in SIZES:
+        for lg in range(20, 25):
+            n = (1 << lg) // args.scale
+            st = torch.full((n,), s, dtype=torch.int64, device="cuda")
+            p = torch.empty_like(st)
+            if s * (1 << lg) > (8 << 30):
+                G.gallatin_reset()
+                a, b = ev(), ev()
+                a.record(stream)
+                G.gallatin_malloc(st, p)
+                b.record(stream)
+                torch.cuda.synchronize()
+                nulls = int((p == 0).sum().item())
+                cap_runs[f"{s}x2^{lg}"] = {"n": n, "nulls": nulls, "granted": n - nulls, "malloc_ms": a.elapsed_time(b),
+                                           "granted_bytes": (n - nulls) * s}
+                G.gallatin_free(p)
+                continue
+            mm, fm = [], []
+            for _ in range(reps + 1):
+                G.gallatin_reset()
+                a, b, c = ev(), ev(), ev()
+                a.record(stream)
+                G.gallatin_malloc(st, p)
+                b.record(stream)
+                G.gallatin_free(p)
+                c.record(stream)
+                torch.cuda.synchronize()
+                mm.append(a.elapsed_time(b))
+                fm.append(b.elapsed_time(c))
+            mm, fm = mm[1:], fm[1:]
+            m, f = statistics.median(mm), statistics.median(fm)
+            cells[f"{s}x2^{lg}"] = {"n": n, "malloc_ms": round(m, 5), "free_ms": round(f, 5),
+                                    "malloc_ms_p10_p90": [round(x, 5) for x in pctl(mm)],
+                                    "free_ms_p10_p90": [round(x, 5) for x in pctl(fm)],
+                                    "malloc_ops_s": n / m * 1e3, "free_ops_s": n / f * 1e3}
+            if (1 << lg) == min(1 << 24, (8 << 30) // s):             # the headline cell: warm rounds
+                G.gallatin_reset()
+                G.gallatin_malloc(st, p)
+                G.gallatin_free(p)                                   # the untimed first round
+                wm, wf = [], []
+                for _ in range(reps):
+                    a, b, c = ev(), ev(), ev()
+                    a.record(stream)
+                    G.gallatin_malloc(st, p)
+                    b.record(stream)
+                    G.gallatin_free(p)
+                    c.record(stream)
+                    torch.cuda.synchronize()
+                    wm.append(a.elapsed_time(b))
+                    wf.append(b.elapsed_time(c))
+                warm[str(s)] = {"n": n, "cold_malloc_ms": round(m, 5), "warm_malloc_ms": round(statistics.median(wm), 5),
+                                "cold_free_ms": round(f, 5), "warm_free_ms": round(statistics.median(wf), 5),
+                                "warm_over_cold_malloc": statistics.median(wm) / m}
+            del st, p
+    G.gallatin_reset()
+    return {"workload": "BASELINE configs[1] grid: 16 B..4 KB x 2^20..2^24 threads, 16 GiB heap", "reps": reps,
+            "cells": cells, "capacity_runs": cap_runs, "warm_vs_cold": warm}
+
+
+HOT_N = [1, 4, 9, 18, 37, 74, 148, 256, 302, 1024]       # SURVEY 8(d) PK2: slot-line counts
+
+
+def run_probes(G) -> dict:
+    """SURVEY 8(d) PK1-PK7 on persistent microkernels (probes.cu), same
+    session as the configs.  Rates in operations per second."""
+    def rate(kind, n, param):
+        ms, ops = G.gallatin_probe(kind, n, param)
+        return ops / ms * 1e3
+    w16m = (16 << 20) // 8                       # a 16 MB L2-resident array of u64
+    pk = {"atom_distinct": {
+        "u64_random": rate(1, 1 << 27, w16m), "u32_random": rate(7, 1 << 27, 2 * w16m),
+        "u64_coalesced": rate(8, 1 << 27, w16m), "u32_coalesced": rate(9, 1 << 27, 2 * w16m)}}
+    pk["atom_hot"] = {str(n): rate(2, 1 << 24, n) for n in HOT_N}
+    pk["red_hot"] = {str(n): rate(3, 1 << 24, n) for n in HOT_N}
+    pk["cas_hot"] = {str(n): rate(10, 1 << 22, n) for n in HOT_N}
+    pk["bump_warp_16B"] = rate(4, 1 << 24, 148)
+    pk["bump_cta_16B"] = rate(11, 1 << 24, 148)
+    pk["bump_cta_4KB_4slots"] = rate(11, 1 << 24, 4)
+    pk["fence_acq_rel_per_warp"] = rate(5, 1 << 22, 1)
+    pk["fence_sc_per_warp"] = rate(12, 1 << 22, 1)
+    pk["load_random_8B_L2_16MB"] = rate(13, 1 << 27, w16m)
+    pk["load_random_8B_HBM_4GB"] = rate(13, 1 << 26, (4 << 30) // 8)
+    ms, ops = G.gallatin_probe(6, 1 << 24, 1 << 31)
+    pk["hbm_copy_gbs"] = ops / ms / 1e6
+    pk["units"] = "operations/s (atomics, loads, fences, bump requests); hbm_copy in GB/s"
+    return pk
 
 
 def run_paper_modes(args, G, torch):
@@ -635,13 +829,27 @@ def time_oracle(cells, steps: int):
     return ops, total
 
 
+def host_cpu() -> dict:
+    """The box's host CPU model and core count (north_star: "core count stated")."""
+    model = "unknown"
+    try:
+        for line in open("/proc/cpuinfo"):
+            if line.startswith("model name"):
+                model = line.split(":", 1)[1].strip()
+                break
+    except Exception:
+        pass
+    return {"cpu_model": model, "nproc": os.cpu_count(), "affinity_cores": len(os.sched_getaffinity(0))}
+
+
 def cpu_baseline(args):
     div = 8
     cells = cpu_sample(div)
+    host = host_cpu()
     ops, sec = time_oracle(cells, 1)
     return {"value": ops / sec, "unit": "ops/s", "cores": 1, "kind": "oracle",
-            "sample": f"O2 (oracle/alloc_oracle.c) on every cell of the sweep at 1/{div} of its threads "
-                      f"({ops // 2} mallocs + frees), one pinned host core", "seconds": sec}
+            "sample": f"O2-P (oracle/alloc_paper.c, the paper's policy) on every cell of the sweep at 1/{div} of "
+                      f"its threads ({ops // 2} mallocs + frees), one pinned host core", "seconds": sec, **host}
 
 
 def run_reference(args, rank, world):
@@ -649,6 +857,7 @@ def run_reference(args, rank, world):
         return
     div = 8 * args.scale
     cells = cpu_sample(div)
+    host = host_cpu()
     steps = max(1, min(args.steps, 3))
     for _ in range(min(args.warmup, 1)):
         time_oracle(cells[:1], 1)
@@ -663,7 +872,8 @@ def run_reference(args, rank, world):
         "config": {"workload": "BASELINE configs[1]: single-size sweep 16 B-4 KB, 16 GiB heap; the CPU oracle "
                                f"runs each cell at 1/{div} of its threads", "cells": [[s, n] for s, n in cells]},
         "cpu_baseline": {"value": value, "unit": "ops/s", "cores": 1, "kind": "oracle",
-                         "sample": f"every cell at 1/{div} of its threads, {steps} step(s), one pinned host core"},
+                         "sample": f"O2-P on every cell at 1/{div} of its threads, {steps} step(s), one pinned host core",
+                         **host},
         "e2e": {"value": value, "unit": "ops/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
     }
     print(json.dumps(line))

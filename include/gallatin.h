@@ -200,26 +200,49 @@ int veb_insert(veb_t *h, const uint64_t *d_keys, uint8_t *d_out, uint64_t n, voi
 int veb_delete(veb_t *h, const uint64_t *d_keys, uint8_t *d_out, uint64_t n, void *stream);
 int veb_member(veb_t *h, const uint64_t *d_keys, uint8_t *d_out, uint64_t n, void *stream);
 /* succ(x) = min{y in S, y >= x}; pred(x) = max{y in S, y <= x};
- * UINT64_MAX when none.  Query batches read the tree through the read-only
- * path: no insert/delete may run on the same tree concurrently (different
- * streams) with a query batch. */
+ * UINT64_MAX when none.  By default query batches (member / successor /
+ * predecessor) read the tree through the read-only path: no insert/delete may
+ * run on the same tree concurrently (different streams) with a query batch. */
 int veb_successor(veb_t *h, const uint64_t *d_q, uint64_t *d_out, uint64_t n, void *stream);
 int veb_predecessor(veb_t *h, const uint64_t *d_q, uint64_t *d_out, uint64_t n, void *stream);
+/* on = 1: later query batches read the tree with coherent loads
+ * (ld.relaxed.gpu) and MAY overlap insert/delete batches on other streams
+ * (SURVEY 8(f)3 concurrent mixed batches).  A query then sees each key that
+ * stays present throughout it, and reports only keys present at some moment
+ * during it (bt_successor restarts past a summary bit whose child emptied).
+ * on = 0 (default) = the read-only path, quiescent trees only.  Host-side
+ * flag: takes effect for batches launched after the call. */
+int veb_set_concurrent(veb_t *h, int on);
 /* Image (all levels, level 0 first; bit = element / child non-empty); syncs. */
 int veb_words(const veb_t *h, uint64_t *words);
 int veb_snapshot(const veb_t *h, uint64_t *h_out, uint64_t cap_words, uint64_t *len_words);
 
 /* ------------------------------------------------------ measurement ----- */
-/* Peak probes; each returns the kernel time of one
- * launch in *ms (CUDA events on `stream`) and the operation count in *ops.
- *   kind 1: distinct-address 64-bit atomicAdd with return, over `param` words
- *   kind 2: hot-address atomicAdd with return, one lane per warp, `param` lines
- *   kind 3: as 2 with red (no return)
- *   kind 4: bump ceiling: per warp one atomicAdd(32) on `param` lines and
- *           __shfl_sync + 16 B of HBM I/O per lane (the allocator's lower bound)
- *   kind 5: fence.acq_rel.gpu per warp (ops = warps)
- *   kind 6: HBM copy of `param` bytes (ops = bytes moved, read + write)
- * `n` = threads launched. */
+/* Peak probes (DESIGN.md 5 "Roofline"): persistent
+ * microkernels over all SMs (148 x 8 CTAs x 256 threads) looping over about
+ * `n` operations; each returns the time of one launch in *ms (CUDA events on
+ * `stream`, after an untimed warm-up launch) and the operations it performed
+ * in *ops.  `param` per kind: */
+enum {
+    GALLATIN_PROBE_ATOM_U64_RANDOM = 1,    /* PK1 atom.add.u64 with return, random over param words        */
+    GALLATIN_PROBE_ATOM_HOT = 2,           /* PK2 atom.add.u64 with return by one lane per warp on param
+                                              128 B lines chosen by %smid (the block-buffer pattern)    */
+    GALLATIN_PROBE_RED_HOT = 3,            /* PK3 as 2 with red.add (no return)                             */
+    GALLATIN_PROBE_BUMP_WARP = 4,          /* PK5a one team atomicAdd per warp + 16 B I/O per request, n
+                                              requests, param lines (RegEff-AW analogue)         */
+    GALLATIN_PROBE_FENCE_ACQ_REL = 5,      /* PK7 fence.acq_rel.gpu per warp (ops = fences)                 */
+    GALLATIN_PROBE_HBM_COPY = 6,           /* PK6 HBM copy of param bytes (ops = bytes read + written)      */
+    GALLATIN_PROBE_ATOM_U32_RANDOM = 7,    /* PK1 atom.add.u32, random over param words                     */
+    GALLATIN_PROBE_ATOM_U64_COALESCED = 8, /* PK1 atom.add.u64, thread-consecutive words                    */
+    GALLATIN_PROBE_ATOM_U32_COALESCED = 9, /* PK1 atom.add.u32, thread-consecutive words                    */
+    GALLATIN_PROBE_CAS_HOT = 10,           /* PK4 atom.cas on param hot lines (every CAS counted)           */
+    GALLATIN_PROBE_BUMP_CTA = 11,          /* PK5b the bulk CTA kernel's structure without the allocator:
+                                              one RMW per class per 512-request tile, 16 B I/O per
+                                              request; n requests of 16 B, param slot lines           */
+    GALLATIN_PROBE_FENCE_SC = 12,          /* PK7 fence.sc.gpu per warp                                     */
+    GALLATIN_PROBE_LOAD_RANDOM = 13        /* PK6 random 8 B loads over param words (L2-resident at 16 MB,
+                                              HBM random sectors beyond L2)                             */
+};
 int gallatin_probe(int kind, uint64_t n, uint64_t param, double *ms, double *ops, void *stream);
 
 const char *gallatin_version(void);

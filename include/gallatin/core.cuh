@@ -207,10 +207,12 @@ __device__ inline __noinline__ uint32_t reclaim_idle(const View &v) {
 }
 
 // [dev] A claimer that lost the race for a bit of leaf word `old` retries at a
-// pseudo-random free bit of that same word (seeded by the thread and the
-// attempt) instead of the next one up: k simultaneous claimers -- every slot
-// refilling at a launch's start -- then collide O(1) times each instead of
-// walking the word one loss at a time.  kNone if the word had no free bit.
+// pseudo-random bit among the free bits its failed RMW returned (seeded by the
+// thread and the attempt) instead of the next one up: k simultaneous claimers
+// -- every slot refilling at a launch's start -- then collide O(1) times each
+// instead of walking the word one loss at a time, and they stay in the lowest
+// word with free segments (front-first packing).  kNone if the word
+// had no free bit.
 __device__ __forceinline__ uint64_t claim_retry_hint(uint64_t wi, uint64_t old, uint32_t attempt) {
     if (old == 0) return kNone;
     const uint32_t tid = blockIdx.x * blockDim.x + threadIdx.x;
@@ -241,24 +243,6 @@ __device__ __forceinline__ uint64_t claim_spread(uint64_t s, uint32_t attempt, u
     uint32_t b = (lo + h % (64u - lo)) & ~(claim_align(kmax) - 1);
     if (b < lo) b = lo;
     return (s & ~63ull) | b;
-}
-
-// [dev] The FIRST loss of a segment claim means every concurrent claimer
-// aimed at the same lowest free bit (a launch's first burst: one refill per
-// slot at once); the loser then aims at a pseudo-random bit of the next
-// kSpreadWords leaf words, unseen -- the RMW tells whether it was free --
-// instead of queueing on the one word; later losses use the free bits the
-// RMW returned (claim_retry_hint).  Serially no claim loses.
-constexpr uint32_t kSpreadWords = 4;
-__device__ __forceinline__ uint64_t claim_first_loss(const View &v, uint64_t wi, uint32_t kmax = 1) {
-    const uint32_t tid = blockIdx.x * blockDim.x + threadIdx.x;
-    uint32_t h = tid * 0x9E3779B1u;
-    h ^= h >> 13;
-    h *= 0x85EBCA6Bu;
-    h ^= h >> 16;
-    const uint32_t words = kSpreadWords + kmax / 2;            // room for the windows of every claimer
-    const uint64_t s = ((wi + h % words) << 6) | (((h >> 8) & 63) & ~(claim_align(kmax) - 1));
-    return s < v.nseg ? s : v.nseg - 1;
 }
 
 // successor(0) on the segment tree + claimIndex, front first
@@ -294,7 +278,7 @@ __device__ inline __noinline__ uint64_t claim_front(const View &v) {
             ptx::fence_acq_rel();
             return s;
         }
-        hint = ++attempt == 1 ? claim_first_loss(v, s >> 6) : claim_retry_hint(s >> 6, old, attempt);
+        hint = claim_retry_hint(s >> 6, old, ++attempt);   // a free bit the lost RMW saw, same word
         from = ((s >> 6) + 1) << 6;
     }
 }
@@ -340,7 +324,11 @@ __device__ inline __noinline__ uint64_t claim_front_run(const View &v, uint32_t 
         if (flip) bt_reconcile_up(st, 0, wi);
         if (extra) oom_notify(v);
         if (run == 0) {
-            hint = ++attempt == 1 ? claim_first_loss(v, wi, kmax) : claim_retry_hint(wi, old & ~mask, attempt);
+            // a free bit the lost RMW saw, at a window boundary if one is free
+            // (concurrent windows then do not overlap)
+            const uint32_t al = claim_align(kmax);
+            const uint64_t fr = old & ~mask, at = fr & (al >= 64 ? 1ull : ~0ull / ((1ull << al) - 1));
+            hint = claim_retry_hint(wi, at ? at : fr, ++attempt);
             from = (wi + 1) << 6;
             continue;
         }

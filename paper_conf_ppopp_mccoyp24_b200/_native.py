@@ -96,6 +96,7 @@ def lib() -> ctypes.CDLL:
         "veb_successor": ([vp, vp, vp, u64, vp], i32),
         "veb_predecessor": ([vp, vp, vp, u64, vp], i32),
         "veb_words": ([vp, P64], i32),
+        "veb_set_concurrent": ([vp, i32], i32),
         "veb_snapshot": ([vp, vp, u64, P64], i32),
         "gallatin_probe": ([i32, u64, u64, dp, dp, vp], i32),
         "gallatin_version": ([], ctypes.c_char_p),
@@ -320,6 +321,10 @@ class Veb:
 
     def clear(self, stream=None):
         check(lib().veb_clear(self._h, _stream(stream)), "veb_clear")
+
+    def set_concurrent(self, on: bool = True):
+        """Coherent query loads, so queries may overlap updates (include/gallatin.h)."""
+        check(lib().veb_set_concurrent(self._h, 1 if on else 0), "veb_set_concurrent")
 
     def _flags(self, fn, keys, want_out, stream):
         import torch

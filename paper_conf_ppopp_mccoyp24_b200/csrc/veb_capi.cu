@@ -14,6 +14,7 @@ struct veb {
     uint32_t k;
     BitTree t;
     uint64_t words;
+    int concurrent;       // 1: queries read coherently (ld.relaxed.gpu), may overlap updates
 };
 
 namespace {
@@ -41,11 +42,14 @@ __global__ void __launch_bounds__(kThreads) k_delete(BitTree t, const uint64_t *
     const bool r = bt_delete(t, keys[i]);
     if (out) out[i] = r;
 }
-// Read-only queries, ITEMS per thread: the ITEMS query keys are loaded
-// before any is walked (their HBM latency paid once, not ITEMS times); the
-// tree words come through the read-only path (L1-resident at u <= 2^24).
+// Queries, ITEMS per thread: the ITEMS query keys are loaded before any is
+// walked (their HBM latency paid once, not ITEMS times).  NC: the tree words
+// come through the read-only path (L1-resident at u <= 2^24) -- only while no
+// update runs on the tree; otherwise coherent ld.relaxed.gpu loads
+// (veb_set_concurrent), with which a set summary bit over a just-emptied
+// child restarts the search past it (bt_successor / bt_predecessor).
 enum QueryOp { kMember, kSucc, kPred };
-template <QueryOp OP, int ITEMS, typename OUT>
+template <QueryOp OP, int ITEMS, bool NC, typename OUT>
 __global__ void __launch_bounds__(kThreads) k_query(BitTree t, const uint64_t *__restrict__ q, OUT *__restrict__ out,
                                                     uint64_t n) {
     const uint64_t base = blockIdx.x * (uint64_t)(kThreads * ITEMS) + threadIdx.x;
@@ -59,17 +63,22 @@ __global__ void __launch_bounds__(kThreads) k_query(BitTree t, const uint64_t *_
     for (int k = 0; k < ITEMS; k++) {
         const uint64_t i = base + (uint64_t)kThreads * k;
         if (i >= n) break;
-        if (OP == kMember) out[i] = (OUT)bt_member<true>(t, x[k]);
-        else if (OP == kSucc) out[i] = (OUT)bt_successor<true>(t, x[k]);
-        else out[i] = (OUT)bt_predecessor<true>(t, x[k]);
+        if (OP == kMember) out[i] = (OUT)bt_member<NC>(t, x[k]);
+        else if (OP == kSucc) out[i] = (OUT)bt_successor<NC>(t, x[k]);
+        else out[i] = (OUT)bt_predecessor<NC>(t, x[k]);
     }
 }
-template <QueryOp OP, typename OUT>
-int launch_query(const BitTree &t, const uint64_t *q, OUT *out, uint64_t n, cudaStream_t st) {
+template <QueryOp OP, bool NC, typename OUT>
+void launch_query_nc(const BitTree &t, const uint64_t *q, OUT *out, uint64_t n, cudaStream_t st) {
     if (n >= (1ull << 20))                                    // enough queries to fill every SM 4-deep
-        k_query<OP, 4, OUT><<<(unsigned)((n + 4 * kThreads - 1) / (4 * kThreads)), kThreads, 0, st>>>(t, q, out, n);
+        k_query<OP, 4, NC, OUT><<<(unsigned)((n + 4 * kThreads - 1) / (4 * kThreads)), kThreads, 0, st>>>(t, q, out, n);
     else
-        k_query<OP, 1, OUT><<<grid_for(n), kThreads, 0, st>>>(t, q, out, n);
+        k_query<OP, 1, NC, OUT><<<grid_for(n), kThreads, 0, st>>>(t, q, out, n);
+}
+template <QueryOp OP, typename OUT>
+int launch_query(const veb *h, const uint64_t *q, OUT *out, uint64_t n, cudaStream_t st) {
+    if (h->concurrent) launch_query_nc<OP, false, OUT>(h->t, q, out, n, st);
+    else launch_query_nc<OP, true, OUT>(h->t, q, out, n, st);
     return launch_status();
 }
 }  // namespace
@@ -127,12 +136,18 @@ VEB_BULK(veb_delete, k_delete, uint8_t, false)
         if (!h) return GALLATIN_ERR_INVALID;                                                \
         if (n == 0) return GALLATIN_OK;                                                     \
         if (!d_keys || !d_out) return GALLATIN_ERR_INVALID;                                 \
-        return launch_query<op, out_t>(h->t, d_keys, d_out, n, S(stream));                 \
+        return launch_query<op, out_t>(h, d_keys, d_out, n, S(stream));                    \
     }
 
 VEB_QUERY(veb_member, kMember, uint8_t)
 VEB_QUERY(veb_successor, kSucc, uint64_t)
 VEB_QUERY(veb_predecessor, kPred, uint64_t)
+
+int veb_set_concurrent(veb_t *h, int on) {
+    if (!h || (on != 0 && on != 1)) return GALLATIN_ERR_INVALID;
+    h->concurrent = on;
+    return GALLATIN_OK;
+}
 
 int veb_words(const veb_t *h, uint64_t *words) {
     if (!h || !words) return GALLATIN_ERR_INVALID;

@@ -334,7 +334,7 @@ def test_bulk_kernel_variants(cuda_ok, G, knobs, n):
     shapes (2^21 and 2^23+ pointers), and the policy knobs, on mixed sizes
     with a ragged tail: stamp-verified, accounted, overlap-checked, pristine
     after free-all + drain."""
-    nseg = 1024
+    nseg = 1024 if n < (1 << 22) else 2048       # ~0.9 KB per small request + 1-64 MB every 2^14
     G.gallatin_init(nseg * SEG, **knobs)
     sizes = wg.mixed_sizes(n, p_large=2.0 ** -14)
     assert _bulk_round(G, nseg, sizes) == 0

@@ -23,11 +23,14 @@ def _u64(t):
     return t.cpu().numpy().view(np.uint64)
 
 
-def _run_batches(k, batches):
+def _run_batches(k, batches, concurrent=False):
     """Apply the same homogeneous batches to the GPU tree and to O1; compare
-    every per-op output and the final image."""
+    every per-op output and the final image.  concurrent: the coherent query
+    path (veb_set_concurrent) instead of the read-only one."""
     import paper_conf_ppopp_mccoyp24_b200 as G
     g = G.Veb(k)
+    if concurrent:
+        g.set_concurrent(True)
     o = oracle.Veb(k)
     for op, keys in batches:
         d = _dev(keys)
@@ -50,9 +53,11 @@ def _run_batches(k, batches):
     g.close()
 
 
-def test_config1_veb_parity(cuda_ok):
+@pytest.mark.parametrize("concurrent", [False, True])
+def test_config1_veb_parity(cuda_ok, concurrent):
     """BASELINE configs[0]: 2^16 random insert / successor / delete on a 2^20
-    universe, plus pred/member of the same queries."""
+    universe, plus pred/member of the same queries -- on the
+    read-only and on the coherent (concurrent-mode) query path."""
     w = wg.veb_workload(20, 1 << 16)
     _run_batches(20, [
         (OV_SUCC, w["succ1"]),                     # empty tree: all none
@@ -63,7 +68,7 @@ def test_config1_veb_parity(cuda_ok):
         (OV_DELETE, w["delete"]),
         (OV_SUCC, w["succ2"]),
         (OV_PRED, w["succ2"]),
-    ])
+    ], concurrent=concurrent)
 
 
 def test_bulk_queries_four_per_thread(cuda_ok):
@@ -78,8 +83,9 @@ def test_bulk_queries_four_per_thread(cuda_ok):
     _run_batches(k, [(OV_INSERT, ins), (OV_SUCC, q), (OV_PRED, q), (OV_MEMBER, q)])
 
 
+@pytest.mark.parametrize("concurrent", [False, True])
 @pytest.mark.parametrize("k", [1, 3, 6, 7, 12, 13, 18, 19, 24])
-def test_universe_sizes(cuda_ok, k):
+def test_universe_sizes(cuda_ok, k, concurrent):
     """Every level count (1..5) incl. partial top words; dense and sparse sets."""
     u = 1 << k
     n = min(u, 1 << 15)
@@ -88,7 +94,7 @@ def test_universe_sizes(cuda_ok, k):
     q = np.concatenate([wg.uniform_below(seed ^ 1, 4096, u), np.array([0, u - 1, u, u + 7], dtype=np.uint64)])
     dele = ins[: n // 2]
     _run_batches(k, [(OV_INSERT, ins), (OV_SUCC, q), (OV_PRED, q), (OV_DELETE, dele), (OV_SUCC, q),
-                     (OV_PRED, q), (OV_MEMBER, q), (OV_DELETE, ins), (OV_SUCC, q)])
+                     (OV_PRED, q), (OV_MEMBER, q), (OV_DELETE, ins), (OV_SUCC, q)], concurrent=concurrent)
 
 
 def test_universe_2_32_sampled(cuda_ok):
@@ -152,9 +158,9 @@ def test_concurrent_insert_delete_quiescent_exact(cuda_ok):
 
 @pytest.mark.parametrize("k", [16, 24])
 def test_concurrent_mixed_batches_linearizable(cuda_ok, k):
-    """Concurrent mixed-batch mode: successor / predecessor /
-    member queries race with inserts and deletes of VOLATILE keys on other
-    streams.  Linearizability-style invariants, for every query x:
+    """Concurrent mixed-batch mode (veb_set_concurrent):
+    successor / predecessor / member queries race with inserts and deletes of
+    VOLATILE keys on other streams.  Linearizability-style invariants, for every query x:
     succ(x) is NONE only if no STABLE key (present throughout) is >= x;
     otherwise x <= succ(x) <= the smallest stable key >= x and succ(x) is a
     stable or volatile key (never a key that was never present); pred
@@ -168,6 +174,7 @@ def test_concurrent_mixed_batches_linearizable(cuda_ok, k):
     stable, vol_in, vol_out = keys[:third], keys[third:2 * third], keys[2 * third:]
     q = wg.uniform_below(seed ^ 5, 1 << 20, u)
     g = G.Veb(k)
+    g.set_concurrent(True)            # queries overlap updates: coherent loads (include/gallatin.h)
     g.insert(_dev(np.concatenate([stable, vol_out])), want_out=False)
     torch.cuda.synchronize()
     s1, s2, s3 = torch.cuda.Stream(), torch.cuda.Stream(), torch.cuda.Stream()

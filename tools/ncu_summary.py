@@ -24,6 +24,14 @@ METRICS = [
     ("dram__bytes_write.sum", "DRAM write"),
     ("lts__t_requests_srcunit_tex_op_atom_dot_alu.sum", "L2 atomic requests (ALU)"),
     ("lts__t_requests_srcunit_tex_op_atom_dot_cas.sum", "L2 atomic requests (CAS)"),
+    ("lts__t_requests_op_atom.sum", "L2 atom requests (all)"),
+    ("lts__t_requests_op_red.sum", "L2 red requests"),
+    ("lts__t_requests_op_atom.sum.per_second", "L2 atom requests / s"),
+    ("l1tex__t_requests_pipe_lsu_mem_global_op_atom.sum", "L1 global atom requests (warp instructions)"),
+    ("l1tex__t_sectors_pipe_lsu_mem_global_op_atom.sum", "L1 global atom sectors (address replay = sectors / requests)"),
+    ("smsp__inst_executed_op_global_atom.sum", "global atom instructions executed"),
+    ("l1tex__t_sectors_pipe_lsu_mem_global_op_ld.sum", "global load sectors"),
+    ("lts__t_sectors_srcunit_tex_op_read.sum", "L2 read sectors (from SM)"),
     ("l1tex__t_sectors_pipe_lsu_mem_local_op_st.sum", "local-memory store sectors"),
     ("smsp__thread_inst_executed_per_inst_executed.ratio", "active threads per instruction (divergence)"),
     ("smsp__sass_branch_targets_threads_divergent.sum", "divergent branch targets"),
@@ -63,6 +71,9 @@ def main():
     ap.add_argument("--tag", default="r1")
     ap.add_argument("--cells", default="")
     ap.add_argument("--command", default="python bench.py --steps 2 --warmup 3 --no-extras --no-cpu")
+    ap.add_argument("--capture", default="-k regex:k_bulk ... tools/prof_cells.py",
+                    help="the captured command, for the report header")
+    ap.add_argument("--traffic", action="store_true", help="write profiles/traffic.json (bulk-kernel DRAM bytes)")
     a = ap.parse_args()
     prof = os.path.join(ROOT, "profiles")
     os.makedirs(prof, exist_ok=True)
@@ -81,8 +92,9 @@ def main():
         hdr, units = raw[0], raw[1]
         cells = [c for c in a.cells.split(",") if c]
         lines = [f"# Kernel captures ({a.tag})", "",
-                 f"`ncu --set full --clock-control none --import-source on -k regex:k_bulk ... tools/prof_cells.py {a.cells}`",
-                 "", "One launch per row group (after one warm-up round); cells in order: " + (a.cells or "?"), ""]
+                 f"`ncu --set full --clock-control none --import-source on {a.capture} {a.cells}`",
+                 "", "One launch per row group (after one warm-up round)" +
+                 ("; cells in order: " + a.cells if a.cells else ""), ""]
         traffic = {}
         src = ncu_csv(a.report, "source", ["--print-source", "sass"])
         stalls = []
@@ -98,8 +110,9 @@ def main():
         for n, r in enumerate(raw[2:]):
             name = r[hdr.index("Kernel Name")]
             short = name.split("(")[0].replace("void ", "").replace("<unnamed>::", "")
-            cell = cells[n // 2] if len(cells) * 2 == len(raw) - 2 else "?"
-            lines += [f"## `{short}` (cell {cell} B)", "", "| counter | value |", "|---|---:|"]
+            cell = cells[n // 2] if len(cells) * 2 == len(raw) - 2 else str(n)
+            lines += [f"## `{short}` ({'cell ' + cell + ' B' if cells else 'launch ' + cell})", "",
+                      "| counter | value |", "|---|---:|"]
             for m, label in METRICS:
                 if m in hdr:
                     lines.append(f"| {label} (`{m}`) | {r[hdr.index(m)]} {units[hdr.index(m)]} |")
@@ -111,8 +124,13 @@ def main():
             key = "k_bulk_malloc" if "malloc" in short else ("k_bulk_free" if "free" in short else short)
             traffic.setdefault(key, {})[cell] = tb
             lines.append("")
-        # top stall sites per distinct kernel (ncu aggregates per kernel name)
+        # top stall sites per distinct kernel (ncu aggregates per kernel name;
+        # the source page repeats a kernel once per captured launch: keep one)
+        seen = set()
         for name, rows in stalls:
+            if name in seen:
+                continue
+            seen.add(name)
             si = shdr.index("Warp Stall Sampling (All Samples)")
             tot = sum(int(x[si]) for x in rows) or 1
             top = sorted(range(len(rows)), key=lambda i: -int(rows[i][si]))[:6]
@@ -122,6 +140,8 @@ def main():
                 lines.append(f"| {int(rows[i][si]) / tot:.1%} | `{ctx}` |")
             lines.append("")
         open(os.path.join(prof, f"{a.tag}_kernels.md"), "w").write("\n".join(lines) + "\n")
+        if not a.traffic:
+            return
         tj = {k: (sum(v.values()) / len(v)) for k, v in traffic.items()}
         json.dump({"note": f"DRAM read+write bytes per launch from {a.tag} ncu --set full (mean over captured cells "
                            f"{a.cells})", **tj, "per_cell": traffic}, open(os.path.join(prof, "traffic.json"), "w"),

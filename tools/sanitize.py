@@ -7,7 +7,8 @@ result (so a sanitizer run is also a correctness run):
   veb    -- configs[0] vEB: insert / successor / predecessor / member / delete
             on u = 2^20 vs O1 (the oracle), bit-exact image;
   alloc  -- configs[0] allocator (64 MB heap, 2^16 x 16 B) on the small-batch
-            kernels, and 2^20 mixed 16 B-4 KB requests on the CTA-aggregated
+            kernels, and 2^20 mixed 16 B-4 KB (+ 1-64 MB) requests on a 4 GB
+            heap on the CTA-aggregated
             kernels (shared-memory ranking: the racecheck target), stamp +
             verify, free-all + drain -> pristine;
   replay -- serialized replay of a mixed op list vs O2 (offsets + image);
@@ -67,10 +68,10 @@ def part_alloc():
         _round(4, wg.single_sizes(16, 1 << 16))
     finally:
         G.gallatin_destroy()
-    G.gallatin_init(64 * SEG)
+    G.gallatin_init(256 * SEG)
     try:
-        _round(64, wg.mixed_sizes(1 << 20, p_large=2.0 ** -14))
-        _round(64, wg.single_sizes(64, 1 << 20))
+        _round(256, wg.mixed_sizes(1 << 20, p_large=2.0 ** -14))
+        _round(256, wg.single_sizes(64, 1 << 20))
     finally:
         G.gallatin_destroy()
     print("alloc ok")
