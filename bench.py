@@ -405,10 +405,10 @@ def fractions(line: dict, hbm_peak: float) -> dict:
                     "frac_hbm_free": m["free_ops_s"] * 8 / 1e9 / hbm_peak}
         if pk:
             fr["C3"]["frac_bump"] = m["malloc_ops_s"] / pk["bump_cta_16B"]
-    if "scaling" in line:
+    if "thread_scaling" in line:
         fr["C4"] = {n: {"frac_hbm_malloc": v["malloc_ops_s"] * 16 / 1e9 / hbm_peak,
                         "frac_hbm_free": v["free_ops_s"] * 8 / 1e9 / hbm_peak}
-                    for n, v in line["scaling"]["points"].items()}
+                    for n, v in line["thread_scaling"]["points"].items()}
     if "graph" in line:
         bpe = {"init": 12, "bulk_insert": 12, "bulk_delete": 8, "expansion": 4, "edge_insert": 12, "edge_delete": 8}
         fr["C5"] = {k: {"frac_hbm_min": v["edges_per_s"] * bpe[k] / 1e9 / hbm_peak, "bytes_per_edge_min": bpe[k]}
@@ -440,19 +440,24 @@ def run_extras(args, G, torch, stream):
     e1.record(stream)
     torch.cuda.synchronize()
     succ_ms = e0.elapsed_time(e1) / reps
-    # insert/delete throughput on the same universe
+    # insert/delete throughput on the same universe: R rounds of (clear,
+    # insert the 2^16 keys, delete the 2^16 delete keys), events between the
+    # back-to-back launches, median per launch
     dk = torch.from_numpy(w["delete"].view(np.int64)).cuda()
-    v.clear()
-    e0.record(stream)
-    v.insert(keys, want_out=False)
-    e1.record(stream)
-    torch.cuda.synchronize()
-    ins_ms = e0.elapsed_time(e1)
-    e0.record(stream)
-    v.delete(dk, want_out=False)
-    e1.record(stream)
-    torch.cuda.synchronize()
-    del_ms = e0.elapsed_time(e1)
+    ins_l, del_l = [], []
+    for r in range(12):
+        v.clear()
+        ea, eb, ec = (torch.cuda.Event(enable_timing=True) for _ in range(3))
+        ea.record(stream)
+        v.insert(keys, want_out=False)
+        eb.record(stream)
+        v.delete(dk, want_out=False)
+        ec.record(stream)
+        torch.cuda.synchronize()
+        if r >= 2:
+            ins_l.append(ea.elapsed_time(eb))
+            del_l.append(eb.elapsed_time(ec))
+    ins_ms, del_ms = statistics.median(ins_l), statistics.median(del_l)
     v.close()
     out["veb"] = {"successor_ops_s": nq / succ_ms * 1e3, "successor_queries": nq, "successor_ms": succ_ms,
                   "insert_ops_s": len(w["insert"]) / ins_ms * 1e3, "delete_ops_s": len(w["delete"]) / del_ms * 1e3,
@@ -467,6 +472,8 @@ def run_extras(args, G, torch, stream):
         bk = torch.from_numpy(wg.distinct_below(wg.cell_seed(1, 400 + k), nk, 1 << k).view(np.int64)).cuda()
         bq = torch.from_numpy(wg.uniform_below(wg.cell_seed(1, 500 + k), nq, 1 << k).view(np.int64)).cuda()
         br = torch.empty_like(bq)
+        vb.insert(bk, want_out=False)                 # warm-up round (then cleared)
+        vb.clear()
         e0.record(stream)
         vb.insert(bk, want_out=False)
         e1.record(stream)
@@ -514,7 +521,7 @@ def run_extras(args, G, torch, stream):
 
     out["probes"] = run_probes(G)
     out["grid"] = run_grid(args, G, torch, stream)
-    out["scaling"] = run_scaling(args, G, torch, stream)
+    out["thread_scaling"] = run_scaling(args, G, torch, stream)
     out["graph"] = run_graph(args, G, torch, stream)
     out["paper_modes"] = run_paper_modes(args, G, torch)
     return out

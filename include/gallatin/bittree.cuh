@@ -75,12 +75,29 @@ __device__ inline void bt_reconcile_up(const BitTree &t, uint32_t lvl, uint64_t 
     }
 }
 
+// The setting half of the reconcile: the thread whose RMW made level-lvl word
+// idx non-empty sets its parent bit with a release fence before the RMW, and
+// climbs while its RMWs flip parents from empty.  No re-read loop is needed on
+// this side: if a clearer's RMW on the parent bit comes after ours in the
+// bit's coherence order, it read our release, so the clearer's re-read (after
+// its fence.sc, bt_reconcile_up) sees our child RMW and sets the bit again.
+// One fence.acq_rel per level instead of two fence.sc and a re-read.
+__device__ inline void bt_set_up(const BitTree &t, uint32_t lvl, uint64_t idx) {
+    while (lvl + 1 < t.levels) {
+        ptx::fence_acq_rel();
+        const uint64_t old = ptx::atom_or(t.w + t.off[lvl + 1] + (idx >> 6), 1ull << (idx & 63));
+        if (old != 0) return;
+        lvl++;
+        idx >>= 6;
+    }
+}
+
 // insert(x): S <- S u {x}.  Returns true iff x was newly added.
 __device__ inline bool bt_insert(const BitTree &t, uint64_t x) {
     if (x >= t.nbits) return false;
     const uint64_t bit = 1ull << (x & 63);
     const uint64_t old = ptx::atom_or(t.w + t.off[0] + (x >> 6), bit);
-    if (old == 0) bt_reconcile_up(t, 0, x >> 6);
+    if (old == 0) bt_set_up(t, 0, x >> 6);
     return !(old & bit);
 }
 
@@ -202,7 +219,7 @@ __device__ inline void bt_insert_range(const BitTree &t, uint64_t i, uint64_t k)
         const uint32_t lo = (uint32_t)(x & 63);
         const uint32_t hi = (uint32_t)((end - (wi << 6)) < 64 ? (end - (wi << 6)) : 64);
         const uint64_t old = ptx::atom_or(t.w + t.off[0] + wi, bit_range(lo, hi));
-        if (old == 0) bt_reconcile_up(t, 0, wi);
+        if (old == 0) bt_set_up(t, 0, wi);
         x = (wi << 6) + hi;
     }
 }

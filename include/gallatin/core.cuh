@@ -505,6 +505,14 @@ __device__ inline __noinline__ uint32_t get_run_once(const View &v, uint32_t t, 
         // findSegment; after a lost race, a random other candidate
         const uint64_t s = hint != kNone ? hint : bt_successor<false>(bt, from);
         hint = kNone;
+        // [dev] a run of whole segments takes fresh ones while any is free
+        // rather than a short run from a partly returned segment (the
+        // warm-state refills); serially exact with O2-R's R2
+        if (s != kNone && want >= nb && sw_avail(ptx::ld_relaxed(v.seg_word + s)) < (int32_t)want &&
+            bt_successor<false>(seg_tree(v), 0) != kNone) {
+            const uint32_t k = take_segments(v, t, want, first);
+            if (k) return k;
+        }
         if (s != kNone) {
             // reserve up to `want` blocks of s and validate its tree id in one RMW
             const uint64_t dec = (uint64_t)(-(int64_t)want);

@@ -19,7 +19,9 @@
  *      in ascending order) or from one fresh segment whose other blocks are
  *      published; a run of >= nb blocks takes whole free segments privately
  *      (the lowest free one and the free ones right after it, no ring, no
- *      block tree);
+ *      block tree) -- also when the block tree has a segment but with fewer
+ *      than m blocks available, as long as a segment is free (a partly
+ *      returned segment would give a short run: the warm-state refills);
  *   R3 format-ahead: the reservation that takes a segment below nb/4
  *      available blocks formats one more segment for the tree when no higher
  *      segment of the tree has blocks;
@@ -103,6 +105,9 @@ static uint32_t take_segments(o2_t *a, uint32_t t, uint32_t want, uint32_t *firs
 static uint32_t get_run_once(o2_t *a, uint32_t t, uint32_t want, uint32_t *first) {
     uint32_t nb = nb_of(t);
     uint64_t s = oracle_veb_successor(a->btree[t], 0);              /* findSegment */
+    if (s != NONE64 && want >= nb && (uint32_t)a->avail[s] < want &&
+        oracle_veb_successor(a->segfree, 0) != NONE64)              /* R2: whole segments first */
+        return take_segments(a, t, want, first);
     if (s != NONE64) {
         uint32_t av = (uint32_t)a->avail[s];
         uint32_t got = want < av ? want : av;                       /* reserve */

@@ -30,17 +30,52 @@ int launch_status() {
     return GALLATIN_OK;
 }
 
-__global__ void __launch_bounds__(kThreads) k_insert(BitTree t, const uint64_t *keys, uint8_t *out, uint64_t n) {
-    const uint64_t i = blockIdx.x * (uint64_t)kThreads + threadIdx.x;
-    if (i >= n) return;
-    const bool r = bt_insert(t, keys[i]);
-    if (out) out[i] = r;
-}
-__global__ void __launch_bounds__(kThreads) k_delete(BitTree t, const uint64_t *keys, uint8_t *out, uint64_t n) {
-    const uint64_t i = blockIdx.x * (uint64_t)kThreads + threadIdx.x;
-    if (i >= n) return;
-    const bool r = bt_delete(t, keys[i]);
-    if (out) out[i] = r;
+// Bulk insert / delete, ITEMS keys per thread (keys loaded first, then the
+// ITEMS leaf RMWs issued back to back: several L2 round trips in flight per
+// warp).  The lanes of a warp whose keys share a leaf word combine: one
+// atomicOr / atomicAnd of the OR of their bits by the lowest such lane, the
+// old word broadcast back; of several lanes with the SAME key only the lowest
+// reports (exactly one op per distinct key returns 1, reading A-23).  The
+// lane whose RMW flipped the word's emptiness repairs the summaries: set side
+// bt_set_up (release fence, no re-read), clear side bt_reconcile_up.
+template <bool INSERT, int ITEMS>
+__global__ void __launch_bounds__(kThreads) k_update(BitTree t, const uint64_t *__restrict__ keys, uint8_t *__restrict__ out,
+                                                     uint64_t n) {
+    const uint32_t lane = threadIdx.x & 31;
+    const uint64_t base = blockIdx.x * (uint64_t)(kThreads * ITEMS) + threadIdx.x;
+    uint64_t x[ITEMS];
+#pragma unroll
+    for (int k = 0; k < ITEMS; k++) {
+        const uint64_t i = base + (uint64_t)kThreads * k;
+        x[k] = i < n ? __ldcs(reinterpret_cast<const unsigned long long *>(keys) + i) : kNone;
+    }
+    uint64_t old[ITEMS], bit[ITEMS], msk[ITEMS];
+    unsigned wp[ITEMS];
+#pragma unroll
+    for (int k = 0; k < ITEMS; k++) {
+        const bool valid = x[k] < t.nbits;
+        const uint64_t wi = valid ? x[k] >> 6 : ~0ull - lane;       // invalid keys: a word of their own
+        bit[k] = valid ? 1ull << (x[k] & 63) : 0;
+        wp[k] = __match_any_sync(0xFFFFFFFFu, wi);
+        msk[k] = ((uint64_t)__reduce_or_sync(wp[k], (uint32_t)(bit[k] >> 32)) << 32) |
+                 __reduce_or_sync(wp[k], (uint32_t)bit[k]);
+        old[k] = 0;
+        if (valid && lane == (uint32_t)__ffs((int)wp[k]) - 1)
+            old[k] = INSERT ? ptx::atom_or(t.w + t.off[0] + wi, msk[k]) : ptx::atom_and(t.w + t.off[0] + wi, ~msk[k]);
+    }
+#pragma unroll
+    for (int k = 0; k < ITEMS; k++) {
+        const uint32_t leader = (uint32_t)__ffs((int)wp[k]) - 1;
+        const uint64_t o = __shfl_sync(0xFFFFFFFFu, old[k], (int)leader);
+        const unsigned kp = __match_any_sync(0xFFFFFFFFu, x[k]);
+        const uint64_t i = base + (uint64_t)kThreads * k;
+        const bool valid = bit[k] != 0;
+        if (out && i < n) out[i] = valid && lane == (uint32_t)__ffs((int)kp) - 1 && (INSERT ? !(o & bit[k]) : (o & bit[k]) != 0);
+        if (valid && lane == leader) {
+            if (INSERT && o == 0) bt_set_up(t, 0, x[k] >> 6);                          // empty -> non-empty
+            if (!INSERT && (o & msk[k]) != 0 && (o & ~msk[k]) == 0) bt_reconcile_up(t, 0, x[k] >> 6);   // -> empty
+        }
+    }
 }
 // Queries, ITEMS per thread: the ITEMS query keys are loaded before any is
 // walked (their HBM latency paid once, not ITEMS times).  NC: the tree words
@@ -81,6 +116,14 @@ int launch_query(const veb *h, const uint64_t *q, OUT *out, uint64_t n, cudaStre
     else launch_query_nc<OP, true, OUT>(h->t, q, out, n, st);
     return launch_status();
 }
+template <bool INSERT>
+void launch_update(const BitTree &t, const uint64_t *keys, uint8_t *out, uint64_t n, cudaStream_t st) {
+    if (n >= (1ull << 20))                                    // enough keys to fill every SM 4-deep
+        k_update<INSERT, 4><<<(unsigned)((n + 4 * kThreads - 1) / (4 * kThreads)), kThreads, 0, st>>>(t, keys, out, n);
+    else
+        k_update<INSERT, 1><<<grid_for(n), kThreads, 0, st>>>(t, keys, out, n);
+}
+
 }  // namespace
 
 extern "C" {
@@ -119,17 +162,17 @@ int veb_clear(veb_t *h, void *stream) {
     return GALLATIN_OK;
 }
 
-#define VEB_BULK(name, kern, out_t, need_out)                                               \
-    int name(veb_t *h, const uint64_t *d_keys, out_t *d_out, uint64_t n, void *stream) {   \
+#define VEB_UPDATE(name, insert)                                                           \
+    int name(veb_t *h, const uint64_t *d_keys, uint8_t *d_out, uint64_t n, void *stream) { \
         if (!h) return GALLATIN_ERR_INVALID;                                                \
         if (n == 0) return GALLATIN_OK;                                                     \
-        if (!d_keys || (need_out && !d_out)) return GALLATIN_ERR_INVALID;                   \
-        kern<<<grid_for(n), kThreads, 0, S(stream)>>>(h->t, d_keys, d_out, n);              \
+        if (!d_keys) return GALLATIN_ERR_INVALID;                                           \
+        launch_update<insert>(h->t, d_keys, d_out, n, S(stream));                          \
         return launch_status();                                                             \
     }
 
-VEB_BULK(veb_insert, k_insert, uint8_t, false)
-VEB_BULK(veb_delete, k_delete, uint8_t, false)
+VEB_UPDATE(veb_insert, true)
+VEB_UPDATE(veb_delete, false)
 
 #define VEB_QUERY(name, op, out_t)                                                         \
     int name(veb_t *h, const uint64_t *d_keys, out_t *d_out, uint64_t n, void *stream) {   \

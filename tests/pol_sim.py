@@ -107,6 +107,8 @@ class PolSim:
     def get_run_once(self, t, want):
         """(blocks, first linear index); the paper's GetBlock at want = 1."""
         cand = self.tree_segs(t)
+        if cand and self.runs and want >= nb(t) and len(self.ring[cand[0]]) < want and self.free_segs():
+            cand = []                                             # R2: whole fresh segments first
         if cand:
             s = cand[0]
             av = len(self.ring[s])

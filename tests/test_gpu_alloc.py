@@ -346,7 +346,7 @@ def test_malloc_zero_and_nulls(cuda_ok, G, items):
     """malloc(0) is NULL (reading A-4) in both bulk kernels, next to real
     requests in the same warps and CTA tiles; freeing the NULLs is a no-op
     (P:241); non-power-of-two sizes round up to their class."""
-    nseg = 64
+    nseg = 512                                     # ~2.8 KB per request after rounding: 8 GB heap
     G.gallatin_init(nseg * SEG, bulk_items=items)
     n = (1 << 20) + 17
     rng = np.random.Generator(np.random.PCG64(5))

@@ -36,7 +36,7 @@ def test_block_buffer_slots_match_paper_a40():
 
 
 @pytest.mark.parametrize("knobs", [None, dict(run_max=16, format_ahead=1, prefetch=1),
-                                   dict(run_max=128, prefetch=1)])
+                                   dict(run_max=64, prefetch=1)])
 @pytest.mark.parametrize("size,blocks", [(16, "blocks_per_segment_16B"), (32, "blocks_per_segment_32B")])
 def test_blocks_per_segment_and_in_order_slices(size, blocks, knobs):
     """256 blocks per segment at 16 B, 128 at 32 B; 4096 slices
@@ -341,6 +341,24 @@ def test_whole_segment_runs_taken_privately():
     assert (w >> 22) & 0x3FF == 256 and w & 0x3FFFFF == 256 and w >> 32 == 3   # second run: segment 1
     assert int(d["segtree"][0]) == 0                          # no segment free
     assert a.malloc(16, 0) == (1 << 20) * 16 + 3 * 16 and a.check() == 0
+
+
+def test_whole_segment_runs_prefer_fresh_segments():
+    """R2: a run of >= nb blocks is taken from fresh segments while any is
+    free, not from a partly returned segment of the block tree (which would
+    give a run as short as its available blocks -- the warm-state refills).
+    One 2 KB slot (8 MB blocks, nb = 2), runs of 1 then 2 blocks: the first
+    run is block 0 of segment 0 (block 1 published in the ring), the second
+    run wants 2 >= nb: segment 1 whole, not block 1 of segment 0; a whole
+    8 MB block request (tree 7, want 1 < nb) still takes segment 0's block 1."""
+    a = runs(4, slot_base=1, slot_min=1, run_max=2, run_bytes=32 << 20, run_init=1, run_grow=1)
+    bb = 8 << 20
+    offs = a.malloc_batch(np.full(4096 + 1, 2048, dtype=np.uint64), keydiv=0)
+    assert offs[4095] == 4095 * 2048 and offs[4096] == SEG          # second run: segment 1, not block 1
+    w = int(image_sections(a.image())["slots"][7])
+    assert (w >> 22) & 0x3FF == 2 and w & 0x3FFFFF == 2             # run of 2 from linear block 2
+    assert a.malloc(bb, 0) == bb                                      # block path: segment 0's block 1
+    assert a.check() == 0
 
 
 def test_format_ahead_closed_form():

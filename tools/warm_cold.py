@@ -7,6 +7,8 @@ import statistics
 import sys
 
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+if os.environ.get("GALLATIN_PKG_ROOT"):
+    sys.path.insert(0, os.environ["GALLATIN_PKG_ROOT"])  # A/B against another build of the package
 import torch  # noqa: E402
 
 import paper_conf_ppopp_mccoyp24_b200 as G  # noqa: E402
@@ -31,5 +33,5 @@ for sz in [int(x) for x in (sys.argv[1] if len(sys.argv) > 1 else "16,128,512,40
             if it >= 2:
                 ts.append(a.elapsed_time(b))
         res.setdefault(mode, []).append(round(statistics.median(ts), 4))
-    print(json.dumps({"size": sz, "n": n, **res}), flush=True)
+    print(json.dumps({"pkg": os.environ.get("GALLATIN_PKG_ROOT", "."), "size": sz, "n": n, **res}), flush=True)
 G.gallatin_destroy()
