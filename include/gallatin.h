@@ -85,6 +85,13 @@ typedef struct gallatin_config {
                               block tree confirmed exhausted fails in O(1) until memory comes back; 2 = off (every
                               request repeats the full search with slot trims -- the policy oracle/alloc_runs.c
                               replays exactly) */
+    uint32_t prefill;      /* 0/1 = prefilled block buffer (default; "each block buffer is always
+                              populated"): gallatin_init / gallatin_reset leave every slot holding its first run,
+                              laid out class by class from segment 0 (slot q of class c: blocks
+                              [q*r, (q+1)*r) of the class's segments, r = its first-run length; the class's partly
+                              used last segment keeps its other blocks in its ring and block tree) -- when those
+                              runs fit in half the heap, else the slots start empty and fill on first use (reading
+                              A-19); 2 = off.  gallatin_drain empties the slots (the pristine image). */
 } gallatin_config_t;
 
 int gallatin_init(uint64_t heap_bytes);                 /* defaults for the rest */
@@ -109,8 +116,9 @@ int gallatin_free(void *const *d_ptrs, uint64_t n, void *stream);
 int gallatin_malloc_host(const uint64_t *h_sizes, uint64_t *h_ptrs, uint64_t n, void *stream);
 int gallatin_free_host(const uint64_t *h_ptrs, uint64_t n, void *stream);
 
-/* Pristine state (the paper resets before every run).  Invalidates
- * every outstanding pointer.  Asynchronous on `stream`. */
+/* The initial state (the paper resets before every run): the pristine
+ * image, or with the prefill knob every slot holding its first run.
+ * Invalidates every outstanding pointer.  Asynchronous on `stream`. */
 int gallatin_reset(void *stream);
 
 /* Quiescent only (no malloc/free in flight): retire every block-buffer slot
@@ -140,6 +148,7 @@ typedef struct gallatin_stats {
     uint32_t run_cap[9];         /* max blocks per run per class                    */
     uint32_t slot_base, slot_min, run_max, format_ahead, fence_free, run_init, formatters, prefetch;
     uint32_t run_grow, demand_hint, oom_record;
+    uint32_t prefill_segments;   /* segments a reset carves into prefilled slot runs (0 = none) */
 } gallatin_stats_t;
 int gallatin_stats(gallatin_stats_t *out);               /* synchronizes the device */
 

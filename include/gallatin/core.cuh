@@ -363,8 +363,25 @@ __device__ inline __noinline__ void format_segment(const View &v, uint64_t s, ui
 }
 
 // ---- block return (Alg.4; ring enqueue P:178) --------------------
+// [dev] A segment of one block (4 KB slices: 16 MB blocks) whose block comes
+// back is home at once: one CAS {t, 0 available} -> FREE retires it without
+// the ring enqueue, the table fetch-add and the block-tree repair that the
+// general path runs (its block-tree bit was never set: no RMW ever saw it
+// with a block available).  The same final state as the general path; a
+// failed CAS (a refiller's transient reservation on the word) falls back.
+__device__ __forceinline__ bool return_whole_segment(const View &v, uint64_t s, uint32_t t) {
+    if (ptx::atom_cas(v.seg_word + s, sw_make(t, 0), sw_make(kTreeFree, 0)) != sw_make(t, 0)) return false;
+    ptx::st_relaxed(v.seg_tid + s, kTreeFree);
+    ptx::fence_acq_rel();                                    // table + tree-id copy before the tree bit
+    bt_insert(seg_tree(v), s);
+    oom_notify(v);
+    return true;
+}
+
 __device__ inline __noinline__ void return_block(const View &v, uint32_t gid) {
     const uint64_t s = gid / kMaxBlocks;
+    const uint32_t tid = ptx::ld_relaxed(v.seg_tid + s);
+    if (tid == kTrees - 1 && return_whole_segment(v, s, tid)) return;
     const uint32_t pos = atomicAdd(v.q_tail + s, 1u) & (kMaxBlocks - 1);
     uint16_t *slotp = v.q_entries + s * kMaxBlocks + pos;
     ptx::Backoff wb(3, (s << 32) | pos);

@@ -64,6 +64,16 @@ struct gallatin_device_view {
     uint32_t run_grow;          /* log2 of the run growth factor per refill    */
     uint32_t demand_hint;       /* 1 = bulk refills sized to the launch's demand */
     uint32_t oom_record;        /* 1 = exhaustion record on (DESIGN.md Deviations 11) */
+    /* prefilled block buffer ("always populated"; reading A-19):
+     * 0 segments = reset leaves every slot empty; else class c's slots hold
+     * runs of pf_run[c] blocks laid out from segment pf_base[c] on, slot q at
+     * linear block pf_base[c] * nb(c) + q * pf_run[c]; pf_last[c] is the class's
+     * partly used last segment (0xFFFFFFFF: none), pf_used[c] its blocks in runs */
+    uint32_t pf_segs;
+    uint32_t pf_base[GALLATIN_NUM_TREES];
+    uint32_t pf_run[GALLATIN_NUM_TREES];
+    uint32_t pf_last[GALLATIN_NUM_TREES];
+    uint32_t pf_used[GALLATIN_NUM_TREES];
 };
 typedef struct gallatin_device_view gallatin_device_view_t;
 

@@ -84,7 +84,7 @@ def lib() -> ctypes.CDLL:
             "oracle_veb_image_levels": ([ctypes.c_uint, vp], ctypes.c_uint),
             "o2_create_paper": ([u64, ctypes.c_uint, ctypes.c_uint], vp),
             "o2_create_runs": ([u64, ctypes.c_uint, ctypes.c_uint, ctypes.c_uint, u64, ctypes.c_uint, ctypes.c_uint,
-                                ctypes.c_uint, ctypes.c_uint], vp),
+                                ctypes.c_uint, ctypes.c_uint, ctypes.c_uint], vp),
             "o2_destroy": ([vp], None),
             "o2_nslot": ([vp, ctypes.c_uint], ctypes.c_uint),
             "o2_errors": ([vp], u64),
@@ -189,13 +189,9 @@ class Allocator:
     def __init__(self, nseg: int, slot_base: int = 148, slot_min: int = 4):
         self._h = None
         self.nseg = nseg
-        self._h = self._create(nseg, slot_base, slot_min)
+        self._h = lib().o2_create_paper(nseg, slot_base, slot_min)
         if not self._h:
             raise ValueError("bad allocator parameters")
-
-    @staticmethod
-    def _create(nseg, slot_base, slot_min):
-        return lib().o2_create_paper(nseg, slot_base, slot_min)
 
     def close(self):
         if self._h:
@@ -262,15 +258,16 @@ class RunsAllocator(Allocator):
     runs of consecutive blocks per slot, format-ahead, prefetch, slot trims
     before "no memory".  run_max=1, run_init=1, format_ahead=0, prefetch=0 is
     the paper's one-block buffer; run_grow = log2 of the growth per
-    refill."""
+    refill; prefill=1: every slot starts holding its first run (R7),
+    when those runs fit in half the heap."""
 
     def __init__(self, nseg: int, slot_base: int = 148, slot_min: int = 4, run_max: int = 1,
                  run_bytes: int = 64 << 20, format_ahead: int = 0, run_init: int = 1, prefetch: int = 0,
-                 run_grow: int = 1):
+                 run_grow: int = 1, prefill: int = 0):
         self._h = None
         self.nseg = nseg
         self._h = lib().o2_create_runs(nseg, slot_base, slot_min, run_max, run_bytes, format_ahead, run_init,
-                                       prefetch, run_grow)
+                                       prefetch, run_grow, prefill)
         if not self._h:
             raise ValueError("bad allocator parameters")
 
@@ -279,12 +276,14 @@ PAPER_KNOBS = {"run_max": 1, "run_init": 1, "format_ahead": 0, "prefetch": 0}
 
 
 def is_paper_policy(params: dict) -> bool:
-    """True if the knobs are the paper's one-block buffer."""
-    return all(params.get(k, PAPER_KNOBS[k]) == v for k, v in PAPER_KNOBS.items())
+    """True if the knobs are the paper's one-block buffer, filled on demand."""
+    return all(params.get(k, PAPER_KNOBS[k]) == v for k, v in PAPER_KNOBS.items()) and not params.get("prefill", 0)
 
 
 def model(nseg: int, **params) -> Allocator:
-    """The O2 model for a set of knobs: O2-P for the paper's policy, else O2-R."""
+    """The O2 model for a set of knobs: O2-P for the paper's policy, else O2-R
+    (which at the paper's knobs adds only the prefilled buffer and the slot
+    trims)."""
     if is_paper_policy(params):
         return Allocator(nseg, params.get("slot_base", 148), params.get("slot_min", 4))
     return RunsAllocator(nseg, **params)

@@ -35,7 +35,9 @@
  *      block; a large request retries its claim once after the trims;
  *   R6 segments formatted ahead and never used (all blocks home) go back to
  *      the segment tree before a segment claim reports "all in use", and in
- *      the drain after the slots are retired.
+ *      the drain after the slots are retired;
+ *   R7 prefill (knob): the initial state holds every slot's first run, laid
+ *      out class by class from the front ("always populated").
  * Not modelled: the exhaustion record (Deviations 11) -- a concurrency
  * device, checked on the GPU by invariants and by the paper-policy replays
  * (where it is state-neutral); the serialized replays of this model run the
@@ -170,6 +172,15 @@ static uint32_t get_run(o2_t *a, uint32_t t, uint32_t want, uint32_t *first) {
     return got;
 }
 
+/* R1: the first run of an empty slot of class c */
+uint32_t runs_first_run(const o2_t *a, uint32_t c) {
+    uint32_t fl = a->run_init < 8 ? a->run_init : 8;
+    uint32_t fr = (a->run_init >> c) > fl ? (a->run_init >> c) : fl;
+    if (fr > nb_of(c)) fr = nb_of(c);
+    uint32_t cap = run_cap(a, c);
+    return fr < cap ? fr : cap;
+}
+
 /* R1/R4: Alg.3 with a run per slot */
 static uint64_t malloc_slice(o2_t *a, uint32_t c, uint64_t key) {
     unsigned i = a->slot_off[c] + (unsigned)(key % a->nslot[c]);
@@ -191,13 +202,53 @@ static uint64_t malloc_slice(o2_t *a, uint32_t c, uint64_t key) {
             a->next[i] = SLOT_EMPTY;
             continue;
         }
-        uint32_t fl = a->run_init < 8 ? a->run_init : 8;
-        uint32_t fr = (a->run_init >> c) > fl ? (a->run_init >> c) : fl;
-        if (fr > nb_of(c)) fr = nb_of(c);
-        uint32_t want = m == 0 ? (fr < cap ? fr : cap) : grow;
+        uint32_t want = m == 0 ? runs_first_run(a, c) : grow;
         uint32_t got = get_run(a, c, want, &first);
         if (!got) { a->slot[i] = SLOT_EMPTY; return NONE64; }       /* nullptr */
         a->slot[i] = slot_make(0, got, first);
+    }
+}
+
+/* ---------------------------------------------------------- prefill --- */
+/* R7 prefill ("each block buffer is always populated", reading A-19):
+ * the initial state has every slot, class-major and slot-ascending, holding
+ * its first run (R1) of fr[c] consecutive blocks of its class: the blocks of the class's current segment
+ * in ring order (a fresh segment when it has none left; fr[c] divides nb), or
+ * fr[c] / nb whole fresh segments.  Skipped unless the segments this takes
+ * fit in half the heap (a 64 MB heap cannot hold a buffer, A-19). */
+void runs_prefill(o2_t *a) {
+    uint32_t fr[NUM_BLOCK_TREES];
+    for (unsigned c = 0; c < NUM_BLOCK_TREES; c++) fr[c] = runs_first_run(a, c);
+    uint64_t need = 0;
+    for (unsigned c = 0; c < NUM_BLOCK_TREES; c++)
+        need += ((uint64_t)a->nslot[c] * fr[c] + nb_of(c) - 1) / nb_of(c);
+    if (need > a->nseg / 2) return;
+    for (unsigned c = 0; c < NUM_BLOCK_TREES; c++) {
+        uint32_t nb = nb_of(c);
+        uint64_t s = NONE64;
+        for (unsigned q = 0; q < a->nslot[c]; q++) {
+            uint64_t first;
+            if (fr[c] >= nb) {                                      /* whole segments, all blocks out */
+                for (uint32_t k = 0; k < fr[c] / nb; k++) {
+                    uint64_t x = pol_claim_front(a);
+                    pol_format_segment(a, x, c);
+                    for (uint32_t j = 0; j < nb; j++) ring_pop(&a->ring[x]);
+                    a->avail[x] = 0;
+                    oracle_veb_delete(a->btree[c], x);
+                    if (k == 0) first = x * nb;
+                }
+            } else {
+                if (s == NONE64 || a->avail[s] == 0) {
+                    s = pol_claim_front(a);
+                    pol_format_segment(a, s, c);
+                }
+                first = s * nb + a->ring[s].e[a->ring[s].head];
+                for (uint32_t j = 0; j < fr[c]; j++) ring_pop(&a->ring[s]);
+                a->avail[s] -= (int32_t)fr[c];
+                if (a->avail[s] == 0) oracle_veb_delete(a->btree[c], s);
+            }
+            a->slot[a->slot_off[c] + q] = slot_make(0, fr[c], (uint32_t)first);
+        }
     }
 }
 

@@ -150,7 +150,8 @@ o2_t *o2_create_paper(uint64_t nseg, unsigned slot_base, unsigned slot_min) {
 
 /* O2-R: the deviation model (DESIGN.md Deviations 5). */
 o2_t *o2_create_runs(uint64_t nseg, unsigned slot_base, unsigned slot_min, unsigned run_max, uint64_t run_bytes,
-                     unsigned format_ahead, unsigned run_init, unsigned prefetch, unsigned run_grow) {
+                     unsigned format_ahead, unsigned run_init, unsigned prefetch, unsigned run_grow,
+                     unsigned prefill) {
     if (run_grow < 1 || run_grow > 8 || run_max < 1 || run_max > 512) return NULL;
     o2_t *a = create(nseg, slot_base, slot_min);
     if (!a) return NULL;
@@ -159,6 +160,7 @@ o2_t *o2_create_runs(uint64_t nseg, unsigned slot_base, unsigned slot_min, unsig
     a->run_init = run_init < 1 ? 1 : run_init;
     a->prefetch = prefetch;
     a->run_grow = run_grow;
+    if (prefill) runs_prefill(a);                             /* R7 */
     return a;
 }
 

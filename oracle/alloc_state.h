@@ -105,5 +105,7 @@ void pol_drain(o2_t *a);
 /* O2-R (alloc_runs.c) */
 uint64_t runs_malloc(o2_t *a, uint64_t size, uint64_t key);
 void runs_drain(o2_t *a);
+uint32_t runs_first_run(const o2_t *a, uint32_t c);
+void runs_prefill(o2_t *a);
 
 #endif

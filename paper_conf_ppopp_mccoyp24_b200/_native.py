@@ -30,7 +30,7 @@ class Config(ctypes.Structure):
                 ("slot_min", ctypes.c_uint32), ("run_max", ctypes.c_uint32), ("format_ahead", ctypes.c_uint32),
                 ("fence_free", ctypes.c_uint32), ("bulk_items", ctypes.c_uint32), ("run_init", ctypes.c_uint32),
                 ("prefetch", ctypes.c_uint32), ("run_grow", ctypes.c_uint32), ("demand_hint", ctypes.c_uint32),
-                ("oom_record", ctypes.c_uint32)]
+                ("oom_record", ctypes.c_uint32), ("prefill", ctypes.c_uint32)]
 
 
 class Stats(ctypes.Structure):
@@ -41,7 +41,7 @@ class Stats(ctypes.Structure):
                 ("slot_min", ctypes.c_uint32), ("run_max", ctypes.c_uint32), ("format_ahead", ctypes.c_uint32),
                 ("fence_free", ctypes.c_uint32), ("run_init", ctypes.c_uint32), ("formatters", ctypes.c_uint32),
                 ("prefetch", ctypes.c_uint32), ("run_grow", ctypes.c_uint32), ("demand_hint", ctypes.c_uint32),
-                ("oom_record", ctypes.c_uint32)]
+                ("oom_record", ctypes.c_uint32), ("prefill_segments", ctypes.c_uint32)]
 
 
 def declared_functions() -> list[str]:
@@ -169,12 +169,13 @@ def _empty64(n: int):
 # ------------------------------------------------------------- allocator ---
 def gallatin_init(heap_bytes: int, slot_base: int = 0, slot_min: int = 0, run_max: int = 0, run_bytes: int = 0,
                   format_ahead: int = 0, fence_free: int = 0, bulk_items: int = 0, run_init: int = 0,
-                  prefetch: int = 0, run_grow: int = 0, demand_hint: int = 0, oom_record: int = 0) -> None:
+                  prefetch: int = 0, run_grow: int = 0, demand_hint: int = 0, oom_record: int = 0,
+                  prefill: int = 0) -> None:
     """0 = library default for every knob (include/gallatin.h gallatin_config_t)."""
     cfg = Config(heap_bytes=heap_bytes, run_bytes=run_bytes, slot_base=slot_base, slot_min=slot_min,
                  run_max=run_max, format_ahead=format_ahead, fence_free=fence_free, bulk_items=bulk_items,
                  run_init=run_init, prefetch=prefetch, run_grow=run_grow, demand_hint=demand_hint,
-                 oom_record=oom_record)
+                 oom_record=oom_record, prefill=prefill)
     check(lib().gallatin_init_ex(ctypes.byref(cfg)), "gallatin_init")
 
 
@@ -240,7 +241,7 @@ def gallatin_stats() -> dict:
             "run_cap": list(s.run_cap), "run_bytes": s.run_bytes, "slot_base": s.slot_base, "slot_min": s.slot_min,
             "run_max": s.run_max, "format_ahead": s.format_ahead, "fence_free": s.fence_free,
             "run_init": s.run_init, "formatters": s.formatters, "prefetch": s.prefetch, "run_grow": s.run_grow,
-            "demand_hint": s.demand_hint, "oom_record": s.oom_record}
+            "demand_hint": s.demand_hint, "oom_record": s.oom_record, "prefill_segments": s.prefill_segments}
 
 
 def oracle_params() -> dict:
@@ -248,7 +249,8 @@ def oracle_params() -> dict:
     st = gallatin_stats()
     return {"slot_base": st["slot_base"], "slot_min": st["slot_min"], "run_max": st["run_max"],
             "run_bytes": st["run_bytes"], "format_ahead": 1 if st["format_ahead"] == 1 else 0,
-            "run_init": st["run_init"], "prefetch": st["prefetch"], "run_grow": st["run_grow"]}
+            "run_init": st["run_init"], "prefetch": st["prefetch"], "run_grow": st["run_grow"],
+            "prefill": 1 if st["prefill_segments"] else 0}
 
 
 def gallatin_snapshot() -> np.ndarray:

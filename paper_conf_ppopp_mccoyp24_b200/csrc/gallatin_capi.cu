@@ -72,9 +72,19 @@ int launch_status() {
 }
 
 // ------------------------------------------------------------ kernels ----
+// The state a reset leaves, every word computed from its index: the
+// pristine image (every segment free, trees and table consistent, rings and
+// counters empty) or -- with a prefilled block buffer ("always
+// populated", v.pf_segs > 0) -- the same with segments [0, pf_segs) carved
+// into the slots' first runs, class by class (view.h).
+__device__ __forceinline__ uint32_t pf_class_of(const View &v, uint64_t s) {
+    uint32_t c = 0;
+    while (c + 1 < core::kTrees && s >= v.pf_base[c + 1]) c++;
+    return c;
+}
 __global__ void k_reset() {
     const View &v = c_view;
-    const uint64_t W = v.tree_words, nseg = v.nseg;
+    const uint64_t W = v.tree_words, nseg = v.nseg, pf = v.pf_segs;
     const uint64_t S = v.nslot_total;
     const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
     uint64_t total = nseg * 128;
@@ -83,27 +93,71 @@ __global__ void k_reset() {
     if (9 * 32 > total) total = 9 * 32;
     for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < total; i += stride) {
         if (i < W) {
-            // pristine segment tree: every segment free, summaries consistent
+            // segment tree: leaf bit s set iff pf <= s < nseg; a summary bit
+            // set iff its child covers such a segment
             uint32_t lvl = 0;
             while (lvl + 1 < v.tree_levels && i >= v.level_off[lvl + 1]) lvl++;
             const uint64_t word = i - v.level_off[lvl];
             const uint64_t nbits = lvl == 0 ? nseg : (uint64_t)(v.level_off[lvl] - v.level_off[lvl - 1]);
-            const uint64_t lo = word * 64;
-            const uint64_t cnt = nbits > lo ? (nbits - lo < 64 ? nbits - lo : 64) : 0;
-            v.seg_tree[i] = cnt == 64 ? ~0ull : ((1ull << cnt) - 1);
+            const uint64_t span = 1ull << (6 * lvl);                  // segments per child
+            uint64_t w = 0;
+            for (uint32_t b = 0; b < 64; b++) {
+                const uint64_t ch = word * 64 + b;
+                if (ch < nbits && (ch + 1) * span > pf) w |= 1ull << b;
+            }
+            v.seg_tree[i] = w;
         }
-        if (i < 9 * W) v.block_trees[i] = 0;
+        if (i < 9 * W) {
+            // block tree t holds only its class's partly used prefill segment
+            const uint32_t t = (uint32_t)(i / W), wi = (uint32_t)(i % W);
+            uint64_t w = 0;
+            if (pf && v.pf_last[t] != 0xFFFFFFFFu) {
+                uint32_t lvl = 0;
+                while (lvl + 1 < v.tree_levels && wi >= v.level_off[lvl + 1]) lvl++;
+                const uint64_t idx = (uint64_t)v.pf_last[t] >> (6 * lvl);      // this level's bit index
+                if (wi - v.level_off[lvl] == (idx >> 6)) w = 1ull << (idx & 63);
+            }
+            v.block_trees[i] = w;
+        }
         if (i < nseg) {
-            v.seg_word[i] = core::sw_make(core::kTreeFree, 0);
-            v.seg_tid[i] = core::kTreeFree;
+            uint32_t t = core::kTreeFree;
+            int32_t avail = 0;
+            uint32_t tail = 0;
+            if (i < pf) {
+                t = pf_class_of(v, i);
+                if (i == v.pf_last[t]) avail = (int32_t)(core::nb_of(t) - v.pf_used[t]);
+                tail = (uint32_t)avail;
+            }
+            v.seg_word[i] = core::sw_make(t, t == core::kTreeFree ? 0 : avail);
+            v.seg_tid[i] = t;
             v.q_head[i] = 0;
-            v.q_tail[i] = 0;
+            v.q_tail[i] = tail;
         }
-        if (i < nseg * 64) reinterpret_cast<uint64_t *>(v.q_entries)[i] = ~0ull;
+        if (i < nseg * 64) {
+            uint64_t e = ~0ull;
+            const uint64_t s = i / 64, q0 = (i % 64) * 4;
+            if (s < pf) {
+                const uint32_t t = pf_class_of(v, s);
+                if (s == v.pf_last[t]) {                                 // ring: blocks used..nb-1, ascending
+                    const uint32_t u = v.pf_used[t], cnt = core::nb_of(t) - u;
+                    e = 0;
+                    for (uint32_t k = 0; k < 4; k++)
+                        e |= (uint64_t)(q0 + k < cnt ? (uint16_t)(u + q0 + k) : core::kRingEmpty) << (16 * k);
+                }
+            }
+            reinterpret_cast<uint64_t *>(v.q_entries)[i] = e;
+        }
         if (i < nseg * 128) reinterpret_cast<uint64_t *>(v.block_free)[i] = 0;
         if (i < S * 16) {
-            const uint64_t w = i % 16;
-            v.slots[i] = w <= 1 ? core::kSlotEmpty : 0;
+            const uint64_t w = i % 16, si = i / 16;
+            uint64_t val = w <= 1 ? core::kSlotEmpty : 0;
+            if (pf && w == 0) {
+                uint32_t c = 0;
+                while (c + 1 < core::kTrees && si >= v.slot_off[c + 1]) c++;
+                const uint64_t first = (uint64_t)v.pf_base[c] * core::nb_of(c) + (si - v.slot_off[c]) * v.pf_run[c];
+                val = ((uint64_t)v.pf_run[c] << core::kRunShift) | first;
+            }
+            v.slots[i] = val;
         }
         if (i < 9 * 32) v.fmt_token[i] = 0;
         if (i == 0) *v.err = 0;
@@ -683,7 +737,7 @@ int gallatin_init_ex(const gallatin_config_t *cfg_in) {
     }
     if (cfg.run_max > core::kMaxRun || cfg.fence_free > 2 || cfg.format_ahead > 2) return GALLATIN_ERR_INVALID;
     if (cfg.bulk_items != 0 && cfg.bulk_items != 1 && cfg.bulk_items != 4) return GALLATIN_ERR_INVALID;
-    if (cfg.prefetch > 2 || cfg.demand_hint > 2 || cfg.oom_record > 2) return GALLATIN_ERR_INVALID;
+    if (cfg.prefetch > 2 || cfg.demand_hint > 2 || cfg.oom_record > 2 || cfg.prefill > 2) return GALLATIN_ERR_INVALID;
     if (!cfg.run_grow) cfg.run_grow = 3;
     if (cfg.run_grow > 8) return GALLATIN_ERR_INVALID;
     if (nseg > (1ull << 14)) return GALLATIN_ERR_INVALID;        // 22-bit run index at 64 KB blocks (256 GiB)
@@ -735,6 +789,25 @@ int gallatin_init_ex(const gallatin_config_t *cfg_in) {
     v.fence_free = cfg.fence_free;
     v.demand_hint = cfg.demand_hint == 2 ? 0u : 1u;
     v.oom_record = cfg.oom_record == 2 ? 0u : 1u;
+    // prefilled block buffer: every slot's first run laid out class
+    // by class from segment 0, if it fits in half the heap (reading A-19)
+    {
+        uint64_t seg = 0;
+        for (uint32_t c = 0; c < core::kTrees; c++) {
+            const uint32_t nb = 256u >> c;
+            const uint32_t fl = cfg.run_init < 8 ? cfg.run_init : 8u;
+            const uint32_t fs = (cfg.run_init >> c) > fl ? (cfg.run_init >> c) : fl;
+            uint32_t fr = fs < nb ? fs : nb;
+            if (fr > v.run_cap[c]) fr = v.run_cap[c];
+            const uint64_t blocks = (uint64_t)v.nslot[c] * fr, segs = (blocks + nb - 1) / nb;
+            v.pf_base[c] = (uint32_t)seg;
+            v.pf_run[c] = fr;
+            v.pf_used[c] = (uint32_t)(blocks - (segs - 1) * nb);
+            v.pf_last[c] = v.pf_used[c] < nb ? (uint32_t)(seg + segs - 1) : 0xFFFFFFFFu;
+            seg += segs;
+        }
+        v.pf_segs = (cfg.prefill != 2 && seg <= nseg / 2) ? (uint32_t)seg : 0u;
+    }
 
     // metadata: one allocation, 256 B aligned sections
     uint64_t sz[12] = {W * 8, 9 * W * 8, nseg * 8, nseg * 4, nseg * 4, nseg * 512, nseg * 1024,
@@ -1005,6 +1078,7 @@ int gallatin_stats(gallatin_stats_t *out) {
     out->prefetch = v.prefetch;
     out->demand_hint = v.demand_hint;
     out->oom_record = v.oom_record;
+    out->prefill_segments = v.pf_segs;
     return GALLATIN_OK;
 }
 

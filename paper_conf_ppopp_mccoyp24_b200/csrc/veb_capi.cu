@@ -32,10 +32,14 @@ int launch_status() {
 
 // Bulk insert / delete, ITEMS keys per thread (keys loaded first, then the
 // ITEMS leaf RMWs issued back to back: several L2 round trips in flight per
-// warp).  The lanes of a warp whose keys share a leaf word combine: one
-// atomicOr / atomicAnd of the OR of their bits by the lowest such lane, the
-// old word broadcast back; of several lanes with the SAME key only the lowest
-// reports (exactly one op per distinct key returns 1, reading A-23).  The
+// warp).  When neighbouring lanes' keys share a leaf word (sorted or
+// clustered batches; one shfl + ballot decides per warp and item) the lanes
+// of a warp on one word combine: one atomicOr / atomicAnd of the OR of their
+// bits by the lowest such lane, the old word broadcast back, and of several
+// lanes with the SAME key only the lowest reports.  Otherwise every lane
+// issues its own RMW (random batches: the match would only cost issue
+// slots); equal keys then still report once -- the second RMW sees the bit
+// (exactly one op per distinct key returns 1, reading A-23).  The
 // lane whose RMW flipped the word's emptiness repairs the summaries: set side
 // bt_set_up (release fence, no re-read), clear side bt_reconcile_up.
 template <bool INSERT, int ITEMS>
@@ -51,14 +55,22 @@ __global__ void __launch_bounds__(kThreads) k_update(BitTree t, const uint64_t *
     }
     uint64_t old[ITEMS], bit[ITEMS], msk[ITEMS];
     unsigned wp[ITEMS];
+    bool comb[ITEMS];                                              // warp-uniform per item
 #pragma unroll
     for (int k = 0; k < ITEMS; k++) {
         const bool valid = x[k] < t.nbits;
         const uint64_t wi = valid ? x[k] >> 6 : ~0ull - lane;       // invalid keys: a word of their own
         bit[k] = valid ? 1ull << (x[k] & 63) : 0;
-        wp[k] = __match_any_sync(0xFFFFFFFFu, wi);
-        msk[k] = ((uint64_t)__reduce_or_sync(wp[k], (uint32_t)(bit[k] >> 32)) << 32) |
-                 __reduce_or_sync(wp[k], (uint32_t)bit[k]);
+        const bool adj = __shfl_up_sync(0xFFFFFFFFu, wi, 1) == wi && lane > 0;
+        comb[k] = __ballot_sync(0xFFFFFFFFu, adj) != 0;
+        if (comb[k]) {
+            wp[k] = __match_any_sync(0xFFFFFFFFu, wi);
+            msk[k] = ((uint64_t)__reduce_or_sync(wp[k], (uint32_t)(bit[k] >> 32)) << 32) |
+                     __reduce_or_sync(wp[k], (uint32_t)bit[k]);
+        } else {
+            wp[k] = 1u << lane;
+            msk[k] = bit[k];
+        }
         old[k] = 0;
         if (valid && lane == (uint32_t)__ffs((int)wp[k]) - 1)
             old[k] = INSERT ? ptx::atom_or(t.w + t.off[0] + wi, msk[k]) : ptx::atom_and(t.w + t.off[0] + wi, ~msk[k]);
@@ -66,11 +78,16 @@ __global__ void __launch_bounds__(kThreads) k_update(BitTree t, const uint64_t *
 #pragma unroll
     for (int k = 0; k < ITEMS; k++) {
         const uint32_t leader = (uint32_t)__ffs((int)wp[k]) - 1;
-        const uint64_t o = __shfl_sync(0xFFFFFFFFu, old[k], (int)leader);
-        const unsigned kp = __match_any_sync(0xFFFFFFFFu, x[k]);
+        uint64_t o = old[k];
+        bool first = true;                                          // the lowest lane with this key
+        if (comb[k]) {
+            o = __shfl_sync(0xFFFFFFFFu, old[k], (int)leader);
+            const unsigned kp = __match_any_sync(0xFFFFFFFFu, x[k]);
+            first = lane == (uint32_t)__ffs((int)kp) - 1;
+        }
         const uint64_t i = base + (uint64_t)kThreads * k;
         const bool valid = bit[k] != 0;
-        if (out && i < n) out[i] = valid && lane == (uint32_t)__ffs((int)kp) - 1 && (INSERT ? !(o & bit[k]) : (o & bit[k]) != 0);
+        if (out && i < n) out[i] = valid && first && (INSERT ? !(o & bit[k]) : (o & bit[k]) != 0);
         if (valid && lane == leader) {
             if (INSERT && o == 0) bt_set_up(t, 0, x[k] >> 6);                          // empty -> non-empty
             if (!INSERT && (o & msk[k]) != 0 && (o & ~msk[k]) == 0) bt_reconcile_up(t, 0, x[k] >> 6);   // -> empty

@@ -47,9 +47,9 @@ def classify(size: int):
 
 class PolSim:
     def __init__(self, nseg, slot_base=148, slot_min=4, run_max=1, run_bytes=64 << 20, format_ahead=0, run_init=1,
-                 prefetch=0, run_grow=1):
+                 prefetch=0, run_grow=1, prefill=0):
         self.nseg = nseg
-        self.runs = not (run_max == 1 and run_init == 1 and format_ahead == 0 and prefetch == 0)
+        self.runs = not (run_max == 1 and run_init == 1 and format_ahead == 0 and prefetch == 0 and not prefill)
         self.nslot = [max(slot_base >> c, slot_min, 1) for c in range(TREES)]
         self.off = [sum(self.nslot[:c]) for c in range(TREES)]
         self.run_max, self.run_bytes, self.fa, self.run_init = run_max, run_bytes, format_ahead, run_init
@@ -61,6 +61,31 @@ class PolSim:
         self.slot = [None] * S               # None or [issued, m, first]
         self.next = [None] * S
         self.err = 0
+        if prefill:
+            self.prefill()
+
+    def first_run(self, c):
+        return min(max(self.run_init >> c, min(self.run_init, 8)), nb(c), self.cap(c))
+
+    def prefill(self):
+        """R7 ("always populated"): slot q of class c holds blocks
+        [q r, (q+1) r) of the class's segments (r its first run), the classes'
+        segments laid out one after another from segment 0; the class's partly
+        used last segment keeps the rest, ascending, in its ring -- if all of
+        it fits in half the heap."""
+        runs = [self.first_run(c) for c in range(TREES)]
+        segs = [-(-self.nslot[c] * runs[c] // nb(c)) for c in range(TREES)]
+        if sum(segs) > self.nseg // 2:
+            return
+        base = 0
+        for c in range(TREES):
+            for s in range(base, base + segs[c]):
+                self.tree[s] = c
+            used = self.nslot[c] * runs[c] - (segs[c] - 1) * nb(c)
+            self.ring[base + segs[c] - 1] = deque(range(used, nb(c)))
+            for q in range(self.nslot[c]):
+                self.slot[self.off[c] + q] = [0, runs[c], base * nb(c) + q * runs[c]]
+            base += segs[c]
 
     # ---- the trees, by scan --------------------------------------------
     def free_segs(self):
@@ -195,7 +220,7 @@ class PolSim:
                 self.slot[i], self.next[i] = self.next[i], None
                 continue
             if sl is None:                                        # first run (R1)
-                want = min(max(self.run_init >> c, min(self.run_init, 8)), nb(c), self.cap(c))
+                want = self.first_run(c)
             else:
                 want = min(sl[1] << self.grow, self.cap(c))
             got, first = self.get_run(c, want)

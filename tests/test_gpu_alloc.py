@@ -38,18 +38,20 @@ def G():
 
 
 def _replay_case(G, nseg, run_max, fa, kinds, args, keys, slot_base=16, slot_min=2, run_bytes=32 << 20, pf=None,
-                 run_init=1, run_grow=0, record=None):
-    """GPU serialized replay vs O2: O2-P at the paper's knobs (with the
-    exhaustion record on, where it is state-neutral), O2-R otherwise (the GPU
-    with the record off: O2-R does not model it)."""
+                 run_init=1, run_grow=0, record=None, prefill=False):
+    """GPU serialized replay vs O2: O2-P at the paper's knobs without prefill
+    (with the exhaustion record on, where it is state-neutral), O2-R otherwise
+    (the GPU with the record off: O2-R does not model it)."""
     if pf is None:
         pf = run_max > 1                    # the paper's policy (run_max=1) has no prefetch
-    paper = run_max == 1 and not fa and not pf and run_init == 1
+    paper = run_max == 1 and not fa and not pf and run_init == 1 and not prefill
     if record is None:
         record = paper
     G.gallatin_init(nseg * SEG, slot_base=slot_base, slot_min=slot_min, run_max=run_max, run_bytes=run_bytes,
                     format_ahead=1 if fa else 2, prefetch=1 if pf else 2, run_init=run_init, run_grow=run_grow,
-                    oom_record=1 if record else 2)
+                    oom_record=1 if record else 2, prefill=1 if prefill else 2)
+    if prefill:
+        assert G.gallatin_stats()["prefill_segments"] > 0, "the case must exercise a prefilled buffer"
     out = _u64(G.gallatin_replay(_dev(kinds, np.uint8), _dev(args), _dev(keys)))
     o2 = oracle.model(nseg, **G.oracle_params())
     assert isinstance(o2, oracle.RunsAllocator) != paper
@@ -71,6 +73,31 @@ def test_serialized_replay_matches_oracle(cuda_ok, G, seed, nseg, run_max, fa):
     replay"); run_max=1, fa=0 is the paper's policy."""
     kinds, args, keys = wg.replay_ops(6000, seed + 100, p_free=0.45, p_drain=0.003, nkeys=64)
     _replay_case(G, nseg, run_max, fa, kinds, args, keys)
+
+
+@pytest.mark.parametrize("seed,nseg,run_max,fa,ri,rg", [(21, 24, 1, 0, 1, 1), (22, 32, 16, 1, 4, 1),
+                                                        (23, 48, 256, 1, 16, 3), (24, 40, 512, 0, 256, 3)])
+def test_serialized_replay_prefilled(cuda_ok, G, seed, nseg, run_max, fa, ri, rg):
+    """A prefilled block buffer ("always populated", O2-R R7): init and
+    the replay's drains leave the state O2-R reaches; at the paper's one-block
+    knobs (first case) and with runs; OOM and drains included."""
+    kinds, args, keys = wg.replay_ops(6000, seed + 100, p_free=0.45, p_drain=0.003, nkeys=64)
+    _replay_case(G, nseg, run_max, fa, kinds, args, keys, pf=False, run_init=ri, run_grow=rg, prefill=True)
+
+
+def test_reset_prefills_block_buffer(cuda_ok, G):
+    """gallatin_reset with the prefill knob (default) leaves exactly O2-R's
+    prefilled initial state (R7); drain turns it into the pristine image."""
+    nseg = 1024
+    G.gallatin_init(nseg * SEG)
+    st = G.gallatin_stats()
+    assert st["prefill_segments"] > 0
+    G.gallatin_malloc(_dev(wg.mixed_sizes(1 << 16, p_large=2.0 ** -8)))
+    G.gallatin_reset()
+    o2 = oracle.model(nseg, **G.oracle_params())
+    msg = diff_images(G.gallatin_snapshot(), o2.image())
+    assert not msg, msg
+    _assert_pristine(G, nseg)
 
 
 def test_serialized_replay_block_boundaries(cuda_ok, G):
@@ -109,6 +136,7 @@ def test_serialized_replay_default_knobs(cuda_ok, G):
     nseg = 64
     kinds, args, keys = wg.replay_ops(8000, 141, p_free=0.45, p_drain=0.002, nkeys=148 * 4)
     G.gallatin_init(nseg * SEG, oom_record=2)
+    assert G.gallatin_stats()["prefill_segments"] > 0          # the production default fills the buffer
     st = G.gallatin_stats()
     assert st["slot_base"] == 148 and st["run_max"] == 256 and st["format_ahead"] == 1 and st["run_grow"] == 3
     out = _u64(G.gallatin_replay(_dev(kinds, np.uint8), _dev(args), _dev(keys)))
@@ -279,7 +307,7 @@ def test_host_buffer_api_chunked(cuda_ok, G):
 
 def test_reset_restores_pristine(cuda_ok, G):
     nseg = 8
-    G.gallatin_init(nseg * SEG)
+    G.gallatin_init(nseg * SEG, prefill=2)
     G.gallatin_malloc(_dev(wg.mixed_sizes(1 << 14, p_large=2.0 ** -8)))
     G.gallatin_reset()
     img = G.gallatin_snapshot()

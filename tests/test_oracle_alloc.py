@@ -201,6 +201,10 @@ SIM_CASES = [
     # production-shaped knobs (gallatin_init defaults at 64 segments): 148 slots at 16 B,
     # runs up to 256 blocks / 16 MB, format-ahead, x8 growth, first runs of 4 blocks
     (22, 64, 148, 4, dict(run_max=256, run_bytes=16 << 20, run_init=4, run_grow=3, format_ahead=1)),
+    # prefilled block buffers (R7): the paper's one-block slots, and the production-shaped knobs
+    (23, 32, 16, 2, dict(prefill=1)),
+    (24, 64, 148, 4, dict(run_max=256, run_bytes=16 << 20, run_init=4, run_grow=3, format_ahead=1, prefill=1)),
+    (25, 40, 16, 2, dict(run_max=512, run_init=16, run_grow=3, prefetch=1, prefill=1)),
 ]
 
 
@@ -219,6 +223,8 @@ def test_o2_matches_brute_force_simulation(seed, nseg, sb, sm, knobs):
     sim = PolSim(nseg, sb, sm, **kw)
     a = oracle.model(nseg, slot_base=sb, slot_min=sm, **kw)
     assert isinstance(a, oracle.RunsAllocator) == (knobs is not None)
+    if kw.get("prefill"):
+        assert a.image()[8] != pristine_image(nseg, int(a.image()[4]))[8], "the prefill must apply"
     want = sim.replay(kinds, args, keys)
     got = a.replay(kinds, args, keys)
     bad = np.nonzero(got != want)[0]
@@ -359,6 +365,44 @@ def test_whole_segment_runs_prefer_fresh_segments():
     assert (w >> 22) & 0x3FF == 2 and w & 0x3FFFFF == 2             # run of 2 from linear block 2
     assert a.malloc(bb, 0) == bb                                      # block path: segment 0's block 1
     assert a.check() == 0
+
+
+def test_prefill_layout_closed_form():
+    """R7 ("always populated"): with run_init 64 every class's slots
+    start with runs of min(max(64 >> c, 8), nb(c)) blocks = 64, 32, 16, 8, 8,
+    8, 4, 2, 1 (R1), laid out class by class from segment 0: 4 slots of 16 B
+    fill segment 0; 2 slots x 32 of the 128 32-B blocks use half of segment 1,
+    whose other 64 blocks stay in its ring (ascending) and block tree 1; ...;
+    13 segments in all, the rest free.  The first 16 B request of slot 1 lands
+    at block 64 of segment 0."""
+    a = runs(32, slot_base=4, slot_min=2, run_max=512, run_bytes=1 << 30, run_init=64, prefill=1)
+    d = image_sections(a.image())
+    runs_ = [64, 32, 16, 8, 8, 8, 4, 2, 1]
+    nslot = [4, 2, 2, 2, 2, 2, 2, 2, 2]
+    segs = [-(-n * r // (256 >> c)) for c, (n, r) in enumerate(zip(nslot, runs_))]
+    assert segs == [1, 1, 1, 1, 1, 2, 2, 2, 2]
+    base = np.cumsum([0] + segs)
+    slots = d["slots"]
+    for c in range(9):
+        for q in range(nslot[c]):
+            w = int(slots[sum(nslot[:c]) + q])
+            assert w == (runs_[c] << 22) | (int(base[c]) * (256 >> c) + q * runs_[c]), (c, q, hex(w))
+    assert int(d["segtree"][0]) == ((1 << 32) - 1) & ~((1 << 13) - 1)      # segments 13..31 free
+    assert int(d["segword"][1]) == (1 << 32) | 64 and int(d["btrees"][1][0]) == 1 << 1
+    assert list(d["qentries"][1][:2]) == [64, 65] and int(d["qcount"][1]) == 64
+    assert int(d["segword"][0]) == 0 and int(d["segword"][5]) == (5 << 32)   # full segments: avail 0
+    assert a.malloc(16, 1) == 64 * 65536 and a.check() == 0
+    a.free(64 * 65536)
+    a.drain()
+    assert np.array_equal(a.image(), pristine_image(32, 20))
+
+
+def test_prefill_skipped_when_it_does_not_fit():
+    """R7 / reading A-19: a buffer that would take more than half the heap
+    is not prefilled (a 64 MB heap cannot hold one block of every class for
+    every slot): the initial image is pristine."""
+    a = runs(4, slot_base=148, slot_min=4, run_max=256, run_init=1, prefill=1)
+    assert np.array_equal(a.image(), pristine_image(4, 302))
 
 
 def test_format_ahead_closed_form():
