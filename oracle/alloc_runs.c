@@ -212,24 +212,40 @@ static uint64_t malloc_slice(o2_t *a, uint32_t c, uint64_t key) {
 /* ---------------------------------------------------------- prefill --- */
 /* R7 prefill ("each block buffer is always populated", reading A-19):
  * the initial state has every slot, class-major and slot-ascending, holding
- * its first run (R1) of fr[c] consecutive blocks of its class: the blocks of the class's current segment
- * in ring order (a fresh segment when it has none left; fr[c] divides nb), or
- * fr[c] / nb whole fresh segments.  Skipped unless the segments this takes
- * fit in half the heap (a 64 MB heap cannot hold a buffer, A-19). */
+ * a run of r[c] consecutive blocks of its class: the blocks of the class's
+ * current segment in ring order (a fresh segment when it has none left), or
+ * r[c] / nb whole fresh segments.  r[c] starts at the largest power of two
+ * <= the first run (R1); while the segments this takes exceed nseg / 8, the
+ * class holding the most segments (lowest class on ties) with r[c] > 1 is
+ * halved; if every r[c] is 1 and it still does not fit, nothing is filled. */
+static uint64_t prefill_segs(const o2_t *a, const uint32_t *r, unsigned c) {
+    return ((uint64_t)a->nslot[c] * r[c] + nb_of(c) - 1) / nb_of(c);
+}
+
 void runs_prefill(o2_t *a) {
-    uint32_t fr[NUM_BLOCK_TREES];
-    for (unsigned c = 0; c < NUM_BLOCK_TREES; c++) fr[c] = runs_first_run(a, c);
-    uint64_t need = 0;
-    for (unsigned c = 0; c < NUM_BLOCK_TREES; c++)
-        need += ((uint64_t)a->nslot[c] * fr[c] + nb_of(c) - 1) / nb_of(c);
-    if (need > a->nseg / 2) return;
+    uint32_t r[NUM_BLOCK_TREES];
+    for (unsigned c = 0; c < NUM_BLOCK_TREES; c++) {
+        uint32_t fr = runs_first_run(a, c);
+        r[c] = 1;
+        while (r[c] * 2 <= fr) r[c] *= 2;
+    }
+    for (;;) {
+        uint64_t total = 0;
+        for (unsigned c = 0; c < NUM_BLOCK_TREES; c++) total += prefill_segs(a, r, c);
+        if (total <= a->nseg / 8) break;
+        int big = -1;
+        for (unsigned c = 0; c < NUM_BLOCK_TREES; c++)
+            if (r[c] > 1 && (big < 0 || prefill_segs(a, r, c) > prefill_segs(a, r, (unsigned)big))) big = (int)c;
+        if (big < 0) return;                                        /* does not fit: slots start empty */
+        r[big] /= 2;
+    }
     for (unsigned c = 0; c < NUM_BLOCK_TREES; c++) {
         uint32_t nb = nb_of(c);
         uint64_t s = NONE64;
         for (unsigned q = 0; q < a->nslot[c]; q++) {
-            uint64_t first;
-            if (fr[c] >= nb) {                                      /* whole segments, all blocks out */
-                for (uint32_t k = 0; k < fr[c] / nb; k++) {
+            uint64_t first = 0;
+            if (r[c] >= nb) {                                       /* whole segments, all blocks out */
+                for (uint32_t k = 0; k < r[c] / nb; k++) {
                     uint64_t x = pol_claim_front(a);
                     pol_format_segment(a, x, c);
                     for (uint32_t j = 0; j < nb; j++) ring_pop(&a->ring[x]);
@@ -237,17 +253,17 @@ void runs_prefill(o2_t *a) {
                     oracle_veb_delete(a->btree[c], x);
                     if (k == 0) first = x * nb;
                 }
-            } else {
+            } else {                                                /* r[c] divides nb */
                 if (s == NONE64 || a->avail[s] == 0) {
                     s = pol_claim_front(a);
                     pol_format_segment(a, s, c);
                 }
                 first = s * nb + a->ring[s].e[a->ring[s].head];
-                for (uint32_t j = 0; j < fr[c]; j++) ring_pop(&a->ring[s]);
-                a->avail[s] -= (int32_t)fr[c];
+                for (uint32_t j = 0; j < r[c]; j++) ring_pop(&a->ring[s]);
+                a->avail[s] -= (int32_t)r[c];
                 if (a->avail[s] == 0) oracle_veb_delete(a->btree[c], s);
             }
-            a->slot[a->slot_off[c] + q] = slot_make(0, fr[c], (uint32_t)first);
+            a->slot[a->slot_off[c] + q] = slot_make(0, r[c], (uint32_t)first);
         }
     }
 }

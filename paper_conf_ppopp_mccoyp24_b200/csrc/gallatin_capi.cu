@@ -789,24 +789,42 @@ int gallatin_init_ex(const gallatin_config_t *cfg_in) {
     v.fence_free = cfg.fence_free;
     v.demand_hint = cfg.demand_hint == 2 ? 0u : 1u;
     v.oom_record = cfg.oom_record == 2 ? 0u : 1u;
-    // prefilled block buffer: every slot's first run laid out class
-    // by class from segment 0, if it fits in half the heap (reading A-19)
+    // prefilled block buffer (include/gallatin.h "prefill"): runs of
+    // a power of two <= the first run, the class holding the most segments
+    // halved until the buffer fits in nseg/8 segments, laid out class by class
     {
-        uint64_t seg = 0;
+        uint32_t r[core::kTrees];
         for (uint32_t c = 0; c < core::kTrees; c++) {
             const uint32_t nb = 256u >> c;
             const uint32_t fl = cfg.run_init < 8 ? cfg.run_init : 8u;
             const uint32_t fs = (cfg.run_init >> c) > fl ? (cfg.run_init >> c) : fl;
             uint32_t fr = fs < nb ? fs : nb;
             if (fr > v.run_cap[c]) fr = v.run_cap[c];
-            const uint64_t blocks = (uint64_t)v.nslot[c] * fr, segs = (blocks + nb - 1) / nb;
+            r[c] = 1u << (31 - __builtin_clz(fr));                  // largest power of two <= fr
+        }
+        auto segs_of = [&](uint32_t c) { return ((uint64_t)v.nslot[c] * r[c] + (256u >> c) - 1) / (256u >> c); };
+        bool fits = cfg.prefill != 2;
+        for (;;) {
+            uint64_t total = 0;
+            for (uint32_t c = 0; c < core::kTrees; c++) total += segs_of(c);
+            if (total <= nseg / 8) break;
+            int big = -1;
+            for (uint32_t c = 0; c < core::kTrees; c++)
+                if (r[c] > 1 && (big < 0 || segs_of(c) > segs_of((uint32_t)big))) big = (int)c;
+            if (big < 0) { fits = false; break; }
+            r[big] >>= 1;
+        }
+        uint64_t seg = 0;
+        for (uint32_t c = 0; c < core::kTrees; c++) {
+            const uint32_t nb = 256u >> c;
+            const uint64_t blocks = (uint64_t)v.nslot[c] * r[c], segs = segs_of(c);
             v.pf_base[c] = (uint32_t)seg;
-            v.pf_run[c] = fr;
+            v.pf_run[c] = r[c];
             v.pf_used[c] = (uint32_t)(blocks - (segs - 1) * nb);
             v.pf_last[c] = v.pf_used[c] < nb ? (uint32_t)(seg + segs - 1) : 0xFFFFFFFFu;
             seg += segs;
         }
-        v.pf_segs = (cfg.prefill != 2 && seg <= nseg / 2) ? (uint32_t)seg : 0u;
+        v.pf_segs = fits ? (uint32_t)seg : 0u;
     }
 
     // metadata: one allocation, 256 B aligned sections

@@ -69,23 +69,30 @@ class PolSim:
 
     def prefill(self):
         """R7 ("always populated"): slot q of class c holds blocks
-        [q r, (q+1) r) of the class's segments (r its first run), the classes'
-        segments laid out one after another from segment 0; the class's partly
-        used last segment keeps the rest, ascending, in its ring -- if all of
-        it fits in half the heap."""
-        runs = [self.first_run(c) for c in range(TREES)]
-        segs = [-(-self.nslot[c] * runs[c] // nb(c)) for c in range(TREES)]
-        if sum(segs) > self.nseg // 2:
-            return
+        [q r, (q+1) r) of the class's segments, the classes' segments laid out
+        one after another from segment 0; the class's partly used last segment
+        keeps the rest, ascending, in its ring.  r = the largest power of two
+        <= the first run, then the class with the most segments (lowest on
+        ties, r > 1) halved until all fits in nseg / 8 segments (else none)."""
+        r = [1 << (self.first_run(c).bit_length() - 1) for c in range(TREES)]
+
+        def segs(c):
+            return -(-self.nslot[c] * r[c] // nb(c))
+        while sum(segs(c) for c in range(TREES)) > self.nseg // 8:
+            cand = [c for c in range(TREES) if r[c] > 1]
+            if not cand:
+                return
+            big = max(cand, key=lambda c: (segs(c), -c))
+            r[big] //= 2
         base = 0
         for c in range(TREES):
-            for s in range(base, base + segs[c]):
+            for s in range(base, base + segs(c)):
                 self.tree[s] = c
-            used = self.nslot[c] * runs[c] - (segs[c] - 1) * nb(c)
-            self.ring[base + segs[c] - 1] = deque(range(used, nb(c)))
+            used = self.nslot[c] * r[c] - (segs(c) - 1) * nb(c)
+            self.ring[base + segs(c) - 1] = deque(range(used, nb(c)))
             for q in range(self.nslot[c]):
-                self.slot[self.off[c] + q] = [0, runs[c], base * nb(c) + q * runs[c]]
-            base += segs[c]
+                self.slot[self.off[c] + q] = [0, r[c], base * nb(c) + q * r[c]]
+            base += segs(c)
 
     # ---- the trees, by scan --------------------------------------------
     def free_segs(self):

@@ -202,9 +202,9 @@ SIM_CASES = [
     # runs up to 256 blocks / 16 MB, format-ahead, x8 growth, first runs of 4 blocks
     (22, 64, 148, 4, dict(run_max=256, run_bytes=16 << 20, run_init=4, run_grow=3, format_ahead=1)),
     # prefilled block buffers (R7): the paper's one-block slots, and the production-shaped knobs
-    (23, 32, 16, 2, dict(prefill=1)),
-    (24, 64, 148, 4, dict(run_max=256, run_bytes=16 << 20, run_init=4, run_grow=3, format_ahead=1, prefill=1)),
-    (25, 40, 16, 2, dict(run_max=512, run_init=16, run_grow=3, prefetch=1, prefill=1)),
+    (23, 96, 16, 2, dict(prefill=1)),
+    (24, 256, 148, 4, dict(run_max=256, run_bytes=16 << 20, run_init=4, run_grow=3, format_ahead=1, prefill=1)),
+    (25, 128, 16, 2, dict(run_max=512, run_init=16, run_grow=3, prefetch=1, prefill=1)),
 ]
 
 
@@ -373,9 +373,9 @@ def test_prefill_layout_closed_form():
     8, 4, 2, 1 (R1), laid out class by class from segment 0: 4 slots of 16 B
     fill segment 0; 2 slots x 32 of the 128 32-B blocks use half of segment 1,
     whose other 64 blocks stay in its ring (ascending) and block tree 1; ...;
-    13 segments in all, the rest free.  The first 16 B request of slot 1 lands
-    at block 64 of segment 0."""
-    a = runs(32, slot_base=4, slot_min=2, run_max=512, run_bytes=1 << 30, run_init=64, prefill=1)
+    13 segments in all (<= 128 / 8: no halving), the rest free.  The first
+    16 B request of slot 1 lands at block 64 of segment 0."""
+    a = runs(128, slot_base=4, slot_min=2, run_max=512, run_bytes=1 << 30, run_init=64, prefill=1)
     d = image_sections(a.image())
     runs_ = [64, 32, 16, 8, 8, 8, 4, 2, 1]
     nslot = [4, 2, 2, 2, 2, 2, 2, 2, 2]
@@ -387,20 +387,37 @@ def test_prefill_layout_closed_form():
         for q in range(nslot[c]):
             w = int(slots[sum(nslot[:c]) + q])
             assert w == (runs_[c] << 22) | (int(base[c]) * (256 >> c) + q * runs_[c]), (c, q, hex(w))
-    assert int(d["segtree"][0]) == ((1 << 32) - 1) & ~((1 << 13) - 1)      # segments 13..31 free
+    assert int(d["segtree"][0]) == ((1 << 64) - 1) & ~((1 << 13) - 1) and int(d["segtree"][1]) == (1 << 64) - 1
     assert int(d["segword"][1]) == (1 << 32) | 64 and int(d["btrees"][1][0]) == 1 << 1
     assert list(d["qentries"][1][:2]) == [64, 65] and int(d["qcount"][1]) == 64
     assert int(d["segword"][0]) == 0 and int(d["segword"][5]) == (5 << 32)   # full segments: avail 0
     assert a.malloc(16, 1) == 64 * 65536 and a.check() == 0
     a.free(64 * 65536)
     a.drain()
-    assert np.array_equal(a.image(), pristine_image(32, 20))
+    assert np.array_equal(a.image(), pristine_image(128, 20))
+
+
+def test_prefill_halves_the_largest_class_to_fit():
+    """R7's budget: runs start at the largest power of two <= the first run
+    (256 blocks at 16 B: 2 slots = 2 segments, one segment for each other
+    class: 10 in all); on a 72-segment heap (budget 72 / 8 = 9) the class
+    with the most segments -- 16 B -- is halved once: 2 x 128 blocks in
+    segment 0, classes 1..8 in segments 1..8."""
+    a = runs(72, slot_base=2, slot_min=1, run_max=512, run_bytes=1 << 30, run_init=256, prefill=1)
+    d = image_sections(a.image())
+    assert [int(w) for w in d["slots"][:2]] == [128 << 22, (128 << 22) | 128]
+    assert [int(w) >> 32 for w in d["segword"][:10]] == list(range(9)) + [TREE_FREE]
+    assert int(d["slots"][2]) == (128 << 22) | 128                             # 32 B: 128 blocks of segment 1
+    b = runs(80, slot_base=2, slot_min=1, run_max=512, run_bytes=1 << 30, run_init=256, prefill=1)
+    assert int(image_sections(b.image())["slots"][1]) == (256 << 22) | 256   # budget 10: no halving
+    c = runs(64, slot_base=2, slot_min=1, run_max=512, run_bytes=1 << 30, run_init=256, prefill=1)
+    assert np.array_equal(c.image(), pristine_image(64, 10))                  # 9 segments at least: none
 
 
 def test_prefill_skipped_when_it_does_not_fit():
-    """R7 / reading A-19: a buffer that would take more than half the heap
-    is not prefilled (a 64 MB heap cannot hold one block of every class for
-    every slot): the initial image is pristine."""
+    """R7 / reading A-19: a buffer that cannot fit in nseg / 8 segments even
+    at one block per slot is not prefilled (a 64 MB heap cannot hold one
+    block of every class for every slot): the initial image is pristine."""
     a = runs(4, slot_base=148, slot_min=4, run_max=256, run_init=1, prefill=1)
     assert np.array_equal(a.image(), pristine_image(4, 302))
 
