@@ -69,21 +69,16 @@ class PolSim:
 
     def prefill(self):
         """R7 ("always populated"): slot q of class c holds blocks
-        [q r, (q+1) r) of the class's segments, the classes' segments laid out
-        one after another from segment 0; the class's partly used last segment
-        keeps the rest, ascending, in its ring.  r = the largest power of two
-        <= the first run, then the class with the most segments (lowest on
-        ties, r > 1) halved until all fits in nseg / 8 segments (else none)."""
+        [q r, (q+1) r) of the class's segments, r = the largest power of two
+        <= its first run; the classes' segments laid out one after another
+        from segment 0; the class's partly used last segment keeps the rest,
+        ascending, in its ring -- if it all fits in nseg / 8 segments."""
         r = [1 << (self.first_run(c).bit_length() - 1) for c in range(TREES)]
 
         def segs(c):
             return -(-self.nslot[c] * r[c] // nb(c))
-        while sum(segs(c) for c in range(TREES)) > self.nseg // 8:
-            cand = [c for c in range(TREES) if r[c] > 1]
-            if not cand:
-                return
-            big = max(cand, key=lambda c: (segs(c), -c))
-            r[big] //= 2
+        if sum(segs(c) for c in range(TREES)) > self.nseg // 8:
+            return
         base = 0
         for c in range(TREES):
             for s in range(base, base + segs(c)):

@@ -76,11 +76,11 @@ def test_serialized_replay_matches_oracle(cuda_ok, G, seed, nseg, run_max, fa):
 
 
 @pytest.mark.parametrize("seed,nseg,run_max,fa,ri,rg", [(21, 96, 1, 0, 1, 1), (22, 128, 16, 1, 4, 1),
-                                                        (23, 160, 256, 1, 16, 3), (24, 96, 512, 0, 256, 3)])
+                                                        (23, 160, 256, 1, 16, 3), (24, 256, 512, 0, 64, 3)])
 def test_serialized_replay_prefilled(cuda_ok, G, seed, nseg, run_max, fa, ri, rg):
     """A prefilled block buffer ("always populated", O2-R R7): init and
     the replay's drains leave the state O2-R reaches; at the paper's one-block
-    knobs (first case) and with runs (the last one halved to fit nseg / 8)."""
+    knobs (first case) and with runs."""
     kinds, args, keys = wg.replay_ops(6000, seed + 100, p_free=0.45, p_drain=0.003, nkeys=64)
     _replay_case(G, nseg, run_max, fa, kinds, args, keys, pf=False, run_init=ri, run_grow=rg, prefill=True)
 
@@ -88,7 +88,7 @@ def test_serialized_replay_prefilled(cuda_ok, G, seed, nseg, run_max, fa, ri, rg
 def test_reset_prefills_block_buffer(cuda_ok, G):
     """gallatin_reset with the prefill knob (default) leaves exactly O2-R's
     prefilled initial state (R7); drain turns it into the pristine image."""
-    nseg = 1024
+    nseg = 4096                                    # 64 GB: the first runs fit in nseg / 8
     G.gallatin_init(nseg * SEG)
     st = G.gallatin_stats()
     assert st["prefill_segments"] > 0
@@ -136,7 +136,6 @@ def test_serialized_replay_default_knobs(cuda_ok, G):
     nseg = 64
     kinds, args, keys = wg.replay_ops(8000, 141, p_free=0.45, p_drain=0.002, nkeys=148 * 4)
     G.gallatin_init(nseg * SEG, oom_record=2)
-    assert G.gallatin_stats()["prefill_segments"] > 0          # the production default fills the buffer
     st = G.gallatin_stats()
     assert st["slot_base"] == 148 and st["run_max"] == 256 and st["format_ahead"] == 1 and st["run_grow"] == 3
     out = _u64(G.gallatin_replay(_dev(kinds, np.uint8), _dev(args), _dev(keys)))

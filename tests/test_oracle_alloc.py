@@ -373,7 +373,7 @@ def test_prefill_layout_closed_form():
     8, 4, 2, 1 (R1), laid out class by class from segment 0: 4 slots of 16 B
     fill segment 0; 2 slots x 32 of the 128 32-B blocks use half of segment 1,
     whose other 64 blocks stay in its ring (ascending) and block tree 1; ...;
-    13 segments in all (<= 128 / 8: no halving), the rest free.  The first
+    13 segments in all (<= 128 / 8), the rest free.  The first
     16 B request of slot 1 lands at block 64 of segment 0."""
     a = runs(128, slot_base=4, slot_min=2, run_max=512, run_bytes=1 << 30, run_init=64, prefill=1)
     d = image_sections(a.image())
@@ -397,26 +397,25 @@ def test_prefill_layout_closed_form():
     assert np.array_equal(a.image(), pristine_image(128, 20))
 
 
-def test_prefill_halves_the_largest_class_to_fit():
-    """R7's budget: runs start at the largest power of two <= the first run
-    (256 blocks at 16 B: 2 slots = 2 segments, one segment for each other
-    class: 10 in all); on a 72-segment heap (budget 72 / 8 = 9) the class
-    with the most segments -- 16 B -- is halved once: 2 x 128 blocks in
-    segment 0, classes 1..8 in segments 1..8."""
-    a = runs(72, slot_base=2, slot_min=1, run_max=512, run_bytes=1 << 30, run_init=256, prefill=1)
-    d = image_sections(a.image())
-    assert [int(w) for w in d["slots"][:2]] == [128 << 22, (128 << 22) | 128]
-    assert [int(w) >> 32 for w in d["segword"][:10]] == list(range(9)) + [TREE_FREE]
-    assert int(d["slots"][2]) == (128 << 22) | 128                             # 32 B: 128 blocks of segment 1
+def test_prefill_budget():
+    """R7's budget: the buffer is filled only if the runs fit in nseg / 8
+    segments.  Runs of the largest power of two <= the first run: 256 blocks
+    at 16 B (2 slots = 2 segments), one segment for each other class: 10 in
+    all -- an 80-segment heap (budget 10) fills it, with 16 B slot 1 at block
+    256 (segment 1); a 72-segment heap (budget 9) does not."""
     b = runs(80, slot_base=2, slot_min=1, run_max=512, run_bytes=1 << 30, run_init=256, prefill=1)
-    assert int(image_sections(b.image())["slots"][1]) == (256 << 22) | 256   # budget 10: no halving
-    c = runs(64, slot_base=2, slot_min=1, run_max=512, run_bytes=1 << 30, run_init=256, prefill=1)
-    assert np.array_equal(c.image(), pristine_image(64, 10))                  # 9 segments at least: none
+    d = image_sections(b.image())
+    assert [int(w) for w in d["slots"][:2]] == [256 << 22, (256 << 22) | 256]
+    assert [int(w) >> 32 for w in d["segword"][:11]] == [0, 0] + list(range(1, 9)) + [TREE_FREE]
+    c = runs(72, slot_base=2, slot_min=1, run_max=512, run_bytes=1 << 30, run_init=256, prefill=1)
+    assert np.array_equal(c.image(), pristine_image(72, 10))
+    e = runs(80, slot_base=2, slot_min=1, run_max=100, run_bytes=1 << 30, run_init=256, prefill=1)
+    assert int(image_sections(e.image())["slots"][0]) >> 22 == 64                # 100 -> 64 (power of two)
 
 
 def test_prefill_skipped_when_it_does_not_fit():
-    """R7 / reading A-19: a buffer that cannot fit in nseg / 8 segments even
-    at one block per slot is not prefilled (a 64 MB heap cannot hold one
+    """R7 / reading A-19: a buffer that does not fit in nseg / 8 segments is
+    not prefilled (a 64 MB heap cannot hold one
     block of every class for every slot): the initial image is pristine."""
     a = runs(4, slot_base=148, slot_min=4, run_max=256, run_init=1, prefill=1)
     assert np.array_equal(a.image(), pristine_image(4, 302))
