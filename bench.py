@@ -647,7 +647,7 @@ def run_paper_modes(args, G, torch):
     # fragmentation with the default knobs (runs of blocks per slot) and with
     # the paper's one-block buffer (run_max = run_init = 1, no format-ahead)
     out["fragmentation"] = {"n": (1 << 20) // args.scale}
-    for name, knobs in (("default", {}), ("paper_policy", dict(run_max=1, run_init=1, format_ahead=2, prefetch=2))):
+    for name, knobs in (("default", {}), ("paper_policy", dict(run_max=1, run_init=1, format_ahead=2, prefetch=2, prefill=2))):
         G.gallatin_init(HEAP_C2, **knobs)
         frag = {}
         for size in SIZES:

@@ -206,17 +206,20 @@ __device__ inline __noinline__ uint32_t reclaim_idle(const View &v) {
     return n;
 }
 
-// [dev] A claimer that lost the race for a bit of a leaf word retries at one
-// of the free bits its failed RMW returned (`free`), the (ticket mod
-// popcount)-th: concurrent losers draw consecutive tickets from one counter,
-// so up to popcount of them aim at distinct bits (a hash would collide) and a
-// launch's burst of claims -- every slot refilling at once -- settles in a
-// round or two, while every claimer stays in the lowest word with free
-// segments (front-first packing).  kNone if `free` is empty.
-__device__ __forceinline__ uint64_t claim_retry_hint(const View &v, uint64_t wi, uint64_t free) {
-    if (free == 0) return kNone;
-    uint32_t r = atomicAdd(v.ticket, 1u) % (uint32_t)__popcll((long long)free);
-    uint64_t m = free;
+// [dev] A claimer that lost the race for a bit of leaf word `old` retries at a
+// pseudo-random bit among the free bits its failed RMW returned (seeded by the
+// thread and the attempt) instead of the next one up: k simultaneous claimers
+// -- every slot refilling at a launch's start -- then collide O(1) times each
+// instead of walking the word one loss at a time, and they stay in the lowest
+// word with free segments (front-first packing).  kNone if the word
+// had no free bit.
+__device__ __forceinline__ uint64_t claim_retry_hint(uint64_t wi, uint64_t old, uint32_t attempt) {
+    if (old == 0) return kNone;
+    const uint32_t tid = blockIdx.x * blockDim.x + threadIdx.x;
+    uint32_t h = (tid * 0x9E3779B1u) ^ (attempt * 0x85EBCA6Bu);
+    h ^= h >> 15;
+    uint32_t r = h % (uint32_t)__popcll((long long)old);
+    uint64_t m = old;
     for (; r; r--) m &= m - 1;                                // drop r lowest free bits
     return (wi << 6) + (uint64_t)(__ffsll((long long)m) - 1);
 }
@@ -275,8 +278,7 @@ __device__ inline __noinline__ uint64_t claim_front(const View &v) {
             ptx::fence_acq_rel();
             return s;
         }
-        ++attempt;
-        hint = claim_retry_hint(v, s >> 6, old);            // a free bit the lost RMW saw, same word
+        hint = claim_retry_hint(s >> 6, old, ++attempt);   // a free bit the lost RMW saw, same word
         from = ((s >> 6) + 1) << 6;
     }
 }
@@ -326,8 +328,7 @@ __device__ inline __noinline__ uint64_t claim_front_run(const View &v, uint32_t 
             // (concurrent windows then do not overlap)
             const uint32_t al = claim_align(kmax);
             const uint64_t fr = old & ~mask, at = fr & (al >= 64 ? 1ull : ~0ull / ((1ull << al) - 1));
-            ++attempt;
-            hint = claim_retry_hint(v, wi, at ? at : fr);
+            hint = claim_retry_hint(wi, at ? at : fr, ++attempt);
             from = (wi + 1) << 6;
             continue;
         }
@@ -617,8 +618,8 @@ __device__ inline __noinline__ uint32_t get_run_once(const View &v, uint32_t t, 
             btree_reconcile(v, t, s);
             oom_notify(v);
             from = s + 1;
-            ++attempt;
-            hint = claim_retry_hint(v, s >> 6, ptx::ld_relaxed(bt.w + bt.off[0] + (s >> 6)) & ~(1ull << (s & 63)));
+            hint = claim_retry_hint(s >> 6, ptx::ld_relaxed(bt.w + bt.off[0] + (s >> 6)) & ~(1ull << (s & 63)),
+                                    ++attempt);
             continue;
         }
         if (from != 0) {                                      // re-scan from the front once more

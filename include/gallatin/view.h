@@ -26,8 +26,6 @@
  *   oom         one 128 B line: word 0 = {epoch:32 | searchers:22 | flag:10}
  *               (the exhaustion record, DESIGN.md Deviations 11), word 1 + t =
  *               epoch + 1 at which block tree t was confirmed exhausted
- *   ticket      one 128 B line: a counter that spreads the retries of claimers
- *               that lost a race over the free bits they saw
  */
 #ifndef GALLATIN_VIEW_H_
 #define GALLATIN_VIEW_H_
@@ -51,7 +49,6 @@ struct gallatin_device_view {
     uint32_t *fmt_token;        /* 32 words (128 B) per tree                  */
     unsigned long long *err;
     uint64_t *oom;              /* exhaustion record (1 line)                  */
-    uint32_t *ticket;           /* claim tickets of losing claimers (1 line)   */
     uint32_t tree_levels;       /* L                                           */
     uint32_t tree_words;        /* W                                           */
     uint32_t level_off[GALLATIN_MAX_LEVELS];

@@ -212,21 +212,38 @@ static uint64_t malloc_slice(o2_t *a, uint32_t c, uint64_t key) {
 /* ---------------------------------------------------------- prefill --- */
 /* R7 prefill ("each block buffer is always populated", reading A-19):
  * the initial state has every slot, class-major and slot-ascending, holding
- * a run of r[c] consecutive blocks of its class, r[c] = the largest power of
- * two <= its first run (R1): the blocks of the class's current segment in
- * ring order (a fresh segment when it has none left), or r[c] / nb whole
- * fresh segments -- if the segments this takes fit in nseg / 8, else the
- * slots start empty. */
+ * a run of r[c] consecutive blocks of its class: the blocks of the class's
+ * current segment in ring order (a fresh segment when it has none left), or
+ * r[c] / nb whole fresh segments.  r[c] starts at the largest power of two
+ * <= the first run (R1); while the segments this takes exceed nseg / 8, the
+ * class holding the most segments (lowest class on ties) whose r[c] is above
+ * max(1, nb >> run_grow) is halved (so the slot's first refill still grows
+ * to whole segments); if none can be and it does not fit, the slots start
+ * empty. */
+static uint64_t prefill_segs(const o2_t *a, const uint32_t *r, unsigned c) {
+    return ((uint64_t)a->nslot[c] * r[c] + nb_of(c) - 1) / nb_of(c);
+}
+
 void runs_prefill(o2_t *a) {
     uint32_t r[NUM_BLOCK_TREES];
-    uint64_t total = 0;
     for (unsigned c = 0; c < NUM_BLOCK_TREES; c++) {
         uint32_t fr = runs_first_run(a, c);
         r[c] = 1;
         while (r[c] * 2 <= fr) r[c] *= 2;
-        total += ((uint64_t)a->nslot[c] * r[c] + nb_of(c) - 1) / nb_of(c);
     }
-    if (total > a->nseg / 8) return;
+    for (;;) {
+        uint64_t total = 0;
+        for (unsigned c = 0; c < NUM_BLOCK_TREES; c++) total += prefill_segs(a, r, c);
+        if (total <= a->nseg / 8) break;
+        int big = -1;
+        for (unsigned c = 0; c < NUM_BLOCK_TREES; c++) {
+            uint32_t floor_ = nb_of(c) >> a->run_grow;
+            if (floor_ < 1) floor_ = 1;
+            if (r[c] > floor_ && (big < 0 || prefill_segs(a, r, c) > prefill_segs(a, r, (unsigned)big))) big = (int)c;
+        }
+        if (big < 0) return;                                        /* does not fit: slots start empty */
+        r[big] /= 2;
+    }
     for (unsigned c = 0; c < NUM_BLOCK_TREES; c++) {
         uint32_t nb = nb_of(c);
         uint64_t s = NONE64;

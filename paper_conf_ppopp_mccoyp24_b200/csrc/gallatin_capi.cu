@@ -162,7 +162,6 @@ __global__ void k_reset() {
         if (i < 9 * 32) v.fmt_token[i] = 0;
         if (i == 0) *v.err = 0;
         if (i < 16) v.oom[i] = 0;
-        if (i == 0) *v.ticket = 0;
     }
 }
 
@@ -791,8 +790,8 @@ int gallatin_init_ex(const gallatin_config_t *cfg_in) {
     v.demand_hint = cfg.demand_hint == 2 ? 0u : 1u;
     v.oom_record = cfg.oom_record == 2 ? 0u : 1u;
     // prefilled block buffer (include/gallatin.h "prefill"): every
-    // slot's first run (rounded down to a power of two) laid out class by
-    // class, if all of it fits in nseg/8 segments
+    // slot's first run (rounded down to a power of two), shrunk to fit nseg/8
+    // segments, laid out class by class
     {
         uint32_t r[core::kTrees];
         for (uint32_t c = 0; c < core::kTrees; c++) {
@@ -804,6 +803,22 @@ int gallatin_init_ex(const gallatin_config_t *cfg_in) {
             r[c] = 1u << (31 - __builtin_clz(fr));                  // largest power of two <= fr
         }
         auto segs_of = [&](uint32_t c) { return ((uint64_t)v.nslot[c] * r[c] + (256u >> c) - 1) / (256u >> c); };
+        // over budget: halve the class holding the most segments (lowest class
+        // on ties) whose run is above max(1, nb >> run_grow) -- the refill
+        // after such a run grows to whole segments
+        bool fits = true;
+        for (;;) {
+            uint64_t total = 0;
+            for (uint32_t c = 0; c < core::kTrees; c++) total += segs_of(c);
+            if (total <= nseg / 8) break;
+            int big = -1;
+            for (uint32_t c = 0; c < core::kTrees; c++) {
+                const uint32_t floor_ = ((256u >> c) >> cfg.run_grow) > 1 ? ((256u >> c) >> cfg.run_grow) : 1u;
+                if (r[c] > floor_ && (big < 0 || segs_of(c) > segs_of((uint32_t)big))) big = (int)c;
+            }
+            if (big < 0) { fits = false; break; }
+            r[big] >>= 1;
+        }
         uint64_t seg = 0;
         for (uint32_t c = 0; c < core::kTrees; c++) {
             const uint32_t nb = 256u >> c;
@@ -814,14 +829,14 @@ int gallatin_init_ex(const gallatin_config_t *cfg_in) {
             v.pf_last[c] = v.pf_used[c] < nb ? (uint32_t)(seg + segs - 1) : 0xFFFFFFFFu;
             seg += segs;
         }
-        v.pf_segs = (cfg.prefill != 2 && seg <= nseg / 8) ? (uint32_t)seg : 0u;
+        v.pf_segs = (cfg.prefill != 2 && fits) ? (uint32_t)seg : 0u;
     }
 
     // metadata: one allocation, 256 B aligned sections
-    uint64_t sz[13] = {W * 8, 9 * W * 8, nseg * 8, nseg * 4, nseg * 4, nseg * 512, nseg * 1024,
-                       (uint64_t)off * 128, 9 * 128, 128, nseg * 4, 128, 128};
-    uint64_t total = 0, offs[13];
-    for (int i = 0; i < 13; i++) { offs[i] = total; total += align_up(sz[i], 256); }
+    uint64_t sz[12] = {W * 8, 9 * W * 8, nseg * 8, nseg * 4, nseg * 4, nseg * 512, nseg * 1024,
+                       (uint64_t)off * 128, 9 * 128, 128, nseg * 4, 128};
+    uint64_t total = 0, offs[12];
+    for (int i = 0; i < 12; i++) { offs[i] = total; total += align_up(sz[i], 256); }
     void *meta = nullptr;
     if (cudaMalloc(&meta, total) != cudaSuccess) { cudaGetLastError(); return GALLATIN_ERR_NOMEM; }
     void *heap = nullptr;
@@ -843,7 +858,6 @@ int gallatin_init_ex(const gallatin_config_t *cfg_in) {
     v.err = reinterpret_cast<unsigned long long *>(m + offs[9]);
     v.seg_tid = reinterpret_cast<uint32_t *>(m + offs[10]);
     v.oom = reinterpret_cast<uint64_t *>(m + offs[11]);
-    v.ticket = reinterpret_cast<uint32_t *>(m + offs[12]);
     v.heap = align_up(reinterpret_cast<uint64_t>(heap), core::kSegBytes);   // 16 MiB aligned base
 
     g.init = true;

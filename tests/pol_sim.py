@@ -69,16 +69,22 @@ class PolSim:
 
     def prefill(self):
         """R7 ("always populated"): slot q of class c holds blocks
-        [q r, (q+1) r) of the class's segments, r = the largest power of two
-        <= its first run; the classes' segments laid out one after another
-        from segment 0; the class's partly used last segment keeps the rest,
-        ascending, in its ring -- if it all fits in nseg / 8 segments."""
+        [q r, (q+1) r) of the class's segments, the classes' segments laid out
+        one after another from segment 0; the class's partly used last segment
+        keeps the rest, ascending, in its ring.  r = the largest power of two
+        <= the first run, then -- while it all exceeds nseg / 8 segments --
+        the class with the most segments (lowest on ties) whose r is above
+        max(1, nb >> run_grow) halved; if none can be, nothing is filled."""
         r = [1 << (self.first_run(c).bit_length() - 1) for c in range(TREES)]
 
         def segs(c):
             return -(-self.nslot[c] * r[c] // nb(c))
-        if sum(segs(c) for c in range(TREES)) > self.nseg // 8:
-            return
+        while sum(segs(c) for c in range(TREES)) > self.nseg // 8:
+            cand = [c for c in range(TREES) if r[c] > max(1, nb(c) >> self.grow)]
+            if not cand:
+                return
+            big = max(cand, key=lambda c: (segs(c), -c))
+            r[big] //= 2
         base = 0
         for c in range(TREES):
             for s in range(base, base + segs(c)):

@@ -398,17 +398,24 @@ def test_prefill_layout_closed_form():
 
 
 def test_prefill_budget():
-    """R7's budget: the buffer is filled only if the runs fit in nseg / 8
-    segments.  Runs of the largest power of two <= the first run: 256 blocks
-    at 16 B (2 slots = 2 segments), one segment for each other class: 10 in
-    all -- an 80-segment heap (budget 10) fills it, with 16 B slot 1 at block
-    256 (segment 1); a 72-segment heap (budget 9) does not."""
-    b = runs(80, slot_base=2, slot_min=1, run_max=512, run_bytes=1 << 30, run_init=256, prefill=1)
+    """R7's budget nseg / 8.  Runs start at the largest power of two <= the
+    first run: 256 blocks at 16 B (2 slots = 2 segments), one segment for
+    each other class: 10 in all.  An 80-segment heap (budget 10) takes them
+    as they are (16 B slot 1 at block 256 = segment 1).  On 72 segments
+    (budget 9) the class with the most segments -- 16 B -- is halved once,
+    to 128 >= 256 >> run_grow: both 16 B runs in segment 0.  With run_grow 1
+    the floor is 128 too; on 64 segments (budget 8) nothing can be halved
+    below the floors (each class still needs a segment): no prefill."""
+    b = runs(80, slot_base=2, slot_min=1, run_max=512, run_bytes=1 << 30, run_init=256, run_grow=3, prefill=1)
     d = image_sections(b.image())
     assert [int(w) for w in d["slots"][:2]] == [256 << 22, (256 << 22) | 256]
     assert [int(w) >> 32 for w in d["segword"][:11]] == [0, 0] + list(range(1, 9)) + [TREE_FREE]
-    c = runs(72, slot_base=2, slot_min=1, run_max=512, run_bytes=1 << 30, run_init=256, prefill=1)
-    assert np.array_equal(c.image(), pristine_image(72, 10))
+    h = runs(72, slot_base=2, slot_min=1, run_max=512, run_bytes=1 << 30, run_init=256, run_grow=3, prefill=1)
+    d = image_sections(h.image())
+    assert [int(w) for w in d["slots"][:2]] == [128 << 22, (128 << 22) | 128]
+    assert [int(w) >> 32 for w in d["segword"][:10]] == list(range(9)) + [TREE_FREE]
+    c = runs(64, slot_base=2, slot_min=1, run_max=512, run_bytes=1 << 30, run_init=256, run_grow=1, prefill=1)
+    assert np.array_equal(c.image(), pristine_image(64, 10))
     e = runs(80, slot_base=2, slot_min=1, run_max=100, run_bytes=1 << 30, run_init=256, prefill=1)
     assert int(image_sections(e.image())["slots"][0]) >> 22 == 64                # 100 -> 64 (power of two)
 

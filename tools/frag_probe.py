@@ -12,7 +12,7 @@ if os.environ.get("GALLATIN_PKG_ROOT"):
 import paper_conf_ppopp_mccoyp24_b200 as G  # noqa: E402
 from paper_conf_ppopp_mccoyp24_b200 import experiments as X  # noqa: E402
 
-for name, knobs in (("default", {}), ("paper_policy", dict(run_max=1, run_init=1, format_ahead=2, prefetch=2))):
+for name, knobs in (("default", {}), ("paper_policy", dict(run_max=1, run_init=1, format_ahead=2, prefetch=2, prefill=2))):
     G.gallatin_init(16 << 30, **knobs)
     out = {}
     for sz in [16 << i for i in range(9)]:
