@@ -245,55 +245,17 @@ __device__ __forceinline__ uint64_t claim_spread(uint64_t s, uint32_t attempt, u
     return (s & ~63ull) | b;
 }
 
-// [dev] Rank of an empty slot's first refill: the slot's index when many
-// threads run (a multi-thread launch), kNoRank in a single-thread launch
-// (serialized replay: exactly successor(0)) and for every later refill.  A
-// ranked claimer's FIRST attempt aims at the rank-th free segment counted up
-// from the lowest one (the lowest 8 leaf words, loaded together): the burst
-// of first refills at a cold launch's start -- every slot at once -- then
-// claims distinct segments in one round, packed at the front,
-// instead of all aiming at the lowest bit.  Lone later refills stay exact
-// front-first.
-constexpr uint32_t kNoRank = 0xFFFFFFFFu;
-__device__ __forceinline__ uint32_t launch_rank(uint32_t si) {
-    return (uint64_t)gridDim.x * blockDim.x > 1 ? si : kNoRank;
-}
-__device__ inline uint64_t claim_rank_target(const BitTree &st, uint64_t s0, uint64_t r) {
-    const uint64_t nw = (st.nbits + 63) / 64, wi = s0 >> 6;
-    uint64_t w[8];
-#pragma unroll
-    for (int q = 0; q < 8; q++) w[q] = wi + q < nw ? ptx::ld_relaxed(st.w + st.off[0] + wi + q) : 0ull;
-    w[0] &= ~0ull << (s0 & 63);
-    uint64_t total = 0;
-#pragma unroll
-    for (int q = 0; q < 8; q++) total += (uint64_t)__popcll((long long)w[q]);
-    if (total == 0) return s0;
-    r %= total;
-#pragma unroll
-    for (int q = 0; q < 8; q++) {
-        const uint64_t pc = (uint64_t)__popcll((long long)w[q]);
-        if (r < pc) {
-            uint64_t m = w[q];
-            for (; r; r--) m &= m - 1;
-            return ((wi + q) << 6) + (uint64_t)(__ffsll((long long)m) - 1);
-        }
-        r -= pc;
-    }
-    return s0;
-}
-
 // successor(0) on the segment tree + claimIndex, front first
 // (P:138).  Returns the claimed segment or kNone when every segment is in use.
 // A claimer that loses the race retries elsewhere (claim_retry_hint,
 // claim_spread; serially the first attempt always wins, so this is
 // successor(0)).
-__device__ inline __noinline__ uint64_t claim_front(const View &v, uint32_t rank = kNoRank) {
+__device__ inline __noinline__ uint64_t claim_front(const View &v) {
     const BitTree st = seg_tree(v);
     uint64_t from = 0, hint = kNone;
     uint32_t attempt = 0;
     for (;;) {
         uint64_t s = hint != kNone ? hint : bt_successor<false>(st, from);
-        if (attempt == 0 && rank != kNoRank && s != kNone && rank != 0) s = claim_rank_target(st, s, rank);
         if (hint == kNone && attempt > 0 && s != kNone) {
             s = claim_spread(s, attempt);
             if (s >= v.nseg) s = v.nseg - 1;
@@ -327,15 +289,12 @@ __device__ inline __noinline__ uint64_t claim_front(const View &v, uint32_t rank
 // s is kept and the rest given back.  Concurrent claimers then get disjoint
 // windows instead of interleaving single segments.  *k = segments claimed
 // (serially: s = successor(0) and the free segments that follow it).
-__device__ inline __noinline__ uint64_t claim_front_run(const View &v, uint32_t kmax, uint32_t *k,
-                                                        uint32_t rank = kNoRank) {
+__device__ inline __noinline__ uint64_t claim_front_run(const View &v, uint32_t kmax, uint32_t *k) {
     const BitTree st = seg_tree(v);
     uint64_t from = 0, hint = kNone;
     uint32_t attempt = 0;
     for (;;) {
         uint64_t s = hint != kNone ? hint : bt_successor<false>(st, from);
-        if (attempt == 0 && rank != kNoRank && s != kNone && rank != 0)
-            s = claim_rank_target(st, s, (uint64_t)rank * (kmax < 64 ? kmax : 64));
         if (hint == kNone && attempt > 0 && s != kNone) {
             s = claim_spread(s, attempt, kmax);
             if (s >= v.nseg) s = v.nseg - 1;
@@ -477,15 +436,14 @@ __device__ inline __noinline__ void format_ahead(const View &v, uint32_t t) {
 // [dev] A run covering whole segments takes up to want/nb fresh segments
 // privately (no ring, no block tree): the lowest free one and the free ones
 // that follow it.  Returns the blocks taken (0 if no segment is free).
-__device__ inline __noinline__ uint32_t take_segments(const View &v, uint32_t t, uint32_t want, uint32_t *first,
-                                                      uint32_t rank = kNoRank) {
+__device__ inline __noinline__ uint32_t take_segments(const View &v, uint32_t t, uint32_t want, uint32_t *first) {
     const uint32_t nb = nb_of(t);
     uint32_t k = 0;
     const uint32_t kmax = want / nb;
 #ifdef GALLATIN_TRACE
     const uint64_t tr0 = ptx::globaltimer();
 #endif
-    const uint64_t s0 = claim_front_run(v, kmax, &k, rank);
+    const uint64_t s0 = claim_front_run(v, kmax, &k);
     if (s0 == kNone) return 0;
 #ifdef GALLATIN_TRACE
     const uint32_t attempts = k >> 16;
@@ -552,7 +510,7 @@ __device__ inline __noinline__ bool flux_pending(const View &v, uint32_t t) {
 // -- checked only once the block tree came up empty, with the record loaded
 // at entry, so a refill that finds blocks pays no extra round trip.
 __device__ inline __noinline__ uint32_t get_run_once(const View &v, uint32_t t, uint32_t want, uint32_t *first,
-                                                     bool check_oom = false, uint32_t rank = kNoRank) {
+                                                     bool check_oom = false) {
     const uint64_t oom_r = check_oom ? ptx::ld_relaxed(v.oom) : 0, oom_rec = check_oom ? ptx::ld_relaxed(v.oom + 1 + t) : 0;
     const BitTree bt = block_tree(v, t);
     const uint32_t nb = nb_of(t);
@@ -569,7 +527,7 @@ __device__ inline __noinline__ uint32_t get_run_once(const View &v, uint32_t t, 
         // warm-state refills); serially exact with O2-R's R2
         if (s != kNone && want >= nb && sw_avail(ptx::ld_relaxed(v.seg_word + s)) < (int32_t)want &&
             bt_successor<false>(seg_tree(v), 0) != kNone) {
-            const uint32_t k = take_segments(v, t, want, first, rank);
+            const uint32_t k = take_segments(v, t, want, first);
             if (k) return k;
         }
         if (s != kNone) {
@@ -682,7 +640,7 @@ __device__ inline __noinline__ uint32_t get_run_once(const View &v, uint32_t t, 
             continue;
         }
         if (want >= nb) {
-            const uint32_t k = take_segments(v, t, want, first, rank);
+            const uint32_t k = take_segments(v, t, want, first);
             if (k || !flux_pending(v, t) || flux_retries >= kFluxRetries) return k;   // 0: "No allocations left"
             flux_retries++;
             bo.pause();
@@ -695,7 +653,7 @@ __device__ inline __noinline__ uint32_t get_run_once(const View &v, uint32_t t, 
                 token_release(tok);
                 continue;
             }
-            const uint64_t s1 = claim_front(v, rank);
+            const uint64_t s1 = claim_front(v);
             if (s1 != kNone) format_segment(v, s1, t, want);
             token_release(tok);
             if (s1 == kNone) {
@@ -761,15 +719,14 @@ __device__ inline __noinline__ uint32_t trim_slots(const View &v) {
 // concurrency the retry repeats while trims still find blocks, and once
 // more after an empty trim: a concurrent refiller's trim may just have given
 // the blocks back.  Serially this is one trim and one retry.
-__device__ inline __noinline__ uint32_t get_run(const View &v, uint32_t t, uint32_t want, uint32_t *first,
-                                                uint32_t rank = kNoRank) {
+__device__ inline __noinline__ uint32_t get_run(const View &v, uint32_t t, uint32_t want, uint32_t *first) {
     const bool rec = v.oom_record != 0;
 #ifdef GALLATIN_TRACE
     const uint64_t tr0 = ptx::globaltimer();
-    uint32_t got = get_run_once(v, t, want, first, rec, rank);
+    uint32_t got = get_run_once(v, t, want, first, rec);
     ptx::trace(tr0, ptx::globaltimer(), (3ull << 60) | ((uint64_t)t << 24) | (want << 12) | got);
 #else
-    uint32_t got = get_run_once(v, t, want, first, rec, rank);
+    uint32_t got = get_run_once(v, t, want, first, rec);
 #endif
     if (got || (rec && *first == kOomFast)) return got;       // [dev] exhaustion record
     oom_enter(v);
@@ -815,10 +772,10 @@ __device__ inline __noinline__ bool refill_slot(const View &v, uint32_t si, uint
     uint32_t first = 0;
 #ifdef GALLATIN_TRACE
     const uint64_t t0 = ptx::globaltimer();
-    const uint32_t got = get_run(v, c, want, &first, m_prev == 0 ? launch_rank(si) : kNoRank);
+    const uint32_t got = get_run(v, c, want, &first);
     ptx::trace(t0, ptx::globaltimer(), ((uint64_t)si << 32) | (c << 24) | (want << 12) | got);
 #else
-    const uint32_t got = get_run(v, c, want, &first, m_prev == 0 ? launch_rank(si) : kNoRank);
+    const uint32_t got = get_run(v, c, want, &first);
 #endif
     if (got == 0) {
         ptx::st_relaxed(slot_word(v, si) + 2, 1ull);        // waiters then consult the exhaustion record
