@@ -245,6 +245,26 @@ __device__ __forceinline__ uint64_t claim_spread(uint64_t s, uint32_t attempt, u
     return (s & ~63ull) | b;
 }
 
+// [dev] RUN claims only (a window of kmax >= 2 whole segments, a deviation
+// of ours): the FIRST loss means every concurrent claimer aimed at the same
+// lowest free window (a launch's burst of refills); the loser then aims at a
+// pseudo-random window boundary of the next kSpreadWords + kmax/2 leaf words
+// -- the RMW tells whether it was free -- instead of queueing on one word
+// (4 KB cell: 32 slots x 16-segment windows).  Single-segment claims (the
+// paper's GetSegment, formats) stay in the lowest word with free segments
+// (claim_retry_hint).  Serially no claim loses.
+constexpr uint32_t kSpreadWords = 4;
+__device__ __forceinline__ uint64_t claim_first_loss(const View &v, uint64_t wi, uint32_t kmax = 1) {
+    const uint32_t tid = blockIdx.x * blockDim.x + threadIdx.x;
+    uint32_t h = tid * 0x9E3779B1u;
+    h ^= h >> 13;
+    h *= 0x85EBCA6Bu;
+    h ^= h >> 16;
+    const uint32_t words = kSpreadWords + kmax / 2;            // room for the windows of every claimer
+    const uint64_t s = ((wi + h % words) << 6) | (((h >> 8) & 63) & ~(claim_align(kmax) - 1));
+    return s < v.nseg ? s : v.nseg - 1;
+}
+
 // successor(0) on the segment tree + claimIndex, front first
 // (P:138).  Returns the claimed segment or kNone when every segment is in use.
 // A claimer that loses the race retries elsewhere (claim_retry_hint,
@@ -325,10 +345,11 @@ __device__ inline __noinline__ uint64_t claim_front_run(const View &v, uint32_t 
         if (extra) oom_notify(v);
         if (run == 0) {
             // a free bit the lost RMW saw, at a window boundary if one is free
-            // (concurrent windows then do not overlap)
+            // (concurrent windows then do not overlap); a run claim's first
+            // loss spreads over the next words (claim_first_loss)
             const uint32_t al = claim_align(kmax);
             const uint64_t fr = old & ~mask, at = fr & (al >= 64 ? 1ull : ~0ull / ((1ull << al) - 1));
-            hint = claim_retry_hint(wi, at ? at : fr, ++attempt);
+            hint = (++attempt == 1 && kmax >= 2) ? claim_first_loss(v, wi, kmax) : claim_retry_hint(wi, at ? at : fr, attempt);
             from = (wi + 1) << 6;
             continue;
         }
