@@ -245,14 +245,14 @@ __device__ __forceinline__ uint64_t claim_spread(uint64_t s, uint32_t attempt, u
     return (s & ~63ull) | b;
 }
 
-// [dev] RUN claims only (a window of kmax >= 2 whole segments, a deviation
-// of ours): the FIRST loss means every concurrent claimer aimed at the same
-// lowest free window (a launch's burst of refills); the loser then aims at a
-// pseudo-random window boundary of the next kSpreadWords + kmax/2 leaf words
-// -- the RMW tells whether it was free -- instead of queueing on one word
-// (4 KB cell: 32 slots x 16-segment windows).  Single-segment claims (the
-// paper's GetSegment, formats) stay in the lowest word with free segments
-// (claim_retry_hint).  Serially no claim loses.
+// [dev] RUN claims only (claim_front_run: a slot's run of whole segments, a
+// deviation of ours): the FIRST loss means every concurrent claimer aimed at
+// the same lowest free window (a launch's burst of refills); the loser then
+// aims at a pseudo-random window boundary of the next kSpreadWords + kmax/2
+// leaf words -- the RMW tells whether it was free -- instead of queueing on
+// one word.  The paper's GetSegment (claim_front: formats) stays in the
+// lowest word with free segments (claim_retry_hint).  Serially no claim
+// loses.
 constexpr uint32_t kSpreadWords = 4;
 __device__ __forceinline__ uint64_t claim_first_loss(const View &v, uint64_t wi, uint32_t kmax = 1) {
     const uint32_t tid = blockIdx.x * blockDim.x + threadIdx.x;
@@ -349,7 +349,7 @@ __device__ inline __noinline__ uint64_t claim_front_run(const View &v, uint32_t 
             // loss spreads over the next words (claim_first_loss)
             const uint32_t al = claim_align(kmax);
             const uint64_t fr = old & ~mask, at = fr & (al >= 64 ? 1ull : ~0ull / ((1ull << al) - 1));
-            hint = (++attempt == 1 && kmax >= 2) ? claim_first_loss(v, wi, kmax) : claim_retry_hint(wi, at ? at : fr, attempt);
+            hint = ++attempt == 1 ? claim_first_loss(v, wi, kmax) : claim_retry_hint(wi, at ? at : fr, attempt);
             from = (wi + 1) << 6;
             continue;
         }
