@@ -72,6 +72,8 @@ def test_utilization_closed_form(cuda_ok, G, X, size):
 
 @pytest.mark.parametrize("size", [16, 256, 4096])
 def test_fragmentation_range(cuda_ok, G, X, size):
+    """E7 with the default knobs: every request granted, the range at least
+    the bytes requested and inside the heap, accounting exact, pristine after."""
     nseg = 1024
     G.gallatin_init(nseg * SEG)
     r = X.fragmentation(size, 1 << 20)
@@ -80,6 +82,24 @@ def test_fragmentation_range(cuda_ok, G, X, size):
     assert r["range_bytes"] < nseg * SEG
     usum, ubad = G.gallatin_usable(r["ptrs"], r["sizes"])
     assert ubad == 0 and usum == (1 << 20) * size
+    G.gallatin_free(r["ptrs"])
+    _pristine(G, nseg)
+
+
+def test_fragmentation_paper_policy_front_first(cuda_ok, G, X):
+    """E7 under the paper's one-block policy (run_max = run_init = 1, no
+    format-ahead, slots filled on demand): segments are claimed front first
+     even when 148 slots refill at once -- a loser retries among the
+    free bits its RMW returned, in the lowest word with free segments -- so
+    2^20 16-B requests (16 MB, one segment of slices) stay within the
+    segments the concurrent formatters (<= 32 tokens) and the slots' blocks
+    take: about one leaf word of 64 segments (bound: 80; round 1's spreading
+    over the next words reached 249 segments)."""
+    nseg = 1024
+    G.gallatin_init(nseg * SEG, run_max=1, run_init=1, format_ahead=2, prefetch=2, prefill=2)
+    r = X.fragmentation(16, 1 << 20)
+    assert r["nulls"] == 0
+    assert r["range_bytes"] < 80 * SEG, f"range {r['range_bytes'] / SEG:.1f} segments"
     G.gallatin_free(r["ptrs"])
     _pristine(G, nseg)
 

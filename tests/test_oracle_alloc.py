@@ -234,6 +234,36 @@ def test_o2_matches_brute_force_simulation(seed, nseg, sb, sm, knobs):
     assert (got == NONE).sum() > (kinds == 0).sum() // 20 or nseg >= 64     # OOM exercised on the tiny heaps
 
 
+@pytest.mark.parametrize("mutant", ["lifo_ring", "back_first_blocks", "tree_off_by_one"])
+def test_brute_force_simulation_detects_mutants(mutant, monkeypatch):
+    """The simulation pin has teeth: a plausible mistake in the policy -- a
+    LIFO ring (A-15), block segments taken from the back, a block
+    tree that drops segments with a single block available (off by one in
+    A-16) -- makes the simulation disagree with O2-P on the same op list."""
+    import pol_sim
+    from collections import deque
+
+    if mutant == "lifo_ring":
+        def return_block(self, s, j):
+            self.ring[s].appendleft(j)
+            if len(self.ring[s]) == pol_sim.nb(self.tree[s]):
+                self.tree[s] = pol_sim.FREE
+                self.ring[s] = deque()
+        monkeypatch.setattr(PolSim, "return_block", return_block)
+    elif mutant == "back_first_blocks":
+        monkeypatch.setattr(PolSim, "free_segs", lambda self: [s for s in range(self.nseg - 1, -1, -1)
+                                                               if self.tree[s] == pol_sim.FREE])
+    else:
+        monkeypatch.setattr(PolSim, "tree_segs", lambda self, t: [s for s in range(self.nseg) if self.tree[s] == t
+                                                                  and len(self.ring[s]) > 1])
+    kinds, args, keys = wg.replay_ops(4000, 11, p_free=0.45, p_drain=0.003, nkeys=64)
+    sim = PolSim(3, 16, 2)
+    a = oracle.Allocator(3, 16, 2)
+    same = np.array_equal(sim.replay(kinds, args, keys), a.replay(kinds, args, keys)) and \
+        np.array_equal(sim.image(), a.image())
+    assert not same, f"the {mutant} mutant went unnoticed"
+
+
 @pytest.mark.parametrize("seed,nseg", [(31, 3), (32, 8), (33, 32)])
 def test_runs_model_at_paper_knobs_equals_paper_core(seed, nseg):
     """O2-R with run_max = run_init = 1, no format-ahead, no prefetch is the
