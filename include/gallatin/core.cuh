@@ -724,10 +724,12 @@ __device__ inline __noinline__ uint32_t trim_slots(const View &v) {
                 back += m - m2;
                 break;
             }
-            if (v.prefetch) {
-                const uint64_t nx = ptx::atom_exch(sw + 1, kSlotEmpty);
-                for (uint32_t k = 0; k < run_len(nx); k++) block_freed(v, gid_of(c, (nx & kRunNone) + k), kSlices);
-                back += run_len(nx);
+            {                                                    // a prefetched run (not one in flight)
+                const uint64_t nx = ptx::ld_relaxed(sw + 1);
+                if (run_len(nx) != 0 && ptx::atom_cas(sw + 1, nx, kSlotEmpty) == nx) {
+                    for (uint32_t k = 0; k < run_len(nx); k++) block_freed(v, gid_of(c, (nx & kRunNone) + k), kSlices);
+                    back += run_len(nx);
+                }
             }
         }
     }
@@ -765,23 +767,17 @@ __device__ inline __noinline__ uint32_t get_run(const View &v, uint32_t t, uint3
 // Replace an exhausted run (Alg.3): the run doubles up to the class cap.
 // [dev] `hint` (bulk calls only): the blocks this slot's share of the launch
 // needs (DESIGN.md Deviations 10); the run is at least that long, up to the cap.
-__device__ inline __noinline__ bool refill_slot(const View &v, uint32_t si, uint32_t c, uint32_t m_prev,
-                                                uint32_t hint = 0) {
-    if (v.prefetch) {                                         // [dev] the prefetched run, if any
-        const uint64_t nx = ptx::atom_exch(slot_word(v, si) + 1, kSlotEmpty);
-        if (run_len(nx) != 0) {
-            ptx::st_relaxed(slot_word(v, si) + 2, 0ull);
-            ptx::atom_exch(slot_word(v, si), nx);               // {issued 0, run, first}
-            return true;
-        }
-    }
+// The length of a slot's next run: the first run (halves per class, floor
+// min(run_init, 8), at most one segment) or 2^run_grow times the last, up to
+// the class cap; [dev] at least `hint` blocks (the launch's demand, bulk
+// calls only), rounded up to whole segments above one segment.
+__device__ __forceinline__ uint32_t refill_want(const View &v, uint32_t c, uint32_t m_prev, uint32_t hint) {
     const uint32_t cap = v.run_cap[c];
-    // halves per class, floor min(run_init, 8), at most one segment (nb blocks)
     const uint32_t fl = v.run_init < 8 ? v.run_init : 8u;
     const uint32_t fs = (v.run_init >> c) > fl ? (v.run_init >> c) : fl;
     const uint32_t fr = fs < (256u >> c) ? fs : (256u >> c);
     const uint32_t first_run = fr < cap ? fr : cap;
-    const uint32_t grow = m_prev << v.run_grow;                   // x 2^run_grow per refill
+    const uint32_t grow = m_prev << v.run_grow;
     uint32_t want = m_prev == 0 ? first_run : (grow < cap ? grow : cap);
     if (hint > want) {
         // whole segments once the hint exceeds one (a run of more than nb
@@ -790,6 +786,32 @@ __device__ inline __noinline__ bool refill_slot(const View &v, uint32_t si, uint
         const uint32_t h = hint > nb ? (hint + nb - 1) / nb * nb : hint;
         want = h < cap ? h : cap;
     }
+    return want;
+}
+
+// slot word 1 while a demand prefetch is fetching the run (run length 0: the
+// drain and the trims see no blocks in it)
+constexpr uint64_t kSlotPending = 0x3FFFFEull;
+
+// Replace an exhausted run (Alg.3): the prefetched run if one is
+// waiting in word 1 (or being fetched: wait for it), else a new run.
+__device__ inline __noinline__ bool refill_slot(const View &v, uint32_t si, uint32_t c, uint32_t m_prev,
+                                                uint32_t hint = 0) {
+    {                                                         // [dev] the prefetched run, if any
+        uint64_t *w1 = slot_word(v, si) + 1;
+        uint64_t nx = ptx::ld_relaxed(w1);
+        ptx::Backoff bo(6, si);
+        while (nx == kSlotPending) {
+            bo.pause();
+            nx = ptx::ld_relaxed(w1);
+        }
+        if (run_len(nx) != 0 && ptx::atom_cas(w1, nx, kSlotEmpty) == nx) {
+            ptx::st_relaxed(slot_word(v, si) + 2, 0ull);
+            ptx::atom_exch(slot_word(v, si), nx);               // {issued 0, run, first}
+            return true;
+        }
+    }
+    const uint32_t want = refill_want(v, c, m_prev, hint);
     uint32_t first = 0;
 #ifdef GALLATIN_TRACE
     const uint64_t t0 = ptx::globaltimer();
@@ -822,6 +844,20 @@ __device__ inline __noinline__ void prefetch_slot(const View &v, uint32_t si, ui
     const uint64_t run = ((uint64_t)got << kRunShift) | first;
     if (ptx::atom_cas(slot_word(v, si) + 1, kSlotEmpty, run) != kSlotEmpty)
         for (uint32_t k = 0; k < got; k++) block_freed(v, gid_of(c, (uint64_t)first + k), kSlices);   // raced: give back
+}
+
+// [dev] Demand prefetch (bulk CTA kernel, DESIGN.md Deviations 19): a tile
+// whose slot RMW leaves the run shorter than the launch's estimated demand
+// on the slot fetches the next run into word 1 after its own stores -- one
+// tile per slot wins the EMPTY -> PENDING CAS -- so the run's end swaps it
+// in instead of stalling every CTA of the slot on a refill.
+__device__ inline __noinline__ void demand_prefetch(const View &v, uint32_t si, uint32_t c, uint32_t m,
+                                                    uint32_t hint) {
+    uint64_t *w1 = slot_word(v, si) + 1;
+    if (ptx::atom_cas(w1, kSlotEmpty, kSlotPending) != kSlotEmpty) return;
+    uint32_t first = 0;
+    const uint32_t got = get_run_once(v, c, refill_want(v, c, m, hint), &first);   // never trims other slots
+    ptx::atom_exch(w1, got ? (((uint64_t)got << kRunShift) | first) : kSlotEmpty);
 }
 
 __device__ __forceinline__ void *slice_ptr(const View &v, uint32_t c, uint64_t first, uint64_t idx) {

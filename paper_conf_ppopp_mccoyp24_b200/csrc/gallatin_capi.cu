@@ -347,11 +347,24 @@ __global__ void __launch_bounds__(NT, MINB) k_bulk_malloc_cta(const uint64_t *__
     // address of the run's slice 0, so an item's pointer is one shift-add
     __shared__ uint64_t lim_lo[core::kTrees];
     __shared__ uint64_t run_base[core::kTrees];
+    uint32_t pf_m = 0, pf_hint = 0;                       // demand prefetch duty (thread c < 9)
     if (threadIdx.x < core::kTrees && cnt[threadIdx.x]) {
         const uint32_t c = threadIdx.x;
         const uint64_t old = ptx::atom_add(core::slot_word(v, v.slot_off[c] + key % v.nslot[c]), (uint64_t)cnt[c] << 32);
-        lim_lo[c] = ((uint64_t)(core::run_len(old) << core::kSliceLog2) << 32) | (old >> 32);
+        const uint32_t limit = core::run_len(old) << core::kSliceLog2, issued = (uint32_t)(old >> 32) + cnt[c];
+        lim_lo[c] = ((uint64_t)limit << 32) | (old >> 32);
         run_base[c] = reinterpret_cast<uint64_t>(core::slice_ptr(v, c, old & core::kRunNone, 0));
+        if (v.demand_hint && issued < limit) {
+            // [dev] the launch's demand on this slot (this tile's count x
+            // tiles / slots) exceeds what is left of the run: fetch the next
+            // run now (after this tile's stores), not when the run runs out
+            const uint64_t demand = (uint64_t)cnt[c] * gridDim.x / v.nslot[c];
+            if (demand > limit - issued &&
+                ptx::ld_relaxed(core::slot_word(v, v.slot_off[c] + key % v.nslot[c]) + 1) == core::kSlotEmpty) {
+                pf_m = core::run_len(old);
+                pf_hint = (uint32_t)((demand + core::kSlices - 1) >> core::kSliceLog2);
+            }
+        }
     }
     __syncthreads();
     uint32_t slow = 0;
@@ -382,6 +395,10 @@ __global__ void __launch_bounds__(NT, MINB) k_bulk_malloc_cta(const uint64_t *__
             info[k >> 2] |= (uint64_t)code << (16 * (k & 3));
         }
         if (!(code & 0x1C00u) && (full || i < n)) __stcs(reinterpret_cast<unsigned long long *>(ptrs) + i, p);
+    }
+    if (pf_m) {                                        // before any of this thread's waits
+        const uint32_t c = threadIdx.x;
+        core::demand_prefetch(v, v.slot_off[c] + key % v.nslot[c], c, pf_m, pf_hint);
     }
     const unsigned callers = __ballot_sync(0xFFFFFFFFu, slow != 0);
     if (slow) {
