@@ -355,14 +355,16 @@ __global__ void __launch_bounds__(NT, MINB) k_bulk_malloc_cta(const uint64_t *__
         lim_lo[c] = ((uint64_t)limit << 32) | (old >> 32);
         run_base[c] = reinterpret_cast<uint64_t>(core::slice_ptr(v, c, old & core::kRunNone, 0));
         if (v.demand_hint && issued < limit) {
-            // [dev] the launch's demand on this slot (this tile's count x
-            // tiles / slots) exceeds what is left of the run: fetch the next
-            // run now (after this tile's stores), not when the run runs out
-            const uint64_t demand = (uint64_t)cnt[c] * gridDim.x / v.nslot[c];
-            if (demand > limit - issued &&
+            // [dev] what the rest of the launch will ask of this slot (this
+            // tile's count x the tiles not yet started / slots: CTAs start
+            // in index order) exceeds what is left of the run: fetch the
+            // missing blocks now (after this tile's stores), not when the
+            // run runs out
+            const uint64_t rest = (uint64_t)cnt[c] * (gridDim.x - blockIdx.x) / v.nslot[c];
+            if (rest > limit - issued &&
                 ptx::ld_relaxed(core::slot_word(v, v.slot_off[c] + key % v.nslot[c]) + 1) == core::kSlotEmpty) {
                 pf_m = core::run_len(old);
-                pf_hint = (uint32_t)((demand + core::kSlices - 1) >> core::kSliceLog2);
+                pf_hint = (uint32_t)((rest - (limit - issued) + core::kSlices - 1) >> core::kSliceLog2);
             }
         }
     }
