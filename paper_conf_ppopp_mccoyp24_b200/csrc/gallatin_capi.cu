@@ -360,8 +360,10 @@ __global__ void __launch_bounds__(NT, MINB) k_bulk_malloc_cta(const uint64_t *__
             // in index order) exceeds what is left of the run: fetch the
             // missing blocks now (after this tile's stores), not when the
             // run runs out
+            // -- at least a block short, and not in the launch's last quarter,
+            // where the fetch would only lengthen the tail
             const uint64_t rest = (uint64_t)cnt[c] * (gridDim.x - blockIdx.x) / v.nslot[c];
-            if (rest > limit - issued &&
+            if (rest >= (uint64_t)(limit - issued) + core::kSlices && blockIdx.x < gridDim.x - gridDim.x / 4 &&
                 ptx::ld_relaxed(core::slot_word(v, v.slot_off[c] + key % v.nslot[c]) + 1) == core::kSlotEmpty) {
                 pf_m = core::run_len(old);
                 pf_hint = (uint32_t)((rest - (limit - issued) + core::kSlices - 1) >> core::kSliceLog2);
