@@ -54,6 +54,7 @@ struct gallatin_device_view {
     uint32_t level_off[GALLATIN_MAX_LEVELS];
     uint32_t nslot[GALLATIN_NUM_TREES];
     uint32_t slot_off[GALLATIN_NUM_TREES];
+    float nslot_rcp[GALLATIN_NUM_TREES];  /* 1 / nslot (bulk demand estimates) */
     uint32_t nslot_total;
     uint32_t run_cap[GALLATIN_NUM_TREES];  /* max blocks per slot run, per class */
     uint32_t format_ahead;      /* 1 = format the next segment at nb/4 left   */

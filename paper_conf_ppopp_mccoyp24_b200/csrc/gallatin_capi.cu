@@ -347,27 +347,16 @@ __global__ void __launch_bounds__(NT, MINB) k_bulk_malloc_cta(const uint64_t *__
     // address of the run's slice 0, so an item's pointer is one shift-add
     __shared__ uint64_t lim_lo[core::kTrees];
     __shared__ uint64_t run_base[core::kTrees];
-    uint32_t pf_m = 0, pf_hint = 0;                       // demand prefetch duty (thread c < 9)
+    uint32_t pf_rem = 0, pf_m = 0;                        // thread c < 9: what is left of its run
     if (threadIdx.x < core::kTrees && cnt[threadIdx.x]) {
         const uint32_t c = threadIdx.x;
         const uint64_t old = ptx::atom_add(core::slot_word(v, v.slot_off[c] + key % v.nslot[c]), (uint64_t)cnt[c] << 32);
         const uint32_t limit = core::run_len(old) << core::kSliceLog2, issued = (uint32_t)(old >> 32) + cnt[c];
         lim_lo[c] = ((uint64_t)limit << 32) | (old >> 32);
         run_base[c] = reinterpret_cast<uint64_t>(core::slice_ptr(v, c, old & core::kRunNone, 0));
-        if (v.demand_hint && issued < limit) {
-            // [dev] what the rest of the launch will ask of this slot (this
-            // tile's count x the tiles not yet started / slots: CTAs start
-            // in index order) exceeds what is left of the run: fetch the
-            // missing blocks now (after this tile's stores), not when the
-            // run runs out
-            // -- at least a block short, and not in the launch's last quarter,
-            // where the fetch would only lengthen the tail
-            const uint64_t rest = (uint64_t)cnt[c] * (gridDim.x - blockIdx.x) / v.nslot[c];
-            if (rest >= (uint64_t)(limit - issued) + core::kSlices && blockIdx.x < gridDim.x - gridDim.x / 4 &&
-                ptx::ld_relaxed(core::slot_word(v, v.slot_off[c] + key % v.nslot[c]) + 1) == core::kSlotEmpty) {
-                pf_m = core::run_len(old);
-                pf_hint = (uint32_t)((rest - (limit - issued) + core::kSlices - 1) >> core::kSliceLog2);
-            }
+        if (issued < limit) {
+            pf_rem = limit - issued;
+            pf_m = core::run_len(old);
         }
     }
     __syncthreads();
@@ -400,9 +389,21 @@ __global__ void __launch_bounds__(NT, MINB) k_bulk_malloc_cta(const uint64_t *__
         }
         if (!(code & 0x1C00u) && (full || i < n)) __stcs(reinterpret_cast<unsigned long long *>(ptrs) + i, p);
     }
-    if (pf_m) {                                        // before any of this thread's waits
+    // [dev] demand prefetch (DESIGN.md Deviations 19): what the rest of the
+    // launch will ask of this slot (this tile's count x the tiles not yet
+    // started / slots -- CTAs start in index order) exceeds what is left of
+    // the run by a block or more, the run still covers 16+ tiles (a run about
+    // to end is refilled as usual) and the launch is not in its last quarter
+    // (the fetch would only lengthen the tail): fetch the missing blocks
+    // into the slot's second word now -- before this thread waits on anything
+    if (v.demand_hint && pf_rem >= 16u * cnt[threadIdx.x < core::kTrees ? threadIdx.x : 0] && pf_m &&
+        blockIdx.x < gridDim.x - gridDim.x / 4) {
         const uint32_t c = threadIdx.x;
-        core::demand_prefetch(v, v.slot_off[c] + key % v.nslot[c], c, pf_m, pf_hint);
+        const float rest = (float)cnt[c] * (float)(gridDim.x - blockIdx.x) * v.nslot_rcp[c];
+        if (rest >= (float)(pf_rem + core::kSlices) &&
+            ptx::ld_relaxed(core::slot_word(v, v.slot_off[c] + key % v.nslot[c]) + 1) == core::kSlotEmpty)
+            core::demand_prefetch(v, v.slot_off[c] + key % v.nslot[c], c, pf_m,
+                                  (uint32_t)((rest - (float)pf_rem) * (1.0f / core::kSlices)) + 1u);
     }
     const unsigned callers = __ballot_sync(0xFFFFFFFFu, slow != 0);
     if (slow) {
@@ -776,6 +777,7 @@ int gallatin_init_ex(const gallatin_config_t *cfg_in) {
         if (n < 1) n = 1;
         v.nslot[c] = n;
         v.slot_off[c] = off;
+        v.nslot_rcp[c] = 1.0f / (float)n;
         off += n;
     }
     v.nslot_total = off;
