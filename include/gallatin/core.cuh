@@ -337,7 +337,8 @@ __device__ inline __noinline__ uint64_t claim_front_run(const View &v, uint32_t 
         uint64_t *leaf = st.w + st.off[0] + wi;
         const uint64_t old = ptx::atom_and(leaf, ~mask);
         const uint64_t got = old & mask;
-        const uint32_t run = (uint32_t)__ffsll((long long)~(got >> lo)) - 1;   // 0 if s was lost
+        const uint64_t inv = ~(got >> lo);                 // 0 only if all 64 bits of a word were taken
+        const uint32_t run = inv ? (uint32_t)__ffsll((long long)inv) - 1 : 64u;   // 0 if s was lost
         const uint64_t extra = got & ~bit_range(lo, lo + run);
         bool flip = old != 0 && (old & ~mask) == 0;
         if (extra) flip |= ptx::atom_or(leaf, extra) == 0;
@@ -488,7 +489,8 @@ __device__ inline __noinline__ uint32_t take_segments(const View &v, uint32_t t,
         uint64_t *leaf = st.w + st.off[0] + wi;
         const uint64_t old = ptx::atom_and(leaf, ~mask);
         const uint64_t got = old & mask;
-        const uint32_t run = (uint32_t)__ffsll((long long)~(got >> lo)) - 1;   // prefix length
+        const uint64_t inv = ~(got >> lo);                 // 0 only if all 64 bits of a word were taken
+        const uint32_t run = inv ? (uint32_t)__ffsll((long long)inv) - 1 : 64u;   // prefix length
         const uint64_t extra = got & ~bit_range(lo, lo + run);
         bool flip = old != 0 && (old & ~mask) == 0;
         if (extra) flip |= ptx::atom_or(leaf, extra) == 0;
@@ -965,91 +967,6 @@ __device__ inline __noinline__ void *malloc_block(const View &v, uint32_t t) {
         pending &= ~served;
     }
     return res;
-}
-
-// ---- [dev] combined whole-block requests of the bulk calls (Deviations 20) --
-// A bulk call's (4 KB, 16 MB) requests do not each chain their own GetBlock
-// (a format queued on the tree's formatter tokens every nb requests): each
-// enqueues its output slot on its tree's queue; one leader per tree -- the
-// requester that wins the tree's lock -- serves everything queued with runs
-// of blocks (get_run for the whole backlog: whole segments at once when the
-// backlog covers them) and writes every requester's pointer; requesters wait
-// for their slot and take the lead whenever the lock is free and their entry
-// is still pending, so no entry is stranded.  One requester alone is exactly
-// GetBlock(t).  The serialized replay and the device API keep malloc_block.
-constexpr uint64_t kPtrPending = 1ull;          // never a valid (16 B aligned) pointer
-
-__device__ inline __noinline__ void bq_lead(const View &v, uint32_t t) {
-    uint32_t *tail = v.bq_ctl + t * 64, *lock = tail + 32, *head = tail + 33;
-    uint64_t *items = v.bq_item + (uint64_t)t * GALLATIN_BQ;
-    for (;;) {
-        if (atomicCAS(lock, 0u, 1u) != 0u) return;          // someone else leads
-        ptx::fence_acq_rel();
-        uint32_t h = ptx::ld_relaxed(head), tl = ptx::ld_relaxed(tail);
-        while (h != tl) {
-            uint32_t cnt = tl - h;
-            if (cnt > GALLATIN_BQ / 4) cnt = GALLATIN_BQ / 4;
-            uint32_t first = 0;
-            uint32_t got = get_run(v, t, cnt, &first);
-            const bool none = got == 0;                        // no memory: the whole batch gets NULL
-            if (none) got = cnt;
-            for (uint32_t j = 0; j < got; j++) {
-                uint64_t *e = items + ((h + j) & (GALLATIN_BQ - 1));
-                uint64_t slot = ptx::ld_relaxed(e);
-                ptx::Backoff wb(7, h + j);
-                while (slot == 0) {                            // its enqueue is in flight
-                    wb.pause();
-                    slot = ptx::ld_relaxed(e);
-                }
-                ptx::st_relaxed(e, 0ull);
-                uint64_t p = 0;
-                if (!none) {
-                    atomicExch(v.block_free + gid_of(t, (uint64_t)first + j), kSlices - 1);   // A-2
-                    p = v.heap + (((uint64_t)first + j) << (16 + t));
-                }
-                ptx::fence_acq_rel();                          // block counter before the pointer
-                ptx::st_relaxed(reinterpret_cast<uint64_t *>(slot), p);
-            }
-            h += got;
-            ptx::st_relaxed(head, h);
-            tl = ptx::ld_relaxed(tail);
-        }
-        ptx::fence_acq_rel();
-        atomicExch(lock, 0u);
-        ptx::fence_sc();                                       // pairs with an enqueuer's: one sees the other
-        if (ptx::ld_relaxed(tail) == h) return;
-    }
-}
-
-// Returns the block pointer (NULL: no memory); false if the queue was full
-// (the caller then runs malloc_block itself).
-__device__ inline __noinline__ bool combine_block(const View &v, uint32_t t, uint64_t *slot, void **res) {
-    uint32_t *tail = v.bq_ctl + t * 64, *lock = tail + 32, *head = tail + 33;
-    uint32_t pos = ptx::ld_relaxed(tail);
-    for (;;) {
-        if (pos - ptx::ld_relaxed(head) >= GALLATIN_BQ) return false;   // full
-        const uint32_t o = atomicCAS(tail, pos, pos + 1);
-        if (o == pos) break;
-        pos = o;
-    }
-    ptx::st_relaxed(slot, kPtrPending);
-    uint64_t *e = v.bq_item + (uint64_t)t * GALLATIN_BQ + (pos & (GALLATIN_BQ - 1));
-    ptx::Backoff wb(8, pos);
-    while (ptx::ld_relaxed(e) != 0) wb.pause();                 // the previous lap's entry is being consumed
-    ptx::fence_acq_rel();                                      // the pending mark before the entry
-    ptx::st_relaxed(e, reinterpret_cast<uint64_t>(slot));
-    ptx::fence_sc();
-    bq_lead(v, t);
-    ptx::Backoff bo(9, pos);
-    uint64_t p = ptx::ld_relaxed(slot);
-    while (p == kPtrPending) {
-        bo.pause();
-        if (ptx::ld_relaxed(lock) == 0) bq_lead(v, t);        // nobody leads: serve the backlog
-        p = ptx::ld_relaxed(slot);
-    }
-    ptx::fence_acq_rel();
-    *res = reinterpret_cast<void *>(p);
-    return true;
 }
 
 // >= 16 MB: Alg.1 with treeId >= numBlockTrees: claimMultiple from the back

@@ -23,9 +23,6 @@
  *               word 2 = 1 if the slot's last refill found no memory
  *   fmt_token   9 x 128 B lines: one formatter per block tree
  *   err         u64 error counter (bad frees)
- *   bq_ctl/item whole-block request queues of the bulk calls, one per block
- *               tree (DESIGN.md Deviations 20): tail / lock / head words and
- *               GALLATIN_BQ entries (the requester's output slot address)
  *   oom         one 128 B line: word 0 = {epoch:32 | searchers:22 | flag:10}
  *               (the exhaustion record, DESIGN.md Deviations 11), word 1 + t =
  *               epoch + 1 at which block tree t was confirmed exhausted
@@ -36,7 +33,6 @@
 
 #define GALLATIN_NUM_TREES 9
 #define GALLATIN_MAX_LEVELS 8
-#define GALLATIN_BQ 16384       /* whole-block request queue entries per block tree (bulk calls) */
 
 struct gallatin_device_view {
     uint64_t heap;              /* device address of segment 0                */
@@ -53,8 +49,6 @@ struct gallatin_device_view {
     uint32_t *fmt_token;        /* 32 words (128 B) per tree                  */
     unsigned long long *err;
     uint64_t *oom;              /* exhaustion record (1 line)                  */
-    uint32_t *bq_ctl;           /* per block tree 64 words: [0] tail, [32] lock, [33] head */
-    uint64_t *bq_item;          /* per block tree GALLATIN_BQ entries: the requester's output slot */
     uint32_t tree_levels;       /* L                                           */
     uint32_t tree_words;        /* W                                           */
     uint32_t level_off[GALLATIN_MAX_LEVELS];

@@ -91,10 +91,7 @@ __global__ void k_reset() {
     if (S * 16 > total) total = S * 16;
     if (9 * W > total) total = 9 * W;
     if (9 * 32 > total) total = 9 * 32;
-    if (9ull * GALLATIN_BQ > total) total = 9ull * GALLATIN_BQ;
     for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < total; i += stride) {
-        if (i < 9ull * GALLATIN_BQ) v.bq_item[i] = 0;
-        if (i < 9 * 64) v.bq_ctl[i] = 0;
         if (i < W) {
             // segment tree: leaf bit s set iff pf <= s < nseg; a summary bit
             // set iff its child covers such a segment
@@ -209,13 +206,7 @@ __device__ __noinline__ void bulk_malloc_slow(const uint64_t *sizes, void **ptrs
         const uint64_t sz = sizes[i];
         void *p;
         if (code & 0x800u) {
-            // whole blocks through the tree's request queue (Deviations 20)
-            if (sz > core::kMaxSlice && sz < core::kSegBytes) {
-                if (!core::combine_block(v, core::block_class(sz), reinterpret_cast<uint64_t *>(ptrs) + i, &p))
-                    p = core::malloc_impl(v, sz, key);
-            } else {
-                p = core::malloc_impl(v, sz, key);
-            }
+            p = core::malloc_impl(v, sz, key);
         } else {
             const uint32_t c = core::slice_class(sz);
             if (code & 0x1000u) core::slot_exhausted(v, v.slot_off[c] + key % v.nslot[c], c, 0, ~0u);  // wait
@@ -865,10 +856,10 @@ int gallatin_init_ex(const gallatin_config_t *cfg_in) {
     }
 
     // metadata: one allocation, 256 B aligned sections
-    uint64_t sz[14] = {W * 8, 9 * W * 8, nseg * 8, nseg * 4, nseg * 4, nseg * 512, nseg * 1024,
-                       (uint64_t)off * 128, 9 * 128, 128, nseg * 4, 128, 9 * 256, 9ull * GALLATIN_BQ * 8};
-    uint64_t total = 0, offs[14];
-    for (int i = 0; i < 14; i++) { offs[i] = total; total += align_up(sz[i], 256); }
+    uint64_t sz[12] = {W * 8, 9 * W * 8, nseg * 8, nseg * 4, nseg * 4, nseg * 512, nseg * 1024,
+                       (uint64_t)off * 128, 9 * 128, 128, nseg * 4, 128};
+    uint64_t total = 0, offs[12];
+    for (int i = 0; i < 12; i++) { offs[i] = total; total += align_up(sz[i], 256); }
     void *meta = nullptr;
     if (cudaMalloc(&meta, total) != cudaSuccess) { cudaGetLastError(); return GALLATIN_ERR_NOMEM; }
     void *heap = nullptr;
@@ -890,8 +881,6 @@ int gallatin_init_ex(const gallatin_config_t *cfg_in) {
     v.err = reinterpret_cast<unsigned long long *>(m + offs[9]);
     v.seg_tid = reinterpret_cast<uint32_t *>(m + offs[10]);
     v.oom = reinterpret_cast<uint64_t *>(m + offs[11]);
-    v.bq_ctl = reinterpret_cast<uint32_t *>(m + offs[12]);
-    v.bq_item = reinterpret_cast<uint64_t *>(m + offs[13]);
     v.heap = align_up(reinterpret_cast<uint64_t>(heap), core::kSegBytes);   // 16 MiB aligned base
 
     g.init = true;
@@ -924,7 +913,6 @@ int gallatin_reset(void *stream) {
     if (!g.init) return GALLATIN_ERR_STATE;
     uint64_t n = g.v.nseg * 128;
     if ((uint64_t)g.v.nslot_total * 16 > n) n = (uint64_t)g.v.nslot_total * 16;
-    if (9ull * GALLATIN_BQ > n) n = 9ull * GALLATIN_BQ;
     unsigned grid = grid_for(n);
     if (grid > 148 * 16) grid = 148 * 16;
     k_reset<<<grid, kThreads, 0, S(stream)>>>();

@@ -100,6 +100,24 @@ def test_reset_prefills_block_buffer(cuda_ok, G):
     _assert_pristine(G, nseg)
 
 
+def test_serialized_replay_full_word_window(cuda_ok, G):
+    """A run of 64 whole segments claimed at a leaf-word boundary (all 64 bits
+    of the word in one window): 64 slots of the 4 KB class take segments
+    0..63 with their first one-block runs, then slot 0 exhausts its block and
+    refills with a 64-segment run (growth 2^6) -- segments 64..127.  (A round-1
+    bug read such a window's consecutive prefix as 2^16 - 1 segments.)"""
+    nseg = 256
+    n1, n2 = 64, 4096 + 3
+    kinds = np.zeros(n1 + n2 + 2, dtype=np.uint8)
+    args = np.full(n1 + n2 + 2, 4096, dtype=np.uint64)
+    keys = np.concatenate([np.arange(n1), np.zeros(n2 + 2, dtype=np.int64)]).astype(np.uint64)
+    kinds[-2], args[-2] = 1, n1 + n2 - 1                   # free the first slice of the 64-segment run
+    kinds[-1], args[-1] = 2, 0                             # drain
+    out = _replay_case(G, nseg, 512, False, kinds, args, keys, slot_base=64, slot_min=64, run_bytes=64 << 24,
+                       pf=False, run_init=1, run_grow=6)
+    assert out[n1 + n2 - 1] == 64 * SEG + 3 * 4096         # the 4th slice of slot 0's run at segment 64
+
+
 def test_serialized_replay_block_boundaries(cuda_ok, G):
     """Exactly-full blocks and runs, exhausted slots and refills with a single
     slot per class (every request hits the same slot)."""
