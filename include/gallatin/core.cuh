@@ -800,6 +800,9 @@ constexpr uint64_t kSlotPending = 0x3FFFFEull;
 __device__ inline __noinline__ bool refill_slot(const View &v, uint32_t si, uint32_t c, uint32_t m_prev,
                                                 uint32_t hint = 0) {
     {                                                         // [dev] the prefetched run, if any
+#ifdef GALLATIN_TRACE
+        const uint64_t ts0 = ptx::globaltimer();
+#endif
         uint64_t *w1 = slot_word(v, si) + 1;
         uint64_t nx = ptx::ld_relaxed(w1);
         ptx::Backoff bo(6, si);
@@ -810,6 +813,9 @@ __device__ inline __noinline__ bool refill_slot(const View &v, uint32_t si, uint
         if (run_len(nx) != 0 && ptx::atom_cas(w1, nx, kSlotEmpty) == nx) {
             ptx::st_relaxed(slot_word(v, si) + 2, 0ull);
             ptx::atom_exch(slot_word(v, si), nx);               // {issued 0, run, first}
+#ifdef GALLATIN_TRACE
+            ptx::trace(ts0, ptx::globaltimer(), (11ull << 60) | ((uint64_t)si << 32) | run_len(nx));
+#endif
             return true;
         }
     }
@@ -881,6 +887,16 @@ __device__ inline __noinline__ bool slot_exhausted(const View &v, uint32_t si, u
     const uint32_t m = run_len(old);
     if (idx == (m << kSliceLog2)) return refill_slot(v, si, c, m);
     ptx::Backoff bo(1, si);
+#ifdef GALLATIN_TRACE
+    const uint64_t tw0 = ptx::globaltimer();
+    struct TraceEnd {
+        uint64_t t0, si;
+        __device__ ~TraceEnd() {
+            if ((threadIdx.x & 31) == (uint32_t)(__ffs((int)__activemask()) - 1))
+                ptx::trace(t0, ptx::globaltimer(), (10ull << 60) | (si << 32));
+        }
+    } trace_end{tw0, si};
+#endif
     for (;;) {
         // the slot word and its failed-refill flag share a sector (one round trip)
         const uint64_t w = ptx::ld_relaxed(slot_word(v, si));

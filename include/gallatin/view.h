@@ -65,6 +65,7 @@ struct gallatin_device_view {
     uint32_t run_grow;          /* log2 of the run growth factor per refill    */
     uint32_t demand_hint;       /* 1 = bulk refills sized to the launch's demand */
     uint32_t oom_record;        /* 1 = exhaustion record on (DESIGN.md Deviations 11) */
+    uint32_t nsm;               /* SMs of the device (slot keys are %smid mod nslot) */
     /* prefilled block buffer ("always populated"; reading A-19):
      * 0 segments = reset leaves every slot empty; else class c's slots hold
      * runs of pf_run[c] blocks laid out from segment pf_base[c] on, slot q at

@@ -285,6 +285,116 @@ __global__ void __launch_bounds__(kThreads, 5) k_bulk_malloc(const uint64_t *__r
     if (slow) bulk_malloc_slow(sizes, ptrs, n, base, key, slow, &info, ITEMS, callers);
 }
 
+// The slow remainder of one k_bulk_malloc_cta tile (called by every thread
+// of the tile, or by none).  Thread c_me < 9 serves class c_me: its slot si,
+// the tile's my_cnt requests of the class, the RMW's lo/run (my_lo, my_m),
+// duty = this tile drew the run's end.
+template <int ITEMS, int NT>
+__device__ __noinline__ void tile_slow(const uint64_t *sizes, void **ptrs, uint64_t base, uint32_t key,
+                                       const uint32_t *cr, uint32_t pend, uint32_t big, uint32_t pfd,
+                                       const uint32_t *cnt, uint64_t *lim_lo, uint64_t *run_base, uint32_t *roff,
+                                       uint32_t *failed) {
+    const View &v = c_view;
+    // [dev] prefetch duties (knob prefetch=1): the item that drew the middle of a run
+    for (int k = 0; k < ITEMS; k++) {
+        if (!((pfd >> k) & 1)) continue;
+        const uint32_t c = cr[k] & 0xFFu;
+        core::prefetch_slot(v, v.slot_off[c] + key % v.nslot[c], c, (uint32_t)(lim_lo[c] >> 32) >> core::kSliceLog2);
+    }
+    const uint32_t c_me = (threadIdx.x & 31) * (NT / 32) + (threadIdx.x >> 5);
+    const bool cls_thread = c_me < core::kTrees;
+    uint32_t my_cnt = cls_thread ? cnt[c_me] : 0u;
+    const uint64_t ll0 = my_cnt ? lim_lo[c_me] : 0ull;
+    uint32_t my_lo = (uint32_t)ll0, my_limit = (uint32_t)(ll0 >> 32), my_m = my_limit >> core::kSliceLog2;
+    const uint32_t si = cls_thread ? v.slot_off[c_me] + key % v.nslot[c_me] : 0u;
+    bool duty = my_cnt && my_lo <= my_limit && my_limit < my_lo + my_cnt;
+    // Refill duty (Alg.3: the request that draws the end replaces
+    // the run) -- discharged by the class thread before it ever waits, so no
+    // tile waits on a refill while holding one.  [dev] The refill is sized to
+    // this slot's share of the launch (demand hint, DESIGN.md Deviations 10).
+    bool dutyfail = false;
+    const uint32_t hint_of = cls_thread && v.demand_hint
+                                 ? (uint32_t)(((uint64_t)my_cnt * gridDim.x / v.nslot[c_me] + core::kSlices - 1) >>
+                                              core::kSliceLog2)
+                                 : 0u;
+    if (duty) dutyfail = !core::refill_slot(v, si, c_me, my_m, hint_of);
+    // [dev] demand prefetch (DESIGN.md Deviations 19): what the rest of the
+    // launch will ask of this slot (this tile's count x the tiles not yet
+    // started / slots -- CTAs start in index order) exceeds what is left of
+    // the run by a block or more, the run still covers 16+ tiles (a run about
+    // to end is refilled as usual) and the launch is not in its last quarter
+    // (the fetch would only lengthen the tail): fetch the missing blocks
+    // into the slot's second word now -- before this thread waits on anything
+    if (cls_thread && v.demand_hint && my_cnt && my_lo + my_cnt < my_limit &&
+        my_limit - (my_lo + my_cnt) >= 16u * my_cnt && blockIdx.x < gridDim.x - gridDim.x / 4) {
+        const uint32_t pf_rem = my_limit - (my_lo + my_cnt);
+        const float rest = (float)my_cnt * (float)(gridDim.x - blockIdx.x) * v.nslot_rcp[c_me];
+        if (rest >= (float)(pf_rem + core::kSlices) && ptx::ld_relaxed(core::slot_word(v, si) + 1) == core::kSlotEmpty)
+            core::demand_prefetch(v, si, c_me, my_m, (uint32_t)((rest - (float)pf_rem) * (1.0f / core::kSlices)) + 1u);
+    }
+    // Rounds: the class thread retires what the last round served, waits for
+    // the slot's refill (another tile's duty), takes the tile's remaining
+    // requests of its class with ONE more RMW, and the items retry -- one RMW
+    // and one barrier per round for the whole tile, not one per warp and item.
+    bool still = my_cnt && (dutyfail || my_lo + my_cnt > my_limit);
+    while (__syncthreads_or(still)) {
+        duty = false;
+        if (still) {
+            const uint32_t served = my_lo < my_limit ? min(my_limit - my_lo, my_cnt) : 0u;
+            if (dutyfail) {
+                failed[c_me] = 1;                             // the team's refill found no memory
+                my_cnt = 0;
+            } else {
+                roff[c_me] += served;
+                my_cnt -= served;
+                // wait for the refill; false: tree c is recorded exhausted [dev]
+                if (!core::slot_exhausted(v, si, c_me, 0, ~0u)) {
+                    failed[c_me] = 1;
+                    my_cnt = 0;
+                } else {
+                    const uint64_t old = ptx::atom_add(core::slot_word(v, si), (uint64_t)my_cnt << 32);
+                    my_m = core::run_len(old);
+                    my_limit = my_m << core::kSliceLog2;
+                    my_lo = (uint32_t)(old >> 32);
+                    lim_lo[c_me] = ((uint64_t)my_limit << 32) | my_lo;
+                    run_base[c_me] = reinterpret_cast<uint64_t>(core::slice_ptr(v, c_me, old & core::kRunNone, 0));
+                    duty = my_lo <= my_limit && my_limit < my_lo + my_cnt;
+                }
+            }
+        }
+        __syncthreads();
+        for (int k = 0; k < ITEMS; k++) {
+            if (!((pend >> k) & 1)) continue;
+            const uint64_t i = base + (uint64_t)NT * k;
+            const uint32_t c = cr[k] & 0xFFu;
+            if (failed[c]) {
+                __stcs(reinterpret_cast<unsigned long long *>(ptrs) + i, 0ull);   // heap exhausted: NULL
+                pend &= ~(1u << k);
+                continue;
+            }
+            const uint64_t ll = lim_lo[c];
+            const uint32_t limit = (uint32_t)(ll >> 32);
+            const uint32_t idx = (uint32_t)ll + (cr[k] >> 8) - roff[c];
+            if (idx < limit) {
+                __stcs(reinterpret_cast<unsigned long long *>(ptrs) + i,
+                       run_base[c] + ((uint64_t)idx << (core::kMinSliceLog2 + c)));
+                pend &= ~(1u << k);
+            }
+        }
+        dutyfail = duty && !core::refill_slot(v, si, c_me, my_m, hint_of);
+        still = my_cnt && (dutyfail || my_lo + my_cnt > my_limit);
+    }
+    // whole blocks and segment runs: the device path, per lane
+    if (big) {
+        for (int k = 0; k < ITEMS; k++) {
+            if (!((big >> k) & 1)) continue;
+            const uint64_t i = base + (uint64_t)NT * k;
+            __stcs(reinterpret_cast<unsigned long long *>(ptrs) + i,
+                   reinterpret_cast<unsigned long long>(core::malloc_impl(v, sizes[i], key)));
+        }
+    }
+}
+
 // Bulk malloc with CTA-level aggregation: every warp of a CTA runs on one SM,
 // hence uses one block-buffer slot per class; the CTA's requests of a class
 // are counted in shared memory (one shared atomic per warp team) and ONE
@@ -299,10 +409,7 @@ __global__ void __launch_bounds__(NT, MINB) k_bulk_malloc_cta(const uint64_t *__
     const uint32_t lane = threadIdx.x & 31;
     const uint64_t base = blockIdx.x * (uint64_t)(NT * ITEMS) + threadIdx.x;
 #ifdef GALLATIN_TRACE
-    if (threadIdx.x == 0 && (blockIdx.x == 0 || blockIdx.x == gridDim.x - 1)) {
-        const uint64_t tk = ptx::globaltimer();
-        ptx::trace(tk, tk, (7ull << 60) | blockIdx.x);
-    }
+    const uint64_t tk0 = ptx::globaltimer();
 #endif
     const uint32_t key = ptx::smid();
     if (threadIdx.x < core::kTrees) cnt[threadIdx.x] = 0;
@@ -343,76 +450,80 @@ __global__ void __launch_bounds__(NT, MINB) k_bulk_malloc_cta(const uint64_t *__
         cr[k] = c | ((__shfl_sync(0xFFFFFFFFu, b, (int)leader) + (uint32_t)__popc(peers & lt)) << 8);
     }
     __syncthreads();
-    // per class: the slot RMW's {limit : 32 | first index : 32} and the
-    // address of the run's slice 0, so an item's pointer is one shift-add
+    // Class c is served by thread (c % warps) * 32 + c / warps (one per warp
+    // in turn: refills of different classes run in different warps).  Per
+    // class, shared: the slot RMW's {limit : 32 | first index : 32}, the
+    // address of the run's slice 0 (an item's pointer is one shift-add), the
+    // rank of the lowest request still unserved, and a failed flag.
     __shared__ uint64_t lim_lo[core::kTrees];
     __shared__ uint64_t run_base[core::kTrees];
-    uint32_t pf_rem = 0, pf_m = 0;                        // thread c < 9: what is left of its run
-    if (threadIdx.x < core::kTrees && cnt[threadIdx.x]) {
-        const uint32_t c = threadIdx.x;
-        const uint64_t old = ptx::atom_add(core::slot_word(v, v.slot_off[c] + key % v.nslot[c]), (uint64_t)cnt[c] << 32);
-        const uint32_t limit = core::run_len(old) << core::kSliceLog2, issued = (uint32_t)(old >> 32) + cnt[c];
-        lim_lo[c] = ((uint64_t)limit << 32) | (old >> 32);
-        run_base[c] = reinterpret_cast<uint64_t>(core::slice_ptr(v, c, old & core::kRunNone, 0));
-        if (issued < limit) {
-            pf_rem = limit - issued;
-            pf_m = core::run_len(old);
+    __shared__ uint32_t roff[core::kTrees];
+    __shared__ uint32_t failed[core::kTrees];
+    constexpr uint32_t NW = NT / 32;
+    const uint32_t c_me = lane * NW + (threadIdx.x >> 5);
+    const bool cls_thread = c_me < core::kTrees;
+    bool cls_slow = false;      // this class thread has a refill duty or a demand prefetch
+    if (cls_thread) {
+        roff[c_me] = 0;
+        failed[c_me] = 0;
+        const uint32_t my_cnt = cnt[c_me];
+        if (my_cnt) {
+            const uint64_t old = ptx::atom_add(core::slot_word(v, v.slot_off[c_me] + key % v.nslot[c_me]),
+                                               (uint64_t)my_cnt << 32);
+            const uint32_t my_limit = core::run_len(old) << core::kSliceLog2, my_lo = (uint32_t)(old >> 32);
+            lim_lo[c_me] = ((uint64_t)my_limit << 32) | my_lo;
+            run_base[c_me] = reinterpret_cast<uint64_t>(core::slice_ptr(v, c_me, old & core::kRunNone, 0));
+            cls_slow = my_lo + my_cnt > my_limit ||                  // requests past the run's end
+                       (v.prefetch && my_lo <= (my_limit >> 1) && (my_limit >> 1) < my_lo + my_cnt) ||
+                       (v.demand_hint && my_limit - (my_lo + my_cnt) >= 16u * my_cnt &&
+                        blockIdx.x < gridDim.x - gridDim.x / 4 &&
+                        (float)my_cnt * (float)(gridDim.x - blockIdx.x) * v.nslot_rcp[c_me] >=
+                            (float)(my_limit - (my_lo + my_cnt) + core::kSlices));   // demand prefetch (tile_slow)
         }
     }
-    __syncthreads();
-    uint32_t slow = 0;
-    uint64_t info[(ITEMS + 3) / 4];
+    bool big_any = false;
 #pragma unroll
-    for (int q = 0; q < (ITEMS + 3) / 4; q++) info[q] = 0;
+    for (int k = 0; k < ITEMS; k++) big_any |= (cr[k] & 0xFFu) == 0xFFu;
+    // the tile's slow remainder is known here, before any store: the fast
+    // path ends with its stores (no barrier behind them)
+    const bool slow_tile = __syncthreads_or(cls_slow || big_any);
+    // items whose slice lies inside the run are stored now; the rest wait in
+    // `pend` for the tile's next round (bit k: item k)
+    uint32_t pend = 0, big = 0, pfd = 0;
 #pragma unroll
     for (int k = 0; k < ITEMS; k++) {
         const uint64_t i = base + (uint64_t)NT * k;
         const uint32_t c = cr[k] & 0xFFu;
-        uint64_t p = 0;
-        uint32_t code = 0;
         if (c < core::kTrees) {
             const uint64_t ll = lim_lo[c];
             const uint32_t limit = (uint32_t)(ll >> 32);
             const uint32_t idx = (uint32_t)ll + (cr[k] >> 8);
             if (idx < limit) {
-                p = run_base[c] + ((uint64_t)idx << (core::kMinSliceLog2 + c));
-                if (v.prefetch && idx == (limit >> 1)) code = 0x2000u | (limit >> core::kSliceLog2);   // prefetch duty
+                __stcs(reinterpret_cast<unsigned long long *>(ptrs) + i,
+                       run_base[c] + ((uint64_t)idx << (core::kMinSliceLog2 + c)));
+                if (v.prefetch && idx == (limit >> 1)) pfd |= 1u << k;
             } else {
-                code = idx == limit ? (0x400u | (limit >> core::kSliceLog2)) : 0x1000u;
+                pend |= 1u << k;
             }
         } else if (c == 0xFFu) {
-            code = 0x800u;
+            big |= 1u << k;                                   // a whole block or segments
+        } else if (full || i < n) {
+            __stcs(reinterpret_cast<unsigned long long *>(ptrs) + i, 0ull);   // malloc(0): NULL
         }
-        if (code) {
-            slow |= 1u << k;
-            info[k >> 2] |= (uint64_t)code << (16 * (k & 3));
-        }
-        if (!(code & 0x1C00u) && (full || i < n)) __stcs(reinterpret_cast<unsigned long long *>(ptrs) + i, p);
     }
-    // [dev] demand prefetch (DESIGN.md Deviations 19): what the rest of the
-    // launch will ask of this slot (this tile's count x the tiles not yet
-    // started / slots -- CTAs start in index order) exceeds what is left of
-    // the run by a block or more, the run still covers 16+ tiles (a run about
-    // to end is refilled as usual) and the launch is not in its last quarter
-    // (the fetch would only lengthen the tail): fetch the missing blocks
-    // into the slot's second word now -- before this thread waits on anything
-    if (v.demand_hint && pf_rem >= 16u * cnt[threadIdx.x < core::kTrees ? threadIdx.x : 0] && pf_m &&
-        blockIdx.x < gridDim.x - gridDim.x / 4) {
-        const uint32_t c = threadIdx.x;
-        const float rest = (float)cnt[c] * (float)(gridDim.x - blockIdx.x) * v.nslot_rcp[c];
-        if (rest >= (float)(pf_rem + core::kSlices) &&
-            ptx::ld_relaxed(core::slot_word(v, v.slot_off[c] + key % v.nslot[c]) + 1) == core::kSlotEmpty)
-            core::demand_prefetch(v, v.slot_off[c] + key % v.nslot[c], c, pf_m,
-                                  (uint32_t)((rest - (float)pf_rem) * (1.0f / core::kSlices)) + 1u);
-    }
-    const unsigned callers = __ballot_sync(0xFFFFFFFFu, slow != 0);
-    if (slow) {
-        uint64_t spill[(ITEMS + 3) / 4];                  // addressed copy only on the slow path
+    // the rest -- refill duties, demand prefetch, further rounds, blocks and
+    // segments -- only if some thread of the tile has any of it (its frame
+    // is not the fast path's)
+    if (slow_tile) {
+        uint32_t crs[ITEMS];
 #pragma unroll
-        for (int q = 0; q < (ITEMS + 3) / 4; q++) spill[q] = info[q];
-        bulk_malloc_slow(sizes, ptrs, n, base, key, slow, spill, ITEMS, callers, NT,
-                         v.demand_hint ? cnt : nullptr, gridDim.x);
+        for (int k = 0; k < ITEMS; k++) crs[k] = cr[k];
+        tile_slow<ITEMS, NT>(sizes, ptrs, base, key, crs, pend, big, pfd, cnt, lim_lo, run_base, roff, failed);
     }
+#ifdef GALLATIN_TRACE
+    __syncthreads();
+    if (threadIdx.x == 0) ptx::trace(tk0, ptx::globaltimer(), (7ull << 60) | blockIdx.x);   // CTA start, end
+#endif
 }
 
 __device__ __noinline__ void free_slow(const View &v, uint64_t p) {
@@ -812,6 +923,7 @@ int gallatin_init_ex(const gallatin_config_t *cfg_in) {
     v.fence_free = cfg.fence_free;
     v.demand_hint = cfg.demand_hint == 2 ? 0u : 1u;
     v.oom_record = cfg.oom_record == 2 ? 0u : 1u;
+    v.nsm = (uint32_t)sms;
     // prefilled block buffer (include/gallatin.h "prefill"): every
     // slot's first run (rounded down to a power of two), shrunk to fit nseg/8
     // segments, laid out class by class

@@ -4,7 +4,7 @@ sys.path.insert(0, os.getcwd())
 import numpy as np, torch
 import paper_conf_ppopp_mccoyp24_b200 as G
 import workload_gen as wg
-G.gallatin_init(64 << 30)
+G.gallatin_init(64 << 30, **json.loads(os.environ.get('GALLATIN_CFG', '{}')))
 for name, kw in [("mixed", {}), ("no_large", dict(p_large=0.0)), ("large_only", None), ("segment_only", 1),
                  ("block_only", 2)]:
     if kw is None or isinstance(kw, int):

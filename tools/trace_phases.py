@@ -18,7 +18,7 @@ import paper_conf_ppopp_mccoyp24_b200 as G  # noqa: E402
 sizes = [int(x) for x in (sys.argv[1] if len(sys.argv) > 1 else "16,512,4096").split(",")]
 L = G.lib()
 L.gallatin_debug_trace.argtypes = [ctypes.c_void_p, ctypes.c_uint64, ctypes.POINTER(ctypes.c_uint64)]
-G.gallatin_init(16 << 30)
+G.gallatin_init(16 << 30, **(json.loads(os.environ.get('GALLATIN_CFG', '{}'))))
 cap = 1 << 20
 buf = torch.zeros(3 * cap, dtype=torch.int64, device="cuda")
 for sz in sizes:
@@ -40,9 +40,19 @@ for sz in sizes:
     t0 = t[:, 0].astype(np.int64)
     base = t0[tag == 7].min() if (tag == 7).any() else t0.min()
     out = {"size": sz, "kernel_ms": round(e0.elapsed_time(e1), 4)}
+    if (tag == 8).any():
+        out["plan_segments"] = int(t[tag == 8, 2][0] & np.uint64(0xFFFFFFFF))
     if (tag == 7).sum() >= 2:
-        out["cta_start_span_us"] = round((t0[tag == 7].max() - t0[tag == 7].min()) / 1e3, 1)
-    for g_ in (0, 1, 2, 3):
+        m7 = tag == 7
+        out["cta_start_span_us"] = round((t0[m7].max() - t0[m7].min()) / 1e3, 1)
+        end7 = (t[m7, 1].astype(np.int64) - base) / 1e3
+        dur7 = (t[m7, 1] - t[m7, 0]).astype(np.float64) / 1e3
+        bid = (t[m7, 2] & np.uint64(0xFFFFFFFF)).astype(np.int64)
+        out["cta_end_us_p50_p90_p99_max"] = [round(float(np.percentile(end7, q)), 1) for q in (50, 90, 99, 100)]
+        out["cta_dur_us_p50_p90_p99_max"] = [round(float(np.percentile(dur7, q)), 2) for q in (50, 90, 99, 100)]
+        slow = np.argsort(-dur7)[:5]
+        out["slowest_ctas"] = [[int(bid[i]), round(float((t0[m7][i] - base) / 1e3), 1), round(float(dur7[i]), 1)] for i in slow]
+    for g_ in (0, 1, 2, 3, 8, 10, 11):
         m = tag == g_
         if not m.any():
             continue
