@@ -26,6 +26,9 @@
  *   oom         one 128 B line: word 0 = {epoch:32 | searchers:22 | flag:10}
  *               (the exhaustion record, DESIGN.md Deviations 11), word 1 + t =
  *               epoch + 1 at which block tree t was confirmed exhausted
+ *   bigq        the whole-block and segment requests a bulk malloc launch
+ *               defers to its batch kernel (k_big): bigq_cap x {&ptrs[i],
+ *               size}; bigq_ctl = {owner tag, count} (one line)
  */
 #ifndef GALLATIN_VIEW_H_
 #define GALLATIN_VIEW_H_
@@ -49,6 +52,9 @@ struct gallatin_device_view {
     uint32_t *fmt_token;        /* 32 words (128 B) per tree                  */
     unsigned long long *err;
     uint64_t *oom;              /* exhaustion record (1 line)                  */
+    uint64_t *bigq;             /* bulk launches' deferred whole-block / segment requests:
+                                   bigq_cap pairs {&ptrs[i], size} (DESIGN.md Deviations 20) */
+    uint32_t *bigq_ctl;         /* one 128 B line: [0] owner launch tag (0 = free), [1] entries */
     uint32_t tree_levels;       /* L                                           */
     uint32_t tree_words;        /* W                                           */
     uint32_t level_off[GALLATIN_MAX_LEVELS];
@@ -66,6 +72,7 @@ struct gallatin_device_view {
     uint32_t demand_hint;       /* 1 = bulk refills sized to the launch's demand */
     uint32_t oom_record;        /* 1 = exhaustion record on (DESIGN.md Deviations 11) */
     uint32_t nsm;               /* SMs of the device (slot keys are %smid mod nslot) */
+    uint32_t bigq_cap;
     /* prefilled block buffer ("always populated"; reading A-19):
      * 0 segments = reset leaves every slot empty; else class c's slots hold
      * runs of pf_run[c] blocks laid out from segment pf_base[c] on, slot q at

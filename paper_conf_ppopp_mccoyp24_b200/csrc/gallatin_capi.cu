@@ -7,6 +7,7 @@
 #include <cuda_runtime.h>
 #include <stdint.h>
 #include <stdio.h>
+#include <stdlib.h>
 #include <string.h>
 
 #include <vector>
@@ -40,6 +41,8 @@ struct State {
     uint64_t scratch_bytes = 0;
     // host-array calls: copy-in / copy-out streams and per-chunk events
     cudaStream_t cin = nullptr, cout = nullptr;
+    uint32_t launch_tag = 0;                          // bulk malloc launches (deferred-request queue owner)
+    bool pdl = true;
     cudaEvent_t ev_in[kMaxChunks] = {}, ev_k[kMaxChunks] = {};
 };
 State g;
@@ -162,6 +165,7 @@ __global__ void k_reset() {
         if (i < 9 * 32) v.fmt_token[i] = 0;
         if (i == 0) *v.err = 0;
         if (i < 16) v.oom[i] = 0;
+        if (i < 2) v.bigq_ctl[i] = 0;
     }
 }
 
@@ -285,6 +289,22 @@ __global__ void __launch_bounds__(kThreads, 5) k_bulk_malloc(const uint64_t *__r
     if (slow) bulk_malloc_slow(sizes, ptrs, n, base, key, slow, &info, ITEMS, callers);
 }
 
+// [dev] Deferred big requests (DESIGN.md Deviations 20): a bulk launch's
+// whole-block and segment requests go into one device queue -- claimed by the
+// launch's tag (concurrent launches on other streams find it taken and serve
+// theirs inline) -- and the batch kernel k_big that follows the launch serves
+// them together.  Returns false (serve inline) if the queue is another
+// launch's or full.
+__device__ __noinline__ bool defer_big(const View &v, uint32_t tag, uint64_t addr, uint64_t size) {
+    const uint32_t own = atomicCAS(v.bigq_ctl, 0u, tag);
+    if (own != 0u && own != tag) return false;
+    const uint32_t q = atomicAdd(v.bigq_ctl + 1, 1u);
+    if (q >= v.bigq_cap) return false;
+    v.bigq[2 * (uint64_t)q] = addr;
+    v.bigq[2 * (uint64_t)q + 1] = size;
+    return true;
+}
+
 // The slow remainder of one k_bulk_malloc_cta tile (called by every thread
 // of the tile, or by none).  Thread c_me < 9 serves class c_me: its slot si,
 // the tile's my_cnt requests of the class, the RMW's lo/run (my_lo, my_m),
@@ -293,7 +313,7 @@ template <int ITEMS, int NT>
 __device__ __noinline__ void tile_slow(const uint64_t *sizes, void **ptrs, uint64_t base, uint32_t key,
                                        const uint32_t *cr, uint32_t pend, uint32_t big, uint32_t pfd,
                                        const uint32_t *cnt, uint64_t *lim_lo, uint64_t *run_base, uint32_t *roff,
-                                       uint32_t *failed) {
+                                       uint32_t *failed, bool rounds, uint32_t tag) {
     const View &v = c_view;
     // [dev] prefetch duties (knob prefetch=1): the item that drew the middle of a run
     for (int k = 0; k < ITEMS; k++) {
@@ -336,9 +356,9 @@ __device__ __noinline__ void tile_slow(const uint64_t *sizes, void **ptrs, uint6
     // the slot's refill (another tile's duty), takes the tile's remaining
     // requests of its class with ONE more RMW, and the items retry -- one RMW
     // and one barrier per round for the whole tile, not one per warp and item.
+    // (rounds is CTA-uniform: no class past its run's end -> no duty, no round, no barrier)
     bool still = my_cnt && (dutyfail || my_lo + my_cnt > my_limit);
-    while (__syncthreads_or(still)) {
-        duty = false;
+    while (rounds && __syncthreads_or(still)) {
         if (still) {
             const uint32_t served = my_lo < my_limit ? min(my_limit - my_lo, my_cnt) : 0u;
             if (dutyfail) {
@@ -358,7 +378,11 @@ __device__ __noinline__ void tile_slow(const uint64_t *sizes, void **ptrs, uint6
                     my_lo = (uint32_t)(old >> 32);
                     lim_lo[c_me] = ((uint64_t)my_limit << 32) | my_lo;
                     run_base[c_me] = reinterpret_cast<uint64_t>(core::slice_ptr(v, c_me, old & core::kRunNone, 0));
+                    // a duty is discharged at once, before the barrier: a
+                    // sibling class thread may be waiting in this phase for a
+                    // refill whose holder waits for this one (no cycle)
                     duty = my_lo <= my_limit && my_limit < my_lo + my_cnt;
+                    dutyfail = duty && !core::refill_slot(v, si, c_me, my_m, hint_of);
                 }
             }
         }
@@ -381,7 +405,6 @@ __device__ __noinline__ void tile_slow(const uint64_t *sizes, void **ptrs, uint6
                 pend &= ~(1u << k);
             }
         }
-        dutyfail = duty && !core::refill_slot(v, si, c_me, my_m, hint_of);
         still = my_cnt && (dutyfail || my_lo + my_cnt > my_limit);
     }
     // whole blocks and segment runs: the device path, per lane
@@ -389,8 +412,17 @@ __device__ __noinline__ void tile_slow(const uint64_t *sizes, void **ptrs, uint6
         for (int k = 0; k < ITEMS; k++) {
             if (!((big >> k) & 1)) continue;
             const uint64_t i = base + (uint64_t)NT * k;
+            // [dev] deferred to the launch's batch kernel (k_big) while the
+            // queue is this launch's and has room (DESIGN.md Deviations 20)
+            if (tag && defer_big(v, tag, reinterpret_cast<uint64_t>(ptrs + i), sizes[i])) continue;
+#ifdef GALLATIN_TRACE
+            const uint64_t tb0 = ptx::globaltimer();
+#endif
             __stcs(reinterpret_cast<unsigned long long *>(ptrs) + i,
                    reinterpret_cast<unsigned long long>(core::malloc_impl(v, sizes[i], key)));
+#ifdef GALLATIN_TRACE
+            ptx::trace(tb0, ptx::globaltimer(), (12ull << 60) | (sizes[i] >> 20));
+#endif
         }
     }
 }
@@ -403,16 +435,21 @@ __device__ __noinline__ void tile_slow(const uint64_t *sizes, void **ptrs, uint6
 // Item k of thread t is request blockIdx*256*ITEMS + k*256 + t.
 template <int ITEMS, int MINB = 5, int NT = kThreads>
 __global__ void __launch_bounds__(NT, MINB) k_bulk_malloc_cta(const uint64_t *__restrict__ sizes,
-                                                                  void **__restrict__ ptrs, uint64_t n) {
+                                                                  void **__restrict__ ptrs, uint64_t n,
+                                                                  uint32_t tag) {
     const View &v = c_view;
     __shared__ uint32_t cnt[core::kTrees];
+    __shared__ uint32_t tile_flags;
     const uint32_t lane = threadIdx.x & 31;
     const uint64_t base = blockIdx.x * (uint64_t)(NT * ITEMS) + threadIdx.x;
 #ifdef GALLATIN_TRACE
     const uint64_t tk0 = ptx::globaltimer();
 #endif
     const uint32_t key = ptx::smid();
+    // the launch's batch kernel (k_big) may become resident once every tile has started
+    asm volatile("griddepcontrol.launch_dependents;");
     if (threadIdx.x < core::kTrees) cnt[threadIdx.x] = 0;
+    if (threadIdx.x == 32) tile_flags = 0;
     // a tile entirely inside the array needs no per-item range checks (CTA-uniform)
     const bool full = (blockIdx.x + 1ull) * (NT * ITEMS) <= n;
     // per item: class (0..8 slice class, 0xFE nothing to do, 0xFF block or
@@ -462,7 +499,8 @@ __global__ void __launch_bounds__(NT, MINB) k_bulk_malloc_cta(const uint64_t *__
     constexpr uint32_t NW = NT / 32;
     const uint32_t c_me = lane * NW + (threadIdx.x >> 5);
     const bool cls_thread = c_me < core::kTrees;
-    bool cls_slow = false;      // this class thread has a refill duty or a demand prefetch
+    bool cls_over = false;      // requests of this class past the run's end: the tile needs rounds
+    bool cls_slow = false;      // this class thread has a prefetch or a demand prefetch to do
     if (cls_thread) {
         roff[c_me] = 0;
         failed[c_me] = 0;
@@ -473,8 +511,8 @@ __global__ void __launch_bounds__(NT, MINB) k_bulk_malloc_cta(const uint64_t *__
             const uint32_t my_limit = core::run_len(old) << core::kSliceLog2, my_lo = (uint32_t)(old >> 32);
             lim_lo[c_me] = ((uint64_t)my_limit << 32) | my_lo;
             run_base[c_me] = reinterpret_cast<uint64_t>(core::slice_ptr(v, c_me, old & core::kRunNone, 0));
-            cls_slow = my_lo + my_cnt > my_limit ||                  // requests past the run's end
-                       (v.prefetch && my_lo <= (my_limit >> 1) && (my_limit >> 1) < my_lo + my_cnt) ||
+            cls_over = my_lo + my_cnt > my_limit;
+            cls_slow = (v.prefetch && my_lo <= (my_limit >> 1) && (my_limit >> 1) < my_lo + my_cnt) ||
                        (v.demand_hint && my_limit - (my_lo + my_cnt) >= 16u * my_cnt &&
                         blockIdx.x < gridDim.x - gridDim.x / 4 &&
                         (float)my_cnt * (float)(gridDim.x - blockIdx.x) * v.nslot_rcp[c_me] >=
@@ -486,7 +524,10 @@ __global__ void __launch_bounds__(NT, MINB) k_bulk_malloc_cta(const uint64_t *__
     for (int k = 0; k < ITEMS; k++) big_any |= (cr[k] & 0xFFu) == 0xFFu;
     // the tile's slow remainder is known here, before any store: the fast
     // path ends with its stores (no barrier behind them)
-    const bool slow_tile = __syncthreads_or(cls_slow || big_any);
+    if (cls_over) atomicOr(&tile_flags, 1u);
+    if (cls_slow || big_any) atomicOr(&tile_flags, 2u);
+    __syncthreads();
+    const uint32_t slow_tile = tile_flags;                    // bit 0: rounds, bit 1: barrier-free slow work
     // items whose slice lies inside the run are stored now; the rest wait in
     // `pend` for the tile's next round (bit k: item k)
     uint32_t pend = 0, big = 0, pfd = 0;
@@ -518,12 +559,268 @@ __global__ void __launch_bounds__(NT, MINB) k_bulk_malloc_cta(const uint64_t *__
         uint32_t crs[ITEMS];
 #pragma unroll
         for (int k = 0; k < ITEMS; k++) crs[k] = cr[k];
-        tile_slow<ITEMS, NT>(sizes, ptrs, base, key, crs, pend, big, pfd, cnt, lim_lo, run_base, roff, failed);
+        tile_slow<ITEMS, NT>(sizes, ptrs, base, key, crs, pend, big, pfd, cnt, lim_lo, run_base, roff, failed,
+                             slow_tile & 1, tag);
     }
 #ifdef GALLATIN_TRACE
     __syncthreads();
     if (threadIdx.x == 0) ptx::trace(tk0, ptx::globaltimer(), (7ull << 60) | blockIdx.x);   // CTA start, end
 #endif
+}
+
+// ---- the batch kernel of a bulk malloc launch's deferred big requests ------
+// [dev] (DESIGN.md Deviations 20).  One CTA, after the launch (stream order):
+//   1. rank every request within its block tree (4 KB < size < 16 MB: one
+//      whole block of tree t, reading A-2) and sum the segment requests' k;
+//   2. ONE claim of consecutive free segments from the front for all the
+//      trees' blocks (tree after tree, ceil(requests / nb) segments each,
+//      taken privately like a whole-segment run, O2-R R2; a tree's partly
+//      used last segment keeps the rest of its blocks in its ring and block
+//      tree, initSegment P:125) and ONE claimMultiple from the back (P:110-113,
+//      P:138) of the sum of the segment requests' k -- both as one atomicAnd
+//      per leaf word, the words spread over a warp's lanes;
+//   3. every request's pointer in rank order (a block's free counter preset
+//      to 4095, reading A-2; a segment run's table entries, P:143 / P:235).
+// A claim that finds no such range (fragmented or nearly full heap) leaves
+// its requests to the per-request device path (malloc_impl: GetBlock /
+// claimMultiple, NULL on exhaustion).
+constexpr int kBigThreads = 1024;
+constexpr uint32_t kBigCap = 8192;
+constexpr uint32_t kMaxLeafWords = 256;                      // nseg <= 2^14 (gallatin_init_ex)
+
+__device__ __noinline__ void *big_inline(const View &v, uint64_t size) { return core::malloc_impl(v, size, 0u); }
+
+// lowest start of k consecutive set bits among the nw words of lw (shared
+// copy of the segment tree's leaves); kNone if none
+__device__ uint64_t lowest_run_of(const uint64_t *lw, uint64_t nw, uint64_t k) {
+    uint64_t run = 0, start = 0;
+    for (uint64_t wi = 0; wi < nw; wi++) {
+        const uint64_t x = lw[wi], base = wi << 6;
+        if (x == ~0ull) {
+            if (!run) start = base;
+            run += 64;
+            if (run >= k) return start;
+            continue;
+        }
+        const uint32_t tr = (uint32_t)__ffsll((long long)~x) - 1;   // ones at the bottom continue the run
+        if (tr) {
+            if (!run) start = base;
+            run += tr;
+            if (run >= k) return start;
+        }
+        run = 0;
+        uint64_t rest = x & (~0ull << tr);                          // bit tr is 0
+        while (rest) {
+            const uint32_t lo = (uint32_t)__ffsll((long long)rest) - 1;
+            const uint64_t sh = rest >> lo;
+            const uint32_t len = (uint32_t)__ffsll((long long)~sh) - 1;
+            if (len >= k) return base + lo;
+            if (lo + len == 64) {                                      // continues into the next word
+                run = len;
+                start = base + lo;
+                break;
+            }
+            rest &= ~bit_range(lo, lo + len);
+        }
+    }
+    return kNone;
+}
+
+// Claim [i0, i0+k) of the segment tree, one atomicAnd per leaf word spread
+// over the lanes of the calling warp; on a conflict every bit taken is given
+// back (claimMultiple, for the whole range at once).  Summary repair
+// of the words the claim emptied runs in parallel, one lane per word.
+__device__ bool claim_range_warp(const BitTree &st, uint64_t i0, uint64_t k, uint32_t lane) {
+    const uint64_t w0 = i0 >> 6, w1 = (i0 + k - 1) >> 6;
+    constexpr int R = (int)(kMaxLeafWords / 32);
+    uint64_t old[R], msk[R];
+    bool ok = true;
+#pragma unroll
+    for (int r = 0; r < R; r++) {
+        const uint64_t wi = w0 + lane + 32u * r;
+        msk[r] = 0;
+        old[r] = 0;
+        if (wi <= w1) {
+            const uint32_t lo = wi == w0 ? (uint32_t)(i0 & 63) : 0u;
+            const uint32_t hi = wi == w1 ? (uint32_t)((i0 + k - 1) & 63) + 1 : 64u;
+            msk[r] = bit_range(lo, hi);
+            old[r] = ptx::atom_and(st.w + st.off[0] + wi, ~msk[r]);
+            ok &= (old[r] & msk[r]) == msk[r];
+        }
+    }
+    ok = __all_sync(0xFFFFFFFFu, ok);
+#pragma unroll
+    for (int r = 0; r < R; r++) {
+        if (!msk[r]) continue;
+        const uint64_t wi = w0 + lane + 32u * r;
+        bool flip = (old[r] & ~msk[r]) == 0 && (old[r] & msk[r]) != 0;   // our RMW emptied the word
+        if (!ok && (old[r] & msk[r])) flip |= ptx::atom_or(st.w + st.off[0] + wi, old[r] & msk[r]) == 0;
+        if (flip) bt_reconcile_up(st, 0, wi);
+    }
+    return ok;
+}
+
+__global__ void __launch_bounds__(kBigThreads, 1) k_big(uint32_t tag) {
+    const View &v = c_view;
+    __shared__ uint32_t own, nq;
+    __shared__ uint32_t tcnt[core::kTrees], tsegs[core::kTrees], tbase[core::kTrees];
+    __shared__ uint32_t ksum;
+    __shared__ uint64_t front, back;                  // claimed ranges (kNone: serve inline)
+    __shared__ uint64_t leaf[kMaxLeafWords];
+    __shared__ uint32_t erank[kBigCap];               // tree << 28 | rank, or 0xF << 28 | segment offset
+    const uint32_t tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+    // launched as the bulk malloc kernel's programmatic dependent: resident
+    // before that kernel ends, it waits here for its completion (and memory)
+    asm volatile("griddepcontrol.wait;" ::: "memory");
+    if (tid == 0) {
+        own = ptx::ld_relaxed(v.bigq_ctl);
+        const uint32_t c = ptx::ld_relaxed(v.bigq_ctl + 1);
+        nq = c < v.bigq_cap ? c : v.bigq_cap;
+        ksum = 0;
+        front = kNone;
+        back = kNone;
+    }
+    if (tid < core::kTrees) tcnt[tid] = 0;
+    __syncthreads();
+    if (own != tag) return;                                   // nothing of this launch's was deferred
+    const uint32_t n = nq;
+#ifdef GALLATIN_TRACE
+    const uint64_t tb0 = ptx::globaltimer();
+#endif
+    const BitTree st = core::seg_tree(v);
+    const uint64_t nw = (v.nseg + 63) / 64;
+    if (tid < nw) leaf[tid] = ptx::ld_relaxed(st.w + st.off[0] + tid);
+    // 1. ranks
+    for (uint32_t e = tid; e < n; e += kBigThreads) {
+        const uint64_t size = v.bigq[2 * (uint64_t)e + 1];
+        if (size < core::kSegBytes) {
+            const uint32_t t = core::block_class(size);
+            erank[e] = (t << 28) | atomicAdd(&tcnt[t], 1u);
+        } else {
+            const uint64_t k = (size >> core::kSegLog2) + ((size & (core::kSegBytes - 1)) != 0);
+            erank[e] = k <= v.nseg ? ((0xFu << 28) | atomicAdd(&ksum, (uint32_t)k)) : 0xFFFFFFFFu;
+        }
+    }
+    __syncthreads();
+#ifdef GALLATIN_TRACE
+    if (tid == 0) ptx::trace(tb0, ptx::globaltimer(), (13ull << 60) | 1);
+#endif
+    uint64_t T = 0;                                           // segments for the trees' blocks
+#pragma unroll
+    for (uint32_t t = 0; t < core::kTrees; t++) {
+        const uint32_t sg = (tcnt[t] + core::nb_of(t) - 1) / core::nb_of(t);
+        if (tid == 0) {
+            tsegs[t] = sg;
+            tbase[t] = (uint32_t)T;                           // offset from `front` for now
+        }
+        T += sg;
+    }
+    // 2. the two claims (warp 0: front, warp 1: back), each retried once on a lost race
+    if (warp == 0 && T) {
+        for (int attempt = 0; attempt < 2; attempt++) {
+            uint64_t s0 = lane == 0 ? lowest_run_of(leaf, nw, T) : 0;
+            s0 = __shfl_sync(0xFFFFFFFFu, s0, 0);
+            if (s0 == kNone) break;
+            if (claim_range_warp(st, s0, T, lane)) {
+                if (lane == 0) front = s0;
+                break;
+            }
+            for (uint64_t w = lane; w < nw; w += 32) leaf[w] = ptx::ld_relaxed(st.w + st.off[0] + w);
+            __syncwarp();
+        }
+    }
+    if (warp == 1 && ksum) {
+        for (int attempt = 0; attempt < 2; attempt++) {
+            uint64_t s0 = lane == 0 ? bt_find_highest_run(st, ksum) : 0;
+            s0 = __shfl_sync(0xFFFFFFFFu, s0, 0);
+            if (s0 == kNone) break;
+            if (claim_range_warp(st, s0, ksum, lane)) {
+                if (lane == 0) back = s0;
+                break;
+            }
+        }
+    }
+    __syncthreads();
+#ifdef GALLATIN_TRACE
+    if (tid == 0) ptx::trace(tb0, ptx::globaltimer(), (13ull << 60) | 2);
+#endif
+    // the trees' segments, taken privately ({t, 0 available}, tree-id copy);
+    // a tree's partly used last segment: the rest of its blocks into its ring
+    const uint64_t fr = front;
+    if (fr != kNone) {
+        for (uint64_t x = tid; x < T; x += kBigThreads) {
+            uint32_t t = 0;
+            while (x >= (uint64_t)tbase[t] + tsegs[t]) t++;
+            const uint64_t s = fr + x;
+            const uint32_t nb = core::nb_of(t), used = tcnt[t] - (tsegs[t] - 1) * nb;
+            if (x == (uint64_t)tbase[t] + tsegs[t] - 1 && used < nb) {
+                uint16_t *e = v.q_entries + s * core::kMaxBlocks;
+                for (uint32_t q = 0; q < nb - used; q++) e[q] = (uint16_t)(used + q);
+                ptx::st_relaxed(v.q_head + s, 0u);
+                ptx::st_relaxed(v.q_tail + s, nb - used);
+            }
+            ptx::st_relaxed(v.seg_tid + s, t);
+            ptx::atom_add(v.seg_word + s, core::sw_retree(core::kTreeFree, t));
+        }
+        ptx::fence_acq_rel();
+    }
+    // 3. pointers
+    for (uint32_t e = tid; e < n; e += kBigThreads) {
+        const uint32_t er = erank[e];
+        const uint64_t addr = v.bigq[2 * (uint64_t)e];
+        void *p = nullptr;
+        if (er == 0xFFFFFFFFu) {
+            p = nullptr;                                      // more segments than the heap
+        } else if ((er >> 28) < core::kTrees) {
+            const uint32_t t = er >> 28, r = er & 0x0FFFFFFFu;
+            if (fr != kNone) {
+                const uint64_t lin = (fr + tbase[t]) * core::nb_of(t) + r;
+                atomicExch(v.block_free + core::gid_of(t, lin), core::kSlices - 1);   // reading A-2
+                p = reinterpret_cast<void *>(v.heap + (lin << (16 + t)));
+            } else {
+                p = big_inline(v, v.bigq[2 * (uint64_t)e + 1]);
+            }
+        } else {
+            const uint64_t size = v.bigq[2 * (uint64_t)e + 1];
+            const uint64_t k = (size >> core::kSegLog2) + ((size & (core::kSegBytes - 1)) != 0);
+            if (back != kNone) {
+                const uint64_t i = back + (er & 0x0FFFFFFFu);
+                ptx::st_relaxed(v.seg_tid + i, core::kTrees + (uint32_t)k);
+                for (uint64_t m = 1; m < k; m++) ptx::st_relaxed(v.seg_tid + i + m, core::kTreeCont);
+                ptx::atom_add(v.seg_word + i, core::sw_retree(core::kTreeFree, core::kTrees + (uint32_t)k));
+                for (uint64_t m = 1; m < k; m++)
+                    ptx::atom_add(v.seg_word + i + m, core::sw_retree(core::kTreeFree, core::kTreeCont));
+                ptx::fence_acq_rel();
+                p = reinterpret_cast<void *>(v.heap + (i << core::kSegLog2));
+            } else {
+                p = big_inline(v, size);
+            }
+        }
+        *reinterpret_cast<uint64_t *>(addr) = reinterpret_cast<uint64_t>(p);
+    }
+#ifdef GALLATIN_TRACE
+    __syncthreads();
+    if (tid == 0) ptx::trace(tb0, ptx::globaltimer(), (13ull << 60) | 3);
+#endif
+    // the rest of each partly used segment becomes available (joins its block tree)
+    if (fr != kNone && tid < core::kTrees && tsegs[tid]) {
+        const uint32_t t = tid, nb = core::nb_of(t), used = tcnt[t] - (tsegs[t] - 1) * nb;
+        if (used < nb) {
+            const uint64_t s = fr + tbase[t] + tsegs[t] - 1;
+            const uint64_t old = ptx::atom_add(v.seg_word + s, (uint64_t)(nb - used));
+            core::seg_after_rmw(v, s, old, old + (nb - used));
+            core::oom_notify(v);
+        }
+    }
+    __syncthreads();
+#ifdef GALLATIN_TRACE
+    if (tid == 0) ptx::trace(tb0, ptx::globaltimer(), (15ull << 60) | n);
+#endif
+    if (tid == 0) {                                           // the queue is free for the next launch
+        ptx::st_relaxed(v.bigq_ctl + 1, 0u);
+        ptx::fence_acq_rel();
+        ptx::st_relaxed(v.bigq_ctl, 0u);
+    }
 }
 
 __device__ __noinline__ void free_slow(const View &v, uint64_t p) {
@@ -968,10 +1265,10 @@ int gallatin_init_ex(const gallatin_config_t *cfg_in) {
     }
 
     // metadata: one allocation, 256 B aligned sections
-    uint64_t sz[12] = {W * 8, 9 * W * 8, nseg * 8, nseg * 4, nseg * 4, nseg * 512, nseg * 1024,
-                       (uint64_t)off * 128, 9 * 128, 128, nseg * 4, 128};
-    uint64_t total = 0, offs[12];
-    for (int i = 0; i < 12; i++) { offs[i] = total; total += align_up(sz[i], 256); }
+    uint64_t sz[14] = {W * 8, 9 * W * 8, nseg * 8, nseg * 4, nseg * 4, nseg * 512, nseg * 1024,
+                       (uint64_t)off * 128, 9 * 128, 128, nseg * 4, 128, (uint64_t)kBigCap * 16, 128};
+    uint64_t total = 0, offs[14];
+    for (int i = 0; i < 14; i++) { offs[i] = total; total += align_up(sz[i], 256); }
     void *meta = nullptr;
     if (cudaMalloc(&meta, total) != cudaSuccess) { cudaGetLastError(); return GALLATIN_ERR_NOMEM; }
     void *heap = nullptr;
@@ -993,10 +1290,17 @@ int gallatin_init_ex(const gallatin_config_t *cfg_in) {
     v.err = reinterpret_cast<unsigned long long *>(m + offs[9]);
     v.seg_tid = reinterpret_cast<uint32_t *>(m + offs[10]);
     v.oom = reinterpret_cast<uint64_t *>(m + offs[11]);
+    v.bigq = reinterpret_cast<uint64_t *>(m + offs[12]);
+    v.bigq_ctl = reinterpret_cast<uint32_t *>(m + offs[13]);
+    v.bigq_cap = kBigCap;
     v.heap = align_up(reinterpret_cast<uint64_t>(heap), core::kSegBytes);   // 16 MiB aligned base
 
     g.init = true;
     g.device = dev;
+    {
+        const char *e = getenv("GALLATIN_PDL");
+        g.pdl = !(e && e[0] == '0');
+    }
     g.cfg = cfg;
     g.heap_raw = heap;
     g.meta = meta;
@@ -1036,9 +1340,26 @@ int gallatin_malloc(const uint64_t *d_sizes, void **d_ptrs, uint64_t n, void *st
     if (n == 0) return GALLATIN_OK;
     if (!d_sizes || !d_ptrs || n > (1ull << 40)) return GALLATIN_ERR_INVALID;
     const uint32_t items = g.cfg.bulk_items ? g.cfg.bulk_items : (n >= (uint64_t)kItemsMin ? 4u : 1u);
-    if (items == 4)   // 128-thread CTAs, 4 requests per thread, one slot RMW per class per CTA
-        k_bulk_malloc_cta<4, 10, 128><<<(unsigned)((n + 511) / 512), 128, 0, S(stream)>>>(d_sizes, d_ptrs, n);
-    else
+    if (items == 4) {  // 128-thread CTAs, 4 requests per thread, one slot RMW per class per CTA
+        // the launch's tag claims the deferred-request queue; its batch kernel follows
+        if (++g.launch_tag == 0) g.launch_tag = 1;
+        k_bulk_malloc_cta<4, 10, 128><<<(unsigned)((n + 511) / 512), 128, 0, S(stream)>>>(d_sizes, d_ptrs, n,
+                                                                                       g.launch_tag);
+        const int rc = launch_status();
+        if (rc) return rc;
+        // programmatic dependent launch: k_big's launch overlaps the tail of
+        // the malloc kernel; it waits for that kernel with griddepcontrol.wait
+        cudaLaunchConfig_t lc = {};
+        lc.gridDim = dim3(1);
+        lc.blockDim = dim3(kBigThreads);
+        lc.stream = S(stream);
+        cudaLaunchAttribute at[1];
+        at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+        at[0].val.programmaticStreamSerializationAllowed = 1;
+        lc.attrs = at;
+        lc.numAttrs = g.pdl ? 1 : 0;
+        CUDA_TRY(cudaLaunchKernelEx(&lc, k_big, g.launch_tag));
+    } else
         k_bulk_malloc<1><<<grid_for(n), kThreads, 0, S(stream)>>>(d_sizes, d_ptrs, n);
     return launch_status();
 }

@@ -1,6 +1,8 @@
 """C3 mixed workload broken down: which requests make the malloc slow."""
 import sys, os, json, statistics
 sys.path.insert(0, os.getcwd())
+if os.environ.get('GALLATIN_PKG_ROOT'):
+    sys.path.insert(0, os.environ['GALLATIN_PKG_ROOT'])
 import numpy as np, torch
 import paper_conf_ppopp_mccoyp24_b200 as G
 import workload_gen as wg
