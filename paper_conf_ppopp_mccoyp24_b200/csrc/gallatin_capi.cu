@@ -626,11 +626,44 @@ __device__ uint64_t lowest_run_of(const uint64_t *lw, uint64_t nw, uint64_t k) {
     return kNone;
 }
 
+// Warp-parallel fast path of lowest_run_of / bt_find_highest_run: if the k
+// bits from the lowest set bit (back = false) or ending at the highest set
+// bit (back = true) are all set, their start; else kNone (the caller scans).
+__device__ uint64_t edge_run_warp(const uint64_t *lw, uint64_t nw, uint64_t k, bool back, uint32_t lane) {
+    uint64_t edge = kNone;
+    for (uint64_t b = 0; b < nw && edge == kNone; b += 32) {
+        const uint64_t wi = back ? nw - 1 - (b + lane) : b + lane;
+        const uint64_t x = (b + lane < nw) ? lw[wi] : 0ull;
+        const unsigned any = __ballot_sync(0xFFFFFFFFu, x != 0);
+        if (any) {
+            const uint32_t src = (uint32_t)__ffs((int)any) - 1;
+            const uint64_t xs = __shfl_sync(0xFFFFFFFFu, x, (int)src);
+            const uint64_t ws = back ? nw - 1 - (b + src) : b + src;
+            edge = (ws << 6) + (back ? 63 - (uint64_t)__clzll((long long)xs) : (uint64_t)(__ffsll((long long)xs) - 1));
+        }
+    }
+    if (edge == kNone) return kNone;
+    if (back && edge + 1 < k) return kNone;
+    const uint64_t i0 = back ? edge + 1 - k : edge;
+    if (i0 + k > nw * 64) return kNone;
+    const uint64_t w0 = i0 >> 6, w1 = (i0 + k - 1) >> 6;
+    bool ok = true;
+    for (uint64_t wi = w0 + lane; wi <= w1; wi += 32) {
+        const uint32_t lo = wi == w0 ? (uint32_t)(i0 & 63) : 0u;
+        const uint32_t hi = wi == w1 ? (uint32_t)((i0 + k - 1) & 63) + 1 : 64u;
+        const uint64_t m = bit_range(lo, hi);
+        ok &= (lw[wi] & m) == m;
+    }
+    return __all_sync(0xFFFFFFFFu, ok) ? i0 : kNone;
+}
+
 // Claim [i0, i0+k) of the segment tree, one atomicAnd per leaf word spread
 // over the lanes of the calling warp; on a conflict every bit taken is given
-// back (claimMultiple, for the whole range at once).  Summary repair
-// of the words the claim emptied runs in parallel, one lane per word.
-__device__ bool claim_range_warp(const BitTree &st, uint64_t i0, uint64_t k, uint32_t lane) {
+// back (claimMultiple, for the whole range at once).  On success the
+// words this lane's RMWs emptied are left in *emptied (bit r: word w0 + lane
+// + 32 r): their summary repair (bt_reconcile_up) is the caller's, later --
+// a stale summary over an empty word only makes a search restart.
+__device__ bool claim_range_warp(const BitTree &st, uint64_t i0, uint64_t k, uint32_t lane, uint32_t *emptied) {
     const uint64_t w0 = i0 >> 6, w1 = (i0 + k - 1) >> 6;
     constexpr int R = (int)(kMaxLeafWords / 32);
     uint64_t old[R], msk[R];
@@ -649,15 +682,26 @@ __device__ bool claim_range_warp(const BitTree &st, uint64_t i0, uint64_t k, uin
         }
     }
     ok = __all_sync(0xFFFFFFFFu, ok);
+    *emptied = 0;
 #pragma unroll
     for (int r = 0; r < R; r++) {
         if (!msk[r]) continue;
         const uint64_t wi = w0 + lane + 32u * r;
         bool flip = (old[r] & ~msk[r]) == 0 && (old[r] & msk[r]) != 0;   // our RMW emptied the word
-        if (!ok && (old[r] & msk[r])) flip |= ptx::atom_or(st.w + st.off[0] + wi, old[r] & msk[r]) == 0;
+        if (ok) {
+            if (flip) *emptied |= 1u << r;
+            continue;
+        }
+        if (old[r] & msk[r]) flip |= ptx::atom_or(st.w + st.off[0] + wi, old[r] & msk[r]) == 0;
         if (flip) bt_reconcile_up(st, 0, wi);
     }
     return ok;
+}
+
+// the summary repair claim_range_warp left to its caller
+__device__ __forceinline__ void claim_range_repair(const BitTree &st, uint64_t i0, uint32_t lane, uint32_t emptied) {
+    for (; emptied; emptied &= emptied - 1)
+        bt_reconcile_up(st, 0, (i0 >> 6) + lane + 32u * (uint32_t)(__ffs((int)emptied) - 1));
 }
 
 __global__ void __launch_bounds__(kBigThreads, 1) k_big(uint32_t tag) {
@@ -716,12 +760,18 @@ __global__ void __launch_bounds__(kBigThreads, 1) k_big(uint32_t tag) {
         T += sg;
     }
     // 2. the two claims (warp 0: front, warp 1: back), each retried once on a lost race
+    uint32_t emptied = 0;
+    uint64_t claimed = kNone;
     if (warp == 0 && T) {
         for (int attempt = 0; attempt < 2; attempt++) {
-            uint64_t s0 = lane == 0 ? lowest_run_of(leaf, nw, T) : 0;
-            s0 = __shfl_sync(0xFFFFFFFFu, s0, 0);
+            uint64_t s0 = edge_run_warp(leaf, nw, T, false, lane);   // the free segments from the lowest on
+            if (s0 == kNone) {
+                s0 = lane == 0 ? lowest_run_of(leaf, nw, T) : 0;
+                s0 = __shfl_sync(0xFFFFFFFFu, s0, 0);
+            }
             if (s0 == kNone) break;
-            if (claim_range_warp(st, s0, T, lane)) {
+            if (claim_range_warp(st, s0, T, lane, &emptied)) {
+                claimed = s0;
                 if (lane == 0) front = s0;
                 break;
             }
@@ -731,10 +781,14 @@ __global__ void __launch_bounds__(kBigThreads, 1) k_big(uint32_t tag) {
     }
     if (warp == 1 && ksum) {
         for (int attempt = 0; attempt < 2; attempt++) {
-            uint64_t s0 = lane == 0 ? bt_find_highest_run(st, ksum) : 0;
-            s0 = __shfl_sync(0xFFFFFFFFu, s0, 0);
+            uint64_t s0 = edge_run_warp(leaf, nw, ksum, true, lane);   // the free segments up to the highest
+            if (s0 == kNone) {
+                s0 = lane == 0 ? bt_find_highest_run(st, ksum) : 0;
+                s0 = __shfl_sync(0xFFFFFFFFu, s0, 0);
+            }
             if (s0 == kNone) break;
-            if (claim_range_warp(st, s0, ksum, lane)) {
+            if (claim_range_warp(st, s0, ksum, lane, &emptied)) {
+                claimed = s0;
                 if (lane == 0) back = s0;
                 break;
             }
@@ -764,7 +818,23 @@ __global__ void __launch_bounds__(kBigThreads, 1) k_big(uint32_t tag) {
         }
         ptx::fence_acq_rel();
     }
-    // 3. pointers
+    __syncthreads();
+    // summaries over the words the claims emptied (warps 0-1), the rest of
+    // each tree's partly used segment made available -- it joins the tree's
+    // block tree (warp 2) -- and the pointers, all at once
+    if (claimed != kNone) claim_range_repair(st, claimed, lane, emptied);
+    if (warp == 2 && fr != kNone && lane < core::kTrees && tsegs[lane]) {
+        const uint32_t t = lane, nb = core::nb_of(t), used = tcnt[t] - (tsegs[t] - 1) * nb;
+        if (used < nb) {
+            const uint64_t s = fr + tbase[t] + tsegs[t] - 1;
+            ptx::fence_acq_rel();                             // the ring entries (another thread's) before the count
+            const uint64_t old = ptx::atom_add(v.seg_word + s, (uint64_t)(nb - used));
+            core::seg_after_rmw(v, s, old, old + (nb - used));
+            core::oom_notify(v);
+        }
+    }
+    // 3. pointers (read by the caller after this kernel: its end orders the
+    // table writes before them)
     for (uint32_t e = tid; e < n; e += kBigThreads) {
         const uint32_t er = erank[e];
         const uint64_t addr = v.bigq[2 * (uint64_t)e];
@@ -775,7 +845,7 @@ __global__ void __launch_bounds__(kBigThreads, 1) k_big(uint32_t tag) {
             const uint32_t t = er >> 28, r = er & 0x0FFFFFFFu;
             if (fr != kNone) {
                 const uint64_t lin = (fr + tbase[t]) * core::nb_of(t) + r;
-                atomicExch(v.block_free + core::gid_of(t, lin), core::kSlices - 1);   // reading A-2
+                ptx::st_relaxed(v.block_free + core::gid_of(t, lin), core::kSlices - 1);   // reading A-2 (block is ours)
                 p = reinterpret_cast<void *>(v.heap + (lin << (16 + t)));
             } else {
                 p = big_inline(v, v.bigq[2 * (uint64_t)e + 1]);
@@ -790,27 +860,12 @@ __global__ void __launch_bounds__(kBigThreads, 1) k_big(uint32_t tag) {
                 ptx::atom_add(v.seg_word + i, core::sw_retree(core::kTreeFree, core::kTrees + (uint32_t)k));
                 for (uint64_t m = 1; m < k; m++)
                     ptx::atom_add(v.seg_word + i + m, core::sw_retree(core::kTreeFree, core::kTreeCont));
-                ptx::fence_acq_rel();
                 p = reinterpret_cast<void *>(v.heap + (i << core::kSegLog2));
             } else {
                 p = big_inline(v, size);
             }
         }
         *reinterpret_cast<uint64_t *>(addr) = reinterpret_cast<uint64_t>(p);
-    }
-#ifdef GALLATIN_TRACE
-    __syncthreads();
-    if (tid == 0) ptx::trace(tb0, ptx::globaltimer(), (13ull << 60) | 3);
-#endif
-    // the rest of each partly used segment becomes available (joins its block tree)
-    if (fr != kNone && tid < core::kTrees && tsegs[tid]) {
-        const uint32_t t = tid, nb = core::nb_of(t), used = tcnt[t] - (tsegs[t] - 1) * nb;
-        if (used < nb) {
-            const uint64_t s = fr + tbase[t] + tsegs[t] - 1;
-            const uint64_t old = ptx::atom_add(v.seg_word + s, (uint64_t)(nb - used));
-            core::seg_after_rmw(v, s, old, old + (nb - used));
-            core::oom_notify(v);
-        }
     }
     __syncthreads();
 #ifdef GALLATIN_TRACE
