@@ -457,10 +457,23 @@ def run_extras(args, G, torch, stream):
         if r >= 2:
             ins_l.append(ea.elapsed_time(eb))
             del_l.append(eb.elapsed_time(ec))
-    ins_ms, del_ms = statistics.median(ins_l), statistics.median(del_l)
+    ins_ms_eager, del_ms_eager = statistics.median(ins_l), statistics.median(del_l)
+
+    def vbody(mark):
+        v.clear()
+        mark()
+        v.insert(keys, want_out=False)
+        mark()
+        v.delete(dk, want_out=False)
+        mark()
+    il, dl = graph_phases(torch, vbody, 10)
+    ins_ms, del_ms = statistics.median(il), statistics.median(dl)
     v.close()
     out["veb"] = {"successor_ops_s": nq / succ_ms * 1e3, "successor_queries": nq, "successor_ms": succ_ms,
                   "insert_ops_s": len(w["insert"]) / ins_ms * 1e3, "delete_ops_s": len(w["delete"]) / del_ms * 1e3,
+                  "insert_ms": ins_ms, "delete_ms": del_ms, "insert_ms_eager": ins_ms_eager,
+                  "delete_ms_eager": del_ms_eager,
+                  "insert_delete_timing": "graph-replayed rounds (device time); *_eager: events around eager launches",
                   "universe": "2^20", "keys": len(w["insert"]),
                   "successor_hbm_gbs": nq * 16 / succ_ms / 1e6}
 
@@ -512,9 +525,13 @@ def run_extras(args, G, torch, stream):
         if it >= 3:
             mm.append(a.elapsed_time(b))
             fm.append(b.elapsed_time(c))
-    m, f = statistics.median(mm), statistics.median(fm)
+    me, fe = statistics.median(mm), statistics.median(fm)
+    m, f = malloc_free_graph(G, torch, sizes, p)
     out["mixed"] = {"threads": n, "malloc_ops_s": n / m * 1e3, "free_ops_s": n / f * 1e3,
                     "combined_ops_s": 2 * n / (m + f) * 1e3, "malloc_ms": m, "free_ms": f,
+                    "malloc_ms_eager": me, "free_ms_eager": fe,
+                    "timing": "medians of 7 reset+malloc+free rounds replayed as one CUDA graph; *_eager: events "
+                              "around eager launches",
                     "workload": "BASELINE configs[2]: 16 B-4 KB powers of two + p=2^-12 large 1-64 MB, 64 GiB heap"}
     G.gallatin_destroy()
     G.gallatin_init(HEAP_C2)
@@ -530,7 +547,8 @@ def run_extras(args, G, torch, stream):
 def run_grid(args, G, torch, stream) -> dict:
     """BASELINE configs[1] as a full grid: every size 16 B..4 KB
     x n = 2^20..2^24 threads on the 16 GiB heap.  The 39 cells with s*n <= 8 GiB
-    are timed (reset before every repetition, P:283; median and p10/p90 of 5);
+    are timed (reset before every repetition; median and p10/p90 of 5
+    rounds replayed as one CUDA graph, `graph_phases`);
     the 6 others are capacity runs (one call asking more than the heap holds:
     NULL count and time).  At the headline n of every size, warm rounds (no
     reset, after one untimed round) are timed beside the cold ones."""
@@ -554,19 +572,14 @@ def run_grid(args, G, torch, stream) -> dict:
                                            "granted_bytes": (n - nulls) * s}
                 G.gallatin_free(p)
                 continue
-            mm, fm = [], []
-            for _ in range(reps + 1):
+            def cold(mark):
                 G.gallatin_reset()
-                a, b, c = ev(), ev(), ev()
-                a.record(stream)
+                mark()
                 G.gallatin_malloc(st, p)
-                b.record(stream)
+                mark()
                 G.gallatin_free(p)
-                c.record(stream)
-                torch.cuda.synchronize()
-                mm.append(a.elapsed_time(b))
-                fm.append(b.elapsed_time(c))
-            mm, fm = mm[1:], fm[1:]
+                mark()
+            mm, fm = graph_phases(torch, cold, reps)
             m, f = statistics.median(mm), statistics.median(fm)
             cells[f"{s}x2^{lg}"] = {"n": n, "malloc_ms": round(m, 5), "free_ms": round(f, 5),
                                     "malloc_ms_p10_p90": [round(x, 5) for x in pctl(mm)],
@@ -576,17 +589,14 @@ def run_grid(args, G, torch, stream) -> dict:
                 G.gallatin_reset()
                 G.gallatin_malloc(st, p)
                 G.gallatin_free(p)                                   # the untimed first round
-                wm, wf = [], []
-                for _ in range(reps):
-                    a, b, c = ev(), ev(), ev()
-                    a.record(stream)
+
+                def warm_round(mark):
+                    mark()
                     G.gallatin_malloc(st, p)
-                    b.record(stream)
+                    mark()
                     G.gallatin_free(p)
-                    c.record(stream)
-                    torch.cuda.synchronize()
-                    wm.append(a.elapsed_time(b))
-                    wf.append(b.elapsed_time(c))
+                    mark()
+                wm, wf = graph_phases(torch, warm_round, reps)
                 warm[str(s)] = {"n": n, "cold_malloc_ms": round(m, 5), "warm_malloc_ms": round(statistics.median(wm), 5),
                                 "cold_free_ms": round(f, 5), "warm_free_ms": round(statistics.median(wf), 5),
                                 "warm_over_cold_malloc": statistics.median(wm) / m}
@@ -668,6 +678,48 @@ def run_paper_modes(args, G, torch):
     return out
 
 
+def graph_phases(torch, body, reps: int):
+    """Device time of each phase of body(mark), run `reps` times back to back as
+    ONE CUDA graph (no host launch gaps inside the timed region; the timing
+    events are graph nodes), replayed once to upload and once timed.  Phase i
+    runs from the i-th to the (i+1)-th mark() of a rep; returns
+    [[ms of phase i in rep r for r] for i]."""
+    marks = []
+
+    def mark():
+        e = torch.cuda.Event(enable_timing=True, external=True)
+        e.record(torch.cuda.current_stream())
+        marks.append(e)
+
+    g = torch.cuda.CUDAGraph()
+    cap = torch.cuda.Stream()
+    cap.wait_stream(torch.cuda.current_stream())
+    with torch.cuda.graph(g, stream=cap):
+        for _ in range(reps):
+            body(mark)
+    g.replay()
+    torch.cuda.synchronize()
+    g.replay()
+    torch.cuda.synchronize()
+    per = len(marks) // reps
+    res = [[marks[r * per + i].elapsed_time(marks[r * per + i + 1]) for r in range(reps)] for i in range(per - 1)]
+    del g
+    return res
+
+
+def malloc_free_graph(G, torch, st, p, reps: int = 7):
+    """(malloc ms, free ms) medians of reset + malloc + free, graph-timed."""
+    def body(mark):
+        G.gallatin_reset()
+        mark()
+        G.gallatin_malloc(st, p)
+        mark()
+        G.gallatin_free(p)
+        mark()
+    mm, fm = graph_phases(torch, body, reps)
+    return statistics.median(mm), statistics.median(fm)
+
+
 def run_scaling(args, G, torch, stream):
     """BASELINE configs[3]: 64 B mallocs then frees at 2^10 .. 2^26 threads on the
     16 GiB heap (reset before each run); median of 5 runs per point."""
@@ -689,9 +741,10 @@ def run_scaling(args, G, torch, stream):
             if it >= 2:
                 mm.append(a.elapsed_time(b))
                 fm.append(b.elapsed_time(c))
-        m, f = statistics.median(mm), statistics.median(fm)
+        me, fe = statistics.median(mm), statistics.median(fm)
+        m, f = malloc_free_graph(G, torch, st, p)
         pts[str(n)] = {"malloc_ms": round(m, 5), "free_ms": round(f, 5), "malloc_ops_s": n / m * 1e3,
-                       "free_ops_s": n / f * 1e3}
+                       "free_ops_s": n / f * 1e3, "malloc_ms_eager": round(me, 5), "free_ms_eager": round(fe, 5)}
         del st, p
     # the paper's other scaling sizes (16, 512, 8192 B) up to its 2^20 threads
     paper = {}
@@ -716,12 +769,17 @@ def run_scaling(args, G, torch, stream):
                 if it >= 2:
                     mm.append(a.elapsed_time(b))
                     fm.append(b.elapsed_time(c))
-            m, f = statistics.median(mm), statistics.median(fm)
+            me, fe = statistics.median(mm), statistics.median(fm)
+            m, f = malloc_free_graph(G, torch, st, p)
             pp[str(n)] = {"malloc_ms": round(m, 5), "free_ms": round(f, 5), "malloc_ops_s": n / m * 1e3,
-                          "free_ops_s": n / f * 1e3}
+                          "free_ops_s": n / f * 1e3, "malloc_ms_eager": round(me, 5), "free_ms_eager": round(fe, 5)}
         paper[str(size)] = pp
     return {"workload": "BASELINE configs[3]: 64 B, 2^10..2^26 threads (every 4th power), 16 GiB heap, "
-                        "independent per-GPU heap under torchrun", "points": pts,
+                        "independent per-GPU heap under torchrun",
+            "timing": "malloc_ms/free_ms: medians of 7 reset+malloc+free rounds replayed as one CUDA graph "
+                      "(device time, no host launch gap); *_eager: the same calls with events around eager "
+                      "launches (host ctypes launch latency included)",
+            "points": pts,
             "paper_sizes": {"workload": "P:329 sizes 16/512/8192 B at 2^10..2^20 threads (every 2nd power)",
                             "points": paper}}
 

@@ -513,7 +513,10 @@ __global__ void __launch_bounds__(NT, MINB) k_bulk_malloc_cta(const uint64_t *__
             run_base[c_me] = reinterpret_cast<uint64_t>(core::slice_ptr(v, c_me, old & core::kRunNone, 0));
             cls_over = my_lo + my_cnt > my_limit;
             cls_slow = (v.prefetch && my_lo <= (my_limit >> 1) && (my_limit >> 1) < my_lo + my_cnt) ||
-                       (v.demand_hint && my_limit - (my_lo + my_cnt) >= 16u * my_cnt &&
+                       // (checked by the tile whose draw crosses a 4-block mark only: every
+                       // check reads the slot's second word, a round trip the tile waits for)
+                       (v.demand_hint && (my_lo >> 14) != ((my_lo + my_cnt) >> 14) &&
+                        my_limit - (my_lo + my_cnt) >= 16u * my_cnt &&
                         blockIdx.x < gridDim.x - gridDim.x / 4 &&
                         (float)my_cnt * (float)(gridDim.x - blockIdx.x) * v.nslot_rcp[c_me] >=
                             (float)(my_limit - (my_lo + my_cnt) + core::kSlices));   // demand prefetch (tile_slow)

@@ -25,8 +25,10 @@ for sz in sizes:
     n = min(1 << 24, (8 << 30) // sz)
     st = torch.full((n,), sz, dtype=torch.int64, device="cuda")
     p = torch.empty_like(st)
+    warm = os.environ.get("TRACE_WARM") == "1"
     for rep in range(3):
-        G.gallatin_reset()
+        if not (warm and rep > 0):
+            G.gallatin_reset()
         torch.cuda.synchronize()
         L.gallatin_debug_trace(buf.data_ptr(), cap, None)
         e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
