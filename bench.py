@@ -207,15 +207,24 @@ def run_ours(args, rank, world, local):
 
     # the K timed steps as one CUDA graph (same launches, no host launch gaps
     # between the step's 27 kernels), replayed once untimed to upload it
-    graph = None
+    # Two graphs of the same K steps: `graph` (no timing nodes) is the timed
+    # region of `value`; `graph_ev` adds an event node around every malloc and
+    # free call and is replayed afterwards for the per-kernel times (event
+    # nodes sit on the critical path between kernels: ms_per_step_with_events)
+    graph = graph_ev = None
     if args.graph:
         graph = torch.cuda.CUDAGraph()
+        graph_ev = torch.cuda.CUDAGraph()
         cap = torch.cuda.Stream()
         cap.wait_stream(stream)
         with torch.cuda.graph(graph, stream=cap):
             for _ in range(args.steps):
+                step(False, cap)
+        with torch.cuda.graph(graph_ev, stream=cap):
+            for _ in range(args.steps):
                 step(True, cap)
         graph.replay()
+        graph_ev.replay()
         torch.cuda.synchronize()
     clk = ClockSampler(local)
     d.barrier()
@@ -235,6 +244,13 @@ def run_ours(args, rank, world, local):
     d.barrier()
     ms_local = t0.elapsed_time(t1)
     value, ms, total_ops = aggregate(d, ops_per_step * args.steps, ms_local)
+    ms_ev = None
+    if graph_ev is not None:                       # the per-kernel event times
+        t0.record(stream)
+        graph_ev.replay()
+        t1.record(stream)
+        torch.cuda.synchronize()
+        ms_ev = t0.elapsed_time(t1) / args.steps
 
     # per-kernel times (the roofline's dominant kernel)
     m_ms = [a.elapsed_time(b) for a, b in zip(ev["m0"], ev["m1"])]
@@ -294,9 +310,11 @@ def run_ours(args, rank, world, local):
         line = {
             "metric": "malloc+free ops/s per B200 (single-size sweep 16 B-4 KB)",
             "value": value, "unit": "ops/s", "n_gpus": world, "steps": args.steps, "warmup": max(args.warmup, 3),
-            "ms_per_step": ms / args.steps, "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
+            "ms_per_step": ms / args.steps, "ms_per_step_with_events": ms_ev,
+            "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
             "dtype": "u64", "data": "synthetic",
-            "config": {"launch": "one CUDA graph of the K timed steps" if args.graph else "eager",
+            "config": {"launch": ("one CUDA graph of the K timed steps (per-kernel times from a second graph "
+                                  "with event nodes around each call)") if args.graph else "eager",
                        "workload": "BASELINE configs[1]: single-size sweep 16 B-4 KB, n_s=min(2^24, 8GiB/s) threads, "
                                    "16 GiB heap, reset+malloc+free per size" + (f" (1/{args.scale} scale)" if args.scale > 1 else ""),
                        "heap_bytes": HEAP_C2, "cells": [[s, n] for s, n in cells],
@@ -311,7 +329,7 @@ def run_ours(args, rank, world, local):
                          "algorithmic_bytes_per_op": bytes_per_op, "peak_source": peak_src},
             "clocks": clocks,
             "e2e": e2e,
-            "gpu_launches": 27 * args.steps,
+            "gpu_launches": 36 * args.steps,             # per cell: k_reset, k_bulk_malloc_cta, k_big, k_bulk_free_w
             "cpu_baseline": cpu,
         }
         line.update(extras)
