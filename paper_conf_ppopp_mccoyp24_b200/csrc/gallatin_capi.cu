@@ -90,25 +90,25 @@ __global__ void k_reset() {
     const uint64_t W = v.tree_words, nseg = v.nseg, pf = v.pf_segs;
     const uint64_t S = v.nslot_total;
     const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
-    uint64_t total = nseg * 128;
-    if (S * 16 > total) total = S * 16;
+    // one thread per 16 B of the largest arrays (block counters: 64 per
+    // segment, ring entries: 32 per segment, slot lines: 8 per slot)
+    uint64_t total = nseg * 64;
+    if (S * 8 > total) total = S * 8;
     if (9 * W > total) total = 9 * W;
     if (9 * 32 > total) total = 9 * 32;
+    const uint4 ones = make_uint4(~0u, ~0u, ~0u, ~0u), zeros = make_uint4(0u, 0u, 0u, 0u);
     for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < total; i += stride) {
         if (i < W) {
             // segment tree: leaf bit s set iff pf <= s < nseg; a summary bit
-            // set iff its child covers such a segment
+            // set iff its child covers such a segment: children ch of this
+            // word with ch < nbits and (ch + 1) * span > pf, i.e. ch >= pf / span
             uint32_t lvl = 0;
             while (lvl + 1 < v.tree_levels && i >= v.level_off[lvl + 1]) lvl++;
             const uint64_t word = i - v.level_off[lvl];
             const uint64_t nbits = lvl == 0 ? nseg : (uint64_t)(v.level_off[lvl] - v.level_off[lvl - 1]);
-            const uint64_t span = 1ull << (6 * lvl);                  // segments per child
-            uint64_t w = 0;
-            for (uint32_t b = 0; b < 64; b++) {
-                const uint64_t ch = word * 64 + b;
-                if (ch < nbits && (ch + 1) * span > pf) w |= 1ull << b;
-            }
-            v.seg_tree[i] = w;
+            const uint64_t lo_ch = pf >> (6 * lvl);
+            const uint64_t lo = lo_ch > word * 64 ? lo_ch : word * 64, hi = nbits < word * 64 + 64 ? nbits : word * 64 + 64;
+            v.seg_tree[i] = lo < hi ? bit_range((uint32_t)(lo - word * 64), (uint32_t)(hi - word * 64)) : 0ull;
         }
         if (i < 9 * W) {
             // block tree t holds only its class's partly used prefill segment
@@ -136,31 +136,40 @@ __global__ void k_reset() {
             v.q_head[i] = 0;
             v.q_tail[i] = tail;
         }
-        if (i < nseg * 64) {
-            uint64_t e = ~0ull;
-            const uint64_t s = i / 64, q0 = (i % 64) * 4;
+        if (i < nseg * 32) {                                             // ring entries, 8 per thread
+            uint4 e = ones;
+            const uint64_t s = i / 32;
             if (s < pf) {
                 const uint32_t t = pf_class_of(v, s);
                 if (s == v.pf_last[t]) {                                 // ring: blocks used..nb-1, ascending
-                    const uint32_t u = v.pf_used[t], cnt = core::nb_of(t) - u;
-                    e = 0;
-                    for (uint32_t k = 0; k < 4; k++)
-                        e |= (uint64_t)(q0 + k < cnt ? (uint16_t)(u + q0 + k) : core::kRingEmpty) << (16 * k);
+                    const uint32_t u = v.pf_used[t], cnt = core::nb_of(t) - u, q0 = (uint32_t)(i % 32) * 8;
+                    uint32_t h[4];
+#pragma unroll
+                    for (uint32_t k = 0; k < 4; k++) {
+                        const uint32_t a0 = q0 + 2 * k, a1 = a0 + 1;
+                        h[k] = (a0 < cnt ? (u + a0) : core::kRingEmpty) | ((a1 < cnt ? (u + a1) : core::kRingEmpty) << 16);
+                    }
+                    e = make_uint4(h[0], h[1], h[2], h[3]);
                 }
             }
-            reinterpret_cast<uint64_t *>(v.q_entries)[i] = e;
+            reinterpret_cast<uint4 *>(v.q_entries)[i] = e;
         }
-        if (i < nseg * 128) reinterpret_cast<uint64_t *>(v.block_free)[i] = 0;
-        if (i < S * 16) {
-            const uint64_t w = i % 16, si = i / 16;
-            uint64_t val = w <= 1 ? core::kSlotEmpty : 0;
-            if (pf && w == 0) {
-                uint32_t c = 0;
-                while (c + 1 < core::kTrees && si >= v.slot_off[c + 1]) c++;
-                const uint64_t first = (uint64_t)v.pf_base[c] * core::nb_of(c) + (si - v.slot_off[c]) * v.pf_run[c];
-                val = ((uint64_t)v.pf_run[c] << core::kRunShift) | first;
+        if (i < nseg * 64) reinterpret_cast<uint4 *>(v.block_free)[i] = zeros;
+        if (i < S * 8) {                                                 // slot lines: words 2j, 2j + 1
+            const uint64_t j = i % 8, si = i / 8;
+            uint64_t w0 = 0, w1 = 0;
+            if (j == 0) {
+                w0 = core::kSlotEmpty;
+                w1 = core::kSlotEmpty;
+                if (pf) {
+                    uint32_t c = 0;
+                    while (c + 1 < core::kTrees && si >= v.slot_off[c + 1]) c++;
+                    const uint64_t first = (uint64_t)v.pf_base[c] * core::nb_of(c) + (si - v.slot_off[c]) * v.pf_run[c];
+                    w0 = ((uint64_t)v.pf_run[c] << core::kRunShift) | first;
+                }
             }
-            v.slots[i] = val;
+            reinterpret_cast<uint4 *>(v.slots)[i] =
+                make_uint4((uint32_t)w0, (uint32_t)(w0 >> 32), (uint32_t)w1, (uint32_t)(w1 >> 32));
         }
         if (i < 9 * 32) v.fmt_token[i] = 0;
         if (i == 0) *v.err = 0;
@@ -1385,8 +1394,8 @@ int gallatin_destroy(void) {
 
 int gallatin_reset(void *stream) {
     if (!g.init) return GALLATIN_ERR_STATE;
-    uint64_t n = g.v.nseg * 128;
-    if ((uint64_t)g.v.nslot_total * 16 > n) n = (uint64_t)g.v.nslot_total * 16;
+    uint64_t n = g.v.nseg * 64;
+    if ((uint64_t)g.v.nslot_total * 8 > n) n = (uint64_t)g.v.nslot_total * 8;
     unsigned grid = grid_for(n);
     if (grid > 148 * 16) grid = 148 * 16;
     k_reset<<<grid, kThreads, 0, S(stream)>>>();
