@@ -43,6 +43,7 @@ struct State {
     cudaStream_t cin = nullptr, cout = nullptr;
     uint32_t launch_tag = 0;                          // bulk malloc launches (deferred-request queue owner)
     bool pdl = true;
+    bool defer_big = true;
     cudaEvent_t ev_in[kMaxChunks] = {}, ev_k[kMaxChunks] = {};
 };
 State g;
@@ -1367,6 +1368,8 @@ int gallatin_init_ex(const gallatin_config_t *cfg_in) {
     {
         const char *e = getenv("GALLATIN_PDL");
         g.pdl = !(e && e[0] == '0');
+        const char *b = getenv("GALLATIN_DEFER_BIG");             // measurement: 0 = serve big requests inline
+        g.defer_big = !(b && b[0] == '0');
     }
     g.cfg = cfg;
     g.heap_raw = heap;
@@ -1410,10 +1413,10 @@ int gallatin_malloc(const uint64_t *d_sizes, void **d_ptrs, uint64_t n, void *st
     if (items == 4) {  // 128-thread CTAs, 4 requests per thread, one slot RMW per class per CTA
         // the launch's tag claims the deferred-request queue; its batch kernel follows
         if (++g.launch_tag == 0) g.launch_tag = 1;
-        k_bulk_malloc_cta<4, 10, 128><<<(unsigned)((n + 511) / 512), 128, 0, S(stream)>>>(d_sizes, d_ptrs, n,
-                                                                                       g.launch_tag);
+        k_bulk_malloc_cta<4, 10, 128><<<(unsigned)((n + 511) / 512), 128, 0, S(stream)>>>(
+            d_sizes, d_ptrs, n, g.defer_big ? g.launch_tag : 0u);
         const int rc = launch_status();
-        if (rc) return rc;
+        if (rc || !g.defer_big) return rc;
         // programmatic dependent launch: k_big's launch overlaps the tail of
         // the malloc kernel; it waits for that kernel with griddepcontrol.wait
         cudaLaunchConfig_t lc = {};
