@@ -521,3 +521,84 @@ def test_oom_record_cleared_by_frees(cuda_ok, G):
     assert got3 >= nseg * SEG // 1024 - G.gallatin_stats()["nslot"][6] * 4096
     G.gallatin_free(r)
     _assert_pristine(G, nseg)
+
+
+# ---- the batch kernel of deferred big requests (k_big, DESIGN.md Deviations 21) ----
+def _check_live(G, nseg, sizes_list, ptrs_list):
+    """stamp / verify / usable / overlap over the union of several launches' pointers."""
+    base = G.gallatin_stats()["heap_base"]
+    ps, us = [], []
+    for sizes, ptrs in zip(sizes_list, ptrs_list):
+        d = _dev(sizes)
+        G.gallatin_stamp(ptrs, d)
+        assert G.gallatin_verify(ptrs, d) == 0, "stamp-verify found overwritten words"
+        usable = torch.empty_like(ptrs)
+        usum, ubad = G.gallatin_usable(ptrs, d, usable)
+        assert ubad == 0
+        p = _u64(ptrs)
+        live = p != 0
+        want = int(sum(class_size(int(s)) * int(c) for s, c in zip(*np.unique(sizes[live], return_counts=True))))
+        assert usum == want
+        ps.append(p[live])
+        us.append(_u64(usable)[live])
+    p, u = np.concatenate(ps), np.concatenate(us)
+    order = np.argsort(p)
+    assert np.all(p[order][:-1] + u[order][:-1] <= p[order][1:]), "overlapping allocations"
+    assert np.all((p - np.uint64(base)) < np.uint64(nseg * SEG))
+
+
+def test_deferred_big_requests_two_streams(cuda_ok, G):
+    """Two bulk launches with whole-block and segment requests run at once on
+    two streams: one claims the deferred-request queue, the other finds it
+    taken and serves its big requests inline; every request is granted,
+    disjoint, stamp-verified and accounted; free-all + drain is pristine."""
+    nseg = 2048
+    G.gallatin_init(nseg * SEG)
+    n = (1 << 20) + 77                                   # the CTA kernel (>= 606,208 requests)
+    sizes = [wg.mixed_sizes(n, seed=wg.cell_seed(3, 70 + k), p_large=2.0 ** -12) for k in range(2)]
+    d = [_dev(s) for s in sizes]
+    streams = [torch.cuda.Stream(), torch.cuda.Stream()]
+    for s in streams:
+        s.wait_stream(torch.cuda.current_stream())
+    ptrs = []
+    for k in range(2):
+        with torch.cuda.stream(streams[k]):
+            ptrs.append(G.gallatin_malloc(d[k], stream=streams[k].cuda_stream))
+    torch.cuda.synchronize()
+    assert all(int((p == 0).sum().item()) == 0 for p in ptrs)
+    assert sum(int((s > 4096).sum()) for s in sizes) > 300   # both launches carry big requests
+    _check_live(G, nseg, sizes, ptrs)
+    for p in ptrs:
+        G.gallatin_free(p)
+    torch.cuda.synchronize()
+    _assert_pristine(G, nseg)
+
+
+def test_deferred_queue_overflow(cuda_ok, G):
+    """More big requests than the queue holds (8192): the rest are served
+    inline by their tiles; everything granted, disjoint, pristine after."""
+    nseg = 1024
+    G.gallatin_init(nseg * SEG)
+    n = 1 << 20
+    sizes = wg.single_sizes(64, n).copy()
+    idx = wg.distinct_below(wg.cell_seed(3, 80), 12000, n).astype(np.int64)
+    sizes[idx] = 65537                                   # 128 KB blocks of tree 1 (12000 x 128 KB = 1.5 GB)
+    assert _bulk_round(G, nseg, sizes) == 0
+    _assert_pristine(G, nseg)
+
+
+def test_deferred_big_near_exhaustion(cuda_ok, G):
+    """Segment and block requests that do not all fit (a 1 GB heap, 100 x 16 MB
+    + 200 x 1 MB + 2^20 x 16 B): the batch claims fail, the per-request path
+    grants what fits and returns NULL for the rest; the granted ones are
+    disjoint and verified, and free-all + drain is pristine."""
+    nseg = 64
+    G.gallatin_init(nseg * SEG)
+    n = 1 << 20
+    sizes = wg.single_sizes(16, n).copy()
+    idx = wg.distinct_below(wg.cell_seed(3, 81), 300, n).astype(np.int64)
+    sizes[idx[:100]] = 16 << 20
+    sizes[idx[100:]] = 1 << 20
+    nulls = _bulk_round(G, nseg, sizes)
+    assert 0 < nulls <= 300
+    _assert_pristine(G, nseg)
