@@ -134,7 +134,9 @@ def main():
             si = shdr.index("Warp Stall Sampling (All Samples)")
             tot = sum(int(x[si]) for x in rows) or 1
             top = sorted(range(len(rows)), key=lambda i: -int(rows[i][si]))[:6]
-            lines += [f"### Top stall sites: `{name.split('(')[0]}`", "", "| share | SASS (stalled instruction; its producer precedes it) |", "|---:|---|"]
+            full = name.replace("void ", "").replace("<unnamed>::", "").replace("(anonymous namespace)::", "")
+            lines += [f"### Top stall sites: `{full[:140]}` (every captured launch of this kernel, aggregated)", "",
+                      "| share | SASS (stalled instruction; its producer precedes it) |", "|---:|---|"]
             for i in top:
                 ctx = " ⟵ ".join(rows[j][1].strip()[:60] for j in range(i, max(-1, i - 3), -1))
                 lines.append(f"| {int(rows[i][si]) / tot:.1%} | `{ctx}` |")
