@@ -86,6 +86,14 @@ def main():
                  "| kernel | launches | total µs | mean µs | share |", "|---|---:|---:|---:|---:|"]
         for k, v in sorted(agg.items(), key=lambda x: -sum(x[1])):
             lines.append(f"| `{k[:70]}` | {len(v)} | {sum(v):.1f} | {sum(v) / len(v):.2f} | {sum(v) / tot:.1%} |")
+        # the kernels of the bench's timed step only (the list above also holds
+        # the untimed warm-up gate, post-run drain / stats and the RMW count)
+        timed = {k: v for k, v in agg.items() if k.startswith(("k_reset", "k_bulk_malloc", "k_big", "k_bulk_free"))}
+        tt = sum(sum(v) for v in timed.values()) or 1.0
+        lines += ["", "Kernels of the timed step only (reset, malloc, batch kernel, free):", "",
+                  "| kernel | launches | total µs | mean µs | share of the step's kernels |", "|---|---:|---:|---:|---:|"]
+        for k, v in sorted(timed.items(), key=lambda x: -sum(x[1])):
+            lines.append(f"| `{k[:70]}` | {len(v)} | {sum(v):.1f} | {sum(v) / len(v):.2f} | {sum(v) / tt:.1%} |")
         open(os.path.join(prof, f"{a.tag}_launches.md"), "w").write("\n".join(lines) + "\n")
     if a.report:
         raw = ncu_csv(a.report, "raw")
