@@ -103,7 +103,12 @@ int gallatin_is_initialized(void);                      /* 1 / 0 */
 /* Bulk malloc (Alg. 3 -> 2 -> 1): d_ptrs[i] = malloc(d_sizes[i]) by
  * one GPU thread per request.  Size 0 and exhaustion give NULL.  Sizes
  * <= 4096 B are slices (16 B .. 4 KB powers of two); (4 KB, 16 MB)
- * whole blocks; >= 16 MB whole contiguous segments. */
+ * whole blocks; >= 16 MB whole contiguous segments.
+ * From 606,208 requests on the call is two kernels on `stream`: the bulk
+ * kernel, and a one-CTA batch kernel that serves the launch's whole-block and
+ * segment requests together (DESIGN.md Deviations 21; a launch running
+ * concurrently with another one's batch serves its own inline).  Every
+ * d_ptrs[i] is written when the stream reaches the end of the call. */
 int gallatin_malloc(const uint64_t *d_sizes, void **d_ptrs, uint64_t n, void *stream);
 
 /* Bulk free (Alg. 4).  NULL entries are ignored.  A pointer outside
