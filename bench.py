@@ -183,9 +183,10 @@ def run_ours(args, rank, world, local):
             if record:
                 e = torch.cuda.Event(enable_timing=True, external=ext); e.record(cur); ev["m0"].append(e)
             G.gallatin_malloc(st, p)
-            if record:
-                e = torch.cuda.Event(enable_timing=True, external=ext); e.record(cur); ev["m1"].append(e)
-                e = torch.cuda.Event(enable_timing=True, external=ext); e.record(cur); ev["f0"].append(e)
+            if record:                                   # one event node ends the malloc and starts the free
+                e = torch.cuda.Event(enable_timing=True, external=ext); e.record(cur)
+                ev["m1"].append(e)
+                ev["f0"].append(e)
             G.gallatin_free(p)
             if record:
                 e = torch.cuda.Event(enable_timing=True, external=ext); e.record(cur); ev["f1"].append(e)
