@@ -486,15 +486,34 @@ __global__ void __launch_bounds__(NT, MINB) k_bulk_malloc_cta(const uint64_t *__
         cr[k] = s - 1 < core::kMaxSlice ? sc : (s == 0 ? 0xFEu : 0xFFu);   // branch-free slice_class
     }
     __syncthreads();
-    const uint32_t lt = ptx::lanemask_lt();
+    // A warp whose 32 x ITEMS requests are all of one slice class (single-size
+    // launches: every warp) takes 32 x ITEMS consecutive ranks of its class
+    // with one shared atomic -- any bijection onto [0, count) serves (the tile
+    // ranks are only offsets into the run) -- instead of one match, shared
+    // atomic and shuffle per item; the item pass then reads its class's run
+    // once.  Other warps rank per item by warp teams.
+    const uint32_t cw = __shfl_sync(0xFFFFFFFFu, cr[0], 0);
+    bool mine = cw < core::kTrees;
 #pragma unroll
-    for (int k = 0; k < ITEMS; k++) {
-        const uint32_t c = cr[k];
-        const unsigned peers = __match_any_sync(0xFFFFFFFFu, c);
-        const uint32_t leader = (uint32_t)__ffs((int)peers) - 1;
+    for (int k = 0; k < ITEMS; k++) mine &= cr[k] == cw;
+    const bool uni = __all_sync(0xFFFFFFFFu, mine);
+    if (uni) {
         uint32_t b = 0;
-        if (c < core::kTrees && lane == leader) b = atomicAdd(&cnt[c], (uint32_t)__popc(peers));
-        cr[k] = c | ((__shfl_sync(0xFFFFFFFFu, b, (int)leader) + (uint32_t)__popc(peers & lt)) << 8);
+        if (lane == 0) b = atomicAdd(&cnt[cw], 32u * ITEMS);
+        b = __shfl_sync(0xFFFFFFFFu, b, 0) + lane;
+#pragma unroll
+        for (int k = 0; k < ITEMS; k++) cr[k] = cw | ((b + 32u * k) << 8);
+    } else {
+        const uint32_t lt = ptx::lanemask_lt();
+#pragma unroll
+        for (int k = 0; k < ITEMS; k++) {
+            const uint32_t c = cr[k];
+            const unsigned peers = __match_any_sync(0xFFFFFFFFu, c);
+            const uint32_t leader = (uint32_t)__ffs((int)peers) - 1;
+            uint32_t b = 0;
+            if (c < core::kTrees && lane == leader) b = atomicAdd(&cnt[c], (uint32_t)__popc(peers));
+            cr[k] = c | ((__shfl_sync(0xFFFFFFFFu, b, (int)leader) + (uint32_t)__popc(peers & lt)) << 8);
+        }
     }
     __syncthreads();
     // Class c is served by thread (c % warps) * 32 + c / warps (one per warp
@@ -544,6 +563,21 @@ __global__ void __launch_bounds__(NT, MINB) k_bulk_malloc_cta(const uint64_t *__
     // items whose slice lies inside the run are stored now; the rest wait in
     // `pend` for the tile's next round (bit k: item k)
     uint32_t pend = 0, big = 0, pfd = 0;
+    if (uni) {                                            // one class: its run read once
+        const uint64_t ll = lim_lo[cw], rb = run_base[cw];
+        const uint32_t limit = (uint32_t)(ll >> 32);
+#pragma unroll
+        for (int k = 0; k < ITEMS; k++) {
+            const uint32_t idx = (uint32_t)ll + (cr[k] >> 8);
+            if (idx < limit) {
+                __stcs(reinterpret_cast<unsigned long long *>(ptrs) + base + (uint64_t)NT * k,
+                       rb + ((uint64_t)idx << (core::kMinSliceLog2 + cw)));
+                if (v.prefetch && idx == (limit >> 1)) pfd |= 1u << k;
+            } else {
+                pend |= 1u << k;
+            }
+        }
+    } else
 #pragma unroll
     for (int k = 0; k < ITEMS; k++) {
         const uint64_t i = base + (uint64_t)NT * k;
