@@ -17,5 +17,5 @@ timeout 900 ncu --set full --metrics $M --clock-control none --import-source on 
     -o gpurun_out/prof_veb -f python tools/prof_extra.py veb > gpurun_out/ncu_veb.log 2>&1; echo "ncu veb rc=$?"
 timeout 900 ncu --set full --metrics $M --clock-control none --import-source on -k regex:"k_bulk|k_big" -s 3 -c 3 \
     -o gpurun_out/prof_mixed -f python tools/prof_extra.py mixed > gpurun_out/ncu_mixed.log 2>&1; echo "ncu mixed rc=$?"
-timeout 1500 ncu --set full --metrics $M --clock-control none --import-source on -k regex:"k_(count|grow|copy|scatter|hash|list|shrink|expand|edge)" -c 40 \
+timeout 1500 ncu --set full --metrics $M --clock-control none --import-source on -k regex:"k_(count|grow|copy|scatter|hash|list|shrink|expand|edge|delete|free_all)" -c 60 \
     -o gpurun_out/prof_graph -f python tools/prof_extra.py graph > gpurun_out/ncu_graph.log 2>&1; echo "ncu graph rc=$?"
