@@ -854,12 +854,6 @@ __global__ void __launch_bounds__(kBigThreads, 1) k_big(uint32_t tag) {
             while (x >= (uint64_t)tbase[t] + tsegs[t]) t++;
             const uint64_t s = fr + x;
             const uint32_t nb = core::nb_of(t), used = tcnt[t] - (tsegs[t] - 1) * nb;
-            if (x == (uint64_t)tbase[t] + tsegs[t] - 1 && used < nb) {
-                uint16_t *e = v.q_entries + s * core::kMaxBlocks;
-                for (uint32_t q = 0; q < nb - used; q++) e[q] = (uint16_t)(used + q);
-                ptx::st_relaxed(v.q_head + s, 0u);
-                ptx::st_relaxed(v.q_tail + s, nb - used);
-            }
             ptx::st_relaxed(v.seg_tid + s, t);
             ptx::atom_add(v.seg_word + s, core::sw_retree(core::kTreeFree, t));
         }
@@ -874,10 +868,22 @@ __global__ void __launch_bounds__(kBigThreads, 1) k_big(uint32_t tag) {
         const uint32_t t = lane, nb = core::nb_of(t), used = tcnt[t] - (tsegs[t] - 1) * nb;
         if (used < nb) {
             const uint64_t s = fr + tbase[t] + tsegs[t] - 1;
-            ptx::fence_acq_rel();                             // the ring entries (another thread's) before the count
-            const uint64_t old = ptx::atom_add(v.seg_word + s, (uint64_t)(nb - used));
-            core::seg_after_rmw(v, s, old, old + (nb - used));
-            core::oom_notify(v);
+            // the rest of the segment's blocks, consecutive: a run for the
+            // next-run word of class t's first slot when that word is free
+            // (one CAS; it is swapped in at the slot's next refill, trims and
+            // the drain give it back like any fetched run), else into the
+            // segment's ring and block tree (initSegment)
+            const uint64_t run = ((uint64_t)(nb - used) << core::kRunShift) | (s * nb + used);
+            if (ptx::atom_cas(core::slot_word(v, v.slot_off[t]) + 1, core::kSlotEmpty, run) != core::kSlotEmpty) {
+                uint16_t *e = v.q_entries + s * core::kMaxBlocks;
+                for (uint32_t q = 0; q < nb - used; q++) e[q] = (uint16_t)(used + q);
+                ptx::st_relaxed(v.q_head + s, 0u);
+                ptx::st_relaxed(v.q_tail + s, nb - used);
+                ptx::fence_acq_rel();                         // ring entries before the count
+                const uint64_t old = ptx::atom_add(v.seg_word + s, (uint64_t)(nb - used));
+                core::seg_after_rmw(v, s, old, old + (nb - used));
+                core::oom_notify(v);
+            }
         }
     }
     // 3. pointers (read by the caller after this kernel: its end orders the
