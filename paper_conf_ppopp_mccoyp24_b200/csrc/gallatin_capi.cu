@@ -641,6 +641,25 @@ __device__ __noinline__ void *big_inline(const View &v, uint64_t size) { return 
 // copy of the segment tree's leaves); kNone if none
 __device__ uint64_t lowest_run_of(const uint64_t *lw, uint64_t nw, uint64_t k) {
     uint64_t run = 0, start = 0;
+    if (k > 64) {
+        // a run longer than a word is the leading ones of one word, whole
+        // words, and the trailing ones of another: O(1) per word
+        for (uint64_t wi = 0; wi < nw; wi++) {
+            const uint64_t x = lw[wi], base = wi << 6;
+            if (x == ~0ull) {
+                if (!run) start = base;
+                run += 64;
+                if (run >= k) return start;
+                continue;
+            }
+            const uint32_t tr = (uint32_t)__ffsll((long long)~x) - 1;
+            if (run + tr >= k) return start;
+            const uint32_t lead = (uint32_t)__clzll((long long)~x);          // ones from bit 63 down
+            run = lead;
+            start = base + 64 - lead;
+        }
+        return kNone;
+    }
     for (uint64_t wi = 0; wi < nw; wi++) {
         const uint64_t x = lw[wi], base = wi << 6;
         if (x == ~0ull) {
