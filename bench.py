@@ -615,7 +615,7 @@ def run_grid(args, G, torch, stream) -> dict:
                     mark()
                     G.gallatin_free(p)
                     mark()
-                wm, wf = graph_phases(torch, warm_round, reps)
+                wm, wf = graph_phases(torch, warm_round, 2 * reps - 1)         # warm state drifts: 9 rounds
                 warm[str(s)] = {"n": n, "cold_malloc_ms": round(m, 5), "warm_malloc_ms": round(statistics.median(wm), 5),
                                 "cold_free_ms": round(f, 5), "warm_free_ms": round(statistics.median(wf), 5),
                                 "warm_over_cold_malloc": statistics.median(wm) / m}
