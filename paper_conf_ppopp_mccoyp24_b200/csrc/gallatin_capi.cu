@@ -865,14 +865,13 @@ __global__ void __launch_bounds__(kBigThreads, 1) k_big(uint32_t tag) {
     if (tid == 0) ptx::trace(tb0, ptx::globaltimer(), (13ull << 60) | 2);
 #endif
     // the trees' segments, taken privately ({t, 0 available}, tree-id copy);
-    // a tree's partly used last segment: the rest of its blocks into its ring
+    // (a tree's partly used last segment too: its other blocks are placed below)
     const uint64_t fr = front;
     if (fr != kNone) {
         for (uint64_t x = tid; x < T; x += kBigThreads) {
             uint32_t t = 0;
             while (x >= (uint64_t)tbase[t] + tsegs[t]) t++;
             const uint64_t s = fr + x;
-            const uint32_t nb = core::nb_of(t), used = tcnt[t] - (tsegs[t] - 1) * nb;
             ptx::st_relaxed(v.seg_tid + s, t);
             ptx::atom_add(v.seg_word + s, core::sw_retree(core::kTreeFree, t));
         }
