@@ -28,6 +28,8 @@ import time
 
 ROOT = os.path.dirname(os.path.abspath(__file__))
 sys.path.insert(0, ROOT)
+if os.environ.get("GALLATIN_PKG_ROOT"):            # same-box A/B of another build (tools/ab_build.sh)
+    sys.path.insert(0, os.environ["GALLATIN_PKG_ROOT"])
 
 import numpy as np  # noqa: E402
 
