@@ -325,7 +325,7 @@ def run_ours(args, rank, world, local):
                        "l2": "no flush: each step reads %.2f GiB of sizes + writes/reads the pointer array (> 126 MB L2)" % (
                            sum(8 * n for _, n in cells) / 2 ** 30)},
             "malloc_ops_s": malloc_ops_s, "free_ops_s": free_ops_s, "per_size": per_cell, "rmw_counts": rmw,
-            "roofline": {"bound": "hbm", "kernel": "k_bulk_malloc_cta<4,10,128>" if dominant == "malloc" else "k_bulk_free_w<4,64,32>", "achieved": achieved, "peak": hbm_peak,
+            "roofline": {"bound": "hbm", "kernel": "k_bulk_malloc_cta<4,16,128>" if dominant == "malloc" else "k_bulk_free_w<4,64,32>", "achieved": achieved, "peak": hbm_peak,
                          "unit": "GB/s", "frac": achieved / hbm_peak, "traffic": traffic,
                          "traffic_algorithmic": bytes_per_op * (1 << 24),
                          "traffic_note": "DRAM bytes of one 2^24-thread launch (16 B cell, profiles/r1_kernels.md)",

@@ -1471,7 +1471,7 @@ int gallatin_malloc(const uint64_t *d_sizes, void **d_ptrs, uint64_t n, void *st
     if (items == 4) {  // 128-thread CTAs, 4 requests per thread, one slot RMW per class per CTA
         // the launch's tag claims the deferred-request queue; its batch kernel follows
         if (++g.launch_tag == 0) g.launch_tag = 1;
-        k_bulk_malloc_cta<4, 10, 128><<<(unsigned)((n + 511) / 512), 128, 0, S(stream)>>>(
+        k_bulk_malloc_cta<4, 16, 128><<<(unsigned)((n + 511) / 512), 128, 0, S(stream)>>>(
             d_sizes, d_ptrs, n, g.defer_big ? g.launch_tag : 0u);
         const int rc = launch_status();
         if (rc || !g.defer_big) return rc;
