@@ -325,7 +325,7 @@ def run_ours(args, rank, world, local):
                        "l2": "no flush: each step reads %.2f GiB of sizes + writes/reads the pointer array (> 126 MB L2)" % (
                            sum(8 * n for _, n in cells) / 2 ** 30)},
             "malloc_ops_s": malloc_ops_s, "free_ops_s": free_ops_s, "per_size": per_cell, "rmw_counts": rmw,
-            "roofline": {"bound": "hbm", "kernel": "k_bulk_malloc_cta<4,16,128>" if dominant == "malloc" else "k_bulk_free_w<4,64,32>", "achieved": achieved, "peak": hbm_peak,
+            "roofline": {"bound": "hbm", "kernel": "k_bulk_malloc_cta<8,10,128>" if dominant == "malloc" else "k_bulk_free_w<4,64,32>", "achieved": achieved, "peak": hbm_peak,
                          "unit": "GB/s", "frac": achieved / hbm_peak, "traffic": traffic,
                          "traffic_algorithmic": bytes_per_op * (1 << 24),
                          "traffic_note": "DRAM bytes of one 2^24-thread launch (16 B cell, profiles/r1_kernels.md)",
@@ -350,7 +350,7 @@ def pctl(xs):
 def count_rmws(G, torch, cells, size_t, ptrs) -> dict:
     """Per cell, the L2 RMWs the bulk kernels issue at minimum (SURVEY 8(d)
     "Algorithmic work per unit"): malloc = one slot RMW per class per
-    512-request CTA tile (single size: ceil(n / 512)); free = one counter RMW
+    1024-request CTA tile (single size: ceil(n / 1024)); free = one counter RMW
     per (warp, block) team, counted from the pointers one malloc returns (lane
     l of warp w frees ptrs[128 w + 32 k + l]: teams per 32-pointer row)."""
     base = G.gallatin_stats()["heap_base"]
@@ -366,7 +366,7 @@ def count_rmws(G, torch, cells, size_t, ptrs) -> dict:
         g = torch.sort(g.view(rows, 32), dim=1).values
         teams = int(((g[:, 1:] != g[:, :-1]).sum() + rows).item())
         G.gallatin_free(p)
-        out[str(s)] = {"malloc_slot_rmws": (n + 511) // 512, "free_team_rmws": teams, "nslot": G.gallatin_stats()["nslot"][c]}
+        out[str(s)] = {"malloc_slot_rmws": (n + 1023) // 1024, "free_team_rmws": teams, "nslot": G.gallatin_stats()["nslot"][c]}
     torch.cuda.synchronize()
     G.gallatin_reset()
     return out

@@ -73,7 +73,7 @@ typedef struct gallatin_config {
     uint32_t fence_free;
     uint32_t bulk_items;   /* bulk kernels: 0 = auto (4 from 606,208 requests on, else 1); 1 = one request per
                               thread and one slot RMW per warp team (k_bulk_malloc<1> / k_bulk_free<1>); 4 = four
-                              per thread, one slot RMW per class per 512-request CTA tile (k_bulk_malloc_cta) and
+                              per thread (eight in the malloc), one slot RMW per class per 1024-request CTA tile (k_bulk_malloc_cta) and
                               the warp-team free with 32-bit block ids (k_bulk_free_w) */
     uint32_t run_init;     /* first run of an empty slot of class c: min(max(run_init >> c, min(run_init, 8)), 256 >> c) blocks (default: the largest power of two <= 256 whose first runs over all slots fit in half the heap) */
     uint32_t prefetch;     /* 1 = fetch the next run at the middle of the current one; 0/2 = off (default) */

@@ -1468,10 +1468,10 @@ int gallatin_malloc(const uint64_t *d_sizes, void **d_ptrs, uint64_t n, void *st
     if (n == 0) return GALLATIN_OK;
     if (!d_sizes || !d_ptrs || n > (1ull << 40)) return GALLATIN_ERR_INVALID;
     const uint32_t items = g.cfg.bulk_items ? g.cfg.bulk_items : (n >= (uint64_t)kItemsMin ? 4u : 1u);
-    if (items == 4) {  // 128-thread CTAs, 4 requests per thread, one slot RMW per class per CTA
+    if (items == 4) {  // 128-thread CTAs, 8 requests per thread, one slot RMW per class per CTA
         // the launch's tag claims the deferred-request queue; its batch kernel follows
         if (++g.launch_tag == 0) g.launch_tag = 1;
-        k_bulk_malloc_cta<4, 16, 128><<<(unsigned)((n + 511) / 512), 128, 0, S(stream)>>>(
+        k_bulk_malloc_cta<8, 10, 128><<<(unsigned)((n + 1023) / 1024), 128, 0, S(stream)>>>(
             d_sizes, d_ptrs, n, g.defer_big ? g.launch_tag : 0u);
         const int rc = launch_status();
         if (rc || !g.defer_big) return rc;

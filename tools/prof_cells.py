@@ -4,6 +4,8 @@ import os
 import sys
 
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+if os.environ.get("GALLATIN_PKG_ROOT"):
+    sys.path.insert(0, os.environ["GALLATIN_PKG_ROOT"])  # another build of the package
 import torch  # noqa: E402
 
 import paper_conf_ppopp_mccoyp24_b200 as G  # noqa: E402
