@@ -254,53 +254,6 @@ __device__ inline bool bt_claim_range(const BitTree &t, uint64_t i, uint64_t k) 
     return ok;
 }
 
-// Lowest start i >= from such that [i, i+k) is all set (first fit), by an
-// ascending walk over the leaf words (8 loads in flight at a time); kNone if
-// no such run is visible.  Leaf reads are relaxed: the claim re-validates.
-__device__ inline uint64_t bt_find_lowest_run(const BitTree &t, uint64_t k, uint64_t from) {
-    if (k == 0 || from >= t.nbits || t.nbits - from < k) return kNone;
-    const uint64_t nw = (t.nbits + 63) / 64;
-    uint64_t run = 0, start = 0;
-    uint64_t batch[8];
-    for (uint64_t wi = from >> 6; wi < nw; wi++) {
-        const uint32_t slot = (uint32_t)((wi - (from >> 6)) & 7);
-        if (slot == 0) {
-#pragma unroll
-            for (int q = 0; q < 8; q++) batch[q] = wi + q < nw ? ptx::ld_relaxed(t.w + t.off[0] + wi + q) : 0ull;
-        }
-        uint64_t x = batch[slot];
-        if (wi == (from >> 6)) x &= ~0ull << (from & 63);            // nothing below from
-        const uint64_t base = wi << 6;
-        if (x == ~0ull) {
-            if (!run) start = base;
-            run += 64;
-            if (run >= k) return start;
-            continue;
-        }
-        const uint32_t tr = (uint32_t)__ffsll((long long)~x) - 1;   // ones at the bottom continue the run
-        if (tr) {
-            if (!run) start = base;
-            run += tr;
-            if (run >= k) return start;
-        }
-        run = 0;
-        uint64_t rest = x & (~0ull << tr);                          // bit tr is 0
-        while (rest) {
-            const uint32_t lo = (uint32_t)__ffsll((long long)rest) - 1;
-            const uint64_t sh = rest >> lo;
-            const uint32_t len = (uint32_t)__ffsll((long long)~sh) - 1;
-            if (len >= k) return base + lo;
-            if (lo + len == 64) {                                      // continues into the next word
-                run = len;
-                start = base + lo;
-                break;
-            }
-            rest &= ~bit_range(lo, lo + len);
-        }
-    }
-    return kNone;
-}
-
 // Highest start i such that [i, i+k) is all set (first fit from the back,
 // P:138 / reading A-17), by a top-down walk over the leaf words; kNone if no
 // such run is visible.  Leaf reads are relaxed: the claim re-validates.

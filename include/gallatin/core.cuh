@@ -465,7 +465,7 @@ __device__ inline __noinline__ uint32_t take_segments(const View &v, uint32_t t,
 #ifdef GALLATIN_TRACE
     const uint64_t tr0 = ptx::globaltimer();
 #endif
-    uint64_t s0 = claim_front_run(v, kmax, &k);
+    const uint64_t s0 = claim_front_run(v, kmax, &k);
     if (s0 == kNone) return 0;
 #ifdef GALLATIN_TRACE
     const uint32_t attempts = k >> 16;
@@ -498,20 +498,6 @@ __device__ inline __noinline__ uint32_t take_segments(const View &v, uint32_t t,
         if (extra) oom_notify(v);
         k += run;
         if (lo + run < hi) break;                         // the free run ended here
-    }
-    // [dev] a run from the lowest free segment shorter than half of what was
-    // asked (a fragmented heap: the warm state, where the slots' undrawn run
-    // remainders pin segments) is traded for the lowest window of kmax free
-    // segments, if there is one -- the short run goes back (O2-R R2; serially
-    // exact)
-    if (2 * k < kmax) {
-        const uint64_t w = bt_find_lowest_run(st, kmax, s0 + k);
-        if (w != kNone && bt_claim_range(st, w, kmax)) {
-            bt_insert_range(st, s0, k);
-            oom_notify(v);
-            s0 = w;
-            k = kmax;
-        }
     }
     // tree ids (table words and the read-mostly copies) for the free path;
     // both are read only through a pointer this run hands out, so one fence

@@ -19,9 +19,7 @@
  *      in ascending order) or from one fresh segment whose other blocks are
  *      published; a run of >= nb blocks takes whole free segments privately
  *      (the lowest free one and the free ones right after it, no ring, no
- *      block tree; if that run is under half of want / nb segments, the
- *      lowest window of want / nb free segments instead, when there is one)
- *      -- also when the block tree has a segment but with fewer
+ *      block tree) -- also when the block tree has a segment but with fewer
  *      than m blocks available, as long as a segment is free (a partly
  *      returned segment would give a short run: the warm-state refills);
  *   R3 format-ahead: the reservation that takes a segment below nb/4
@@ -90,25 +88,13 @@ static void format_keep(o2_t *a, uint64_t s, uint32_t t, uint32_t keep) {
 
 /* R2: up to want / nb consecutive free segments from the front, privately */
 static uint32_t take_segments(o2_t *a, uint32_t t, uint32_t want, uint32_t *first) {
-    uint32_t nb = nb_of(t), kmax = want / nb;
+    uint32_t nb = nb_of(t);
     uint64_t s0 = claim_front(a);
     if (s0 == NONE64) return 0;
     uint32_t k = 1;
-    while (k < kmax && s0 + k < a->nseg && oracle_veb_member(a->segfree, s0 + k)) {
+    while (k < want / nb && s0 + k < a->nseg && oracle_veb_member(a->segfree, s0 + k)) {
         oracle_veb_delete(a->segfree, s0 + k);
         k++;
-    }
-    if (2 * k < kmax) {                 /* under half of what was asked: the lowest window of kmax free segments */
-        for (uint64_t w = s0 + k; w + kmax <= a->nseg; w++) {
-            uint32_t q = 0;
-            while (q < kmax && oracle_veb_member(a->segfree, w + q)) q++;
-            if (q < kmax) { w += q; continue; }
-            for (uint32_t j = 0; j < k; j++) oracle_veb_insert(a->segfree, s0 + j);   /* the short run back */
-            for (uint32_t j = 0; j < kmax; j++) oracle_veb_delete(a->segfree, w + j);
-            s0 = w;
-            k = kmax;
-            break;
-        }
     }
     for (uint32_t q = 0; q < k; q++) format_keep(a, s0 + q, t, nb);
     *first = (uint32_t)(s0 * nb);

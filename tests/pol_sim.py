@@ -167,19 +167,10 @@ class PolSim:
             s0 = self.claim_front()
             if s0 is None:
                 return 0, 0
-            k, kmax = 1, want // nb(t)
-            while k < kmax and s0 + k < self.nseg and self.tree[s0 + k] == FREE:
+            k = 1
+            while k < want // nb(t) and s0 + k < self.nseg and self.tree[s0 + k] == FREE:
                 self.tree[s0 + k] = "claimed"
                 k += 1
-            if 2 * k < kmax:                                      # R2: the lowest window of kmax free ones
-                w = next((w for w in range(s0 + k, self.nseg - kmax + 1)
-                          if all(self.tree[w + q] == FREE for q in range(kmax))), None)
-                if w is not None:
-                    for q in range(k):
-                        self.tree[s0 + q] = FREE
-                    for q in range(kmax):
-                        self.tree[w + q] = "claimed"
-                    s0, k = w, kmax
             for q in range(k):
                 self.tree[s0 + q] = t
                 self.ring[s0 + q] = deque()

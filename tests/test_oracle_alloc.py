@@ -397,30 +397,6 @@ def test_whole_segment_runs_prefer_fresh_segments():
     assert a.check() == 0
 
 
-def test_whole_segment_runs_take_the_lowest_full_window():
-    """R2 on a fragmented heap: a run of >= nb blocks whose run from the
-    lowest free segment is under half of want / nb segments takes the lowest
-    window of want / nb free segments instead (the short run goes back).  One
-    4 KB slot (a block = a segment), runs of 1, 2, 4, 8 blocks: segment 0,
-    segments 1-2, segments 3-6; segment 1's 4096 slices are then freed (it
-    retires: the lowest free segment is 1, followed by the used segment 2);
-    the 8-block run then starts at segment 7 (the lowest window of 8 free
-    segments: 7-14), not at segment 1; segment 1 stays free."""
-    a = runs(16, slot_base=1, slot_min=1, run_max=8, run_bytes=128 << 20, run_init=1, run_grow=1)
-    offs = a.malloc_batch(np.full(7 * 4096, 4096, dtype=np.uint64), keydiv=0)
-    assert np.array_equal(offs, np.arange(7 * 4096, dtype=np.uint64) * np.uint64(4096))   # segments 0..6 in order
-    a.free_batch(offs[4096:2 * 4096])                                 # segment 1 comes home
-    d = image_sections(a.image())
-    assert int(d["segtree"][0]) & 0xFFFF == 0b1111111110000010        # free: 1 and 7..15
-    nxt = a.malloc(4096, 0)                                           # run 4 exhausted: refill wants 8
-    assert nxt == 7 * SEG
-    d = image_sections(a.image())
-    assert int(d["segtree"][0]) & 0xFFFF == 0b1000000000000010       # 1 and 15 free; 7..14 the new run
-    w = int(d["slots"][8])
-    assert (w >> 22) & 0x3FF == 8 and w & 0x3FFFFF == 7              # run of 8 from linear block 7
-    assert a.check() == 0
-
-
 def test_prefill_layout_closed_form():
     """R7 ("always populated"): with run_init 64 every class's slots
     start with runs of min(max(64 >> c, 8), nb(c)) blocks = 64, 32, 16, 8, 8,
